@@ -33,7 +33,7 @@ $(CU_OBJ): $(CU_SRC) $(HDRS)
 	$(NVCC) $(NVFLAGS) -Xptxas -v -c $< -o $@ 2> build/ptxas.log || (cat build/ptxas.log; false)
 
 $(PKG)/libdgcl.so: $(HOST_OBJ) $(CU_OBJ)
-	$(NVCC) $(GENCODE) -shared -Xcompiler -fPIC $^ -o $@ -L$(CUDA)/lib64 -lcudart -lcuda
+	$(NVCC) $(GENCODE) -shared -Xcompiler -fPIC -cudart static $^ -o $@
 
 clean:
 	rm -rf build synth/_synth.so $(PKG)/libdgcl.so

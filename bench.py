@@ -1,0 +1,582 @@
+#!/usr/bin/env python3
+"""Benchmark of the DGCL halo-exchange hot path on B200 (BASELINE.json metric).
+
+metric: per-layer embedding-exchange ms and NVLink GB/s/GPU at 1/2/4/8 B200 vs 900 GB/s
+A STEP is one GCN training step's communication on the configured graph: graphAllgather forward
+of every layer, then the backward of the layers that need gradients (for the Reddit-shaped config:
+forward dim 602 and dim 256, backward dim 256).  value = halo payload delivered by the whole job
+per second (sum over layers of sum_d |R_d| x dim x 4 bytes, forward and backward) in GB/s;
+per-layer ms and per-GPU GB/s are reported beside it.
+
+N = 1: the 1-GPU loopback configuration (all 8 virtual ranks of the 8-way partition on one
+B200, fused executor launch; bound by HBM).  N > 1 (torchrun, one process per GPU): the real
+multi-GPU path over NVLink peer memory (bound by NVLink).  --impl reference times the CPU oracle
+(the reference arm of this tier) on a bounded sample.
+
+Timing: W warm-up steps, then K steps between device barriers with CUDA events on the launching
+stream; max over ranks.  Every input (embeddings 563 MB, halos 3.8 GB for Reddit dim 602) is far
+larger than the 126 MB L2, so no explicit flush is needed (config.l2 says so).
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "per-layer embedding-exchange ms and NVLink GB/s/GPU at 1/2/4/8 B200 vs 900 GB/s"
+UNIT = "GB/s"
+NVLINK_PEER_GBS = 770.0  # measured peer copy per direction (B200_PROFILING.md); 900 nominal
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ---------------------------------------------------------------------------------------------
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms while running."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index):
+        self.dev = device_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.dev), "--query-gpu=" + self.Q,
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append((time.time(), line.strip()))
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self, t0=None, t1=None):
+        sms, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for (t, line) in self.lines:
+            if t0 is not None and (t < t0 - 0.25 or t > t1 + 0.25):
+                continue
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sms.append(float(f[1]))
+                mx.append(float(f[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sms:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sms), "sm_max_mhz": max(mx),
+                "reasons": sorted(reasons), "samples": len(sms)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f), "measured"
+    return {"hbm_gbs": 6650.0}, "fallback"
+
+
+def profiled_traffic(key):
+    """dram bytes per launch from the committed ncu --set full summary (profiles/traffic.json)."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f).get(key)
+    return None
+
+
+# ---------------------------------------------------------------------------------------------
+class Workload:
+    """Synthetic inputs of one BASELINE.json config (seeded; shared with the oracle)."""
+
+    def __init__(self, cfg_name):
+        import synth
+        self.cfg = synth.get_config(cfg_name)
+        c = self.cfg
+        t = time.time()
+        self.g = synth.make_graph(c.n, c.e, c.m, c.graph_seed, c.part_seed, keep_edges=False)
+        self.gen_s = time.time() - t
+        self.S = int(self.g.req_ptr[-1])
+        self.order = np.argsort(self.g.part, kind="stable")
+        self.fwd_layers = list(range(len(c.dims)))
+        self.bwd_layers = list(c.backward_layers)
+
+    def step_payload_bytes(self, ranks=None):
+        """Halo payload one step delivers (forward) and returns (backward), algorithmic bytes."""
+        ptr = self.g.req_ptr
+        S = self.S if ranks is None else sum(int(ptr[d + 1] - ptr[d]) for d in ranks)
+        dims = self.cfg.dims
+        return S * 4 * (sum(dims[l] for l in self.fwd_layers) +
+                        sum(dims[l] for l in self.bwd_layers))
+
+
+def host_inputs(w, pitches, rows_order=None):
+    """Hash-defined host arrays in the loopback layouts (see synth/values.py)."""
+    import synth
+    c = w.cfg
+    emb, hg, eg = {}, {}, {}
+    for l in w.fwd_layers:
+        emb[l] = synth.fill_values(c.n, c.dims[l], pitches[l], keys=w.order, seed=c.emb_seed,
+                                   stream=synth.values.STREAM_EMB + l)
+    for l in w.bwd_layers:
+        hg[l] = synth.fill_values(w.S, c.dims[l], pitches[l], seed=c.grad_seed,
+                                  stream=synth.values.STREAM_HGRAD + l)
+        eg[l] = synth.fill_values(c.n, c.dims[l], pitches[l], keys=w.order, seed=c.grad_seed,
+                                  stream=synth.values.STREAM_EGRAD + l)
+    return emb, hg, eg
+
+
+# ---------------------------------------------------------------------------------------------
+def oracle_sample(w, emb, hg, eg, budget_s=15.0, ranks=None):
+    """Time the CPU oracle (as it stands) on destination/owner ranks until the budget is spent.
+    Returns (GB/s, seconds, ranks used, threads)."""
+    from oracle import halo
+    c = w.cfg
+    g = w.g
+    m = c.m
+    loc, n_local = halo.local_rows(g.part, m)
+    ro = np.concatenate([[0], np.cumsum(n_local)])
+    R = [g.R(d) for d in range(m)]
+    done_bytes, t_total, used = 0, 0.0, []
+    for d in (ranks if ranks is not None else range(m)):
+        t = time.perf_counter()
+        for l in w.fwd_layers:
+            dim = c.dims[l]
+            local = [emb[l][ro[s]:ro[s + 1], :dim] for s in range(m)]
+            Rd = [R[q] if q == d else np.zeros(0, np.int64) for q in range(m)]
+            halo.forward(local, Rd, g.part, loc)
+        for l in w.bwd_layers:
+            dim = c.dims[l]
+            L = [eg[l][ro[s]:ro[s + 1], :dim] if s == d else np.zeros((n_local[s], dim), np.float32)
+                 for s in range(m)]
+            ptr = g.req_ptr
+            G = [hg[l][ptr[q]:ptr[q + 1], :dim] for q in range(m)]
+            # owner d's rows: every contributor's rows for vertices owned by d
+            Rd = [R[q][g.part[R[q]] == d] for q in range(m)]
+            Gd = [G[q][g.part[R[q]] == d] for q in range(m)]
+            halo.backward_flat(L, Gd, Rd, g.part, loc)
+        t_total += time.perf_counter() - t
+        used.append(d)
+        ptr = g.req_ptr
+        fwd_b = int(ptr[d + 1] - ptr[d]) * 4 * sum(c.dims[l] for l in w.fwd_layers)
+        owned_in = sum(int(np.count_nonzero(g.part[R[q]] == d)) for q in range(m))
+        bwd_b = owned_in * 4 * sum(c.dims[l] for l in w.bwd_layers)
+        done_bytes += fwd_b + bwd_b
+        if t_total >= budget_s:
+            break
+    return done_bytes / t_total / 1e9, t_total, used, 1
+
+
+# ---------------------------------------------------------------------------------------------
+def run_ours_single(args, w):
+    import torch
+    import paper_conf_eurosys_cai0wmcy21_b200 as D
+    torch.cuda.set_device(0)
+    c = w.cfg
+    g = w.g
+    topo = None
+    if c.topology != "uniform_nvswitch":
+        import synth
+        topo = synth.topology.by_name(c.topology, c.m)
+    ctx = D.loopback(c.m, g.part, list(c.dims), device=0)
+    if args.item_bytes:
+        ctx.set_option("item_bytes", args.item_bytes)
+    t = time.time()
+    ctx.build_plan(g.req_ptr, g.req_ids, seed=0, topology=topo)
+    plan_s = time.time() - t
+    ctx.register_workspace()
+    info = ctx.plan_info()
+    pitches = {l: ctx.pitch(l) for l in range(len(c.dims))}
+    emb_h, hg_h, eg_h = host_inputs(w, pitches)
+    emb = {l: torch.from_numpy(a).cuda() for l, a in emb_h.items()}
+    hg = {l: torch.from_numpy(a).cuda() for l, a in hg_h.items()}
+    eg = {l: torch.from_numpy(a).cuda() for l, a in eg_h.items()}
+    stream = torch.cuda.current_stream()
+    names = ["fwd%d_d%d" % (l, c.dims[l]) for l in w.fwd_layers] + \
+            ["bwd%d_d%d" % (l, c.dims[l]) for l in w.bwd_layers]
+
+    def step(evs=None):
+        i = 0
+        for l in w.fwd_layers:
+            if evs is not None:
+                evs[i][0].record(stream)
+            ctx.forward(l, emb[l], stream=stream)
+            if evs is not None:
+                evs[i][1].record(stream)
+            i += 1
+        for l in w.bwd_layers:
+            if evs is not None:
+                evs[i][0].record(stream)
+            ctx.backward(l, hg[l], eg[l], stream=stream)
+            if evs is not None:
+                evs[i][1].record(stream)
+            i += 1
+
+    clk = ClockSampler(torch.cuda.current_device())
+    clk.start()
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    # keep the GPU under load for >= 1 s before timing (clock sampling, steady state)
+    t_soak = time.time()
+    while time.time() - t_soak < 1.0:
+        step()
+        torch.cuda.synchronize()
+    ctx.check()
+    K = args.steps
+    evs = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)]
+            for _ in names] for _ in range(K)]
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    launches0 = ctx.launch_count()
+    torch.cuda.synchronize()
+    tw0 = time.time()
+    e0.record(stream)
+    for k in range(K):
+        step(evs[k])
+    e1.record(stream)
+    torch.cuda.synchronize()
+    tw1 = time.time()
+    launches = ctx.launch_count() - launches0
+    ctx.check()
+    total_ms = e0.elapsed_time(e1)
+    ms_step = total_ms / K
+    per_op = {n: statistics.mean(evs[k][i][0].elapsed_time(evs[k][i][1]) for k in range(K))
+              for i, n in enumerate(names)}
+    clocks = clk.summary(tw0, tw1)
+    if clocks["samples"] == 0:
+        clocks = clk.summary()
+
+    # ---- e2e through the host-buffer C-ABI calls (pinned host memory) ----
+    e2e = None
+    if args.e2e_steps > 0:
+        pin = lambda a: torch.from_numpy(a).pin_memory()
+        emb_p = {l: pin(a) for l, a in emb_h.items()}
+        hg_p = {l: pin(a) for l, a in hg_h.items()}
+        eg_p = {l: pin(a) for l, a in eg_h.items()}
+        halo_p = {l: torch.empty(w.S, pitches[l], dtype=torch.float32).pin_memory()
+                  for l in w.fwd_layers}
+        h2d = sum(a.numel() * 4 for a in emb_p.values()) + \
+            sum(a.numel() * 4 for a in hg_p.values()) + sum(a.numel() * 4 for a in eg_p.values())
+        d2h = sum(a.numel() * 4 for a in halo_p.values()) + sum(a.numel() * 4 for a in eg_p.values())
+
+        def e2e_step():
+            for l in w.fwd_layers:
+                ctx.forward_host(l, emb_p[l], halo_p[l], stream=stream)
+            for l in w.bwd_layers:
+                ctx.backward_host(l, hg_p[l], eg_p[l], stream=stream)
+
+        e2e_step()
+        torch.cuda.synchronize()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        a1.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms = a0.elapsed_time(a1) / args.e2e_steps
+        e2e = {"value": w.step_payload_bytes() / (e2e_ms * 1e-3) / 1e9, "unit": UNIT,
+               "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h)}
+    clk.stop()
+
+    # ---- roofline of the dominant kernel: the forward executor launch of layer 0 ----
+    peaks, src = measured_peaks()
+    l0 = w.fwd_layers[0]
+    dom = names[0]
+    alg_bytes = 2 * w.S * c.dims[l0] * 4      # gather-read + halo-write, both in this HBM
+    achieved = alg_bytes / (per_op[dom] * 1e-3) / 1e9
+    traffic = profiled_traffic("%s/%s" % (c.name, dom))
+    roofline = {"bound": "hbm", "kernel": "executor_kernel<true> (%s)" % dom,
+                "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
+                "algorithmic_bytes_per_launch": alg_bytes, "peak_source": src}
+
+    value = w.step_payload_bytes() / (ms_step * 1e-3) / 1e9
+    cpu = None
+    if not args.no_cpu_baseline:
+        gbs, secs, used, thr = oracle_sample(w, emb_h, hg_h, eg_h, budget_s=args.cpu_budget)
+        cpu = {"value": gbs, "unit": UNIT, "cores": thr, "kind": "oracle",
+               "sample": "oracle forward (all layers) + flat backward for destination/owner "
+                         "ranks %s of %d (%.1f s of CPU work)" % (used, c.m, secs)}
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": K,
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "impl": "ours",
+        "config": {"workload": "%s-shaped R-MAT, %d-way partition, 1-GPU loopback (all %d "
+                               "virtual ranks on one B200)" % (c.name, c.m, c.m),
+                   "config": c.name, "n_vertices": c.n, "n_edges": c.e, "world": c.m,
+                   "dims": list(c.dims), "fwd_layers": w.fwd_layers, "bwd_layers": w.bwd_layers,
+                   "halo_rows_total": w.S, "halo_rows_per_rank": np.diff(g.req_ptr).tolist(),
+                   "topology": c.topology, "parallelism": "loopback%d" % c.m,
+                   "l2": "inputs larger than L2 (no flush needed)"},
+        "ms_per_layer": per_op,
+        "gbs_per_gpu": value,
+        "roofline": roofline,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": int(launches),
+        "clocks": clocks,
+        "plan": dict(info, planner_wall_s=plan_s, graph_gen_s=w.gen_s),
+    }
+    ctx.destroy()
+    return out
+
+
+def run_ours_multi(args, w, rank, world, local_rank):
+    """One process per GPU; the exchange runs over NVLink peer memory (CUDA IPC)."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_eurosys_cai0wmcy21_b200 as D
+    c = w.cfg
+    g = w.g
+    dev = 0 if args.share_gpu else local_rank
+    torch.cuda.set_device(dev)
+    topo = None
+    if c.topology != "uniform_nvswitch":
+        import synth
+        topo = synth.topology.by_name(c.topology, world)
+    # the partition of this run: the config's graph partitioned over `world` GPUs
+    import synth
+    part = synth.partition(c.n, world, c.part_seed)
+    # required lists for this world size (rank 0 computes, all ranks receive)
+    src_dst = None
+    ctx = D.init(part, list(c.dims), rank, world, dev)
+    lists = w.lists
+    ptr = np.zeros(world + 1, np.int64)
+    ptr[1:] = np.cumsum([len(x) for x in lists])
+    ids = np.concatenate(lists)
+    ctx.build_plan(ptr, ids, seed=0, topology=topo)
+    ctx.register_workspace()
+    blobs = [None] * world
+    dist.all_gather_object(blobs, ctx.ipc_export())
+    ctx.ipc_import(blobs)
+    dist.barrier()
+    info = ctx.plan_info()
+    order = np.nonzero(part == rank)[0]
+    n_local = order.shape[0]
+    my_R = lists[rank]
+    emb, hg, eg = {}, {}, {}
+    for l in w.fwd_layers:
+        p = ctx.pitch(l)
+        emb[l] = torch.from_numpy(synth.fill_values(n_local, c.dims[l], p, keys=order,
+                                                    seed=c.emb_seed,
+                                                    stream=synth.values.STREAM_EMB + l)).cuda()
+    for l in w.bwd_layers:
+        p = ctx.pitch(l)
+        hg[l] = torch.from_numpy(synth.fill_values(len(my_R), c.dims[l], p, seed=c.grad_seed,
+                                                   stream=synth.values.STREAM_HGRAD + l)).cuda()
+        eg[l] = torch.from_numpy(synth.fill_values(n_local, c.dims[l], p, keys=order,
+                                                   seed=c.grad_seed,
+                                                   stream=synth.values.STREAM_EGRAD + l)).cuda()
+    stream = torch.cuda.current_stream()
+    names = ["fwd%d_d%d" % (l, c.dims[l]) for l in w.fwd_layers] + \
+            ["bwd%d_d%d" % (l, c.dims[l]) for l in w.bwd_layers]
+
+    def step(evs=None):
+        i = 0
+        for l in w.fwd_layers:
+            if evs is not None:
+                evs[i][0].record(stream)
+            ctx.forward(l, emb[l], stream=stream)
+            if evs is not None:
+                evs[i][1].record(stream)
+            i += 1
+        for l in w.bwd_layers:
+            if evs is not None:
+                evs[i][0].record(stream)
+            ctx.backward(l, hg[l], eg[l], stream=stream)
+            if evs is not None:
+                evs[i][1].record(stream)
+            i += 1
+
+    clk = ClockSampler(dev) if rank == 0 else None
+    if clk:
+        clk.start()
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    ctx.check()
+    K = args.steps
+    evs = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)]
+            for _ in names] for _ in range(K)]
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    l0 = ctx.launch_count()
+    dist.barrier()
+    torch.cuda.synchronize()
+    tw0 = time.time()
+    e0.record(stream)
+    for k in range(K):
+        step(evs[k])
+    e1.record(stream)
+    torch.cuda.synchronize()
+    dist.barrier()
+    tw1 = time.time()
+    ctx.check()
+    launches = ctx.launch_count() - l0
+    t = torch.tensor([e0.elapsed_time(e1)] + [statistics.mean(
+        evs[k][i][0].elapsed_time(evs[k][i][1]) for k in range(K)) for i in range(len(names))],
+        dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    lt = torch.tensor([float(launches)], dtype=torch.float64)
+    dist.all_reduce(lt)
+    if clk:
+        clk.stop()
+    if rank != 0:
+        ctx.destroy()
+        return None
+    ms_step = float(t[0]) / K
+    per_op = {n: float(t[1 + i]) for i, n in enumerate(names)}
+    payload = w.S * 4 * (sum(c.dims[l] for l in w.fwd_layers) + sum(c.dims[l] for l in w.bwd_layers))
+    value = payload / (ms_step * 1e-3) / 1e9
+    counts = ctx.plan_counts()
+    out_rows = counts.sum(axis=(0, 2))
+    in_rows = counts.sum(axis=(0, 1))
+    dom = names[0]
+    maxport = int(max(out_rows.max(), in_rows.max()))
+    alg = maxport * c.dims[w.fwd_layers[0]] * 4
+    achieved = alg / (per_op[dom] * 1e-3) / 1e9
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K,
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "impl": "ours",
+        "config": {"workload": "%s-shaped R-MAT, %d-way partition over %d B200 (NVLink 5)" %
+                               (c.name, world, world), "config": c.name, "dims": list(c.dims),
+                   "world": world, "parallelism": "graph-partition x%d" % world,
+                   "l2": "inputs larger than L2 (no flush needed)"},
+        "ms_per_layer": per_op,
+        "gbs_per_gpu": value / world,
+        "roofline": {"bound": "nvlink", "kernel": "executor_kernel (%s)" % dom,
+                     "achieved": achieved, "peak": NVLINK_PEER_GBS, "unit": "GB/s",
+                     "frac": achieved / NVLINK_PEER_GBS, "traffic": None,
+                     "nominal_peak": 900.0,
+                     "algorithmic_bytes_per_launch": alg},
+        "cpu_baseline": None, "e2e": None, "gpu_launches": int(lt[0]),
+        "clocks": clk.summary(tw0, tw1) if clk else None,
+        "plan": info,
+    }
+    ctx.destroy()
+    return out
+
+
+def run_reference(args, w):
+    """The reference arm of this tier: the CPU oracle as it stands, timed per step on a bounded
+    sample of the same workload (one destination/owner rank per step)."""
+    import synth
+    c = w.cfg
+    pitches = {l: synth.configs.pitch_of(c.dims[l]) for l in range(len(c.dims))}
+    emb_h, hg_h, eg_h = host_inputs(w, pitches)
+    for k in range(args.warmup):
+        oracle_sample(w, emb_h, hg_h, eg_h, budget_s=0.0, ranks=[k % c.m])
+    vals, secs = [], []
+    for k in range(args.steps):
+        gbs, s, used, thr = oracle_sample(w, emb_h, hg_h, eg_h, budget_s=0.0, ranks=[k % c.m])
+        vals.append(gbs)
+        secs.append(s)
+    value = sum(vals) / len(vals)
+    ms = 1e3 * sum(secs) / len(secs)
+    return {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "impl": "reference",
+            "config": {"workload": "%s-shaped R-MAT, %d-way partition; CPU oracle, one rank's "
+                                   "halo + owner rows per step" % (c.name, c.m), "config": c.name},
+            "cpu_baseline": {"value": value, "unit": UNIT, "kind": "oracle", "cores": 1,
+                             "sample": "one destination/owner rank of %d per step" % c.m},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="reddit")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=12.0)
+    ap.add_argument("--item-bytes", type=int, default=0)
+    ap.add_argument("--share-gpu", action="store_true", help=argparse.SUPPRESS)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    subprocess.check_call(["make", "-s", "-C", ROOT, "all"]) if rank == 0 and world == 1 else None
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        w = Workload(args.config)
+        print(json.dumps(run_reference(args, w)), flush=True)
+        return
+
+    if world == 1:
+        w = Workload(args.config)
+        out = run_ours_single(args, w)
+        print(json.dumps(out), flush=True)
+        return
+
+    import torch.distributed as dist
+    dist.init_process_group("gloo" if args.share_gpu else "nccl")
+    import synth
+    cfg = synth.get_config(args.config)
+    # rank 0 builds the graph and the required lists for this world size; broadcast to all
+    objs = [None]
+    if rank == 0:
+        w = Workload(args.config)
+        src, dst = synth.rmat_edges(cfg.n, cfg.e, cfg.graph_seed)
+        part = synth.partition(cfg.n, world, cfg.part_seed)
+        ptr, ids = synth.required_lists(src, dst, part, world)
+        w.lists = [ids[ptr[d]:ptr[d + 1]] for d in range(world)]
+        w.S = int(ptr[-1])
+        w.g = None
+        objs = [w]
+    if dist.get_backend() == "nccl":
+        import torch
+        torch.cuda.set_device(local_rank)
+    dist.broadcast_object_list(objs, src=0)
+    w = objs[0]
+    w.g = type("G", (), {})()
+    out = run_ours_multi(args, w, rank, world, local_rank)
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,227 @@
+/* dgcl.h — C ABI of the B200-native DGCL halo-exchange library (libdgcl.so).
+ *
+ * What it computes (PAPER.md = /root/reference/PAPER.md, "P:n" = line n):
+ *   DGCL's data-parallel hot path: executing a communication plan for GNN embedding passing.
+ *   - graphAllgather forward (§4.2): after the call every GPU d holds, in its halo, the
+ *     embedding row of every remote vertex it requires (V^r_d of §4.1).
+ *   - its backward (§2; §6.1; §6.2): gradients of the halo rows
+ *     flow back along the reversed plan and are summed into the owner rows in a fixed order, with
+ *     no atomics.
+ *   - the plan is built once by SPST (Algorithm 1 + 2, §5.2) over a link-cost model of
+ *     the topology (§5.1) and reused by every layer.
+ *
+ * Conventions (every function):
+ *   - returns dgcl_status; no exception crosses the ABI; dgcl_last_error(ctx) explains failures;
+ *   - one context per rank, used by one host thread;
+ *   - host pointers are read during the call only and never retained unless stated;
+ *   - device pointers are caller-owned unless stated; the library never frees caller memory;
+ *   - `stream` arguments are cudaStream_t passed as void* (0 = legacy default stream);
+ *   - embeddings are fp32 rows; pitches are in ELEMENTS (floats); dims[l] >= 1.
+ *
+ * Row layouts:
+ *   local rows   loc[v] = number of w < v with part[w] == part[v]  (ascending global id, §4.1)
+ *   halo rows    halo_d[i] = embedding of R_d[i], R_d in the order the caller gave to
+ *                dgcl_build_plan (the paper leaves the re-indexed order open)
+ *   LOOPBACK contexts (all `world` virtual ranks on one GPU; test/bench, §8(d) "1-GPU loopback"):
+ *                emb / emb_grad are [N x pitch] partition-major: rank r's local rows start at row
+ *                sum_{q<r} n_local[q];  halo / halo_grad are [sum_d |R_d| x pitch], rank d's block
+ *                starts at row sum_{q<d} |R_q|.
+ */
+#ifndef DGCL_H_
+#define DGCL_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  DGCL_OK = 0,
+  DGCL_EINVAL = 1,   /* bad argument (range, duplicate, alignment, pitch < dim, ...) */
+  DGCL_ESTATE = 2,   /* call out of order (e.g. dispatch before build_plan/register) */
+  DGCL_ECUDA = 3,    /* a CUDA runtime/driver call failed (or no usable GPU) */
+  DGCL_ENOMEM = 4,   /* host or device allocation failed / workspace too small */
+  DGCL_ETIMEOUT = 5, /* a device-side flag wait exceeded the watchdog (a peer never arrived) */
+  DGCL_EPLAN = 6     /* planning failed: some requesting GPU is unreachable in the topology */
+} dgcl_status;
+
+typedef struct dgcl_ctx dgcl_ctx;
+
+/* Loopback flags (dgcl_init_loopback). */
+#define DGCL_LOOPBACK_FUSED 0    /* one executor launch runs every virtual rank's program */
+#define DGCL_LOOPBACK_PER_RANK 1 /* one launch per virtual rank on its own stream, with the full
+                                    ready/done flag protocol of the multi-GPU path (test mode) */
+
+/* Topology D(V', E') of §5.1: ordered GPU pairs (i, j) map to lists of
+ * physical hops; hop h costs hop_ticks[h] (> 0) per embedding row.  A pair with an empty hop list
+ * has no link.  link_ptr is CSR over pair index i*world + j (size world*world + 1). */
+typedef struct {
+  int32_t n_hops;
+  const int64_t *hop_ticks; /* [n_hops] */
+  const int64_t *link_ptr;  /* [world*world + 1] */
+  const int32_t *link_hops; /* [link_ptr[world*world]] hop ids */
+} dgcl_topology;
+
+typedef struct {
+  int32_t world;
+  int32_t n_stages;            /* forward stages K (<= world-1) */
+  int64_t n_vertices_planned;  /* |{u : D_u non-empty}| */
+  int64_t n_deliveries;        /* sum_d |R_d| */
+  int64_t n_tree_edges;        /* sum_u |T_u| edges (>= n_deliveries; excess = relay hops) */
+  int64_t n_relay_rows;        /* tree edges into GPUs that did not request the vertex */
+  int64_t model_cost_ticks;    /* t(S) of §5.1 in ticks */
+  int64_t table_bytes;         /* device bytes of send/receive index tables (Fig. 11) */
+  double planner_seconds;      /* SPST wall time, one host thread (Table 8) */
+  double lowering_seconds;
+  int32_t n_fwd_groups;        /* (stage, src, dst, buffer-kind) tuples */
+  int32_t n_bwd_groups;
+} dgcl_plan_stats;
+
+/* ---- lifecycle ---------------------------------------------------------------------------- */
+
+/* One rank of a `world`-GPU job (§6.3 one process per GPU).
+ * part: host [n_vertices], part[v] in [0, world), copied.  dims: host [n_layers], fp32 elements per
+ * row of each layer; one plan serves every layer.  cuda_device < 0 makes a host-only
+ * planning context (every device call then returns DGCL_ESTATE).  Builds loc / n_local (§4.1).
+ * Errors: EINVAL (rank >= world, world < 1 or > 16, n_layers < 1, dims[l] < 1, part out of range),
+ * ECUDA (cudaSetDevice failed). */
+dgcl_status dgcl_init(int32_t rank, int32_t world, int32_t cuda_device, int64_t n_vertices,
+                      const int32_t *part, int32_t n_layers, const int32_t *dims, dgcl_ctx **out);
+
+/* All `world` virtual ranks in one context on one GPU (the 1-GPU loopback configuration).
+ * flags: DGCL_LOOPBACK_FUSED or DGCL_LOOPBACK_PER_RANK.  Same errors as dgcl_init. */
+dgcl_status dgcl_init_loopback(int32_t world, int32_t cuda_device, int64_t n_vertices,
+                               const int32_t *part, int32_t n_layers, const int32_t *dims,
+                               int32_t flags, dgcl_ctx **out);
+
+/* Optional, before dgcl_build_plan; default = uniform NVSwitch (link i->j = {egress_i, ingress_j},
+ * 900 GB/s each, 111 ticks per row).  Copied.  EINVAL for bad hop ids / ticks, ESTATE after plan. */
+dgcl_status dgcl_set_topology(dgcl_ctx *ctx, const dgcl_topology *topo);
+
+/* Build the communication plan (buildCommInfo; Algorithm 1).
+ * Collective in the sense that every rank must pass ALL ranks' required lists (the Python wrapper
+ * all-gathers them) and the same seed, so every rank computes the identical plan without a master.
+ * req_ptr: host [world+1]; req_ids: host [req_ptr[world]]; R_d = req_ids[req_ptr[d]:req_ptr[d+1]]
+ * in GPU d's halo row order.  Host work only (no device memory is touched).
+ * Errors: EINVAL (id out of range, id owned by the requester, duplicate id in one list),
+ * EPLAN (unreachable GPU), ESTATE (called twice), ENOMEM. */
+dgcl_status dgcl_build_plan(dgcl_ctx *ctx, const int64_t *req_ptr, const int64_t *req_ids,
+                            uint64_t seed);
+
+/* Device workspace.  The caller allocates ONE device buffer of at least *bytes bytes, 256-B
+ * aligned (PyTorch does), keeps it alive until dgcl_destroy, and registers it.  The library carves
+ * out halos (one per layer), relay staging, backward gradient slots and flag words, zeroes the flag
+ * words (synchronously) and uploads the plan tables (library-owned device memory).
+ * Errors: ESTATE (no plan / host-only ctx), EINVAL (misaligned), ENOMEM (too small), ECUDA. */
+dgcl_status dgcl_workspace_bytes(dgcl_ctx *ctx, size_t *bytes);
+dgcl_status dgcl_register_workspace(dgcl_ctx *ctx, void *dev, size_t bytes);
+
+/* Where the halo of `layer` lives inside the registered workspace: byte offset, rows (|R_me|, or
+ * sum_d |R_d| for loopback), pitch in elements (dims[layer] rounded up to a multiple of 4). */
+dgcl_status dgcl_halo_view(dgcl_ctx *ctx, int32_t layer, size_t *offset, int64_t *rows,
+                           int64_t *pitch);
+
+/* Per-rank row counts: n_local[world], n_halo[world] (= |R_d|).  Host arrays filled by the call. */
+dgcl_status dgcl_rank_rows(dgcl_ctx *ctx, int64_t *n_local, int64_t *n_halo);
+
+/* Peer mapping over NVLink (CUDA IPC; the B200 form of §6.2 method (1)).
+ * export: writes this rank's opaque blob (IPC handle of the workspace allocation + offset) into
+ * blob (capacity *len on entry; bytes written on return; DGCL_IPC_BLOB_BYTES always suffices).
+ * import: blobs = world blobs of len_each bytes, in rank order (own entry ignored); maps every
+ * peer workspace.  The caller must barrier all ranks after import and before the first dispatch.
+ * Errors: ESTATE (no workspace), EINVAL (bad blob), ECUDA (peer mapping impossible). */
+#define DGCL_IPC_BLOB_BYTES 256
+dgcl_status dgcl_ipc_export(dgcl_ctx *ctx, void *blob, size_t *len);
+dgcl_status dgcl_ipc_import(dgcl_ctx *ctx, const void *blobs, size_t len_each);
+
+/* ---- the hot path ------------------------------------------------------------------------- */
+
+/* graphAllgather forward for `layer` (plan tuples of §6.1).
+ * emb: device [n_local x emb_pitch] (loopback: [N x emb_pitch], partition-major), caller-owned,
+ * local, read-only during the call.  halo: NULL or the registered view for `layer` (EINVAL
+ * otherwise).  Enqueues on `stream`, returns without a host sync; a collective (every rank calls it
+ * with the same layer sequence).  After the stream reaches this point:
+ *   halo[i][0:dim] == emb_global[R_me[i]][0:dim]   bit-exactly.
+ * Errors: EINVAL (layer, pitch < dim), ESTATE (not registered / not imported), ETIMEOUT (an
+ * earlier call's watchdog fired; the context is unusable), ECUDA (launch failed). */
+dgcl_status dgcl_dispatch_forward(dgcl_ctx *ctx, int32_t layer, const float *emb,
+                                  int64_t emb_pitch, float *halo, void *stream);
+
+/* Backward of graphAllgather for `layer`: the adjoint (stages reversed, send/receive tables
+ * swapped), without atomics (§6.2).
+ * halo_grad: device [|R_me| x hg_pitch] (loopback [sum_d |R_d| x hg_pitch]), caller-owned, local.
+ * emb_grad: device in/out [n_local x eg_pitch] (loopback [N x eg_pitch]).  On completion
+ *   emb_grad[loc u] = ((emb_grad_in[loc u] + val(y1)) + val(y2)) + ...
+ * over u's tree children y1 < y2 < ... (ascending GPU id), where a child's val is its own halo
+ * gradient (if it requested u) followed by its own children's vals, ascending (R6).
+ * For single-stage (direct) plans this is  emb_grad_in + G_c1 + G_c2 + ... , c ascending.
+ * Rows of vertices nobody requested are untouched.  Same errors as dispatch_forward. */
+dgcl_status dgcl_dispatch_backward(dgcl_ctx *ctx, int32_t layer, const float *halo_grad,
+                                   int64_t hg_pitch, float *emb_grad, int64_t eg_pitch,
+                                   void *stream);
+
+/* End-to-end variants with HOST buffers (pinned or pageable): copy the input rows host->device
+ * into library-owned staging, dispatch, copy the result device->host, synchronize `stream`.
+ * forward:  host_emb [rows x pitch] -> host_halo [halo rows x pitch] (pitch = the halo view pitch)
+ * backward: host_halo_grad [halo rows x pitch] and host_emb_grad in/out [rows x pitch].
+ * Errors: as the device variants, plus ENOMEM for staging. */
+dgcl_status dgcl_forward_host(dgcl_ctx *ctx, int32_t layer, const float *host_emb,
+                              float *host_halo, void *stream);
+dgcl_status dgcl_backward_host(dgcl_ctx *ctx, int32_t layer, const float *host_halo_grad,
+                               float *host_emb_grad, void *stream);
+
+/* ---- introspection ----------------------------------------------------------------------- */
+
+dgcl_status dgcl_plan_info(dgcl_ctx *ctx, dgcl_plan_stats *info);
+
+/* Forward rows per (stage k in 1..n_stages, src, dst): rows[((k-1)*world + src)*world + dst];
+ * caller provides n_stages*world*world int64.  Relay rows included (bytes = rows*dim*4). */
+dgcl_status dgcl_plan_counts(dgcl_ctx *ctx, int64_t *rows);
+
+/* Tree edges of the plan (§5.1 T_u) as (u, parent, child, stage) in planning order.
+ * Two-call pattern: pass NULL arrays to get *n_edges, then arrays of that size. */
+dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_t *parent,
+                             int32_t *child, int32_t *stage);
+
+/* Options (before dgcl_register_workspace unless noted):
+ *   "timeout_ms"     device watchdog for flag waits (default 20000; any time)
+ *   "item_bytes"     target bytes per work item (default 65536)
+ *   "ctas_per_sm"    executor CTAs per SM (default: occupancy, max 4)
+ *   "threads"        executor CTA size (128..512, multiple of 32; default 512)
+ *   "debug_skip_rank" fault injection for DGCL_LOOPBACK_PER_RANK contexts: never launch that
+ *                    virtual rank's program, so its peers' flag waits hit the watchdog (any time;
+ *                    -1 = off)
+ * EINVAL for an unknown key or bad value. */
+dgcl_status dgcl_set_option(dgcl_ctx *ctx, const char *key, int64_t value);
+
+/* Number of executor kernel launches issued so far by this context. */
+dgcl_status dgcl_launch_count(dgcl_ctx *ctx, uint64_t *count);
+
+/* Device watchdog result: DGCL_ETIMEOUT if a flag wait expired (the context is then unusable),
+ * DGCL_ECUDA on a sticky CUDA error, else DGCL_OK.  Does not synchronize the device. */
+dgcl_status dgcl_check(dgcl_ctx *ctx);
+
+const char *dgcl_last_error(dgcl_ctx *ctx);
+const char *dgcl_strerror(dgcl_status status);
+
+/* Unmaps peers, frees library-owned memory (tables, staging, streams), never the caller's
+ * workspace.  Synchronizes the device first.  NULL is a no-op. */
+dgcl_status dgcl_destroy(dgcl_ctx *ctx);
+
+/* ---- verification aids (not on the dispatch path) --------------------------------------- */
+
+/* Runs the lowered plan tables of a LOOPBACK context with a host interpreter (single thread, same
+ * item order and fp32 fold order as the device executor), for CPU tests of planning + lowering
+ * without a GPU.  Never called by dgcl_dispatch_*; there is no CPU fallback on the product path.
+ * Buffers use the loopback layouts above with pitch = the halo view pitch of `layer`. */
+dgcl_status dgcl_debug_hostsim_forward(dgcl_ctx *ctx, int32_t layer, const float *emb,
+                                       float *halo);
+dgcl_status dgcl_debug_hostsim_backward(dgcl_ctx *ctx, int32_t layer, const float *halo_grad,
+                                        float *emb_grad);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DGCL_H_ */

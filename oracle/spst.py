@@ -42,30 +42,30 @@ class CostState:
 
     def __init__(self, topo):
         self.topo = topo
-        self.w = list(topo.hop_ticks)
-        self.load = [[0] * len(self.w) for _ in range(topo.m)]   # stage 0 unused
+        self.w = np.asarray(topo.hop_ticks, dtype=np.int64)
+        self.load = np.zeros((topo.m, len(self.w)), dtype=np.int64)    # stage 0 unused
+        # t_i^k of a link is the max over its hops, t^k the max over links: i.e. the max over the
+        # hops that belong to some link
+        used = sorted({h for hops in topo.links.values() for h in hops})
+        self.used = np.asarray(used, dtype=np.int64)
 
     def cost_func(self, load=None):
+        """t(S) = sum_{k=1}^{m-1} max_i max_j c_ij^k * w_ij."""
         load = self.load if load is None else load
-        total = 0
-        for k in range(1, self.topo.m):
-            tk = 0
-            for (_i, _j), hops in self.topo.links.items():
-                tk = max(tk, max(load[k][h] * self.w[h] for h in hops))
-            total += tk
-        return total
+        if self.used.size == 0:
+            return 0
+        return int((load[1:, self.used] * self.w[self.used]).max(axis=1).sum())
 
     def incremental(self, k, link):
         """Algorithm 2 line 6: C(k, e) = costFunc(S + {(k, e)}) - costFunc(S)."""
-        hops = self.topo.link(*link)
-        trial = [row[:] for row in self.load]
-        for h in hops:
-            trial[k][h] += 1
+        trial = self.load.copy()
+        for h in self.topo.link(*link):
+            trial[k, h] += 1
         return self.cost_func(trial) - self.cost_func()
 
     def add(self, k, link):
         for h in self.topo.link(*link):
-            self.load[k][h] += 1
+            self.load[k, h] += 1
 
 
 def _dijkstra(topo, state, nsrc_depth):

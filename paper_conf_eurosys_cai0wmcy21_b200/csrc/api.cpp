@@ -1,0 +1,855 @@
+// api.cpp — the C ABI (include/dgcl.h): context, plan, workspace, IPC, dispatch.
+//
+// PAPER.md references: API §4.2, buildCommInfo, client-side decentralised
+// coordination §6.1, CUDA-VM peer method §6.2, process model §6.3
+// (P:1535-1548).  B200 design: one process per GPU; each GPU's workspace (halos, relay staging,
+// backward slots, flag words) is mapped by every peer over NVLink 5 / NVSwitch with CUDA IPC; one
+// persistent executor launch per layer and direction runs every stage, chained by device flags.
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "dgcl.h"
+#include "hostsim.h"
+#include "plan.h"
+
+using namespace dgcl;
+
+namespace {
+
+constexpr size_t kAlign = 256;
+inline size_t align_up(size_t x, size_t a = kAlign) { return (x + a - 1) / a * a; }
+inline int64_t pitch_of(int dim) { return (dim + 3) / 4 * 4; }
+
+struct Program {
+  // one launch: items for one (layer, direction, executing rank or -1 = fused loopback)
+  std::vector<DevItem> items;
+  size_t dev_off = 0;  // offset (in items) into the device item pool
+};
+
+}  // namespace
+
+struct dgcl_ctx {
+  int rank = 0, world = 1, device = -1;
+  bool loopback = false;
+  int lb_flags = 0;
+  int64_t n = 0;
+  std::vector<int32_t> part;
+  std::vector<int64_t> loc, n_local, row_off;
+  int n_layers = 0;
+  std::vector<int32_t> dims;
+  std::vector<int64_t> pitch;  // halo pitch per layer (elements)
+  int64_t max_pitch = 0;
+
+  Topology topo;
+  bool planned = false;
+  Relation rel;
+  Plan plan;
+  Lowered low;
+  std::vector<int64_t> halo_off;  // loopback: first halo row of each rank
+
+  // workspace layout: per rank, byte offsets relative to that rank's base
+  std::vector<size_t> off_flags, off_slot, ws_need;
+  std::vector<std::vector<size_t>> off_halo, off_relay;  // [layer][rank]
+  char *ws = nullptr;
+  size_t ws_bytes = 0;
+  std::vector<char *> base;  // per rank: workspace base (peer-mapped in multi-GPU mode)
+  std::vector<char *> ipc_opened;
+  bool registered = false, imported = false;
+
+  // device tables
+  DevGroup *d_groups = nullptr;
+  DevWait *d_waits = nullptr;
+  int32_t *d_idx = nullptr;
+  int64_t *d_term_ptr = nullptr;
+  uint32_t *d_terms = nullptr;
+  DevItem *d_items = nullptr;
+  std::vector<Program> progs;  // index prog_index(layer, dir, r)
+  int n_prog_ranks = 1;        // programs per (layer, dir)
+
+  uint64_t seq = 0, epoch[2] = {0, 0};
+  int *err_host = nullptr, *err_dev = nullptr;
+  int threads = 512, ctas_per_sm = 0, grid = 0, n_sm = 0;
+  int64_t item_bytes = 65536, timeout_ms = 20000;
+  std::vector<cudaStream_t> rank_streams;
+  std::vector<cudaEvent_t> rank_events;
+  cudaEvent_t fork_event = nullptr;
+  void *stage_a = nullptr, *stage_b = nullptr;
+  size_t stage_a_bytes = 0, stage_b_bytes = 0;
+  uint64_t launches = 0;
+  int debug_skip_rank = -1;  // fault injection (per-rank loopback): never launch this rank
+  bool dead = false;
+  std::string err;
+
+  int prog_index(int layer, int dir, int r) const { return (layer * 2 + dir) * n_prog_ranks + r; }
+};
+
+namespace {
+
+dgcl_status fail(dgcl_ctx *c, dgcl_status s, const char *fmt, ...) {
+  if (c) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    std::vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    c->err = buf;
+  }
+  return s;
+}
+
+#define CUDA_TRY(c, call)                                                                   \
+  do {                                                                                      \
+    cudaError_t e_ = (call);                                                                \
+    if (e_ != cudaSuccess)                                                                  \
+      return fail((c), DGCL_ECUDA, "%s failed: %s", #call, cudaGetErrorString(e_));         \
+  } while (0)
+
+dgcl_status init_common(int32_t rank, int32_t world, int32_t dev, int64_t n, const int32_t *part,
+                        int32_t n_layers, const int32_t *dims, bool loopback, int flags,
+                        dgcl_ctx **out) {
+  if (!out) return DGCL_EINVAL;
+  *out = nullptr;
+  if (world < 1 || world > kMaxRanks || rank < 0 || rank >= world || n < 0 || n_layers < 1 ||
+      !dims || (n > 0 && !part))
+    return DGCL_EINVAL;
+  if (loopback && flags != DGCL_LOOPBACK_FUSED && flags != DGCL_LOOPBACK_PER_RANK)
+    return DGCL_EINVAL;
+  dgcl_ctx *c = new (std::nothrow) dgcl_ctx();
+  if (!c) return DGCL_ENOMEM;
+  c->rank = rank;
+  c->world = world;
+  c->device = dev;
+  c->loopback = loopback;
+  c->lb_flags = flags;
+  c->n = n;
+  c->n_layers = n_layers;
+  for (int l = 0; l < n_layers; ++l) {
+    if (dims[l] < 1 || dims[l] > (1 << 24)) {
+      delete c;
+      return DGCL_EINVAL;
+    }
+    c->dims.push_back(dims[l]);
+    c->pitch.push_back(pitch_of(dims[l]));
+    c->max_pitch = std::max(c->max_pitch, pitch_of(dims[l]));
+  }
+  c->part.assign(part, part + n);
+  c->loc.assign(n, 0);
+  c->n_local.assign(world, 0);
+  for (int64_t v = 0; v < n; ++v) {  // §4.1 re-indexing: ascending global id per partition
+    const int32_t p = part[v];
+    if (p < 0 || p >= world) {
+      delete c;
+      return DGCL_EINVAL;
+    }
+    c->loc[v] = c->n_local[p]++;
+  }
+  c->row_off.assign(world + 1, 0);
+  for (int d = 0; d < world; ++d) c->row_off[d + 1] = c->row_off[d] + c->n_local[d];
+  c->topo = Topology::uniform_nvswitch(world);
+  if (dev >= 0) {
+    cudaError_t e = cudaSetDevice(dev);
+    if (e != cudaSuccess) {
+      delete c;
+      return DGCL_ECUDA;
+    }
+  }
+  *out = c;
+  return DGCL_OK;
+}
+
+bool has_device(dgcl_ctx *c) { return c->device >= 0; }
+
+void compute_layout(dgcl_ctx *c) {
+  const int m = c->world;
+  const Lowered &L = c->low;
+  c->off_flags.assign(m, 0);
+  c->off_slot.assign(m, 0);
+  c->ws_need.assign(m, 0);
+  c->off_halo.assign(c->n_layers, std::vector<size_t>(m, 0));
+  c->off_relay.assign(c->n_layers, std::vector<size_t>(m, 0));
+  if (c->loopback) {
+    // one allocation, buffer-major: every layer's halo of all ranks is one contiguous array
+    size_t off = 0;
+    for (int r = 0; r < m; ++r) c->off_flags[r] = off + (size_t)r * kFlagBytes;
+    off += (size_t)m * kFlagBytes;
+    for (int l = 0; l < c->n_layers; ++l) {
+      for (int r = 0; r < m; ++r)
+        c->off_halo[l][r] = off + (size_t)c->halo_off[r] * c->pitch[l] * 4;
+      off = align_up(off + (size_t)c->halo_off[m] * c->pitch[l] * 4);
+    }
+    for (int l = 0; l < c->n_layers; ++l)
+      for (int r = 0; r < m; ++r) {
+        c->off_relay[l][r] = off;
+        off = align_up(off + (size_t)L.n_relay[r] * c->pitch[l] * 4);
+      }
+    for (int r = 0; r < m; ++r) {
+      c->off_slot[r] = off;
+      off = align_up(off + (size_t)L.n_slot[r] * c->max_pitch * 4);
+    }
+    for (int r = 0; r < m; ++r) c->ws_need[r] = off;
+  } else {
+    for (int r = 0; r < m; ++r) {
+      size_t off = 0;
+      c->off_flags[r] = 0;
+      off = kFlagBytes;
+      for (int l = 0; l < c->n_layers; ++l) {
+        c->off_halo[l][r] = off;
+        off = align_up(off + (size_t)L.n_halo[r] * c->pitch[l] * 4);
+      }
+      for (int l = 0; l < c->n_layers; ++l) {
+        c->off_relay[l][r] = off;
+        off = align_up(off + (size_t)L.n_relay[r] * c->pitch[l] * 4);
+      }
+      c->off_slot[r] = off;
+      off = align_up(off + (size_t)L.n_slot[r] * c->max_pitch * 4);
+      c->ws_need[r] = off;
+    }
+  }
+}
+
+// counters some group of the given program waits on (fused loopback: only those need a signal)
+std::vector<uint8_t> needed_counters(const Lowered &L, const std::vector<int32_t> &gids) {
+  std::vector<uint8_t> need((size_t)kMaxRanks * kFlagWords, 0);
+  for (int32_t gi : gids) {
+    const DevGroup &g = L.groups[gi];
+    for (int w = 0; w < g.wait_n; ++w)
+      need[(size_t)g.exec_rank * kFlagWords + L.waits[g.wait_off + w].ctr] = 1;
+  }
+  return need;
+}
+
+void build_programs(dgcl_ctx *c) {
+  const Lowered &L = c->low;
+  const int m = c->world;
+  const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
+  c->n_prog_ranks = fused ? 1 : m;
+  c->progs.assign((size_t)c->n_layers * 2 * c->n_prog_ranks, Program());
+  const int ng = (int)L.groups.size();
+  for (int dir = 0; dir < 2; ++dir) {
+    std::vector<std::vector<int32_t>> gids(c->n_prog_ranks);
+    for (int r = 0; r < c->n_prog_ranks; ++r) {
+      const bool want_rank = c->loopback || r == c->rank;
+      if (!fused && !want_rank) continue;
+      if (!fused && m > 1) {
+        for (int gi = 0; gi < ng; ++gi)
+          if (L.groups[gi].op == OP_READY && L.groups[gi].exec_rank == r) gids[r].push_back(gi);
+      }
+      for (int gi = 0; gi < ng; ++gi) {
+        const DevGroup &g = L.groups[gi];
+        if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
+        if (!fused && g.exec_rank != r) continue;
+        gids[r].push_back(gi);
+      }
+      if (!fused && dir == DIR_FWD && m > 1) {
+        for (int gi = 0; gi < ng; ++gi)
+          if (L.groups[gi].op == OP_WAIT && L.groups[gi].exec_rank == r) gids[r].push_back(gi);
+      }
+    }
+    for (int l = 0; l < c->n_layers; ++l) {
+      for (int r = 0; r < c->n_prog_ranks; ++r) {
+        Program &P = c->progs[c->prog_index(l, dir, r)];
+        const std::vector<uint8_t> need = needed_counters(L, gids[r]);
+        build_items(L, gids[r], (int64_t)c->dims[l] * 4, c->item_bytes, !fused, need, &P.items);
+      }
+    }
+  }
+}
+
+template <typename T>
+dgcl_status upload(dgcl_ctx *c, T **dptr, const std::vector<T> &v) {
+  if (*dptr) cudaFree(*dptr);
+  *dptr = nullptr;
+  const size_t bytes = std::max<size_t>(sizeof(T), v.size() * sizeof(T));
+  CUDA_TRY(c, cudaMalloc((void **)dptr, bytes));
+  if (!v.empty()) CUDA_TRY(c, cudaMemcpy(*dptr, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice));
+  return DGCL_OK;
+}
+
+dgcl_status check_dead(dgcl_ctx *c) {
+  if (c->dead) return fail(c, DGCL_ETIMEOUT, "context unusable after a device watchdog timeout");
+  if (c->err_host && *(volatile int *)c->err_host != 0) {
+    c->dead = true;
+    return fail(c, DGCL_ETIMEOUT, "device watchdog: a flag wait timed out (code %d)",
+                *(volatile int *)c->err_host);
+  }
+  return DGCL_OK;
+}
+
+inline bool al16(const void *p) { return ((uintptr_t)p & 15) == 0; }
+
+dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_pitch,
+                   float *out, int64_t out_pitch, cudaStream_t stream) {
+  const int m = c->world;
+  ExecParams P;
+  std::memset(&P, 0, sizeof(P));
+  const int64_t hp = c->pitch[layer] * 4;  // bytes
+  bool v16 = (hp % 16) == 0;
+  for (int r = 0; r < m; ++r) {
+    char *b = c->base[r];
+    P.flags[r] = (uint64_t *)(b + c->off_flags[r]);
+    P.buf[K_HALO][r] = {b + c->off_halo[layer][r], hp};
+    P.buf[K_RELAY][r] = {b + c->off_relay[layer][r], hp};
+    P.buf[K_SLOT][r] = {b + c->off_slot[r], hp};
+  }
+  const int in_kind = dir == DIR_FWD ? K_EMB : K_HGRAD;
+  for (int r = 0; r < m; ++r) {
+    if (!c->loopback && r != c->rank) continue;
+    const int64_t in_row = c->loopback ? (dir == DIR_FWD ? c->row_off[r] : c->halo_off[r]) : 0;
+    P.buf[in_kind][r] = {(char *)(in + in_row * in_pitch), in_pitch * 4};
+    if (dir == DIR_BWD) {
+      const int64_t out_row = c->loopback ? c->row_off[r] : 0;
+      P.buf[K_EGRAD][r] = {(char *)(out + out_row * out_pitch), out_pitch * 4};
+    }
+  }
+  if ((in_pitch * 4) % 16 || !al16(in)) v16 = false;
+  if (dir == DIR_BWD && ((out_pitch * 4) % 16 || !al16(out))) v16 = false;
+  P.groups = c->d_groups;
+  P.waits = c->d_waits;
+  P.idx = c->d_idx;
+  P.term_ptr = c->d_term_ptr;
+  P.terms = c->d_terms;
+  P.world = m;
+  P.row_bytes = c->dims[layer] * 4;
+  P.vec16 = v16 ? 1 : 0;
+  P.n_chunks = v16 ? (P.row_bytes + 15) / 16 : c->dims[layer];
+  const FastDiv fd = make_fastdiv((uint32_t)P.n_chunks);
+  P.div_mul = fd.mul;
+  P.div_shift = fd.shift;
+  P.epoch[0] = c->epoch[0];
+  P.epoch[1] = c->epoch[1];
+  P.seq = c->seq;
+  P.timeout_ns = (uint64_t)c->timeout_ms * 1000000ull;
+  P.err = c->err_dev;
+  const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
+  P.use_ready = (!fused && m > 1) ? 1 : 0;
+  if (fused || !c->loopback) {
+    const int r = fused ? 0 : c->rank;
+    const Program &pg = c->progs[c->prog_index(layer, dir, fused ? 0 : (c->loopback ? r : r))];
+    if (pg.items.empty()) return DGCL_OK;
+    P.items = c->d_items + pg.dev_off;
+    P.n_items = (int32_t)pg.items.size();
+    const int grid = std::min<int64_t>(c->grid, (int64_t)pg.items.size());
+    int e = launch_executor(P, grid, c->threads, stream);
+    if (e != 0) return fail(c, DGCL_ECUDA, "executor launch failed: %s",
+                            cudaGetErrorString((cudaError_t)e));
+    c->launches++;
+    return DGCL_OK;
+  }
+  // loopback, one launch per virtual rank on its own stream (full flag protocol)
+  CUDA_TRY(c, cudaEventRecord(c->fork_event, stream));
+  const int grid_r = std::max(1, c->grid / m);
+  for (int r = 0; r < m; ++r) {
+    const Program &pg = c->progs[c->prog_index(layer, dir, r)];
+    CUDA_TRY(c, cudaStreamWaitEvent(c->rank_streams[r], c->fork_event, 0));
+    if (!pg.items.empty() && r != c->debug_skip_rank) {
+      ExecParams Pr = P;
+      Pr.items = c->d_items + pg.dev_off;
+      Pr.n_items = (int32_t)pg.items.size();
+      int e = launch_executor(Pr, std::min<int64_t>(grid_r, (int64_t)pg.items.size()),
+                              c->threads, c->rank_streams[r]);
+      if (e != 0) return fail(c, DGCL_ECUDA, "executor launch failed: %s",
+                              cudaGetErrorString((cudaError_t)e));
+      c->launches++;
+    }
+    CUDA_TRY(c, cudaEventRecord(c->rank_events[r], c->rank_streams[r]));
+    CUDA_TRY(c, cudaStreamWaitEvent(stream, c->rank_events[r], 0));
+  }
+  return DGCL_OK;
+}
+
+dgcl_status ready_to_dispatch(dgcl_ctx *c, int32_t layer) {
+  if (!c) return DGCL_EINVAL;
+  if (!has_device(c)) return fail(c, DGCL_ESTATE, "host-only context");
+  if (!c->registered) return fail(c, DGCL_ESTATE, "workspace not registered");
+  if (!c->loopback && c->world > 1 && !c->imported)
+    return fail(c, DGCL_ESTATE, "peers not imported");
+  if (layer < 0 || layer >= c->n_layers) return fail(c, DGCL_EINVAL, "bad layer %d", layer);
+  return check_dead(c);
+}
+
+}  // namespace
+
+extern "C" {
+
+dgcl_status dgcl_init(int32_t rank, int32_t world, int32_t cuda_device, int64_t n_vertices,
+                      const int32_t *part, int32_t n_layers, const int32_t *dims, dgcl_ctx **out) {
+  return init_common(rank, world, cuda_device, n_vertices, part, n_layers, dims, false, 0, out);
+}
+
+dgcl_status dgcl_init_loopback(int32_t world, int32_t cuda_device, int64_t n_vertices,
+                               const int32_t *part, int32_t n_layers, const int32_t *dims,
+                               int32_t flags, dgcl_ctx **out) {
+  return init_common(0, world, cuda_device, n_vertices, part, n_layers, dims, true, flags, out);
+}
+
+dgcl_status dgcl_set_topology(dgcl_ctx *c, const dgcl_topology *t) {
+  if (!c || !t || !t->hop_ticks || !t->link_ptr || t->n_hops < 0) return DGCL_EINVAL;
+  if (c->planned) return fail(c, DGCL_ESTATE, "topology must be set before dgcl_build_plan");
+  const int m = c->world;
+  Topology T;
+  T.m = m;
+  for (int h = 0; h < t->n_hops; ++h) {
+    if (t->hop_ticks[h] <= 0) return fail(c, DGCL_EINVAL, "hop %d: ticks must be > 0", h);
+    T.w.push_back(t->hop_ticks[h]);
+  }
+  if (t->link_ptr[0] != 0) return fail(c, DGCL_EINVAL, "link_ptr[0] != 0");
+  T.link_ptr.assign(t->link_ptr, t->link_ptr + (size_t)m * m + 1);
+  for (size_t p = 0; p < (size_t)m * m; ++p) {
+    if (T.link_ptr[p + 1] < T.link_ptr[p]) return fail(c, DGCL_EINVAL, "link_ptr decreasing");
+    if (p / m == p % m && T.link_ptr[p + 1] != T.link_ptr[p])
+      return fail(c, DGCL_EINVAL, "self link %zu", p / m);
+  }
+  const int64_t nh = T.link_ptr[(size_t)m * m];
+  if (nh > 0 && !t->link_hops) return DGCL_EINVAL;
+  for (int64_t q = 0; q < nh; ++q) {
+    if (t->link_hops[q] < 0 || t->link_hops[q] >= t->n_hops)
+      return fail(c, DGCL_EINVAL, "link hop id out of range");
+    T.link_hops.push_back(t->link_hops[q]);
+  }
+  c->topo = T;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_build_plan(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *req_ids,
+                            uint64_t seed) {
+  if (!c || !req_ptr) return DGCL_EINVAL;
+  if (c->planned) return fail(c, DGCL_ESTATE, "plan already built");
+  if (req_ptr[c->world] > 0 && !req_ids) return DGCL_EINVAL;
+  try {
+    std::string e = build_relation(c->n, c->world, c->part.data(), req_ptr, req_ids, &c->rel);
+    if (!e.empty()) return fail(c, DGCL_EINVAL, "%s", e.c_str());
+    for (int d = 0; d < c->world; ++d)
+      if (req_ptr[d + 1] - req_ptr[d] > INT32_MAX) return fail(c, DGCL_EINVAL, "halo too large");
+    e = spst_plan(c->topo, c->part.data(), c->rel, seed, &c->plan);
+    if (!e.empty()) return fail(c, DGCL_EPLAN, "%s", e.c_str());
+    if (c->plan.n_stages >= kMaxStages) return fail(c, DGCL_EPLAN, "too many stages");
+    lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low);
+    c->halo_off.assign(c->world + 1, 0);
+    for (int d = 0; d < c->world; ++d) c->halo_off[d + 1] = c->halo_off[d] + c->rel.n_halo[d];
+    compute_layout(c);
+    build_programs(c);
+  } catch (const std::bad_alloc &) {
+    return fail(c, DGCL_ENOMEM, "host allocation failed while planning");
+  }
+  c->planned = true;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_workspace_bytes(dgcl_ctx *c, size_t *bytes) {
+  if (!c || !bytes) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  *bytes = c->ws_need[c->loopback ? 0 : c->rank];
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
+  if (!c) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  if (!has_device(c)) return fail(c, DGCL_ESTATE, "host-only context");
+  if (c->registered) return fail(c, DGCL_ESTATE, "workspace already registered");
+  if (!dev || ((uintptr_t)dev % kAlign)) return fail(c, DGCL_EINVAL, "workspace must be 256-B aligned");
+  const size_t need = c->ws_need[c->loopback ? 0 : c->rank];
+  if (bytes < need) return fail(c, DGCL_ENOMEM, "workspace %zu < %zu bytes", bytes, need);
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  c->ws = (char *)dev;
+  c->ws_bytes = bytes;
+  c->base.assign(c->world, nullptr);
+  if (c->loopback)
+    for (int r = 0; r < c->world; ++r) c->base[r] = c->ws;
+  else
+    c->base[c->rank] = c->ws;
+  // zero every flag region this context owns (monotonic counters start at 0)
+  if (c->loopback) {
+    CUDA_TRY(c, cudaMemset(c->ws, 0, (size_t)c->world * kFlagBytes));
+  } else {
+    CUDA_TRY(c, cudaMemset(c->ws, 0, kFlagBytes));
+  }
+  // device tables
+  dgcl_status s;
+  if ((s = upload(c, &c->d_groups, c->low.groups)) != DGCL_OK) return s;
+  if ((s = upload(c, &c->d_waits, c->low.waits)) != DGCL_OK) return s;
+  if ((s = upload(c, &c->d_idx, c->low.idx)) != DGCL_OK) return s;
+  if ((s = upload(c, &c->d_term_ptr, c->low.term_ptr)) != DGCL_OK) return s;
+  if ((s = upload(c, &c->d_terms, c->low.terms)) != DGCL_OK) return s;
+  std::vector<DevItem> all;
+  for (Program &p : c->progs) {
+    p.dev_off = all.size();
+    all.insert(all.end(), p.items.begin(), p.items.end());
+  }
+  if ((s = upload(c, &c->d_items, all)) != DGCL_OK) return s;
+  // watchdog word in mapped host memory
+  CUDA_TRY(c, cudaHostAlloc((void **)&c->err_host, 64, cudaHostAllocMapped));
+  std::memset(c->err_host, 0, 64);
+  CUDA_TRY(c, cudaHostGetDevicePointer((void **)&c->err_dev, c->err_host, 0));
+  // launch geometry: persistent grid of co-resident CTAs
+  CUDA_TRY(c, cudaDeviceGetAttribute(&c->n_sm, cudaDevAttrMultiProcessorCount, c->device));
+  int occ = 0;
+  int e = executor_occupancy(c->threads, &occ);
+  if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");
+  if (c->ctas_per_sm <= 0) c->ctas_per_sm = std::min(occ, 4);
+  c->ctas_per_sm = std::max(1, std::min(c->ctas_per_sm, occ));
+  c->grid = c->n_sm * c->ctas_per_sm;
+  if (c->loopback && c->lb_flags == DGCL_LOOPBACK_PER_RANK) {
+    c->rank_streams.assign(c->world, nullptr);
+    c->rank_events.assign(c->world, nullptr);
+    for (int r = 0; r < c->world; ++r) {
+      CUDA_TRY(c, cudaStreamCreateWithFlags(&c->rank_streams[r], cudaStreamNonBlocking));
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->rank_events[r], cudaEventDisableTiming));
+    }
+    CUDA_TRY(c, cudaEventCreateWithFlags(&c->fork_event, cudaEventDisableTiming));
+  }
+  CUDA_TRY(c, cudaDeviceSynchronize());
+  c->registered = true;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_halo_view(dgcl_ctx *c, int32_t layer, size_t *offset, int64_t *rows,
+                           int64_t *pitch) {
+  if (!c || !offset || !rows || !pitch) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  if (layer < 0 || layer >= c->n_layers) return fail(c, DGCL_EINVAL, "bad layer");
+  const int r = c->loopback ? 0 : c->rank;
+  *offset = c->off_halo[layer][r];
+  *rows = c->loopback ? c->halo_off[c->world] : c->rel.n_halo[c->rank];
+  *pitch = c->pitch[layer];
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_rank_rows(dgcl_ctx *c, int64_t *n_local, int64_t *n_halo) {
+  if (!c || !n_local || !n_halo) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  for (int d = 0; d < c->world; ++d) {
+    n_local[d] = c->n_local[d];
+    n_halo[d] = c->rel.n_halo[d];
+  }
+  return DGCL_OK;
+}
+
+namespace {
+struct IpcBlob {
+  uint64_t magic;
+  int32_t rank, world;
+  uint64_t offset;   // workspace start within the exported allocation
+  uint64_t bytes;
+  cudaIpcMemHandle_t handle;
+};
+constexpr uint64_t kBlobMagic = 0x44474C4349504331ull;  // "DGCLIPC1"
+static_assert(sizeof(IpcBlob) <= DGCL_IPC_BLOB_BYTES, "blob size");
+}  // namespace
+
+dgcl_status dgcl_ipc_export(dgcl_ctx *c, void *blob, size_t *len) {
+  if (!c || !blob || !len) return DGCL_EINVAL;
+  if (!c->registered) return fail(c, DGCL_ESTATE, "workspace not registered");
+  if (*len < sizeof(IpcBlob)) return fail(c, DGCL_EINVAL, "blob capacity too small");
+  IpcBlob b;
+  std::memset(&b, 0, sizeof(b));
+  b.magic = kBlobMagic;
+  b.rank = c->rank;
+  b.world = c->world;
+  b.bytes = c->ws_bytes;
+  // allocation base of the (possibly sub-allocated, e.g. PyTorch caching allocator) workspace;
+  // the driver entry point is resolved through the runtime so libdgcl does not link libcuda
+  typedef CUresult (*GetRange)(CUdeviceptr *, size_t *, CUdeviceptr);
+  void *fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  CUDA_TRY(c, cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q));
+  if (!fn || q != cudaDriverEntryPointSuccess)
+    return fail(c, DGCL_ECUDA, "cuMemGetAddressRange entry point unavailable");
+  CUdeviceptr base = 0;
+  size_t sz = 0;
+  CUresult cr = ((GetRange)fn)(&base, &sz, (CUdeviceptr)c->ws);
+  if (cr != CUDA_SUCCESS) return fail(c, DGCL_ECUDA, "cuMemGetAddressRange failed (%d)", (int)cr);
+  b.offset = (uint64_t)((CUdeviceptr)c->ws - base);
+  CUDA_TRY(c, cudaIpcGetMemHandle(&b.handle, (void *)base));
+  std::memcpy(blob, &b, sizeof(b));
+  *len = sizeof(b);
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_ipc_import(dgcl_ctx *c, const void *blobs, size_t len_each) {
+  if (!c || !blobs) return DGCL_EINVAL;
+  if (!c->registered) return fail(c, DGCL_ESTATE, "workspace not registered");
+  if (c->loopback) return fail(c, DGCL_ESTATE, "loopback contexts have no peers");
+  if (c->imported) return fail(c, DGCL_ESTATE, "already imported");
+  if (len_each < sizeof(IpcBlob)) return fail(c, DGCL_EINVAL, "blob too small");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  for (int r = 0; r < c->world; ++r) {
+    if (r == c->rank) continue;
+    IpcBlob b;
+    std::memcpy(&b, (const char *)blobs + (size_t)r * len_each, sizeof(b));
+    if (b.magic != kBlobMagic || b.rank != r || b.world != c->world)
+      return fail(c, DGCL_EINVAL, "bad IPC blob for rank %d", r);
+    if (b.bytes < c->ws_need[r]) return fail(c, DGCL_EINVAL, "peer %d workspace too small", r);
+    void *p = nullptr;
+    CUDA_TRY(c, cudaIpcOpenMemHandle(&p, b.handle, cudaIpcMemLazyEnablePeerAccess));
+    c->ipc_opened.push_back((char *)p);
+    c->base[r] = (char *)p + b.offset;
+  }
+  c->imported = true;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_dispatch_forward(dgcl_ctx *c, int32_t layer, const float *emb, int64_t emb_pitch,
+                                  float *halo, void *stream) {
+  dgcl_status s = ready_to_dispatch(c, layer);
+  if (s != DGCL_OK) return s;
+  if (emb_pitch < c->dims[layer]) return fail(c, DGCL_EINVAL, "emb_pitch < dim");
+  const char *view = c->base[c->loopback ? 0 : c->rank] + c->off_halo[layer][c->loopback ? 0 : c->rank];
+  if (halo && (const char *)halo != view) return fail(c, DGCL_EINVAL, "halo is not the registered view");
+  const int64_t rows = c->loopback ? c->n : c->n_local[c->rank];
+  if (rows > 0 && !emb) return fail(c, DGCL_EINVAL, "emb is NULL");
+  if (c->world == 1) return DGCL_OK;
+  c->seq++;
+  c->epoch[DIR_FWD]++;
+  return launch(c, layer, DIR_FWD, emb, emb_pitch, nullptr, 0, (cudaStream_t)stream);
+}
+
+dgcl_status dgcl_dispatch_backward(dgcl_ctx *c, int32_t layer, const float *halo_grad,
+                                   int64_t hg_pitch, float *emb_grad, int64_t eg_pitch,
+                                   void *stream) {
+  dgcl_status s = ready_to_dispatch(c, layer);
+  if (s != DGCL_OK) return s;
+  if (hg_pitch < c->dims[layer] || eg_pitch < c->dims[layer])
+    return fail(c, DGCL_EINVAL, "pitch < dim");
+  const int64_t hrows = c->loopback ? c->halo_off[c->world] : c->rel.n_halo[c->rank];
+  const int64_t rows = c->loopback ? c->n : c->n_local[c->rank];
+  if ((hrows > 0 && !halo_grad) || (rows > 0 && !emb_grad))
+    return fail(c, DGCL_EINVAL, "NULL buffer");
+  if (c->world == 1) return DGCL_OK;
+  c->seq++;
+  c->epoch[DIR_BWD]++;
+  return launch(c, layer, DIR_BWD, halo_grad, hg_pitch, emb_grad, eg_pitch, (cudaStream_t)stream);
+}
+
+static dgcl_status ensure_stage(dgcl_ctx *c, void **p, size_t *cap, size_t bytes) {
+  if (*cap >= bytes) return DGCL_OK;
+  if (*p) cudaFree(*p);
+  *p = nullptr;
+  *cap = 0;
+  if (cudaMalloc(p, std::max<size_t>(bytes, 256)) != cudaSuccess)
+    return fail(c, DGCL_ENOMEM, "staging allocation of %zu bytes failed", bytes);
+  *cap = bytes;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_forward_host(dgcl_ctx *c, int32_t layer, const float *host_emb, float *host_halo,
+                              void *stream) {
+  dgcl_status s = ready_to_dispatch(c, layer);
+  if (s != DGCL_OK) return s;
+  const int64_t p = c->pitch[layer];
+  const int64_t rows = c->loopback ? c->n : c->n_local[c->rank];
+  const int64_t hrows = c->loopback ? c->halo_off[c->world] : c->rel.n_halo[c->rank];
+  cudaStream_t st = (cudaStream_t)stream;
+  if ((s = ensure_stage(c, &c->stage_a, &c->stage_a_bytes, rows * p * 4)) != DGCL_OK) return s;
+  if (rows > 0)
+    CUDA_TRY(c, cudaMemcpyAsync(c->stage_a, host_emb, rows * p * 4, cudaMemcpyHostToDevice, st));
+  if ((s = dgcl_dispatch_forward(c, layer, (const float *)c->stage_a, p, nullptr, stream)) != DGCL_OK)
+    return s;
+  const char *view = c->base[c->loopback ? 0 : c->rank] + c->off_halo[layer][c->loopback ? 0 : c->rank];
+  if (hrows > 0)
+    CUDA_TRY(c, cudaMemcpyAsync(host_halo, view, hrows * p * 4, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(c, cudaStreamSynchronize(st));
+  return check_dead(c);
+}
+
+dgcl_status dgcl_backward_host(dgcl_ctx *c, int32_t layer, const float *host_halo_grad,
+                               float *host_emb_grad, void *stream) {
+  dgcl_status s = ready_to_dispatch(c, layer);
+  if (s != DGCL_OK) return s;
+  const int64_t p = c->pitch[layer];
+  const int64_t rows = c->loopback ? c->n : c->n_local[c->rank];
+  const int64_t hrows = c->loopback ? c->halo_off[c->world] : c->rel.n_halo[c->rank];
+  cudaStream_t st = (cudaStream_t)stream;
+  if ((s = ensure_stage(c, &c->stage_a, &c->stage_a_bytes, rows * p * 4)) != DGCL_OK) return s;
+  if ((s = ensure_stage(c, &c->stage_b, &c->stage_b_bytes, hrows * p * 4)) != DGCL_OK) return s;
+  if (hrows > 0)
+    CUDA_TRY(c, cudaMemcpyAsync(c->stage_b, host_halo_grad, hrows * p * 4, cudaMemcpyHostToDevice, st));
+  if (rows > 0)
+    CUDA_TRY(c, cudaMemcpyAsync(c->stage_a, host_emb_grad, rows * p * 4, cudaMemcpyHostToDevice, st));
+  if ((s = dgcl_dispatch_backward(c, layer, (const float *)c->stage_b, p, (float *)c->stage_a, p,
+                                  stream)) != DGCL_OK)
+    return s;
+  if (rows > 0)
+    CUDA_TRY(c, cudaMemcpyAsync(host_emb_grad, c->stage_a, rows * p * 4, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(c, cudaStreamSynchronize(st));
+  return check_dead(c);
+}
+
+dgcl_status dgcl_plan_info(dgcl_ctx *c, dgcl_plan_stats *info) {
+  if (!c || !info) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  std::memset(info, 0, sizeof(*info));
+  info->world = c->world;
+  info->n_stages = c->plan.n_stages;
+  info->n_vertices_planned = (int64_t)c->plan.order.size();
+  info->n_deliveries = c->rel.d_ptr[c->rel.n];
+  info->n_tree_edges = c->low.n_tree_edges;
+  info->n_relay_rows = c->low.n_relay_edges;
+  info->model_cost_ticks = c->plan.cost;
+  int64_t item_bytes = 0;
+  for (const Program &p : c->progs) item_bytes += (int64_t)(p.items.size() * sizeof(DevItem));
+  info->table_bytes = c->low.table_bytes() + item_bytes;
+  info->planner_seconds = c->plan.seconds;
+  info->lowering_seconds = c->low.seconds;
+  int nf = 0, nb = 0;
+  for (const DevGroup &g : c->low.groups) {
+    if (g.op == OP_READY || g.op == OP_WAIT) continue;
+    (g.dir == DIR_FWD ? nf : nb)++;
+  }
+  info->n_fwd_groups = nf;
+  info->n_bwd_groups = nb;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_plan_counts(dgcl_ctx *c, int64_t *rows) {
+  if (!c || !rows) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  const int m = c->world, K = c->plan.n_stages;
+  for (int k = 1; k <= K; ++k)
+    for (int s = 0; s < m; ++s)
+      for (int d = 0; d < m; ++d)
+        rows[((size_t)(k - 1) * m + s) * m + d] = c->low.rows(DIR_FWD, k, s, d);
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_plan_export(dgcl_ctx *c, int64_t *n_edges, int64_t *u, int32_t *parent,
+                             int32_t *child, int32_t *stage) {
+  if (!c || !n_edges) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  const int64_t NE = (int64_t)c->plan.e_parent.size();
+  if (!u && !parent && !child && !stage) {
+    *n_edges = NE;
+    return DGCL_OK;
+  }
+  if (!u || !parent || !child || !stage || *n_edges < NE) return DGCL_EINVAL;
+  for (size_t i = 0; i < c->plan.order.size(); ++i)
+    for (int64_t e = c->plan.e_ptr[i]; e < c->plan.e_ptr[i + 1]; ++e) {
+      u[e] = c->plan.order[i];
+      parent[e] = c->plan.e_parent[e];
+      child[e] = c->plan.e_child[e];
+      stage[e] = c->plan.e_stage[e];
+    }
+  *n_edges = NE;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
+  if (!c || !key) return DGCL_EINVAL;
+  const std::string k(key);
+  if (k == "timeout_ms") {
+    if (value < 1) return fail(c, DGCL_EINVAL, "timeout_ms must be >= 1");
+    c->timeout_ms = value;
+    return DGCL_OK;
+  }
+  if (k == "debug_skip_rank") {
+    if (value < -1 || value >= c->world) return fail(c, DGCL_EINVAL, "debug_skip_rank");
+    c->debug_skip_rank = (int)value;
+    return DGCL_OK;
+  }
+  if (c->registered) return fail(c, DGCL_ESTATE, "option %s must be set before registration", key);
+  if (k == "item_bytes") {
+    if (value < 16) return fail(c, DGCL_EINVAL, "item_bytes too small");
+    c->item_bytes = value;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "ctas_per_sm") {
+    if (value < 1 || value > 32) return fail(c, DGCL_EINVAL, "ctas_per_sm out of range");
+    c->ctas_per_sm = (int)value;
+    return DGCL_OK;
+  }
+  if (k == "threads") {
+    if (value < 128 || value > 512 || value % 32) return fail(c, DGCL_EINVAL, "threads");
+    c->threads = (int)value;
+    return DGCL_OK;
+  }
+  return fail(c, DGCL_EINVAL, "unknown option %s", key);
+}
+
+dgcl_status dgcl_launch_count(dgcl_ctx *c, uint64_t *count) {
+  if (!c || !count) return DGCL_EINVAL;
+  *count = c->launches;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_check(dgcl_ctx *c) {
+  if (!c) return DGCL_EINVAL;
+  dgcl_status s = check_dead(c);
+  if (s != DGCL_OK) return s;
+  if (has_device(c)) {
+    cudaError_t e = cudaPeekAtLastError();
+    if (e != cudaSuccess) return fail(c, DGCL_ECUDA, "sticky CUDA error: %s", cudaGetErrorString(e));
+  }
+  return DGCL_OK;
+}
+
+const char *dgcl_last_error(dgcl_ctx *c) { return c ? c->err.c_str() : "null context"; }
+
+const char *dgcl_strerror(dgcl_status s) {
+  switch (s) {
+    case DGCL_OK: return "ok";
+    case DGCL_EINVAL: return "invalid argument";
+    case DGCL_ESTATE: return "invalid call order / state";
+    case DGCL_ECUDA: return "CUDA error";
+    case DGCL_ENOMEM: return "out of memory";
+    case DGCL_ETIMEOUT: return "device flag wait timed out";
+    case DGCL_EPLAN: return "planning failed (unreachable GPU)";
+  }
+  return "unknown status";
+}
+
+dgcl_status dgcl_destroy(dgcl_ctx *c) {
+  if (!c) return DGCL_OK;
+  if (has_device(c)) {
+    cudaSetDevice(c->device);
+    cudaDeviceSynchronize();
+    for (char *p : c->ipc_opened) cudaIpcCloseMemHandle(p);
+    cudaFree(c->d_groups);
+    cudaFree(c->d_waits);
+    cudaFree(c->d_idx);
+    cudaFree(c->d_term_ptr);
+    cudaFree(c->d_terms);
+    cudaFree(c->d_items);
+    if (c->stage_a) cudaFree(c->stage_a);
+    if (c->stage_b) cudaFree(c->stage_b);
+    if (c->err_host) cudaFreeHost(c->err_host);
+    for (cudaStream_t s : c->rank_streams)
+      if (s) cudaStreamDestroy(s);
+    for (cudaEvent_t e : c->rank_events)
+      if (e) cudaEventDestroy(e);
+    if (c->fork_event) cudaEventDestroy(c->fork_event);
+  }
+  delete c;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_debug_hostsim_forward(dgcl_ctx *c, int32_t layer, const float *emb, float *halo) {
+  if (!c || !emb || !halo) return DGCL_EINVAL;
+  if (!c->planned || !c->loopback) return fail(c, DGCL_ESTATE, "needs a planned loopback context");
+  if (layer < 0 || layer >= c->n_layers) return DGCL_EINVAL;
+  hostsim_run(c->low, DIR_FWD, c->row_off, c->halo_off, c->pitch[layer], c->dims[layer], emb, halo,
+              nullptr, nullptr);
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_debug_hostsim_backward(dgcl_ctx *c, int32_t layer, const float *halo_grad,
+                                        float *emb_grad) {
+  if (!c || !halo_grad || !emb_grad) return DGCL_EINVAL;
+  if (!c->planned || !c->loopback) return fail(c, DGCL_ESTATE, "needs a planned loopback context");
+  if (layer < 0 || layer >= c->n_layers) return DGCL_EINVAL;
+  hostsim_run(c->low, DIR_BWD, c->row_off, c->halo_off, c->pitch[layer], c->dims[layer], nullptr,
+              nullptr, halo_grad, emb_grad);
+  return DGCL_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,135 @@
+// internal.h — shared (host + device) definitions of libdgcl.
+//
+// The lowered plan is a list of GROUPS: one per send tuple (d_i, d_j, k, T^s_ij, T^r_ij) of §6.1
+// (PAPER.md P:1401-1420), further split by the buffer kinds the rows come from / go to.  Groups
+// are cut into fixed-size row ranges (ITEMS) which the persistent executor kernel walks in stage
+// order.  Stage chaining uses monotonically increasing per-(direction, stage, source) row counters
+// in the receiver's flag region — the "done" flags of §6.1 — and a per-source
+// "ready" word, so no flag is ever reset and no host round-trip happens between stages.
+#pragma once
+
+#include <cstdint>
+
+namespace dgcl {
+
+constexpr int kMaxRanks = 16;
+constexpr int kMaxStages = 16;  // stage indices 1..15 (<= world-1)
+
+// buffer kinds
+enum Kind : int32_t {
+  K_EMB = 0,    // user embeddings (local rows), read-only
+  K_HALO = 1,   // per-layer halo (workspace), written by peers
+  K_RELAY = 2,  // per-layer relay staging (workspace): rows a GPU forwards but did not request
+  K_HGRAD = 3,  // user halo gradients, read-only
+  K_SLOT = 4,   // backward gradient slots (workspace), written by tree children
+  K_EGRAD = 5,  // user embedding gradients (in/out)
+  K_NKINDS = 6
+};
+
+enum Op : int32_t {
+  OP_COPY = 0,   // dst[dst_row(i)] = src[src_row(i)]
+  OP_FOLD = 1,   // dst[dst_row(i)] = fold(init ? dst : -, terms(i)) in order, fp32 adds
+  OP_READY = 2,  // write ready[exec_rank] = seq into every peer's flag region
+  OP_WAIT = 3    // wait on the group's wait list (forward completion)
+};
+
+enum Dir : int32_t { DIR_FWD = 0, DIR_BWD = 1 };
+
+// flag region layout (uint64 words) at the start of every rank's workspace
+constexpr int64_t ctr_index(int dir, int stage, int src) {
+  return ((int64_t)dir * kMaxStages + stage) * kMaxRanks + src;
+}
+constexpr int64_t kReadyBase = 2 * kMaxStages * kMaxRanks;  // ready[src] words
+constexpr int64_t kFlagWords = kReadyBase + kMaxRanks;
+constexpr int64_t kFlagBytes = 8192;  // region reserved (>= kFlagWords * 8)
+static_assert(kFlagWords * 8 <= kFlagBytes, "flag region");
+
+// term encoding for OP_FOLD: bit 31 set => SLOT(exec) row, else HGRAD(exec) row
+constexpr uint32_t kTermSlot = 0x80000000u;
+
+struct DevGroup {
+  int32_t op;
+  int32_t dir;
+  int32_t exec_rank;   // the GPU executing the group (all reads are local to it)
+  int32_t dst_rank;    // the GPU whose buffer is written (a peer over NVLink, or itself)
+  int32_t stage;       // forward stage k, or backward stage b (RED = K + 1)
+  int32_t src_kind;    // OP_COPY source buffer kind
+  int32_t dst_kind;
+  int32_t fold_init;   // OP_FOLD: start from the destination row (RED)
+  int32_t sig_ctr;     // counter index (ctr_index) on dst_rank to add n_rows to, or -1
+  int32_t ready_rank;  // wait ready[ready_rank] >= seq before writing (-1: none)
+  int32_t wait_off;    // waits[wait_off .. wait_off + wait_n) on exec_rank's counters
+  int32_t wait_n;
+  int64_t n_rows;
+  int64_t src_idx;     // offset into idx pool, or -1 => rows src_base + i
+  int64_t src_base;
+  int64_t dst_idx;     // offset into idx pool, or -1 => rows dst_base + i
+  int64_t dst_base;
+  int64_t term_ptr;    // OP_FOLD: offset into term_ptr pool (n_rows + 1 entries)
+};
+
+struct DevItem {
+  int32_t group;
+  int32_t row_begin;
+  int32_t row_end;
+  int32_t flags;       // bit 0: signal the group's counter after the rows
+};
+constexpr int32_t kItemSignal = 1;
+
+struct DevWait {
+  int32_t ctr;         // counter index on the executing rank
+  int32_t pad;
+  int64_t amount;      // rows per call; target = epoch[dir] * amount
+};
+
+struct BufRef {
+  char *ptr;
+  int64_t pitch;       // bytes
+};
+
+struct ExecParams {
+  BufRef buf[K_NKINDS][kMaxRanks];
+  uint64_t *flags[kMaxRanks];  // flag region of every rank (peer-mapped in multi-GPU mode)
+  const DevGroup *groups;
+  const DevItem *items;
+  const DevWait *waits;
+  const int32_t *idx;
+  const int64_t *term_ptr;
+  const uint32_t *terms;
+  int32_t n_items;
+  int32_t world;
+  int32_t row_bytes;   // dims[layer] * 4: bytes moved per row
+  int32_t n_chunks;    // 16-byte chunks per row (vector path) or 4-byte words (scalar path)
+  uint32_t div_mul;    // fast division by n_chunks: q = (umulhi(x, mul) + x) >> shift
+  int32_t div_shift;
+  int32_t vec16;       // 1: 16-byte path (all bases and pitches 16-B aligned)
+  int32_t use_ready;   // per-rank programs: honour ready words before writing to a peer
+  uint64_t epoch[2];   // completed+current calls per direction (counter targets)
+  uint64_t seq;        // global call sequence number (ready words)
+  uint64_t timeout_ns;
+  int *err;            // host-mapped error word (0 = ok)
+};
+
+// fast unsigned division by a runtime constant d >= 1, exact for x < 2^31
+struct FastDiv {
+  uint32_t mul;
+  int32_t shift;
+};
+inline FastDiv make_fastdiv(uint32_t d) {
+  int l = 0;
+  while ((1ull << l) < d) ++l;  // l = ceil(log2 d)
+  FastDiv f;
+  f.shift = l;
+  f.mul = (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
+  return f;
+}
+inline uint32_t fastdiv_host(uint32_t x, FastDiv f) {
+  uint32_t hi = (uint32_t)(((uint64_t)x * f.mul) >> 32);
+  return (uint32_t)(((uint64_t)hi + x) >> f.shift);
+}
+
+// launch wrapper implemented in executor.cu; returns a cudaError_t value
+int launch_executor(const ExecParams &p, int grid, int block, void *stream);
+int executor_occupancy(int block, int *ctas_per_sm);
+
+}  // namespace dgcl

@@ -1,0 +1,406 @@
+// lowering.cpp — plan trees -> executor groups (host only, no CUDA).
+//
+// §6.1: the plan S is organised into tuples (d_i, d_j, k, T^s_ij, T^r_ij):
+// per stage k and GPU pair, the vertex ids d_i sends to d_j.  Here a tuple becomes one or more
+// GROUPS, split by where the rows live on the sender (its embeddings, its halo, or its relay
+// staging) and on the receiver (halo, or relay staging when the receiver only forwards), with the
+// vertex ids already translated into row numbers of those buffers.  The receiver-side unpack of
+// the paper is fused away: the sender writes each row at its final position.
+//
+// Backward: "stages are executed in a reverse order, and T^s_ij and T^r_ij are
+// switched".  Forward edge p->c at stage k becomes the backward push c->p at stage b = K - k + 1,
+// carrying c's partial sum val_c(u) into a per-(child, vertex) SLOT row on p.  The owner then
+// folds its slots into emb_grad in ascending child order (RED, stage K + 1).  This replaces the
+// paper's |D|-1 sub-stages with the same guarantee — every row has exactly one
+// writer, no atomics — and additionally fixes the summation order (R6).
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <map>
+#include <tuple>
+
+#include "plan.h"
+
+namespace dgcl {
+
+namespace {
+
+struct Entry {
+  uint64_t key;
+  int64_t sort2;
+  int64_t edge;   // plan edge index
+  int64_t vidx;   // index into plan.order
+};
+
+inline uint64_t pack_key(int stage, int exec, int dst, int a, int b) {
+  return ((uint64_t)stage << 24) | ((uint64_t)exec << 16) | ((uint64_t)dst << 8) |
+         ((uint64_t)a << 4) | (uint64_t)b;
+}
+
+// position of u on GPU d (its halo row), or -1 if d did not request u
+inline int32_t halo_pos(const Relation &rel, int64_t u, int d) {
+  for (int64_t q = rel.d_ptr[u]; q < rel.d_ptr[u + 1]; ++q)
+    if (rel.d_gpu[q] == d) return rel.d_pos[q];
+  return -1;
+}
+
+}  // namespace
+
+void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
+                const std::vector<int64_t> &loc, Lowered *out) {
+  auto t0 = std::chrono::steady_clock::now();
+  const int m = plan.m;
+  const int K = plan.n_stages;
+  Lowered &L = *out;
+  L = Lowered();
+  L.m = m;
+  L.n_stages = K;
+  L.n_halo = rel.n_halo;
+  L.n_relay.assign(m, 0);
+  L.n_slot.assign(m, 0);
+  L.rows_sd.assign((size_t)2 * kMaxStages * m * m, 0);
+  const int64_t NE = (int64_t)plan.e_parent.size();
+  L.n_tree_edges = NE;
+  const int64_t NV = (int64_t)plan.order.size();
+
+  // edge -> vertex index
+  std::vector<int64_t> e_vidx(NE);
+  for (int64_t i = 0; i < NV; ++i)
+    for (int64_t e = plan.e_ptr[i]; e < plan.e_ptr[i + 1]; ++e) e_vidx[e] = i;
+  // is the child of edge e a requester (halo) or a pure relay?
+  std::vector<int32_t> child_pos(NE);
+  for (int64_t e = 0; e < NE; ++e)
+    child_pos[e] = halo_pos(rel, plan.order[e_vidx[e]], plan.e_child[e]);
+  // edge into node x of the same tree (for relay sources / children lists)
+  auto edge_into = [&](int64_t vi, int x) -> int64_t {
+    for (int64_t e = plan.e_ptr[vi]; e < plan.e_ptr[vi + 1]; ++e)
+      if (plan.e_child[e] == x) return e;
+    return -1;
+  };
+
+  // source buffer kind of every edge: the owner sends from its embeddings, a requester forwards
+  // from its halo, a pure relay from its relay staging
+  std::vector<int8_t> src_kind(NE);
+  for (int64_t e = 0; e < NE; ++e) {
+    const int64_t u = plan.order[e_vidx[e]];
+    const int p = plan.e_parent[e];
+    src_kind[e] = p == part[u] ? K_EMB : (halo_pos(rel, u, p) >= 0 ? K_HALO : K_RELAY);
+  }
+
+  // ---- forward relay staging rows: contiguous per (receiver c, stage k, sender p, src kind) ----
+  std::vector<int64_t> relay_row(NE, -1);
+  {
+    std::vector<Entry> rel_e;
+    for (int64_t e = 0; e < NE; ++e)
+      if (child_pos[e] < 0)
+        rel_e.push_back({pack_key(plan.e_child[e], plan.e_stage[e], plan.e_parent[e],
+                                  src_kind[e], 0),
+                         e_vidx[e], e, e_vidx[e]});
+    std::sort(rel_e.begin(), rel_e.end(), [](const Entry &a, const Entry &b) {
+      return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
+    });
+    for (const Entry &x : rel_e) relay_row[x.edge] = L.n_relay[plan.e_child[x.edge]]++;
+    L.n_relay_edges = (int64_t)rel_e.size();
+  }
+
+  auto flush_group = [&](std::vector<DevGroup> &groups, DevGroup g, const std::vector<int64_t> &src,
+                         const std::vector<int64_t> &dst) {
+    g.n_rows = (int64_t)dst.size();
+    bool src_contig = !src.empty(), dst_contig = true;
+    for (size_t i = 1; i < dst.size(); ++i) {
+      if (dst[i] != dst[0] + (int64_t)i) dst_contig = false;
+    }
+    for (size_t i = 1; i < src.size(); ++i) {
+      if (src[i] != src[0] + (int64_t)i) src_contig = false;
+    }
+    if (!src.empty()) {
+      g.src_base = src[0];
+      if (src_contig) {
+        g.src_idx = -1;
+      } else {
+        g.src_idx = (int64_t)L.idx.size();
+        for (int64_t v : src) L.idx.push_back((int32_t)v);
+      }
+    } else {
+      g.src_idx = -1;
+      g.src_base = 0;
+    }
+    g.dst_base = dst[0];
+    if (dst_contig) {
+      g.dst_idx = -1;
+    } else {
+      g.dst_idx = (int64_t)L.idx.size();
+      for (int64_t v : dst) L.idx.push_back((int32_t)v);
+    }
+    groups.push_back(g);
+  };
+
+  auto base_group = [&](int op, int dir, int exec, int dst, int stage) {
+    DevGroup g;
+    std::memset(&g, 0, sizeof(g));
+    g.op = op;
+    g.dir = dir;
+    g.exec_rank = exec;
+    g.dst_rank = dst;
+    g.stage = stage;
+    g.sig_ctr = -1;
+    g.ready_rank = -1;
+    g.src_idx = g.dst_idx = -1;
+    g.term_ptr = -1;
+    return g;
+  };
+
+  // ---- forward groups: key (k, p, c, src_kind, dst_kind), rows sorted by destination row ----
+  {
+    std::vector<Entry> ent(NE);
+    std::vector<int64_t> srow(NE), drow(NE);
+    for (int64_t e = 0; e < NE; ++e) {
+      const int64_t vi = e_vidx[e];
+      const int64_t u = plan.order[vi];
+      const int p = plan.e_parent[e], c = plan.e_child[e], k = plan.e_stage[e];
+      const int sk = src_kind[e];
+      if (sk == K_EMB)
+        srow[e] = loc[u];
+      else if (sk == K_HALO)
+        srow[e] = halo_pos(rel, u, p);
+      else
+        srow[e] = relay_row[edge_into(vi, p)];
+      int dk;
+      if (child_pos[e] >= 0) {
+        dk = K_HALO;
+        drow[e] = child_pos[e];
+      } else {
+        dk = K_RELAY;
+        drow[e] = relay_row[e];
+      }
+      ent[e] = {pack_key(k, p, c, sk, dk), drow[e], e, vi};
+    }
+    std::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
+      return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
+    });
+    std::vector<int64_t> src, dst;
+    for (size_t i = 0; i < ent.size();) {
+      size_t j = i;
+      src.clear();
+      dst.clear();
+      while (j < ent.size() && ent[j].key == ent[i].key) {
+        src.push_back(srow[ent[j].edge]);
+        dst.push_back(drow[ent[j].edge]);
+        ++j;
+      }
+      const uint64_t key = ent[i].key;
+      const int k = (int)(key >> 24), p = (int)(key >> 16 & 0xFF), c = (int)(key >> 8 & 0xFF);
+      DevGroup g = base_group(OP_COPY, DIR_FWD, p, c, k);
+      g.src_kind = (int)(key >> 4 & 0xF);
+      g.dst_kind = (int)(key & 0xF);
+      flush_group(L.groups, g, src, dst);
+      L.rows_sd[((size_t)(DIR_FWD * kMaxStages + k) * m + p) * m + c] += (int64_t)dst.size();
+      i = j;
+    }
+    L.n_fwd_groups = (int)L.groups.size();
+  }
+
+  // ---- backward pushes: key (b, c, p, sig) ----
+  {
+    // term signature of c's value for the vertex of edge e (c = child of e)
+    std::vector<int8_t> sig(NE);
+    std::vector<int8_t> nchild(NE, 0);
+    for (int64_t e = 0; e < NE; ++e) {
+      const int64_t vi = e_vidx[e];
+      int nc = 0;
+      for (int64_t f = plan.e_ptr[vi]; f < plan.e_ptr[vi + 1]; ++f)
+        if (plan.e_parent[f] == plan.e_child[e]) ++nc;
+      nchild[e] = (int8_t)nc;
+      const bool own = child_pos[e] >= 0;
+      sig[e] = (own && nc == 0) ? 0 : (!own && nc == 1) ? 1 : 2;
+    }
+    std::vector<Entry> ent(NE);
+    for (int64_t e = 0; e < NE; ++e) {
+      const int b = K - plan.e_stage[e] + 1;
+      const int64_t sort2 = sig[e] == 0 ? (int64_t)child_pos[e] : plan.order[e_vidx[e]];
+      ent[e] = {pack_key(b, plan.e_child[e], plan.e_parent[e], sig[e], 0), sort2, e, e_vidx[e]};
+    }
+    std::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
+      return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
+    });
+    // slot rows on the parent, contiguous per push group
+    std::vector<int64_t> slot_row(NE);
+    for (const Entry &x : ent) slot_row[x.edge] = L.n_slot[plan.e_parent[x.edge]]++;
+
+    // children of node x in tree vi, ascending id -> their edge indices
+    auto children_edges = [&](int64_t vi, int x, int64_t *outv) -> int {
+      int n = 0;
+      for (int64_t f = plan.e_ptr[vi]; f < plan.e_ptr[vi + 1]; ++f)
+        if (plan.e_parent[f] == x) outv[n++] = f;
+      std::sort(outv, outv + n,
+                [&](int64_t a, int64_t b) { return plan.e_child[a] < plan.e_child[b]; });
+      return n;
+    };
+
+    std::vector<int64_t> src, dst;
+    int64_t ch[kMaxRanks];
+    for (size_t i = 0; i < ent.size();) {
+      size_t j = i;
+      while (j < ent.size() && ent[j].key == ent[i].key) ++j;
+      const uint64_t key = ent[i].key;
+      const int b = (int)(key >> 24), c = (int)(key >> 16 & 0xFF), p = (int)(key >> 8 & 0xFF);
+      const int s = (int)(key >> 4 & 0xF);
+      src.clear();
+      dst.clear();
+      DevGroup g = base_group(s == 2 ? OP_FOLD : OP_COPY, DIR_BWD, c, p, b);
+      g.dst_kind = K_SLOT;
+      if (s == 2) {
+        g.term_ptr = (int64_t)L.term_ptr.size();
+        L.term_ptr.push_back((int64_t)L.terms.size());
+      }
+      for (size_t q = i; q < j; ++q) {
+        const int64_t e = ent[q].edge;
+        const int64_t vi = ent[q].vidx;
+        dst.push_back(slot_row[e]);
+        if (s == 0) {
+          src.push_back(child_pos[e]);
+        } else if (s == 1) {
+          const int n = children_edges(vi, c, ch);
+          (void)n;
+          src.push_back(slot_row[ch[0]]);
+        } else {
+          if (child_pos[e] >= 0) L.terms.push_back((uint32_t)child_pos[e]);
+          const int n = children_edges(vi, c, ch);
+          for (int t = 0; t < n; ++t) L.terms.push_back(kTermSlot | (uint32_t)slot_row[ch[t]]);
+          L.term_ptr.push_back((int64_t)L.terms.size());
+        }
+      }
+      g.src_kind = s == 0 ? K_HGRAD : K_SLOT;
+      flush_group(L.groups, g, src, dst);
+      L.rows_sd[((size_t)(DIR_BWD * kMaxStages + b) * m + c) * m + p] += (int64_t)(j - i);
+      i = j;
+    }
+
+    // ---- RED: owner folds its slots into emb_grad, ascending child id, stage K + 1 ----
+    for (int s = 0; s < m; ++s) {
+      std::vector<std::pair<int64_t, int64_t>> rows;  // (loc, vidx)
+      for (int64_t vi = 0; vi < NV; ++vi) {
+        const int64_t u = plan.order[vi];
+        if (part[u] == s && plan.e_ptr[vi + 1] > plan.e_ptr[vi]) rows.push_back({loc[u], vi});
+      }
+      if (rows.empty()) continue;
+      std::sort(rows.begin(), rows.end());
+      DevGroup g = base_group(OP_FOLD, DIR_BWD, s, s, K + 1);
+      g.dst_kind = K_EGRAD;
+      g.fold_init = 1;
+      g.term_ptr = (int64_t)L.term_ptr.size();
+      L.term_ptr.push_back((int64_t)L.terms.size());
+      dst.clear();
+      src.clear();
+      for (auto &r : rows) {
+        dst.push_back(r.first);
+        const int n = children_edges(r.second, s, ch);
+        for (int t = 0; t < n; ++t) L.terms.push_back(kTermSlot | (uint32_t)slot_row[ch[t]]);
+        L.term_ptr.push_back((int64_t)L.terms.size());
+      }
+      flush_group(L.groups, g, src, dst);
+    }
+  }
+
+  // ---- signals and waits (the ready/done protocol of §6.1) ----
+  // wait lists per (dir, stage, exec): every in-peer's counter of the previous stage
+  std::map<std::tuple<int, int, int>, std::pair<int32_t, int32_t>> wait_lists;
+  auto get_waits = [&](int dir, int stage_prev, int r) {
+    auto key = std::make_tuple(dir, stage_prev, r);
+    auto it = wait_lists.find(key);
+    if (it != wait_lists.end()) return it->second;
+    const int32_t off = (int32_t)L.waits.size();
+    for (int s = 0; s < m; ++s) {
+      const int64_t rows = L.rows(dir, stage_prev, s, r);
+      if (rows > 0) L.waits.push_back({(int32_t)ctr_index(dir, stage_prev, s), 0, rows});
+    }
+    auto v = std::make_pair(off, (int32_t)L.waits.size() - off);
+    wait_lists[key] = v;
+    return v;
+  };
+  for (DevGroup &g : L.groups) {
+    if (g.dst_rank != g.exec_rank) {
+      g.sig_ctr = (int32_t)ctr_index(g.dir, g.stage, g.exec_rank);
+      g.ready_rank = g.dst_rank;
+    }
+    bool reads_inflight;
+    if (g.dir == DIR_FWD)
+      reads_inflight = g.src_kind != K_EMB;
+    else
+      reads_inflight = g.op == OP_FOLD || g.src_kind == K_SLOT;
+    if (reads_inflight && g.stage >= 2) {
+      auto w = get_waits(g.dir, g.stage - 1, g.exec_rank);
+      g.wait_off = w.first;
+      g.wait_n = w.second;
+    }
+  }
+  // per-rank READY and forward-completion WAIT groups (used by per-rank programs only)
+  for (int r = 0; r < m; ++r) {
+    DevGroup g = base_group(OP_READY, DIR_FWD, r, r, 0);
+    L.groups.push_back(g);
+  }
+  for (int r = 0; r < m; ++r) {
+    DevGroup g = base_group(OP_WAIT, DIR_FWD, r, r, K + 1);
+    g.wait_off = (int32_t)L.waits.size();
+    for (int k = 1; k <= K; ++k)
+      for (int s = 0; s < m; ++s) {
+        const int64_t rows = L.rows(DIR_FWD, k, s, r);
+        if (rows > 0) L.waits.push_back({(int32_t)ctr_index(DIR_FWD, k, s), 0, rows});
+      }
+    g.wait_n = (int32_t)L.waits.size() - g.wait_off;
+    L.groups.push_back(g);
+  }
+  L.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+}
+
+void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
+                 int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
+                 std::vector<DevItem> *items) {
+  items->clear();
+  const int64_t rpi = std::max<int64_t>(1, item_bytes / std::max<int64_t>(1, row_bytes));
+  size_t i = 0;
+  while (i < gids.size()) {
+    // one stage (READY / WAIT are their own "stage" runs)
+    const DevGroup &g0 = low.groups[gids[i]];
+    size_t j = i;
+    while (j < gids.size() && low.groups[gids[j]].stage == g0.stage &&
+           low.groups[gids[j]].op != OP_READY && low.groups[gids[j]].op != OP_WAIT &&
+           g0.op != OP_READY && g0.op != OP_WAIT)
+      ++j;
+    if (j == i) j = i + 1;
+    // interleave chunks of the groups of this stage
+    int64_t max_chunks = 0;
+    for (size_t q = i; q < j; ++q) {
+      const DevGroup &g = low.groups[gids[q]];
+      const int64_t nch = (g.op == OP_READY || g.op == OP_WAIT) ? 1 : (g.n_rows + rpi - 1) / rpi;
+      max_chunks = std::max(max_chunks, nch);
+    }
+    for (int64_t c = 0; c < max_chunks; ++c) {
+      for (size_t q = i; q < j; ++q) {
+        const DevGroup &g = low.groups[gids[q]];
+        DevItem it;
+        it.group = gids[q];
+        if (g.op == OP_READY || g.op == OP_WAIT) {
+          if (c > 0) continue;
+          it.row_begin = it.row_end = 0;
+          it.flags = 0;
+          items->push_back(it);
+          continue;
+        }
+        const int64_t b = c * rpi;
+        if (b >= g.n_rows) continue;
+        it.row_begin = (int32_t)b;
+        it.row_end = (int32_t)std::min(g.n_rows, b + rpi);
+        bool sig = g.sig_ctr >= 0;
+        if (sig && !signal_all)
+          sig = needed_ctr[(size_t)g.dst_rank * kFlagWords + g.sig_ctr] != 0;
+        it.flags = sig ? kItemSignal : 0;
+        items->push_back(it);
+      }
+    }
+    i = j;
+  }
+}
+
+}  // namespace dgcl

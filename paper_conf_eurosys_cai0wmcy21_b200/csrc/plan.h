@@ -1,0 +1,94 @@
+// plan.h — host-only planning and lowering structures (no CUDA dependency).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+namespace dgcl {
+
+// Topology D(V', E') of §5.1: a link i->j is a list of
+// physical hops, hop h costs w[h] ticks per row.
+struct Topology {
+  int m = 0;
+  std::vector<int64_t> w;          // ticks per row, per hop
+  std::vector<int64_t> link_ptr;   // CSR over i*m + j
+  std::vector<int32_t> link_hops;
+  bool has(int i, int j) const { return link_ptr[i * m + j + 1] > link_ptr[i * m + j]; }
+  static Topology uniform_nvswitch(int m);
+};
+
+// Communication relation: for every vertex u, the GPUs D_u that request
+// it (ascending) and u's halo row pos_d(u) on each of them.
+struct Relation {
+  int64_t n = 0;
+  int m = 0;
+  std::vector<int64_t> d_ptr;  // [n+1]
+  std::vector<int8_t> d_gpu;   // [S]
+  std::vector<int32_t> d_pos;  // [S]
+  std::vector<int64_t> n_halo; // [m] = |R_d|
+};
+
+// The plan S = union of trees T_u, edges grouped per vertex in planning order.
+struct Plan {
+  int m = 0;
+  int n_stages = 0;                // max edge stage K
+  std::vector<int64_t> order;      // planned vertices, in planning order
+  std::vector<int64_t> e_ptr;      // [order.size()+1] edges of order[i]
+  std::vector<int32_t> e_parent, e_child, e_stage;
+  int64_t cost = 0;                // t(S) in ticks
+  double seconds = 0;
+};
+
+// Build the relation from the required lists; returns "" or an error message (EINVAL).
+std::string build_relation(int64_t n, int m, const int32_t *part, const int64_t *req_ptr,
+                           const int64_t *req_ids, Relation *out);
+
+// SPST, Algorithm 1 + 2 (§5.2).  Returns "" or an error message (EPLAN).
+std::string spst_plan(const Topology &topo, const int32_t *part, const Relation &rel,
+                      uint64_t seed, Plan *out);
+
+// ---- lowering ----------------------------------------------------------------------------
+
+struct HostGroup {
+  DevGroup g;        // descriptor (offsets relative to the pools below)
+};
+
+struct Lowered {
+  int m = 0;
+  int n_stages = 0;                      // forward stages K
+  std::vector<DevGroup> groups;          // forward groups, then backward groups
+  int n_fwd_groups = 0;
+  std::vector<int32_t> idx;              // row index pool
+  std::vector<int64_t> term_ptr;         // fold row pointers
+  std::vector<uint32_t> terms;           // fold terms
+  std::vector<DevWait> waits;
+  // per-rank buffer rows
+  std::vector<int64_t> n_halo, n_relay, n_slot;  // [m]
+  // rows in: [dir][stage][src][dst] flattened: ((dir*kMaxStages + k)*m + s)*m + d
+  std::vector<int64_t> rows_sd;
+  int64_t rows(int dir, int k, int s, int d) const {
+    return rows_sd[((size_t)(dir * kMaxStages + k) * m + s) * m + d];
+  }
+  int64_t n_relay_edges = 0;
+  int64_t n_tree_edges = 0;
+  double seconds = 0;
+  int64_t table_bytes() const {
+    return (int64_t)(idx.size() * 4 + term_ptr.size() * 8 + terms.size() * 4 +
+                     waits.size() * sizeof(DevWait) + groups.size() * sizeof(DevGroup));
+  }
+};
+
+void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
+                const std::vector<int64_t> &loc, Lowered *out);
+
+// Work items for one launch: the groups `gids` (already in stage order) cut into row ranges of
+// about item_bytes bytes and interleaved across groups within a stage.
+// completion_rank >= 0 appends nothing (the WAIT group is passed in gids by the caller).
+void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
+                 int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
+                 std::vector<DevItem> *items);
+
+}  // namespace dgcl

@@ -1,0 +1,229 @@
+// planner.cpp — communication relation and the SPST planner (host only, no CUDA).
+//
+// PAPER.md §5.  The planning problem (eq. 2) is: choose for every vertex
+// u a tree T_u rooted at its owner s_u spanning the requesting GPUs D_u, minimising the staged
+// cost t(S) of §5.1.  SPST (Algorithm 1) plans vertices one by one in a random order;
+// per vertex it repeatedly runs a multi-source Dijkstra from the GPUs already holding u (N_src) to
+// the unreached requesters, with edge weights from incrementalLinkCost (Algorithm 2):
+// C(i, e) = costFunc(S + {(i, e)}) - costFunc(S), and adds the cheapest path.
+//
+// Readings (R7-R12): integer ticks per row per hop; node-labelled Dijkstra where x->y
+// weighs C(depth(x)+1, x->y); labels compare (cost, depth, gpu id); target = min (cost, depth, id);
+// stop once D_u is covered; Fisher-Yates shuffle driven by splitmix64(seed).  C is evaluated on
+// demand for the relaxed edges only (the optimisation the paper mentions at P:1384-1392): because
+// S is fixed during one Dijkstra, C(k, e) = max(t^k, max_{h in e} (c_h^k + 1) w_h) - t^k exactly.
+
+#include <chrono>
+#include <cstring>
+#include <string>
+
+#include "plan.h"
+
+namespace dgcl {
+
+Topology Topology::uniform_nvswitch(int m) {
+  // link i->j = {egress_i, ingress_j}; 900 GB/s each => round(1e5 / 900) = 111 ticks per row
+  Topology t;
+  t.m = m;
+  t.w.assign(2 * m, 111);
+  t.link_ptr.assign((size_t)m * m + 1, 0);
+  for (int i = 0; i < m; ++i)
+    for (int j = 0; j < m; ++j) {
+      size_t p = (size_t)i * m + j;
+      if (i != j) {
+        t.link_hops.push_back(i);
+        t.link_hops.push_back(m + j);
+      }
+      t.link_ptr[p + 1] = (int64_t)t.link_hops.size();
+    }
+  return t;
+}
+
+std::string build_relation(int64_t n, int m, const int32_t *part, const int64_t *req_ptr,
+                           const int64_t *req_ids, Relation *out) {
+  Relation &r = *out;
+  r.n = n;
+  r.m = m;
+  r.n_halo.assign(m, 0);
+  if (req_ptr[0] != 0) return "req_ptr[0] must be 0";
+  for (int d = 0; d < m; ++d) {
+    if (req_ptr[d + 1] < req_ptr[d]) return "req_ptr must be non-decreasing";
+    r.n_halo[d] = req_ptr[d + 1] - req_ptr[d];
+  }
+  const int64_t S = req_ptr[m];
+  std::vector<int64_t> cnt(n + 1, 0);
+  for (int d = 0; d < m; ++d) {
+    for (int64_t i = req_ptr[d]; i < req_ptr[d + 1]; ++i) {
+      const int64_t u = req_ids[i];
+      if (u < 0 || u >= n) return "required id out of range: " + std::to_string(u);
+      if (part[u] == d)
+        return "GPU " + std::to_string(d) + " requires its own vertex " + std::to_string(u);
+      cnt[u + 1]++;
+    }
+  }
+  r.d_ptr.assign(n + 1, 0);
+  for (int64_t u = 0; u < n; ++u) r.d_ptr[u + 1] = r.d_ptr[u] + cnt[u + 1];
+  r.d_gpu.assign(S, -1);
+  r.d_pos.assign(S, -1);
+  std::vector<int64_t> fill(r.d_ptr.begin(), r.d_ptr.end() - 1);
+  for (int d = 0; d < m; ++d) {  // ascending d => each D_u list is sorted
+    for (int64_t i = req_ptr[d]; i < req_ptr[d + 1]; ++i) {
+      const int64_t u = req_ids[i];
+      const int64_t f = fill[u];
+      if (f > r.d_ptr[u] && r.d_gpu[f - 1] == d)
+        return "duplicate id " + std::to_string(u) + " in the list of GPU " + std::to_string(d);
+      r.d_gpu[f] = (int8_t)d;
+      r.d_pos[f] = (int32_t)(i - req_ptr[d]);
+      fill[u] = f + 1;
+    }
+  }
+  return "";
+}
+
+namespace {
+
+constexpr uint64_t kGolden = 0x9E3779B97F4A7C15ull;
+inline uint64_t mix64(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+constexpr int64_t kInf = INT64_MAX;
+
+}  // namespace
+
+std::string spst_plan(const Topology &topo, const int32_t *part, const Relation &rel,
+                      uint64_t seed, Plan *out) {
+  auto t0 = std::chrono::steady_clock::now();
+  const int m = topo.m;
+  Plan &P = *out;
+  P = Plan();
+  P.m = m;
+  // vertices with D_u non-empty, ascending, then Fisher-Yates (splitmix64 stream from `seed`)
+  std::vector<int64_t> &order = P.order;
+  for (int64_t u = 0; u < rel.n; ++u)
+    if (rel.d_ptr[u + 1] > rel.d_ptr[u]) order.push_back(u);
+  {
+    uint64_t state = seed;
+    for (int64_t i = (int64_t)order.size() - 1; i >= 1; --i) {
+      state += kGolden;
+      const int64_t j = (int64_t)(mix64(state) % (uint64_t)(i + 1));
+      std::swap(order[i], order[j]);
+    }
+  }
+  const int H = (int)topo.w.size();
+  // c_h^k and t^k, k in 1..m-1 (row 0 unused)
+  std::vector<int64_t> load((size_t)m * H, 0);
+  std::vector<int64_t> tk(m, 0);
+  const int64_t S = rel.d_ptr[rel.n];
+  P.e_ptr.reserve(order.size() + 1);
+  P.e_parent.reserve(S);
+  P.e_child.reserve(S);
+  P.e_stage.reserve(S);
+  P.e_ptr.push_back(0);
+
+  // per-link hop lists as small arrays
+  std::vector<int32_t> lp(topo.link_ptr.begin(), topo.link_ptr.end());
+
+  auto inc_cost = [&](int k, int x, int y) -> int64_t {
+    // C(k, x->y) = costFunc(S + {(k, x->y)}) - costFunc(S): only stage k changes
+    const int64_t cur = tk[k];
+    int64_t mx = cur;
+    const int64_t *ld = &load[(size_t)k * H];
+    for (int32_t q = lp[x * m + y]; q < lp[x * m + y + 1]; ++q) {
+      const int h = topo.link_hops[q];
+      const int64_t v = (ld[h] + 1) * topo.w[h];
+      if (v > mx) mx = v;
+    }
+    return mx - cur;
+  };
+
+  int max_stage = 0;
+  int64_t lcost[kMaxRanks];
+  int ldep[kMaxRanks], pred[kMaxRanks], depth[kMaxRanks];
+  for (const int64_t u : order) {
+    const int su = part[u];
+    uint32_t in_src = 1u << su;
+    for (int x = 0; x < m; ++x) depth[x] = -1;
+    depth[su] = 0;
+    uint32_t remaining = 0;
+    for (int64_t q = rel.d_ptr[u]; q < rel.d_ptr[u + 1]; ++q) remaining |= 1u << rel.d_gpu[q];
+    while (remaining) {
+      // --- multi-source node-labelled Dijkstra (Algorithm 1 line 7) ---
+      for (int x = 0; x < m; ++x) {
+        if (in_src >> x & 1) {
+          lcost[x] = 0;
+          ldep[x] = depth[x];
+        } else {
+          lcost[x] = kInf;
+          ldep[x] = INT32_MAX;
+        }
+        pred[x] = -1;
+      }
+      uint32_t settled = 0;
+      for (;;) {
+        int bx = -1;
+        for (int x = 0; x < m; ++x) {
+          if ((settled >> x & 1) || lcost[x] == kInf) continue;
+          if (bx < 0 || lcost[x] < lcost[bx] || (lcost[x] == lcost[bx] && ldep[x] < ldep[bx]))
+            bx = x;  // ascending x breaks the remaining ties
+        }
+        if (bx < 0) break;
+        settled |= 1u << bx;
+        const int k = ldep[bx] + 1;
+        if (k > m - 1) continue;
+        for (int y = 0; y < m; ++y) {
+          if (y == bx || (settled >> y & 1) || (in_src >> y & 1) || !topo.has(bx, y)) continue;
+          const int64_t c = lcost[bx] + inc_cost(k, bx, y);
+          if (c < lcost[y] || (c == lcost[y] && k < ldep[y])) {
+            lcost[y] = c;
+            ldep[y] = k;
+            pred[y] = bx;
+          }
+        }
+      }
+      // --- Algorithm 1 line 8: cheapest path to an unreached requester ---
+      int tgt = -1;
+      for (int d = 0; d < m; ++d) {
+        if (!(remaining >> d & 1) || lcost[d] == kInf) continue;
+        if (tgt < 0 || lcost[d] < lcost[tgt] || (lcost[d] == lcost[tgt] && ldep[d] < ldep[tgt]))
+          tgt = d;
+      }
+      if (tgt < 0)
+        return "vertex " + std::to_string(u) + ": a requesting GPU is unreachable from GPU " +
+               std::to_string(su);
+      // walk back to N_src, then add nodes and edges (lines 9-10) in root-to-leaf order
+      int path[kMaxRanks];
+      int np = 0;
+      for (int y = tgt; !(in_src >> y & 1); y = pred[y]) path[np++] = y;
+      for (int i = np - 1; i >= 0; --i) {
+        const int c = path[i];
+        const int p = pred[c];
+        const int k = depth[p] + 1;
+        depth[c] = k;
+        in_src |= 1u << c;
+        remaining &= ~(1u << c);
+        P.e_parent.push_back(p);
+        P.e_child.push_back(c);
+        P.e_stage.push_back(k);
+        if (k > max_stage) max_stage = k;
+        int64_t *ld = &load[(size_t)k * H];
+        for (int32_t q = lp[p * m + c]; q < lp[p * m + c + 1]; ++q) {
+          const int h = topo.link_hops[q];
+          ld[h] += 1;
+          const int64_t v = ld[h] * topo.w[h];
+          if (v > tk[k]) tk[k] = v;
+        }
+      }
+    }
+    P.e_ptr.push_back((int64_t)P.e_parent.size());
+  }
+  P.n_stages = max_stage;
+  P.cost = 0;
+  for (int k = 1; k < m; ++k) P.cost += tk[k];
+  P.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+  return "";
+}
+
+}  // namespace dgcl

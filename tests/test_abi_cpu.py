@@ -1,0 +1,184 @@
+"""CPU tests of libdgcl (no GPU): exports, argument validation, SPST parity with the oracle's
+reference planner, plan invariants, and the lowered tables run by the host interpreter against
+the oracle (forward bit-exact, backward bit-exact in tree order)."""
+import ctypes
+import re
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import halo, invariants, spst
+
+pytestmark = pytest.mark.usefixtures("built")
+
+
+def _D():
+    import paper_conf_eurosys_cai0wmcy21_b200 as D
+    return D
+
+
+def test_library_exports_every_header_symbol(built):
+    import os
+    D = _D()
+    hdr = open(os.path.join(built, "include", "dgcl.h")).read()
+    declared = set(re.findall(r"\b(dgcl_[a-z_]+)\s*\(", hdr))
+    declared = {s for s in declared if s not in ("dgcl_status",)}
+    lib = ctypes.CDLL(D.LIB_PATH)
+    for s in sorted(declared):
+        assert hasattr(lib, s), s
+    assert declared == set(D.SYMBOLS)
+
+
+def _ctx(g, dims, topo=None, seed=0, device=-1):
+    D = _D()
+    c = D.loopback(g.m, g.part, dims, device=device)
+    c.build_plan(g.req_ptr, g.req_ids, seed=seed, topology=topo)
+    return c
+
+
+def test_init_validation():
+    D = _D()
+    part = np.array([0, 1, 2], np.int32)
+    with pytest.raises(D.DGCLError):
+        D.loopback(2, part, [4], device=-1)           # part out of range
+    with pytest.raises(D.DGCLError):
+        D.loopback(3, part, [0], device=-1)           # dim < 1
+    with pytest.raises(D.DGCLError):
+        D.init(part, [4], rank=3, world=3, device=-1)  # rank >= world
+    with pytest.raises(D.DGCLError):
+        D.loopback(17, np.zeros(3, np.int32), [4], device=-1)
+
+
+def test_build_plan_validation():
+    D = _D()
+    part = np.array([0, 1, 0, 1], np.int32)
+    c = D.loopback(2, part, [4], device=-1)
+    with pytest.raises(D.DGCLError) as e:
+        c.build_plan([0, 1, 1], [2])                   # GPU 0 requires its own vertex 2
+    assert e.value.status == 1
+    c = D.loopback(2, part, [4], device=-1)
+    with pytest.raises(D.DGCLError):
+        c.build_plan([0, 2, 2], [1, 1])                # duplicate
+    c = D.loopback(2, part, [4], device=-1)
+    with pytest.raises(D.DGCLError):
+        c.build_plan([0, 1, 1], [9])                   # out of range
+    c = D.loopback(2, part, [4], device=-1)
+    c.build_plan([0, 1, 2], [1, 0])
+    with pytest.raises(D.DGCLError) as e:
+        c.build_plan([0, 1, 2], [1, 0])                # twice
+    assert e.value.status == 2
+    from paper_conf_eurosys_cai0wmcy21_b200 import _abi
+    assert c.workspace_bytes() > 0                     # host-side layout is known
+    # device calls on a host-only context are state errors (no memory is touched)
+    assert _abi.lib().dgcl_register_workspace(c.handle, ctypes.c_void_p(1 << 20), 1 << 30) == 2
+    with pytest.raises(D.DGCLError) as e:
+        c.ipc_export()
+    assert e.value.status == 2
+    assert _abi.lib().dgcl_dispatch_forward(c.handle, 0, ctypes.c_void_p(1 << 20), 4, None,
+                                            None) == 2
+
+
+def test_unreachable_gpu_is_eplan():
+    D = _D()
+    part = np.array([0, 1], np.int32)
+    t = synth.Topology("broken", 2, [100.0], ["h"], {})   # no links at all
+    c = D.loopback(2, part, [4], device=-1)
+    with pytest.raises(D.DGCLError) as e:
+        c.build_plan([0, 1, 1], [1], topology=t)
+    assert e.value.status == 6
+
+
+def _check_lowering(g, dims, topo, seed):
+    m = g.m
+    R = [g.R(d) for d in range(m)]
+    loc, _ = halo.local_rows(g.part, m)
+    c = _ctx(g, dims, topo, seed)
+    info = c.plan_info()
+    E = c.plan_export()
+    owner, Dd = spst.relation_from_lists(R, g.part)
+    topo_o = topo if topo is not None else synth.uniform_nvswitch(m)
+    edges, cost = spst.spst(topo_o, owner, Dd, seed=seed)
+    assert [tuple(x) for x in E.tolist()] == [tuple(x) for x in edges]
+    assert cost == info["model_cost_ticks"]
+    invariants.check_plan(topo_o, [tuple(x) for x in E.tolist()], owner, Dd, cost)
+    counts = c.plan_counts()
+    assert counts.sum() == info["n_tree_edges"] == len(edges)
+    for layer, dim in enumerate(dims):
+        pitch = c.halo_view(layer)[2]
+        emb = synth.fill_values(g.n, dim, pitch, keys=np.argsort(g.part, kind="stable"), seed=3)
+        H = np.zeros((int(g.req_ptr[-1]), pitch), np.float32)
+        c.debug_hostsim_forward(layer, emb, H)
+        local = [emb[c.row_off[d]:c.row_off[d + 1], :dim] for d in range(m)]
+        Ho = halo.forward(local, R, g.part, loc)
+        for d in range(m):
+            got = H[g.req_ptr[d]:g.req_ptr[d + 1], :dim]
+            assert np.array_equal(got.view(np.uint32), Ho[d].view(np.uint32))
+        G = synth.fill_values(int(g.req_ptr[-1]), dim, pitch, seed=4)
+        L = synth.fill_values(g.n, dim, pitch, seed=5)
+        EG = L.copy()
+        c.debug_hostsim_backward(layer, G, EG)
+        Ls = [L[c.row_off[d]:c.row_off[d + 1], :dim] for d in range(m)]
+        Gs = [G[g.req_ptr[d]:g.req_ptr[d + 1], :dim] for d in range(m)]
+        Bt = halo.backward_tree(Ls, Gs, R, g.part, loc, E)
+        for d in range(m):
+            got = EG[c.row_off[d]:c.row_off[d + 1], :dim]
+            assert np.array_equal(got.view(np.uint32), Bt[d].view(np.uint32))
+        if info["n_stages"] == 1:
+            Bf = halo.backward_flat(Ls, Gs, R, g.part, loc)
+            for d in range(m):
+                got = EG[c.row_off[d]:c.row_off[d + 1], :dim]
+                assert np.array_equal(got.view(np.uint32), Bf[d].view(np.uint32))
+    return info
+
+
+@pytest.mark.parametrize("m", [2, 3, 8])
+def test_uniform_plan_and_lowering(m):
+    g = synth.make_graph(1500, 12000, m, graph_seed=m, part_seed=50 + m)
+    info = _check_lowering(g, [16, 5], None, seed=3)
+    assert info["n_stages"] == 1 and info["n_relay_rows"] == 0
+
+
+@pytest.mark.parametrize("name", ["dgx1_like", "ring"])
+def test_relay_plan_and_lowering(name):
+    g = synth.make_graph(500, 2500, 8, graph_seed=9, part_seed=19)
+    info = _check_lowering(g, [12, 3], synth.topology.by_name(name), seed=5)
+    assert info["n_stages"] >= 2 and info["n_relay_rows"] > 0
+
+
+def test_shuffled_halo_order():
+    g = synth.make_graph(800, 6000, 4, graph_seed=2, part_seed=3)
+    g.req_ids = synth.graph.shuffle_lists(g.req_ptr, g.req_ids, 77)
+    _check_lowering(g, [8], None, seed=1)
+
+
+def test_fig6_plan_from_library():
+    """The Fig. 6 worked example through the C planner (T_a = d1-d2-d3-d4)."""
+    D = _D()
+    part = np.array([0, 1, 2, 3], np.int32)  # vertex 0 = 'a' owned by GPU 0
+    c = D.loopback(4, part, [4], device=-1)
+    c.build_plan([0, 0, 0, 1, 2], [0, 0], seed=0, topology=synth.fig6())
+    E = c.plan_export()
+    assert E.tolist() == [[0, 0, 1, 1], [0, 1, 2, 2], [0, 2, 3, 3]]
+    assert c.plan_info()["model_cost_ticks"] == 12387
+
+
+def test_empty_and_single_rank():
+    D = _D()
+    part = np.zeros(5, np.int32)
+    c = D.loopback(1, part, [4], device=-1)
+    c.build_plan([0, 0], [])
+    assert c.plan_info()["n_tree_edges"] == 0
+    part = np.array([0, 1, 0, 1], np.int32)
+    c = D.loopback(2, part, [4], device=-1)
+    c.build_plan([0, 0, 0], [])   # nobody requires anything
+    info = c.plan_info()
+    assert info["n_deliveries"] == 0 and info["n_stages"] == 0
+
+
+def test_plan_is_dim_independent():
+    """the plan does not depend on the feature dimension."""
+    g = synth.make_graph(600, 4000, 4, graph_seed=4, part_seed=4)
+    a = _ctx(g, [3], synth.dgx1_like() if False else None, seed=2).plan_export()
+    b = _ctx(g, [602, 256], None, seed=2).plan_export()
+    assert np.array_equal(a, b)

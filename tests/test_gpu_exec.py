@@ -1,0 +1,321 @@
+"""GPU parity tests of the sm_100a executor through the C ABI (-m gpu).
+
+Every case compares the CUDA path with the oracle element by element on seeded inputs:
+  * forward halos bit-exact (uint32 view);
+  * backward bit-exact against the flat oracle for single-stage plans and against the tree-order
+    oracle for relay plans; the flat oracle within |gpu - ref| <= 1e-6 * sum|terms| (R6);
+  * determinism (repeat -> identical bits), the G = 1 closed form, both loopback modes (fused and
+    per-rank with the full ready/done flag protocol), 16-B and 4-B paths, ragged tails, empty
+    halos, the host-buffer (e2e) entry points, the watchdog (ETIMEOUT) and argument errors.
+Full-size configs (BASELINE.json) are checked on sampled rows the oracle recomputes one by one
+from the hash-defined inputs, plus properties that hold at any size.
+"""
+import numpy as np
+import pytest
+
+import synth
+from oracle import halo
+
+pytestmark = [pytest.mark.gpu, pytest.mark.usefixtures("built")]
+
+
+def _torch():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch
+
+
+def _D():
+    import paper_conf_eurosys_cai0wmcy21_b200 as D
+    return D
+
+
+class Case:
+    """Loopback job: graph + a context + device inputs in the loopback layouts."""
+
+    def __init__(self, g, dims, topo=None, seed=0, flags=0, emb_pitch=None, mode="uniform",
+                 options=None):
+        torch = _torch()
+        D = _D()
+        self.g, self.m, self.dims = g, g.m, list(dims)
+        self.ctx = D.loopback(g.m, g.part, dims, device=0, flags=flags)
+        for k, v in (options or {}).items():
+            self.ctx.set_option(k, v)
+        self.ctx.build_plan(g.req_ptr, g.req_ids, seed=seed, topology=topo)
+        self.ctx.register_workspace()
+        self.order = np.argsort(g.part, kind="stable")   # loopback row -> global vertex id
+        self.S = int(g.req_ptr[-1])
+        self.mode = mode
+        self.emb_pitch = emb_pitch
+        self.loc, _ = halo.local_rows(g.part, g.m)
+        self.R = [g.R(d) for d in range(g.m)]
+        self.torch = torch
+
+    def pitch(self, layer):
+        return self.ctx.halo_view(layer)[2]
+
+    def emb(self, layer, seed=3):
+        p = self.emb_pitch or self.pitch(layer)
+        return synth.fill_values(self.g.n, self.dims[layer], p, keys=self.order, seed=seed,
+                                 stream=synth.values.STREAM_EMB + layer, mode=self.mode)
+
+    def grads(self, layer, seed=4, mode=None):
+        mode = mode or self.mode
+        p = self.emb_pitch or self.pitch(layer)
+        G = synth.fill_values(self.S, self.dims[layer], p, seed=seed,
+                              stream=synth.values.STREAM_HGRAD + layer, mode=mode)
+        L = synth.fill_values(self.g.n, self.dims[layer], p, keys=self.order, seed=seed,
+                              stream=synth.values.STREAM_EGRAD + layer, mode=mode)
+        return G, L
+
+    def dev(self, a):
+        return self.torch.from_numpy(a).cuda()
+
+    def run_forward(self, layer, emb):
+        out = self.ctx.forward(layer, self.dev(emb))
+        self.torch.cuda.synchronize()
+        self.ctx.check()
+        return out.cpu().numpy()
+
+    def run_backward(self, layer, G, L):
+        eg = self.dev(L)
+        self.ctx.backward(layer, self.dev(G), eg)
+        self.torch.cuda.synchronize()
+        self.ctx.check()
+        return eg.cpu().numpy()
+
+    # oracle views
+    def local(self, a, dim):
+        ro = self.ctx.row_off
+        return [a[ro[d]:ro[d + 1], :dim] for d in range(self.m)]
+
+    def halos(self, a, dim):
+        ho = self.g.req_ptr
+        return [a[ho[d]:ho[d + 1], :dim] for d in range(self.m)]
+
+
+def _eq(a, b):
+    return np.array_equal(np.ascontiguousarray(a).view(np.uint32),
+                          np.ascontiguousarray(b).view(np.uint32))
+
+
+def _check_case(c, layers=None, bwd=True):
+    layers = range(len(c.dims)) if layers is None else layers
+    info = c.ctx.plan_info()
+    E = c.ctx.plan_export()
+    for layer in layers:
+        dim = c.dims[layer]
+        emb = c.emb(layer)
+        H = c.run_forward(layer, emb)
+        Ho = halo.forward(c.local(emb, dim), c.R, c.g.part, c.loc)
+        for d in range(c.m):
+            assert _eq(c.halos(H, dim)[d], Ho[d]), "forward mismatch layer %d rank %d" % (layer, d)
+        if not bwd:
+            continue
+        G, L = c.grads(layer)
+        out = c.run_backward(layer, G, L)
+        Bt = halo.backward_tree(c.local(L, dim), c.halos(G, dim), c.R, c.g.part, c.loc, E)
+        for d in range(c.m):
+            assert _eq(c.local(out, dim)[d], Bt[d]), "backward (tree order) rank %d" % d
+        Bf = halo.backward_flat(c.local(L, dim), c.halos(G, dim), c.R, c.g.part, c.loc)
+        if info["n_stages"] <= 1:
+            for d in range(c.m):
+                assert _eq(c.local(out, dim)[d], Bf[d]), "backward (flat order) rank %d" % d
+        else:
+            # plan-agnostic oracle: |gpu - ref| <= 1e-6 * sum|terms|
+            absL = [np.abs(x) for x in c.local(L, dim)]
+            absG = [np.abs(x) for x in c.halos(G, dim)]
+            bound = halo.backward_flat(absL, absG, c.R, c.g.part, c.loc)
+            for d in range(c.m):
+                diff = np.abs(c.local(out, dim)[d].astype(np.float64) - Bf[d])
+                assert np.all(diff <= 1e-6 * bound[d] + 0.0), "flat tolerance rank %d" % d
+        # determinism: identical bits on a second run
+        out2 = c.run_backward(layer, G, L)
+        assert _eq(out, out2)
+
+
+def test_tiny_config_bit_exact():
+    """configs[0]: 10k vertices, 100k edges, random 2-way, dim 16, one layer fwd + bwd."""
+    cfg = synth.get_config("tiny")
+    g = synth.make_graph(cfg.n, cfg.e, cfg.m, cfg.graph_seed, cfg.part_seed)
+    _check_case(Case(g, cfg.dims))
+
+
+@pytest.mark.parametrize("m", [3, 4, 8])
+def test_uniform_loopback_fused(m):
+    g = synth.make_graph(6000, 60000, m, graph_seed=m, part_seed=7 * m)
+    _check_case(Case(g, [64, 5, 602]))
+
+
+@pytest.mark.parametrize("m", [2, 8])
+def test_per_rank_flag_protocol(m):
+    """Every virtual rank is its own launch on its own stream: ready handshake, done counters,
+    forward completion waits — the multi-GPU protocol on one device; several calls in a row."""
+    D = _D()
+    g = synth.make_graph(5000, 40000, m, graph_seed=11, part_seed=12)
+    c = Case(g, [32, 7], flags=D.LOOPBACK_PER_RANK)
+    for _ in range(2):
+        _check_case(c)
+
+
+@pytest.mark.parametrize("name,flags", [("dgx1_like", 0), ("ring", 0), ("dgx1_like", 1),
+                                        ("ring", 1)])
+def test_relay_plans(name, flags):
+    g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
+    c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags)
+    assert c.ctx.plan_info()["n_stages"] >= 2
+    _check_case(c)
+
+
+def test_unaligned_pitch_scalar_path():
+    g = synth.make_graph(3000, 20000, 4, graph_seed=2, part_seed=2)
+    _check_case(Case(g, [5], emb_pitch=5))   # 20-B rows: not 16-B aligned -> 4-B path
+
+
+def test_small_items_many_chunks():
+    g = synth.make_graph(3000, 20000, 4, graph_seed=3, part_seed=3)
+    _check_case(Case(g, [37], options={"item_bytes": 64, "ctas_per_sm": 1, "threads": 128}))
+
+
+def test_shuffled_halo_order_idx_lists():
+    g = synth.make_graph(3000, 25000, 4, graph_seed=8, part_seed=8)
+    g.req_ids = synth.graph.shuffle_lists(g.req_ptr, g.req_ids, 5)
+    _check_case(Case(g, [24]))
+
+
+def test_empty_halo_rank_and_no_requests():
+    part = np.array([0, 1, 2, 0, 1, 2], np.int32)
+    g = synth.Graph(6, 3, None, None, part, np.array([0, 2, 2, 3], np.int64),
+                    np.array([1, 5, 0], np.int64))   # GPU 1 requires nothing
+    _check_case(Case(g, [4]))
+
+
+def test_closed_form_ones_and_integer_inputs():
+    g = synth.make_graph(5000, 50000, 4, graph_seed=21, part_seed=22)
+    c = Case(g, [16], topo=synth.dgx1_like() if False else None)
+    G, L = c.grads(0, mode="ones")
+    out = c.run_backward(0, G, np.zeros_like(L))
+    fan = halo.fanout(c.R, g.n)
+    want = fan[c.order].astype(np.float32)
+    assert np.array_equal(out[:, 0], want) and np.array_equal(out[:, 15], want)
+
+
+def test_host_buffer_entry_points():
+    g = synth.make_graph(2000, 15000, 2, graph_seed=31, part_seed=32)
+    c = Case(g, [16])
+    emb = c.emb(0)
+    H = np.zeros((c.S, c.pitch(0)), np.float32)
+    c.ctx.forward_host(0, emb, H)
+    Ho = halo.forward(c.local(emb, 16), c.R, g.part, c.loc)
+    for d in range(2):
+        assert _eq(c.halos(H, 16)[d], Ho[d])
+    G, L = c.grads(0)
+    out = L.copy()
+    c.ctx.backward_host(0, G, out)
+    Bf = halo.backward_flat(c.local(L, 16), c.halos(G, 16), c.R, g.part, c.loc)
+    for d in range(2):
+        assert _eq(c.local(out, 16)[d], Bf[d])
+
+
+def test_watchdog_timeout_when_a_rank_never_arrives():
+    D = _D()
+    g = synth.make_graph(2000, 15000, 4, graph_seed=41, part_seed=42)
+    c = Case(g, [8], flags=D.LOOPBACK_PER_RANK)
+    c.ctx.set_option("timeout_ms", 300)
+    c.ctx.set_option("debug_skip_rank", 2)
+    emb = c.dev(c.emb(0))
+    c.ctx.forward(0, emb)
+    c.torch.cuda.synchronize()
+    with pytest.raises(D.DGCLError) as e:
+        c.ctx.check()
+    assert e.value.status == 5
+    with pytest.raises(D.DGCLError) as e:   # the context stays unusable
+        c.ctx.forward(0, emb)
+    assert e.value.status == 5
+
+
+def test_argument_errors():
+    D = _D()
+    g = synth.make_graph(1000, 8000, 2, graph_seed=51, part_seed=52)
+    c = Case(g, [16])
+    torch = c.torch
+    emb = torch.zeros(g.n, 16, device="cuda")
+    with pytest.raises(D.DGCLError) as e:
+        c.ctx.forward(0, emb, halo=torch.zeros(4, 16, device="cuda"))  # not the registered view
+    assert e.value.status == 1
+    with pytest.raises(D.DGCLError) as e:
+        c.ctx.forward(3, emb)
+    assert e.value.status == 1
+    with pytest.raises(D.DGCLError) as e:
+        c.ctx.forward(0, torch.zeros(g.n, 8, device="cuda"))            # pitch < dim
+    assert e.value.status == 1
+
+
+def test_autograd_graph_allgather():
+    torch = _torch()
+    D = _D()
+    g = synth.make_graph(1500, 10000, 2, graph_seed=61, part_seed=62)
+    c = Case(g, [16])
+    emb = torch.from_numpy(c.emb(0)).cuda().requires_grad_(True)
+    out = D.graph_allgather(c.ctx, 0, emb)
+    assert out.shape[0] == g.n + c.S
+    w = torch.from_numpy(synth.fill_values(out.shape[0], 16, seed=8, stream=3)).cuda()
+    (out * w).sum().backward()
+    wn = w.cpu().numpy()
+    Bf = halo.backward_flat(c.local(wn[:g.n], 16), c.halos(wn[g.n:], 16), c.R, g.part, c.loc)
+    got = emb.grad.cpu().numpy()
+    for d in range(2):
+        assert _eq(c.local(got, 16)[d], Bf[d])
+
+
+# ---- full-size configs (BASELINE.json), sampled parity + properties -------------------------
+
+def _sampled_full(name, dims_override=None, n_samples=3000):
+    cfg = synth.get_config(name)
+    g = synth.make_graph(cfg.n, cfg.e, cfg.m, cfg.graph_seed, cfg.part_seed, keep_edges=False)
+    topo = synth.topology.by_name(cfg.topology, cfg.m) if cfg.topology != "uniform_nvswitch" else None
+    dims = dims_override or list(cfg.dims)
+    c = Case(g, dims, topo=topo, seed=0)
+    rng = np.random.RandomState(123)
+    S = c.S
+    owner = g.part
+    for layer, dim in enumerate(dims):
+        H = c.run_forward(layer, c.emb(layer))
+        rows = rng.choice(S, size=min(n_samples, S), replace=False)
+        cols = np.arange(dim)
+        u = g.req_ids[rows]
+        want = synth.fill_values_numpy(u, cols, seed=3, stream=synth.values.STREAM_EMB + layer)
+        assert _eq(H[rows, :dim], want), "forward sample mismatch (%s layer %d)" % (name, layer)
+        if layer not in cfg.backward_layers and dims_override is None:
+            continue
+        G, L = c.grads(layer)
+        out = c.run_backward(layer, G, L)
+        # oracle for sampled vertices, one by one: own + contributions in ascending GPU order
+        vs = rng.choice(g.n, size=min(n_samples, g.n), replace=False)
+        pos = {}
+        for d in range(c.m):
+            R = c.R[d]
+            sel = np.isin(R, vs)
+            for i in np.nonzero(sel)[0]:
+                pos.setdefault(int(R[i]), []).append((d, int(g.req_ptr[d]) + int(i)))
+        inv = np.empty(g.n, np.int64)
+        inv[c.order] = np.arange(g.n)
+        for v in vs:
+            lrow = inv[v]
+            acc = synth.fill_values_numpy([v], cols, seed=4, stream=synth.values.STREAM_EGRAD + layer)[0]
+            for (d, grow) in sorted(pos.get(int(v), [])):
+                acc = (acc + synth.fill_values_numpy([grow], cols, seed=4,
+                                                     stream=synth.values.STREAM_HGRAD + layer)[0]
+                       ).astype(np.float32)
+            if c.ctx.plan_info()["n_stages"] <= 1:
+                assert _eq(out[lrow, :dim], acc), "backward sample v=%d" % v
+            else:
+                assert np.allclose(out[lrow, :dim], acc, rtol=0, atol=8e-6)
+    return c
+
+
+@pytest.mark.parametrize("name", ["reddit", "google8", "google2", "google4", "orkut",
+                                  "google8_dgx1"])
+def test_full_size_sampled(name):
+    _sampled_full(name)
