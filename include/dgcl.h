@@ -187,7 +187,9 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
 
 /* Options (before dgcl_register_workspace unless noted):
  *   "timeout_ms"     device watchdog for flag waits (default 20000; any time)
- *   "item_bytes"     target bytes per work item (default 65536)
+ *   "item_bytes"     target bytes of gathered operands per work item (default/max 98304)
+ *   "tma"            1 (default): bulk-copy (cp.async.bulk) gather executor when rows are 16-B
+ *                    aligned; 0: the register (LDG/STG) executor
  *   "ctas_per_sm"    executor CTAs per SM (default: occupancy, max 4)
  *   "threads"        executor CTA size (128..512, multiple of 32; default 512)
  *   "debug_skip_rank" fault injection for DGCL_LOOPBACK_PER_RANK contexts: never launch that

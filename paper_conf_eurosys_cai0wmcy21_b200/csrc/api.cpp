@@ -78,8 +78,9 @@ struct dgcl_ctx {
 
   uint64_t seq = 0, epoch[2] = {0, 0};
   int *err_host = nullptr, *err_dev = nullptr;
-  int threads = 512, ctas_per_sm = 0, grid = 0, n_sm = 0;
-  int64_t item_bytes = 65536, timeout_ms = 20000;
+  int threads = 512, ctas_per_sm = 0, grid = 0, n_sm = 0, tma_ctas = 0, use_tma = 1;
+  int64_t max_fold_slots = 1;
+  int64_t item_bytes = kTmaBufBytes, timeout_ms = 20000;
   std::vector<cudaStream_t> rank_streams;
   std::vector<cudaEvent_t> rank_events;
   cudaEvent_t fork_event = nullptr;
@@ -330,6 +331,12 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   P.seq = c->seq;
   P.timeout_ns = (uint64_t)c->timeout_ms * 1000000ull;
   P.err = c->err_dev;
+  P.row16 = (P.row_bytes + 15) / 16 * 16;
+  P.tma_buf = kTmaBufBytes;
+  // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage
+  P.use_tma = (v16 && c->use_tma && c->tma_ctas > 0 &&
+               c->max_fold_slots * P.row16 <= kTmaBufBytes) ? 1 : 0;
+  const int grid_all = P.use_tma ? c->n_sm * c->tma_ctas : c->grid;
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
   P.use_ready = (!fused && m > 1) ? 1 : 0;
   if (fused || !c->loopback) {
@@ -338,7 +345,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     if (pg.items.empty()) return DGCL_OK;
     P.items = c->d_items + pg.dev_off;
     P.n_items = (int32_t)pg.items.size();
-    const int grid = std::min<int64_t>(c->grid, (int64_t)pg.items.size());
+    const int grid = std::min<int64_t>(grid_all, (int64_t)pg.items.size());
     int e = launch_executor(P, grid, c->threads, stream);
     if (e != 0) return fail(c, DGCL_ECUDA, "executor launch failed: %s",
                             cudaGetErrorString((cudaError_t)e));
@@ -347,7 +354,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   }
   // loopback, one launch per virtual rank on its own stream (full flag protocol)
   CUDA_TRY(c, cudaEventRecord(c->fork_event, stream));
-  const int grid_r = std::max(1, c->grid / m);
+  const int grid_r = std::max(1, grid_all / m);
   for (int r = 0; r < m; ++r) {
     const Program &pg = c->progs[c->prog_index(layer, dir, r)];
     CUDA_TRY(c, cudaStreamWaitEvent(c->rank_streams[r], c->fork_event, 0));
@@ -438,6 +445,7 @@ dgcl_status dgcl_build_plan(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *
     for (int d = 0; d < c->world; ++d) c->halo_off[d + 1] = c->halo_off[d] + c->rel.n_halo[d];
     compute_layout(c);
     build_programs(c);
+    c->max_fold_slots = max_fold_slots(c->low);
   } catch (const std::bad_alloc &) {
     return fail(c, DGCL_ENOMEM, "host allocation failed while planning");
   }
@@ -494,7 +502,7 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   // launch geometry: persistent grid of co-resident CTAs
   CUDA_TRY(c, cudaDeviceGetAttribute(&c->n_sm, cudaDevAttrMultiProcessorCount, c->device));
   int occ = 0;
-  int e = executor_occupancy(c->threads, &occ);
+  int e = executor_occupancy(c->threads, &occ, &c->tma_ctas);
   if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");
   if (c->ctas_per_sm <= 0) c->ctas_per_sm = std::min(occ, 4);
   c->ctas_per_sm = std::max(1, std::min(c->ctas_per_sm, occ));
@@ -761,6 +769,10 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (value < 16) return fail(c, DGCL_EINVAL, "item_bytes too small");
     c->item_bytes = value;
     if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "tma") {
+    c->use_tma = value != 0;
     return DGCL_OK;
   }
   if (k == "ctas_per_sm") {

@@ -108,7 +108,13 @@ struct ExecParams {
   uint64_t seq;        // global call sequence number (ready words)
   uint64_t timeout_ns;
   int *err;            // host-mapped error word (0 = ok)
+  int32_t use_tma;     // 1: bulk-copy (TMA) gather into shared memory, then store from smem
+  int32_t row16;       // row bytes rounded up to 16 (bulk-copy size per row)
+  int32_t tma_buf;     // bytes per shared-memory stage buffer (two stages)
+  int32_t pad1;
 };
+
+constexpr int kTmaBufBytes = 96 * 1024;  // 2 stages -> 192 KB dynamic shared memory per CTA
 
 // fast unsigned division by a runtime constant d >= 1, exact for x < 2^31
 struct FastDiv {
@@ -130,6 +136,6 @@ inline uint32_t fastdiv_host(uint32_t x, FastDiv f) {
 
 // launch wrapper implemented in executor.cu; returns a cudaError_t value
 int launch_executor(const ExecParams &p, int grid, int block, void *stream);
-int executor_occupancy(int block, int *ctas_per_sm);
+int executor_occupancy(int block, int *ctas_per_sm, int *tma_ctas_per_sm);
 
 }  // namespace dgcl

@@ -357,11 +357,15 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
                  int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
                  std::vector<DevItem> *items) {
+  // An item is a row range whose gathered operands fit `item_bytes` (and one shared-memory stage
+  // of the bulk-copy executor): a COPY row costs one row, a FOLD row (1 + #terms) rows.
   items->clear();
-  const int64_t rpi = std::max<int64_t>(1, item_bytes / std::max<int64_t>(1, row_bytes));
+  const int64_t row16 = (row_bytes + 15) / 16 * 16;
+  const int64_t cap = std::max<int64_t>(row16, std::min<int64_t>(item_bytes, kTmaBufBytes));
   size_t i = 0;
+  std::vector<std::vector<int32_t>> bounds;  // per group of the stage: chunk start rows + end
   while (i < gids.size()) {
-    // one stage (READY / WAIT are their own "stage" runs)
+    // one stage (READY / WAIT are their own runs)
     const DevGroup &g0 = low.groups[gids[i]];
     size_t j = i;
     while (j < gids.size() && low.groups[gids[j]].stage == g0.stage &&
@@ -369,30 +373,45 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
            g0.op != OP_READY && g0.op != OP_WAIT)
       ++j;
     if (j == i) j = i + 1;
-    // interleave chunks of the groups of this stage
-    int64_t max_chunks = 0;
+    bounds.assign(j - i, std::vector<int32_t>());
+    size_t max_chunks = 0;
     for (size_t q = i; q < j; ++q) {
       const DevGroup &g = low.groups[gids[q]];
-      const int64_t nch = (g.op == OP_READY || g.op == OP_WAIT) ? 1 : (g.n_rows + rpi - 1) / rpi;
-      max_chunks = std::max(max_chunks, nch);
+      std::vector<int32_t> &b = bounds[q - i];
+      b.push_back(0);
+      if (g.op == OP_COPY) {
+        const int64_t rpi = std::max<int64_t>(1, cap / row16);
+        for (int64_t r = rpi; r < g.n_rows; r += rpi) b.push_back((int32_t)r);
+        b.push_back((int32_t)g.n_rows);
+      } else if (g.op == OP_FOLD) {
+        int64_t acc = 0;
+        for (int64_t r = 0; r < g.n_rows; ++r) {
+          const int64_t slots = low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r] +
+                                (g.fold_init ? 1 : 0);
+          const int64_t cost = slots * row16;
+          if (acc > 0 && acc + cost > cap) {
+            b.push_back((int32_t)r);
+            acc = 0;
+          }
+          acc += cost;
+        }
+        b.push_back((int32_t)g.n_rows);
+      } else {
+        b.push_back(0);  // READY / WAIT: one empty item
+      }
+      max_chunks = std::max(max_chunks, b.size() - 1);
     }
-    for (int64_t c = 0; c < max_chunks; ++c) {
+    // interleave the chunks of the groups of this stage (all peers / sources busy at once)
+    for (size_t c = 0; c < max_chunks; ++c) {
       for (size_t q = i; q < j; ++q) {
         const DevGroup &g = low.groups[gids[q]];
+        const std::vector<int32_t> &b = bounds[q - i];
+        if (c + 1 >= b.size()) continue;
         DevItem it;
         it.group = gids[q];
-        if (g.op == OP_READY || g.op == OP_WAIT) {
-          if (c > 0) continue;
-          it.row_begin = it.row_end = 0;
-          it.flags = 0;
-          items->push_back(it);
-          continue;
-        }
-        const int64_t b = c * rpi;
-        if (b >= g.n_rows) continue;
-        it.row_begin = (int32_t)b;
-        it.row_end = (int32_t)std::min(g.n_rows, b + rpi);
-        bool sig = g.sig_ctr >= 0;
+        it.row_begin = b[c];
+        it.row_end = b[c + 1];
+        bool sig = g.sig_ctr >= 0 && (g.op == OP_COPY || g.op == OP_FOLD);
         if (sig && !signal_all)
           sig = needed_ctr[(size_t)g.dst_rank * kFlagWords + g.sig_ctr] != 0;
         it.flags = sig ? kItemSignal : 0;
@@ -401,6 +420,17 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     }
     i = j;
   }
+}
+
+int64_t max_fold_slots(const Lowered &low) {
+  int64_t mx = 1;
+  for (const DevGroup &g : low.groups) {
+    if (g.op != OP_FOLD) continue;
+    for (int64_t r = 0; r < g.n_rows; ++r)
+      mx = std::max<int64_t>(mx, low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r] +
+                                     (g.fold_init ? 1 : 0));
+  }
+  return mx;
 }
 
 }  // namespace dgcl

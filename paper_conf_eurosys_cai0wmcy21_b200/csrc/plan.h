@@ -91,4 +91,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
                  int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
                  std::vector<DevItem> *items);
 
+// largest number of operand rows one FOLD row gathers (1 + #terms); bounds the bulk-copy stage
+int64_t max_fold_slots(const Lowered &low);
+
 }  // namespace dgcl

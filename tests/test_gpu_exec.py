@@ -142,10 +142,11 @@ def test_tiny_config_bit_exact():
     _check_case(Case(g, cfg.dims))
 
 
-@pytest.mark.parametrize("m", [3, 4, 8])
-def test_uniform_loopback_fused(m):
+@pytest.mark.parametrize("m,tma", [(3, 1), (4, 1), (8, 1), (4, 0), (8, 0)])
+def test_uniform_loopback_fused(m, tma):
+    """tma=1: bulk-copy (cp.async.bulk) gather executor; tma=0: the register (LDG) executor."""
     g = synth.make_graph(6000, 60000, m, graph_seed=m, part_seed=7 * m)
-    _check_case(Case(g, [64, 5, 602]))
+    _check_case(Case(g, [64, 5, 602], options={"tma": tma}))
 
 
 @pytest.mark.parametrize("m", [2, 8])
@@ -159,11 +160,13 @@ def test_per_rank_flag_protocol(m):
         _check_case(c)
 
 
-@pytest.mark.parametrize("name,flags", [("dgx1_like", 0), ("ring", 0), ("dgx1_like", 1),
-                                        ("ring", 1)])
-def test_relay_plans(name, flags):
+@pytest.mark.parametrize("name,flags,tma", [("dgx1_like", 0, 1), ("ring", 0, 1),
+                                            ("dgx1_like", 1, 1), ("ring", 1, 1),
+                                            ("ring", 0, 0), ("dgx1_like", 1, 0)])
+def test_relay_plans(name, flags, tma):
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
-    c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags)
+    c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags,
+             options={"tma": tma})
     assert c.ctx.plan_info()["n_stages"] >= 2
     _check_case(c)
 
