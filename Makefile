@@ -12,8 +12,8 @@ CXXFLAGS := -O3 -std=c++17 -fPIC -Wall -Wextra -Iinclude -I$(CUDA)/include
 CSRC     := $(PKG)/csrc
 HOST_SRC := $(CSRC)/planner.cpp $(CSRC)/lowering.cpp $(CSRC)/api.cpp $(CSRC)/hostsim.cpp
 HOST_OBJ := $(patsubst $(CSRC)/%.cpp,build/%.o,$(HOST_SRC))
-CU_SRC   := $(CSRC)/executor.cu
-CU_OBJ   := build/executor.o
+CU_SRC   := $(CSRC)/executor.cu $(CSRC)/executor_tma.cu
+CU_OBJ   := build/executor.o build/executor_tma.o
 HDRS     := include/dgcl.h $(wildcard $(CSRC)/*.h) $(wildcard $(CSRC)/*.cuh)
 
 .PHONY: all synth dgcl clean
@@ -28,9 +28,9 @@ build/%.o: $(CSRC)/%.cpp $(HDRS)
 	@mkdir -p build
 	$(CXX) $(CXXFLAGS) -c $< -o $@
 
-$(CU_OBJ): $(CU_SRC) $(HDRS)
+build/%.o: $(CSRC)/%.cu $(HDRS)
 	@mkdir -p build
-	$(NVCC) $(NVFLAGS) -Xptxas -v -c $< -o $@ 2> build/ptxas.log || (cat build/ptxas.log; false)
+	$(NVCC) $(NVFLAGS) -Xptxas -v -c $< -o $@ 2> build/$*.ptxas.log || (cat build/$*.ptxas.log; false)
 
 $(PKG)/libdgcl.so: $(HOST_OBJ) $(CU_OBJ)
 	$(NVCC) $(GENCODE) -shared -Xcompiler -fPIC -cudart static $^ -o $@

@@ -1,0 +1,144 @@
+// device_common.cuh — PTX helpers shared by the executor kernels (sm_100a).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "internal.h"
+
+namespace dgcl {
+namespace dev {
+
+constexpr int kUnroll = 4;
+
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(uint64_t *p, uint64_t v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_release_sys_add(uint64_t *p, uint64_t v) {
+  asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+__device__ __forceinline__ int4 ld_nc_v4(const void *p) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ int4 ld_cg_v4(const void *p) {
+  int4 r;
+  asm volatile("ld.global.cg.v4.s32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st_v4(void *p, const int4 &v) {
+  asm volatile("st.global.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ int ld_nc_b32(const void *p) {
+  int r;
+  asm volatile("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ int ld_cg_b32(const void *p) {
+  int r;
+  asm volatile("ld.global.cg.b32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st_b32(void *p, int v) {
+  asm volatile("st.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// partial 16-B chunk (a row's tail, nb in {4, 8, 12}): predicated 4-byte accesses
+template <bool kNC>
+__device__ __forceinline__ int4 ld_part(const char *p, int nb) {
+  int4 r = make_int4(0, 0, 0, 0);
+  r.x = kNC ? ld_nc_b32(p) : ld_cg_b32(p);
+  if (nb > 4) r.y = kNC ? ld_nc_b32(p + 4) : ld_cg_b32(p + 4);
+  if (nb > 8) r.z = kNC ? ld_nc_b32(p + 8) : ld_cg_b32(p + 8);
+  return r;
+}
+__device__ __forceinline__ void st_part(char *p, const int4 &v, int nb) {
+  st_b32(p, v.x);
+  if (nb > 4) st_b32(p + 4, v.y);
+  if (nb > 8) st_b32(p + 8, v.z);
+}
+
+// read-only user inputs (embeddings, halo gradients) take the non-coherent path
+__device__ __forceinline__ bool readonly_kind(int kind) { return kind == K_EMB || kind == K_HGRAD; }
+
+__device__ __forceinline__ float4 as_f4(const int4 &v) {
+  return make_float4(__int_as_float(v.x), __int_as_float(v.y), __int_as_float(v.z),
+                     __int_as_float(v.w));
+}
+__device__ __forceinline__ int4 as_i4(const float4 &a) {
+  return make_int4(__float_as_int(a.x), __float_as_int(a.y), __float_as_int(a.z),
+                   __float_as_int(a.w));
+}
+// one IEEE round-to-nearest fp32 add per lane (never contracted, never reassociated)
+__device__ __forceinline__ void add4(float4 &a, const int4 &b) {
+  a.x = __fadd_rn(a.x, __int_as_float(b.x));
+  a.y = __fadd_rn(a.y, __int_as_float(b.y));
+  a.z = __fadd_rn(a.z, __int_as_float(b.z));
+  a.w = __fadd_rn(a.w, __int_as_float(b.w));
+}
+
+// Spin until *p >= target (acquire, system scope), bounded by the watchdog.
+static __device__ __noinline__ bool wait_geq(const uint64_t *p, uint64_t target, const ExecParams &P,
+                                      int code) {
+  if (ld_acquire_sys(p) >= target) return true;
+  const uint64_t t0 = globaltimer();
+  for (uint32_t it = 1;; ++it) {
+    __nanosleep(64);
+    if (ld_acquire_sys(p) >= target) return true;
+    if ((it & 255) == 0) {
+      if (*(volatile int *)P.err != 0) return false;  // another CTA / peer already failed
+      if (globaltimer() - t0 > P.timeout_ns) {
+        atomicCAS(P.err, 0, code);
+        __threadfence_system();
+        return false;
+      }
+    }
+  }
+}
+
+// counter waits of a group (all of them, blocking)
+__device__ __forceinline__ bool wait_group_sources(const ExecParams &P, const DevGroup &G,
+                                                   int code) {
+  bool ok = true;
+  for (int w = 0; ok && w < G.wait_n; ++w) {
+    const DevWait W = P.waits[G.wait_off + w];
+    ok = wait_geq(P.flags[G.exec_rank] + W.ctr, P.epoch[G.dir] * (uint64_t)W.amount, P, code);
+  }
+  return ok;
+}
+
+// fast division by n_chunks (exact for x < 2^31)
+__device__ __forceinline__ uint32_t fdiv(uint32_t x, const ExecParams &P) {
+  return (__umulhi(x, P.div_mul) + x) >> P.div_shift;
+}
+
+__device__ __forceinline__ int64_t row_of(const int32_t *idx, int64_t base, int64_t i) {
+  return idx ? (int64_t)__ldg(idx + i) : base + i;
+}
+
+// receiver-visible completion of an item: every thread's stores, then one counter add
+__device__ __forceinline__ void release_rows(uint64_t *ctr, uint64_t rows, bool leader) {
+  if (leader) red_release_sys_add(ctr, rows);
+}
+
+}  // namespace dev
+}  // namespace dgcl

@@ -114,7 +114,7 @@ struct ExecParams {
   int32_t pad1;
 };
 
-constexpr int kTmaBufBytes = 96 * 1024;  // 2 stages -> 192 KB dynamic shared memory per CTA
+constexpr int kTmaBufBytes = 48 * 1024;  // per stage; 4 stages -> 192 KB dynamic shared memory per CTA
 
 // fast unsigned division by a runtime constant d >= 1, exact for x < 2^31
 struct FastDiv {
