@@ -74,6 +74,8 @@ struct dgcl_ctx {
   uint32_t *d_terms = nullptr;
   DevItem *d_items = nullptr;
   std::vector<Program> progs;  // index prog_index(layer, dir, r)
+  std::vector<int32_t> host_gids[2];  // group order of the host interpreter per direction
+  bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
   int n_prog_ranks = 1;        // programs per (layer, dir)
 
   uint64_t seq = 0, epoch[2] = {0, 0};
@@ -248,12 +250,32 @@ void build_programs(dgcl_ctx *c) {
       for (int gi = 0; gi < ng; ++gi) {
         const DevGroup &g = L.groups[gi];
         if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
+        if (gi >= L.direct_begin && gi < L.direct_end) continue;
         if (!fused && g.exec_rank != r) continue;
         gids[r].push_back(gi);
       }
       if (!fused && dir == DIR_FWD && m > 1) {
         for (int gi = 0; gi < ng; ++gi)
           if (L.groups[gi].op == OP_WAIT && L.groups[gi].exec_rank == r) gids[r].push_back(gi);
+      }
+    }
+    // fused loopback, single-stage plan: the owner folds its requesters' halo gradients in place
+    const bool direct = fused && dir == DIR_BWD && c->direct_reduce && L.n_stages <= 1 &&
+                        L.direct_end > L.direct_begin;
+    if (direct) {
+      gids[0].clear();
+      for (int gi = L.direct_begin; gi < L.direct_end; ++gi) gids[0].push_back(gi);
+    }
+    // the host interpreter runs the fused-order program of this direction
+    c->host_gids[dir].clear();
+    if (direct) {
+      c->host_gids[dir] = gids[0];
+    } else {
+      for (int gi = 0; gi < ng; ++gi) {
+        const DevGroup &g = L.groups[gi];
+        if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
+        if (gi >= L.direct_begin && gi < L.direct_end) continue;
+        c->host_gids[dir].push_back(gi);
       }
     }
     for (int l = 0; l < c->n_layers; ++l) {
@@ -335,7 +357,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   P.tma_buf = kTmaBufBytes;
   // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage
   P.use_tma = (v16 && c->use_tma && c->tma_ctas > 0 &&
-               c->max_fold_slots * P.row16 <= kTmaBufBytes) ? 1 : 0;
+               c->max_fold_slots * P.row16 <= kTmaOperandBytes) ? 1 : 0;
   const int grid_all = P.use_tma ? c->n_sm * c->tma_ctas : c->grid;
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
   P.use_ready = (!fused && m > 1) ? 1 : 0;
@@ -444,6 +466,8 @@ dgcl_status dgcl_build_plan(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *
     c->halo_off.assign(c->world + 1, 0);
     for (int d = 0; d < c->world; ++d) c->halo_off[d + 1] = c->halo_off[d] + c->rel.n_halo[d];
     compute_layout(c);
+    for (int d = 0; d < c->world; ++d)  // direct-reduce terms hold 28-bit halo rows
+      if (c->rel.n_halo[d] > (int64_t)kTermRowMask) c->direct_reduce = false;
     build_programs(c);
     c->max_fold_slots = max_fold_slots(c->low);
   } catch (const std::bad_alloc &) {
@@ -775,6 +799,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     c->use_tma = value != 0;
     return DGCL_OK;
   }
+  if (k == "direct_reduce") {
+    c->direct_reduce = value != 0;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
   if (k == "ctas_per_sm") {
     if (value < 1 || value > 32) return fail(c, DGCL_EINVAL, "ctas_per_sm out of range");
     c->ctas_per_sm = (int)value;
@@ -849,8 +878,8 @@ dgcl_status dgcl_debug_hostsim_forward(dgcl_ctx *c, int32_t layer, const float *
   if (!c || !emb || !halo) return DGCL_EINVAL;
   if (!c->planned || !c->loopback) return fail(c, DGCL_ESTATE, "needs a planned loopback context");
   if (layer < 0 || layer >= c->n_layers) return DGCL_EINVAL;
-  hostsim_run(c->low, DIR_FWD, c->row_off, c->halo_off, c->pitch[layer], c->dims[layer], emb, halo,
-              nullptr, nullptr);
+  hostsim_run(c->low, c->host_gids[DIR_FWD], c->row_off, c->halo_off, c->pitch[layer],
+              c->dims[layer], emb, halo, nullptr, nullptr);
   return DGCL_OK;
 }
 
@@ -859,8 +888,8 @@ dgcl_status dgcl_debug_hostsim_backward(dgcl_ctx *c, int32_t layer, const float 
   if (!c || !halo_grad || !emb_grad) return DGCL_EINVAL;
   if (!c->planned || !c->loopback) return fail(c, DGCL_ESTATE, "needs a planned loopback context");
   if (layer < 0 || layer >= c->n_layers) return DGCL_EINVAL;
-  hostsim_run(c->low, DIR_BWD, c->row_off, c->halo_off, c->pitch[layer], c->dims[layer], nullptr,
-              nullptr, halo_grad, emb_grad);
+  hostsim_run(c->low, c->host_gids[DIR_BWD], c->row_off, c->halo_off, c->pitch[layer],
+              c->dims[layer], nullptr, nullptr, halo_grad, emb_grad);
   return DGCL_OK;
 }
 

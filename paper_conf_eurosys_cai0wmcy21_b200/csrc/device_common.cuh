@@ -115,13 +115,13 @@ static __device__ __noinline__ bool wait_geq(const uint64_t *p, uint64_t target,
   }
 }
 
-// counter waits of a group (all of them, blocking)
-__device__ __forceinline__ bool wait_group_sources(const ExecParams &P, const DevGroup &G,
-                                                   int code) {
+// counter waits of an item (all of them, blocking): its source rows are final
+__device__ __forceinline__ bool wait_item_sources(const ExecParams &P, const DevItem &I,
+                                                  int code) {
   bool ok = true;
-  for (int w = 0; ok && w < G.wait_n; ++w) {
-    const DevWait W = P.waits[G.wait_off + w];
-    ok = wait_geq(P.flags[G.exec_rank] + W.ctr, P.epoch[G.dir] * (uint64_t)W.amount, P, code);
+  for (int w = 0; ok && w < I.wait_n; ++w) {
+    const DevWait W = P.waits[I.wait_off + w];
+    ok = wait_geq(P.flags[I.exec_rank] + W.ctr, P.epoch[I.dir] * (uint64_t)W.amount, P, code);
   }
   return ok;
 }

@@ -29,19 +29,21 @@ namespace {
 
 constexpr int kMaxFoldPrefetch = 4;
 
+__device__ __forceinline__ const int32_t *idx_of(const ExecParams &P, int64_t enc) {
+  return enc < 0 ? P.idx + ~enc : nullptr;
+}
+
 // ---- OP_COPY, 16-byte path ----------------------------------------------------------------
 template <bool kNC>
-__device__ __forceinline__ void copy_rows_v16(const ExecParams &P, const DevGroup &G,
-                                              int32_t rb, int32_t re) {
-  const char *sbase = P.buf[G.src_kind][G.exec_rank].ptr;
-  const int64_t spitch = P.buf[G.src_kind][G.exec_rank].pitch;
-  char *dbase = P.buf[G.dst_kind][G.dst_rank].ptr;
-  const int64_t dpitch = P.buf[G.dst_kind][G.dst_rank].pitch;
-  const int32_t *sidx = G.src_idx >= 0 ? P.idx + G.src_idx + rb : nullptr;
-  const int32_t *didx = G.dst_idx >= 0 ? P.idx + G.dst_idx + rb : nullptr;
-  const int64_t sb = G.src_base + rb, db = G.dst_base + rb;
+__device__ __forceinline__ void copy_rows_v16(const ExecParams &P, const DevItem &I) {
+  const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
+  const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
+  char *dbase = P.buf[I.dst_kind][I.dst_rank].ptr;
+  const int64_t dpitch = P.buf[I.dst_kind][I.dst_rank].pitch;
+  const int32_t *sidx = idx_of(P, I.src), *didx = idx_of(P, I.dst);
+  const int64_t sb = I.src, db = I.dst;
   const uint32_t nch = (uint32_t)P.n_chunks;
-  const uint32_t total = (uint32_t)(re - rb) * nch;
+  const uint32_t total = (uint32_t)I.rows * nch;
   const int tail = P.row_bytes - (int)(nch - 1) * 16;  // bytes in each row's last chunk (1..16)
   const uint32_t T = blockDim.x;
   for (uint32_t e0 = threadIdx.x; e0 < total; e0 += T * kUnroll) {
@@ -73,17 +75,15 @@ __device__ __forceinline__ void copy_rows_v16(const ExecParams &P, const DevGrou
 
 // ---- OP_COPY, 4-byte path (unaligned pitches) ---------------------------------------------
 template <bool kNC>
-__device__ __forceinline__ void copy_rows_b32(const ExecParams &P, const DevGroup &G,
-                                              int32_t rb, int32_t re) {
-  const char *sbase = P.buf[G.src_kind][G.exec_rank].ptr;
-  const int64_t spitch = P.buf[G.src_kind][G.exec_rank].pitch;
-  char *dbase = P.buf[G.dst_kind][G.dst_rank].ptr;
-  const int64_t dpitch = P.buf[G.dst_kind][G.dst_rank].pitch;
-  const int32_t *sidx = G.src_idx >= 0 ? P.idx + G.src_idx + rb : nullptr;
-  const int32_t *didx = G.dst_idx >= 0 ? P.idx + G.dst_idx + rb : nullptr;
-  const int64_t sb = G.src_base + rb, db = G.dst_base + rb;
+__device__ __forceinline__ void copy_rows_b32(const ExecParams &P, const DevItem &I) {
+  const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
+  const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
+  char *dbase = P.buf[I.dst_kind][I.dst_rank].ptr;
+  const int64_t dpitch = P.buf[I.dst_kind][I.dst_rank].pitch;
+  const int32_t *sidx = idx_of(P, I.src), *didx = idx_of(P, I.dst);
+  const int64_t sb = I.src, db = I.dst;
   const uint32_t nch = (uint32_t)P.n_chunks;
-  const uint32_t total = (uint32_t)(re - rb) * nch;
+  const uint32_t total = (uint32_t)I.rows * nch;
   const uint32_t T = blockDim.x;
   for (uint32_t e0 = threadIdx.x; e0 < total; e0 += T * kUnroll) {
     int v[kUnroll];
@@ -108,27 +108,29 @@ __device__ __forceinline__ void copy_rows_b32(const ExecParams &P, const DevGrou
 
 // load 16 bytes (or the row's valid tail) of term row `term` at column chunk `col`
 template <bool V16>
-__device__ __forceinline__ int4 ld_term(const ExecParams &P, int exec, uint32_t term, uint32_t col,
-                                        int nb) {
-  const bool slot = (term & kTermSlot) != 0;
-  const BufRef &B = slot ? P.buf[K_SLOT][exec] : P.buf[K_HGRAD][exec];
-  const char *p = B.ptr + (int64_t)(term & ~kTermSlot) * B.pitch + (int64_t)col * (V16 ? 16 : 4);
+__device__ __forceinline__ int4 ld_term(const ExecParams &P, int exec, int mode, uint32_t term,
+                                        uint32_t col, int nb) {
+  const bool slot = mode == kTermLocal && (term & kTermSlot) != 0;
+  const BufRef &B = mode == kTermRankHgrad ? P.buf[K_HGRAD][term >> 28]
+                    : slot                 ? P.buf[K_SLOT][exec]
+                                           : P.buf[K_HGRAD][exec];
+  const uint32_t row = mode == kTermRankHgrad ? (term & kTermRowMask) : (term & ~kTermSlot);
+  const char *p = B.ptr + (int64_t)row * B.pitch + (int64_t)col * (V16 ? 16 : 4);
   if (V16 && nb == 16) return slot ? ld_cg_v4(p) : ld_nc_v4(p);
   return slot ? ld_part<false>(p, V16 ? nb : 4) : ld_part<true>(p, V16 ? nb : 4);
 }
 
 // ---- OP_FOLD: dst = ((init + t0) + t1) + ... ----------------------------------------------
 template <bool V16>
-__device__ __forceinline__ void fold_rows(const ExecParams &P, const DevGroup &G, int32_t rb,
-                                          int32_t re) {
-  const BufRef D = P.buf[G.dst_kind][G.dst_rank];
-  const int32_t *didx = G.dst_idx >= 0 ? P.idx + G.dst_idx + rb : nullptr;
-  const int64_t db = G.dst_base + rb;
-  const int64_t *tp = P.term_ptr + G.term_ptr + rb;
+__device__ __forceinline__ void fold_rows(const ExecParams &P, const DevItem &I) {
+  const BufRef D = P.buf[I.dst_kind][I.dst_rank];
+  const int32_t *didx = idx_of(P, I.dst);
+  const int64_t db = I.dst;
+  const int64_t *tp = P.term_ptr + I.tp;
   const uint32_t nch = (uint32_t)P.n_chunks;
-  const uint32_t total = (uint32_t)(re - rb) * nch;
+  const uint32_t total = (uint32_t)I.rows * nch;
   const int tail = V16 ? P.row_bytes - (int)(nch - 1) * 16 : 4;
-  const int exec = G.exec_rank;
+  const int exec = I.exec_rank, mode = I.term_mode;
   for (uint32_t e = threadIdx.x; e < total; e += blockDim.x) {
     const uint32_t r = fdiv(e, P);
     const uint32_t col = e - r * nch;
@@ -137,10 +139,10 @@ __device__ __forceinline__ void fold_rows(const ExecParams &P, const DevGroup &G
     int64_t t = __ldg(tp + r);
     const int64_t t1 = __ldg(tp + r + 1);
     float4 acc;
-    if (G.fold_init) {
+    if (I.fold_init) {
       acc = as_f4(V16 && nb == 16 ? ld_cg_v4(dp) : ld_part<false>(dp, V16 ? nb : 4));
     } else {
-      acc = as_f4(ld_term<V16>(P, exec, __ldg(P.terms + t), col, nb));
+      acc = as_f4(ld_term<V16>(P, exec, mode, __ldg(P.terms + t), col, nb));
       ++t;
     }
     while (t < t1) {
@@ -149,7 +151,7 @@ __device__ __forceinline__ void fold_rows(const ExecParams &P, const DevGroup &G
       const int n = (int)(t1 - t < kMaxFoldPrefetch ? t1 - t : kMaxFoldPrefetch);
 #pragma unroll
       for (int j = 0; j < kMaxFoldPrefetch; ++j)
-        if (j < n) buf[j] = ld_term<V16>(P, exec, __ldg(P.terms + t + j), col, nb);
+        if (j < n) buf[j] = ld_term<V16>(P, exec, mode, __ldg(P.terms + t + j), col, nb);
 #pragma unroll
       for (int j = 0; j < kMaxFoldPrefetch; ++j)
         if (j < n) add4(acc, buf[j]);
@@ -166,40 +168,44 @@ __device__ __forceinline__ void fold_rows(const ExecParams &P, const DevGroup &G
 template <bool V16>
 __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant__ ExecParams P) {
   __shared__ int s_abort;
+  __shared__ DevItem s_item;
   for (int it = blockIdx.x; it < P.n_items; it += gridDim.x) {
-    const DevItem item = P.items[it];
-    const DevGroup &G = P.groups[item.group];
+    if (threadIdx.x < 4)
+      reinterpret_cast<int4 *>(&s_item)[threadIdx.x] =
+          __ldg(reinterpret_cast<const int4 *>(P.items + it) + threadIdx.x);
+    __syncthreads();
+    const DevItem I = s_item;
     if (threadIdx.x == 0) {
       bool ok = true;
-      if (G.op == OP_READY) {
+      if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer
         for (int s = 0; s < P.world; ++s)
-          if (s != G.exec_rank) st_release_sys(P.flags[s] + kReadyBase + G.exec_rank, P.seq);
+          if (s != I.exec_rank) st_release_sys(P.flags[s] + kReadyBase + I.exec_rank, P.seq);
       }
-      if (P.use_ready && G.ready_rank >= 0)
-        ok = wait_geq(P.flags[G.exec_rank] + kReadyBase + G.ready_rank, P.seq, P,
-                      1000 + item.group);
-      if (ok) ok = wait_group_sources(P, G, 100000 + item.group);
+      if (P.use_ready && I.ready_rank >= 0)
+        ok = wait_geq(P.flags[I.exec_rank] + kReadyBase + I.ready_rank, P.seq, P,
+                      1000 + I.group);
+      if (ok) ok = wait_item_sources(P, I, 100000 + I.group);
       s_abort = ok ? 0 : 1;
     }
     __syncthreads();
     if (s_abort) return;  // the watchdog fired; the error word is set, leave the launch
-    if (G.op == OP_COPY) {
-      const bool nc = readonly_kind(G.src_kind);
+    if (I.op == OP_COPY) {
+      const bool nc = readonly_kind(I.src_kind);
       if (V16) {
-        if (nc) copy_rows_v16<true>(P, G, item.row_begin, item.row_end);
-        else copy_rows_v16<false>(P, G, item.row_begin, item.row_end);
+        if (nc) copy_rows_v16<true>(P, I);
+        else copy_rows_v16<false>(P, I);
       } else {
-        if (nc) copy_rows_b32<true>(P, G, item.row_begin, item.row_end);
-        else copy_rows_b32<false>(P, G, item.row_begin, item.row_end);
+        if (nc) copy_rows_b32<true>(P, I);
+        else copy_rows_b32<false>(P, I);
       }
-    } else if (G.op == OP_FOLD) {
-      fold_rows<V16>(P, G, item.row_begin, item.row_end);
+    } else if (I.op == OP_FOLD) {
+      fold_rows<V16>(P, I);
     }
-    if (item.flags & kItemSignal) {
+    if (I.flags & kItemSignal) {
       __threadfence_system();  // this thread's row stores are visible system-wide ...
       __syncthreads();         // ... for every thread of the CTA ...
-      release_rows(P.flags[G.dst_rank] + G.sig_ctr, (uint64_t)(item.row_end - item.row_begin),
+      release_rows(P.flags[I.dst_rank] + I.sig_ctr, (uint64_t)I.rows,
                    threadIdx.x == 0);  // ... before the receiver can observe the count
     }
     __syncthreads();

@@ -1,21 +1,24 @@
 // executor_tma.cu — the bulk-copy (TMA) plan executor, warp-specialised (sm_100a).
 //
-// Same semantics as executor.cu (groups / items / counters, see internal.h), different data
-// movement.  PAPER.md §6.1-6.2: the sender packs rows by its send table and writes
-// them into the receiver's buffer; here the "pack" is a gather of whole rows into shared memory by
-// the Tensor Memory Accelerator, and the "send" is a coalesced 16-B store stream from shared
-// memory to the destination rows (a peer's halo over NVLink 5, or local HBM in loopback).
+// Same semantics as executor.cu (items / counters, see internal.h), different data movement.
+// PAPER.md §6.1-6.2: the sender packs rows by its send table and writes them into
+// the receiver's buffer.  Here the "pack" is a gather of whole rows into shared memory by the
+// Tensor Memory Accelerator (one cp.async.bulk per row), and the "send" is a coalesced 16-B store
+// stream from shared memory to the destination rows (a peer's halo over NVLink 5, or local HBM).
 //
-// Per CTA (one per SM, 512 threads, 4 x 48 KB shared-memory stages):
-//   warp 0 (producer): walks the CTA's items in order; for each data item it resolves the item's
-//     source waits (stage chaining, acquire on the receiver-side counters), waits for a free stage
-//     (mbarrier "empty"), arms the stage's "full" mbarrier with the item's byte count and issues one
-//     cp.async.bulk per gathered row (lanes issue rows lane, lane+32, ...);
-//   warps 1-15 (consumers): wait for the stage to fill, store (COPY) or fold-and-store (FOLD) from
-//     shared memory, publish the item (fence.sys + red.release.sys on the receiver's counter) and
-//     release the stage.
-// Up to 4 items (192 KB) of gathers are in flight per SM while the consumers drain older ones, so
-// HBM / NVLink latency is hidden without holding data in registers.
+// Per CTA (one per SM, 512 threads, 4 x 48 KB stages + 2 x 12 KB metadata buffers):
+//   warp 0 (producer) walks the CTA's items in order with a metadata pipeline — item descriptor
+//     two items ahead (registers), the next item's index windows (source rows, term pointers,
+//     terms) one item ahead (bulk copies into a metadata buffer) — so no dependent global load is
+//     on its critical path.  Per data item it resolves the source waits (stage chaining) and the
+//     destination's ready word, waits for a free stage, writes the item header, arms the stage's
+//     "full" mbarrier with the byte count and issues the row gathers (lane l: rows l, l+32, ...)
+//     plus the consumers' row-table windows;
+//   warps 1-15 (consumers) take stages in order: store (COPY) or fold-and-store (FOLD) from shared
+//     memory, publish (per warp: fence.sys, then red.release.sys of the warp's share of the rows
+//     on the receiver's counter — the shares sum to the item's rows, so no CTA barrier is needed)
+//     and release the stage.  An END header stops them (also used to unwind after a watchdog).
+// Up to 4 x 44 KB of gathers are in flight per SM, hiding HBM / NVLink latency without registers.
 
 #include "device_common.cuh"
 
@@ -26,8 +29,16 @@ using namespace dev;
 namespace {
 
 constexpr int kStages = 4;
-constexpr int kStageBytes = kTmaBufBytes;
-constexpr size_t kSmemBytes = 128 + (size_t)kStages * kStageBytes;
+constexpr int kMetaBytes = 12 * 1024;
+constexpr int kHdrInfo = 64;         // stage: int32 info words after the 64-B item header
+constexpr int kTabTp = 128;          // stage: term_ptr window (FOLD)
+constexpr int kTabDst = 2176;        // stage: destination-row window
+constexpr int kMetaDst = 2048;       // meta: destination rows (FOLD init operand)
+constexpr int kMetaTerms = 4096;     // meta: terms window
+constexpr size_t kMetaOff = 128;
+constexpr size_t kStageOff = kMetaOff + 2 * (size_t)kMetaBytes;
+constexpr size_t kSmemBytes = kStageOff + (size_t)kStages * kTmaBufBytes;
+static_assert(kSmemBytes <= 227 * 1024, "shared memory budget");
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -53,11 +64,8 @@ __device__ __forceinline__ bool mbar_test(uint64_t *b, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
-// wait for phase `parity` of barrier b; gives up (returns false) once *abort is set
-__device__ __forceinline__ bool mbar_wait(uint64_t *b, uint32_t parity, volatile int *abort) {
-  for (uint32_t it = 0;; ++it) {
-    if (mbar_test(b, parity)) return true;
-    if ((it & 63) == 63 && *abort) return false;
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+  while (!mbar_test(b, parity)) {
   }
 }
 __device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t bytes,
@@ -68,140 +76,207 @@ __device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t 
       "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
-__device__ __forceinline__ void fence_proxy_async() {
-  asm volatile("fence.proxy.async;" ::: "memory");
+// generic-proxy accesses (acquired flags, smem reads) before async-proxy bulk copies
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
-// Barrier over the consumer warps that gives up once *abort is set (a hardware bar.sync could
-// hang forever if some consumer left on a watchdog abort).  Returns false on abort.
-__device__ __forceinline__ bool consumer_barrier(unsigned *count, volatile unsigned *gen,
-                                                 unsigned nwarps, volatile int *abort, int lane) {
-  __syncwarp();
-  int ok = 1;
-  if (lane == 0) {
-    const unsigned g = *gen;
-    __threadfence_block();
-    if (atomicAdd(count, 1u) == nwarps - 1) {
-      *count = 0;
-      __threadfence_block();
-      atomicAdd((unsigned *)gen, 1u);
-    } else {
-      while (*gen == g) {
-        if (*abort) {
-          ok = 0;
-          break;
-        }
-      }
-    }
-    __threadfence_block();
-  }
-  ok = __shfl_sync(0xffffffffu, ok, 0);
-  return ok != 0;
+__device__ __forceinline__ void fence_proxy_async_global() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 __device__ __forceinline__ int4 lds_v4(const uint8_t *p) {
   return *reinterpret_cast<const int4 *>(p);
 }
-__device__ __forceinline__ bool is_data_op(int op) { return op == OP_COPY || op == OP_FOLD; }
 
-// bytes of gathered operands of a data item (must equal the sum of the bulk copies issued)
-__device__ __forceinline__ uint32_t item_bytes(const ExecParams &P, const DevGroup &G,
-                                               const DevItem &it) {
-  const int rows = it.row_end - it.row_begin;
-  if (G.op == OP_COPY) return (uint32_t)rows * (uint32_t)P.row16;
-  const int64_t *tp = P.term_ptr + G.term_ptr + it.row_begin;
-  return ((uint32_t)(tp[rows] - tp[0]) + (G.fold_init ? rows : 0)) * (uint32_t)P.row16;
-}
-
-// producer lanes: gather the item's rows into `buf` (lane handles rows lane, lane + 32, ...)
-__device__ __forceinline__ void issue_rows(const ExecParams &P, const DevGroup &G,
-                                           const DevItem &item, uint8_t *buf, uint64_t *bar,
-                                           int lane) {
-  const int32_t rb = item.row_begin;
-  const int rows = item.row_end - rb;
-  const uint32_t r16 = (uint32_t)P.row16;
-  if (G.op == OP_COPY) {
-    const char *sbase = P.buf[G.src_kind][G.exec_rank].ptr;
-    const int64_t spitch = P.buf[G.src_kind][G.exec_rank].pitch;
-    const int32_t *sidx = G.src_idx >= 0 ? P.idx + G.src_idx + rb : nullptr;
-    const int64_t sb = G.src_base + rb;
-    for (int r = lane; r < rows; r += 32)
-      bulk_g2s(buf + (size_t)r * r16, sbase + row_of(sidx, sb, r) * spitch, r16, bar);
-  } else {
-    const int64_t *tp = P.term_ptr + G.term_ptr + rb;
-    const int init = G.fold_init;
-    const int64_t t0 = __ldg(tp);
-    const BufRef D = P.buf[G.dst_kind][G.dst_rank];
-    const int32_t *didx = G.dst_idx >= 0 ? P.idx + G.dst_idx + rb : nullptr;
-    const int64_t db = G.dst_base + rb;
-    const BufRef SL = P.buf[K_SLOT][G.exec_rank];
-    const BufRef HG = P.buf[K_HGRAD][G.exec_rank];
-    for (int r = lane; r < rows; r += 32) {
-      const int64_t ta = __ldg(tp + r), tb = __ldg(tp + r + 1);
-      uint32_t slot = (uint32_t)(ta - t0) + (init ? r : 0);
-      if (init)
-        bulk_g2s(buf + (size_t)(slot++) * r16, D.ptr + row_of(didx, db, r) * D.pitch, r16, bar);
-      for (int64_t t = ta; t < tb; ++t) {
-        const uint32_t term = __ldg(P.terms + t);
-        const BufRef &B = (term & kTermSlot) ? SL : HG;
-        bulk_g2s(buf + (size_t)(slot++) * r16, B.ptr + (int64_t)(term & ~kTermSlot) * B.pitch,
-                 r16, bar);
-      }
-    }
-  }
-}
-
-// consumers: store a gathered COPY item from shared memory (whole 16-B chunks: the destinations
-// are library-owned rows whose pitch covers the rounded-up row)
-__device__ __forceinline__ void store_copy(const ExecParams &P, const DevGroup &G,
-                                           const DevItem &item, const uint8_t *buf, uint32_t tid,
-                                           uint32_t T) {
-  char *dbase = P.buf[G.dst_kind][G.dst_rank].ptr;
-  const int64_t dpitch = P.buf[G.dst_kind][G.dst_rank].pitch;
-  const int32_t rb = item.row_begin;
-  const int32_t *didx = G.dst_idx >= 0 ? P.idx + G.dst_idx + rb : nullptr;
-  const int64_t db = G.dst_base + rb;
-  const uint32_t nch = (uint32_t)P.n_chunks;
-  const uint32_t r16 = (uint32_t)P.row16;
-  const uint32_t total = (uint32_t)(item.row_end - rb) * nch;
-  for (uint32_t e0 = tid; e0 < total; e0 += T * kUnroll) {
+__device__ __forceinline__ DevItem load_item(const DevItem *items, int i) {
+  DevItem d;
+  const int4 *s = reinterpret_cast<const int4 *>(items + i);
+  int4 *o = reinterpret_cast<int4 *>(&d);
 #pragma unroll
-    for (int j = 0; j < kUnroll; ++j) {
-      const uint32_t e = e0 + j * T;
-      if (e < total) {
-        const uint32_t r = fdiv(e, P);
-        const uint32_t col = e - r * nch;
-        st_v4(dbase + row_of(didx, db, r) * dpitch + (int64_t)col * 16,
-              lds_v4(buf + r * r16 + col * 16));
+  for (int q = 0; q < 4; ++q) o[q] = __ldg(s + q);
+  return d;
+}
+
+// 16-B aligned window [a, e) of `n` elements of size `sz` starting at element `off`
+struct Win {
+  int64_t a;       // first element copied (aligned down)
+  uint32_t bytes;  // multiple of 16
+  int32_t skew;    // off - a
+};
+__device__ __forceinline__ Win window(int64_t off, int64_t n, int sz) {
+  const int64_t per = 16 / sz;
+  Win w;
+  w.a = off / per * per;
+  const int64_t e = (off + n + per - 1) / per * per;
+  w.bytes = (uint32_t)((e - w.a) * sz);
+  w.skew = (int32_t)(off - w.a);
+  return w;
+}
+
+// producer lane 0: bulk-copy the metadata the producer needs to issue item I's gathers
+__device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I, uint8_t *meta,
+                                           uint64_t *bar) {
+  uint32_t tx = 0;
+  Win ws = {0, 0, 0}, wd = {0, 0, 0}, wt = {0, 0, 0};
+  if (I.op == OP_COPY && I.src < 0) {
+    ws = window(~I.src, I.rows, 4);
+    tx += ws.bytes;
+  } else if (I.op == OP_FOLD) {
+    ws = window(I.tp, I.rows + 1, 8);
+    wt = window(I.t0, I.nterms, 4);
+    tx += ws.bytes + wt.bytes;
+    if (I.fold_init && I.dst < 0) {
+      wd = window(~I.dst, I.rows, 4);
+      tx += wd.bytes;
+    }
+  }
+  fence_proxy_async_smem();
+  mbar_expect_tx(bar, tx);
+  if (ws.bytes)
+    bulk_g2s(meta, I.op == OP_FOLD ? (const void *)(P.term_ptr + ws.a) : (const void *)(P.idx + ws.a),
+             ws.bytes, bar);
+  if (wd.bytes) bulk_g2s(meta + kMetaDst, P.idx + wd.a, wd.bytes, bar);
+  if (wt.bytes) bulk_g2s(meta + kMetaTerms, P.terms + wt.a, wt.bytes, bar);
+}
+
+// operand bytes of a data item (must equal the sum of the row gathers issued)
+__device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const DevItem &I) {
+  const uint32_t slots =
+      I.op == OP_COPY ? (uint32_t)I.rows : (uint32_t)I.nterms + (I.fold_init ? I.rows : 0);
+  return slots * (uint32_t)P.row16;
+}
+
+// producer warp: header, consumer tables and row gathers of data item I into `st`
+__device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I, uint8_t *st,
+                                           const uint8_t *meta, uint64_t *full, int lane) {
+  const uint32_t r16 = (uint32_t)P.row16;
+  // consumer tables: term_ptr window (FOLD) and destination rows (when not consecutive)
+  Win wtp = {0, 0, 0}, wdst = {0, 0, 0};
+  if (I.op == OP_FOLD) wtp = window(I.tp, I.rows + 1, 8);
+  if (I.dst < 0) wdst = window(~I.dst, I.rows, 4);
+  if (lane < 4) reinterpret_cast<int4 *>(st)[lane] = reinterpret_cast<const int4 *>(&I)[lane];
+  if (lane == 4) {
+    int32_t *info = reinterpret_cast<int32_t *>(st + kHdrInfo);
+    info[0] = wtp.skew;
+    info[1] = wdst.skew;
+  }
+  __syncwarp();  // header and info written before lane 0's arrive publishes the stage
+  if (lane == 0) mbar_expect_tx(full, operand_bytes(P, I) + wtp.bytes + wdst.bytes);
+  __syncwarp();
+  fence_proxy_async_smem();
+  if (lane == 0) {
+    if (wtp.bytes) bulk_g2s(st + kTabTp, P.term_ptr + wtp.a, wtp.bytes, full);
+    if (wdst.bytes) bulk_g2s(st + kTabDst, P.idx + wdst.a, wdst.bytes, full);
+  }
+  uint8_t *ops = st + kStageHdrBytes;
+  if (I.op == OP_COPY) {
+    const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
+    const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
+    const int32_t *sidx = reinterpret_cast<const int32_t *>(meta);
+    const int32_t skew = I.src < 0 ? (int32_t)(~I.src - window(~I.src, I.rows, 4).a) : 0;
+    for (int r = lane; r < I.rows; r += 32) {
+      const int64_t srow = I.src >= 0 ? I.src + r : (int64_t)sidx[skew + r];
+      bulk_g2s(ops + (size_t)r * r16, sbase + srow * spitch, r16, full);
+    }
+  } else {
+    const int64_t *tpm = reinterpret_cast<const int64_t *>(meta);
+    const int32_t tps = (int32_t)(I.tp - window(I.tp, I.rows + 1, 8).a);
+    const uint32_t *tm = reinterpret_cast<const uint32_t *>(meta + kMetaTerms);
+    const int32_t ts = (int32_t)(I.t0 - window(I.t0, I.nterms, 4).a);
+    const int32_t *dm = reinterpret_cast<const int32_t *>(meta + kMetaDst);
+    const int32_t ds = I.dst < 0 ? (int32_t)(~I.dst - window(~I.dst, I.rows, 4).a) : 0;
+    const BufRef D = P.buf[I.dst_kind][I.dst_rank];
+    const BufRef SL = P.buf[K_SLOT][I.exec_rank];
+    const BufRef HG = P.buf[K_HGRAD][I.exec_rank];
+    const int init = I.fold_init;
+    for (int r = lane; r < I.rows; r += 32) {
+      const int64_t ta = tpm[tps + r], tb = tpm[tps + r + 1];
+      uint32_t slot = (uint32_t)(ta - I.t0) + (init ? r : 0);
+      if (init) {
+        const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)dm[ds + r];
+        bulk_g2s(ops + (size_t)(slot++) * r16, D.ptr + drow * D.pitch, r16, full);
+      }
+      for (int64_t t = ta; t < tb; ++t) {
+        const uint32_t term = tm[ts + (t - I.t0)];
+        const BufRef *B;
+        uint32_t row;
+        if (I.term_mode == kTermRankHgrad) {
+          B = &P.buf[K_HGRAD][term >> 28];
+          row = term & kTermRowMask;
+        } else {
+          B = (term & kTermSlot) ? &SL : &HG;
+          row = term & ~kTermSlot;
+        }
+        bulk_g2s(ops + (size_t)(slot++) * r16, B->ptr + (int64_t)row * B->pitch, r16, full);
       }
     }
   }
 }
 
-// consumers: fold a gathered FOLD item from shared memory, operands in list order, and store it
-// (the row's last chunk is stored partially: the destination may be the caller's emb_grad)
-__device__ __forceinline__ void store_fold(const ExecParams &P, const DevGroup &G,
-                                           const DevItem &item, const uint8_t *buf, uint32_t tid,
-                                           uint32_t T) {
-  const BufRef D = P.buf[G.dst_kind][G.dst_rank];
-  const int32_t rb = item.row_begin;
-  const int32_t *didx = G.dst_idx >= 0 ? P.idx + G.dst_idx + rb : nullptr;
-  const int64_t db = G.dst_base + rb;
-  const int64_t *tp = P.term_ptr + G.term_ptr + rb;
-  const int64_t t0 = __ldg(tp);
-  const int init = G.fold_init;
+// consumers: store a gathered COPY item (whole 16-B chunks: the destinations are library-owned
+// rows whose pitch covers the rounded-up row)
+__device__ __forceinline__ void store_copy(const ExecParams &P, const DevItem &I, const uint8_t *st,
+                                           uint32_t tid, uint32_t T) {
+  char *dbase = P.buf[I.dst_kind][I.dst_rank].ptr;
+  const int64_t dpitch = P.buf[I.dst_kind][I.dst_rank].pitch;
   const uint32_t nch = (uint32_t)P.n_chunks;
   const uint32_t r16 = (uint32_t)P.row16;
-  const uint32_t total = (uint32_t)(item.row_end - rb) * nch;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  const uint8_t *ops = st + kStageHdrBytes;
+  if (I.dst >= 0) {
+    char *d0 = dbase + I.dst * dpitch;
+    for (uint32_t e0 = tid; e0 < total; e0 += T * kUnroll) {
+#pragma unroll
+      for (int j = 0; j < kUnroll; ++j) {
+        const uint32_t e = e0 + j * T;
+        if (e < total) {
+          const uint32_t r = fdiv(e, P);
+          const uint32_t col = e - r * nch;
+          st_v4(d0 + (int64_t)r * dpitch + col * 16, lds_v4(ops + r * r16 + col * 16));
+        }
+      }
+    }
+  } else {
+    const int32_t *tab = reinterpret_cast<const int32_t *>(st + kTabDst) +
+                         reinterpret_cast<const int32_t *>(st + kHdrInfo)[1];
+    for (uint32_t e0 = tid; e0 < total; e0 += T * kUnroll) {
+#pragma unroll
+      for (int j = 0; j < kUnroll; ++j) {
+        const uint32_t e = e0 + j * T;
+        if (e < total) {
+          const uint32_t r = fdiv(e, P);
+          const uint32_t col = e - r * nch;
+          st_v4(dbase + (int64_t)tab[r] * dpitch + col * 16, lds_v4(ops + r * r16 + col * 16));
+        }
+      }
+    }
+  }
+}
+
+// consumers: fold a gathered FOLD item (operands in list order) and store it; the row's last
+// chunk is stored partially (the destination may be the caller's emb_grad)
+__device__ __forceinline__ void store_fold(const ExecParams &P, const DevItem &I, const uint8_t *st,
+                                           uint32_t tid, uint32_t T) {
+  const BufRef D = P.buf[I.dst_kind][I.dst_rank];
+  const int32_t *info = reinterpret_cast<const int32_t *>(st + kHdrInfo);
+  const int64_t *tp = reinterpret_cast<const int64_t *>(st + kTabTp) + info[0];
+  const int32_t *tab = reinterpret_cast<const int32_t *>(st + kTabDst) + info[1];
+  const int init = I.fold_init;
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t r16 = (uint32_t)P.row16;
+  const uint32_t total = (uint32_t)I.rows * nch;
   const int tail = P.row_bytes - (int)(nch - 1) * 16;
+  const uint8_t *ops = st + kStageHdrBytes;
   for (uint32_t e = tid; e < total; e += T) {
     const uint32_t r = fdiv(e, P);
     const uint32_t col = e - r * nch;
-    const int64_t ta = __ldg(tp + r), tb = __ldg(tp + r + 1);
-    const uint32_t base = (uint32_t)(ta - t0) + (init ? r : 0);
+    const int64_t ta = tp[r], tb = tp[r + 1];
+    const uint32_t base = (uint32_t)(ta - I.t0) + (init ? r : 0);
     const uint32_t cnt = (uint32_t)(tb - ta) + (init ? 1 : 0);
-    const uint8_t *p = buf + (size_t)base * r16 + col * 16;
+    const uint8_t *p = ops + (size_t)base * r16 + col * 16;
     float4 acc = as_f4(lds_v4(p));
     for (uint32_t j = 1; j < cnt; ++j) add4(acc, lds_v4(p + (size_t)j * r16));
-    char *dp = D.ptr + row_of(didx, db, r) * D.pitch + (int64_t)col * 16;
+    const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
+    char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
     const int nb = col + 1 == nch ? tail : 16;
     if (nb == 16)
       st_v4(dp, as_i4(acc));
@@ -215,10 +290,9 @@ __global__ void __launch_bounds__(512, 1)
   extern __shared__ __align__(128) uint8_t dsmem[];
   uint64_t *full = reinterpret_cast<uint64_t *>(dsmem);
   uint64_t *empty = full + kStages;
-  uint8_t *bufs = dsmem + 128;
-  __shared__ volatile int s_abort;
-  __shared__ unsigned s_bar_count;
-  __shared__ volatile unsigned s_bar_gen;
+  uint64_t *metab = empty + kStages;
+  uint8_t *metas = dsmem + kMetaOff;
+  uint8_t *stages = dsmem + kStageOff;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
   if (threadIdx.x == 0) {
@@ -226,90 +300,106 @@ __global__ void __launch_bounds__(512, 1)
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], n_cons_warps);
     }
-    s_abort = 0;
-    s_bar_count = 0;
-    s_bar_gen = 0;
+    mbar_init(&metab[0], 1);
+    mbar_init(&metab[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
 
   if (warp == 0) {
     // ------------------------------- producer warp -------------------------------------------
-    uint32_t k = 0;
-    for (int it = blockIdx.x; it < P.n_items; it += gridDim.x) {
-      const DevItem item = P.items[it];
-      const DevGroup &G = P.groups[item.group];
-      const int op = G.op;
-      if (op == OP_READY) {
+    const int G = gridDim.x;
+    uint32_t k = 0;  // data items issued (stage sequence)
+    uint32_t m = 0;  // items whose metadata was issued (meta buffer sequence)
+    bool ok = true;
+    int it = blockIdx.x;
+    DevItem d0, d1;
+    if (it < P.n_items) {
+      d0 = load_item(P.items, it);
+      if (lane == 0) issue_meta(P, d0, metas, &metab[0]);
+    }
+    if (it + G < P.n_items) d1 = load_item(P.items, it + G);
+    for (; it < P.n_items; it += G, ++m) {
+      // metadata of the next item and the descriptor of the one after
+      if (it + G < P.n_items && lane == 0)
+        issue_meta(P, d1, metas + ((m + 1) & 1) * kMetaBytes, &metab[(m + 1) & 1]);
+      DevItem d2;
+      if (it + 2 * G < P.n_items) d2 = load_item(P.items, it + 2 * G);
+      const DevItem &I = d0;
+      if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer
         if (lane == 0)
           for (int s = 0; s < P.world; ++s)
-            if (s != G.exec_rank) st_release_sys(P.flags[s] + kReadyBase + G.exec_rank, P.seq);
-        __syncwarp();
-        continue;
-      }
-      if (!is_data_op(op)) continue;
-      int ok = 1;
-      if (lane == 0) ok = wait_group_sources(P, G, 100000 + item.group) ? 1 : 0;
-      ok = __shfl_sync(0xffffffffu, ok, 0);
-      if (!ok) s_abort = 1;
-      if (s_abort) break;
-      const uint32_t stage = k % kStages, use = k / kStages;
-      if (use > 0 && !mbar_wait(&empty[stage], (use - 1) & 1u, &s_abort)) break;
-      if (lane == 0) mbar_expect_tx(&full[stage], item_bytes(P, G, item));
-      __syncwarp();
-      fence_proxy_async();  // acquired sources / released stage -> async-proxy bulk copies
-      issue_rows(P, G, item, bufs + (size_t)stage * kStageBytes, &full[stage], lane);
-      ++k;
-    }
-    if (s_abort) {
-      // drain: never leave with bulk copies still writing this CTA's shared memory
-      for (uint32_t s = 0; s < kStages && s < k; ++s) {
-        const uint32_t uses = (k - 1 - s) / kStages + 1;  // issues on stage s
-        while (!mbar_test(&full[s], (uses - 1) & 1u)) {
+            if (s != I.exec_rank) st_release_sys(P.flags[s] + kReadyBase + I.exec_rank, P.seq);
+      } else if (I.op == OP_WAIT) {
+        // forward completion: the launch ends only once every incoming row landed
+        int w = 1;
+        if (lane == 0) w = wait_item_sources(P, I, 200000 + I.group) ? 1 : 0;
+        ok = __shfl_sync(0xffffffffu, w, 0) != 0;
+        if (!ok) break;
+      } else if (I.op == OP_COPY || I.op == OP_FOLD) {
+        int w = 1;
+        if (lane == 0) {
+          // sources final (stage chaining) and the destination's buffers free (ready word)
+          w = wait_item_sources(P, I, 100000 + I.group) ? 1 : 0;
+          if (w && P.use_ready && I.ready_rank >= 0)
+            w = wait_geq(P.flags[I.exec_rank] + kReadyBase + I.ready_rank, P.seq, P,
+                         1000 + I.group) ? 1 : 0;
         }
+        ok = __shfl_sync(0xffffffffu, w, 0) != 0;
+        if (!ok) break;
+        if (I.wait_n > 0) fence_proxy_async_global();  // acquired peers' rows -> bulk reads
+        mbar_wait(&metab[m & 1], (m >> 1) & 1u);
+        const uint32_t stage = k % kStages, use = k / kStages;
+        if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
+        issue_item(P, I, stages + (size_t)stage * kTmaBufBytes, metas + (m & 1) * kMetaBytes,
+                   &full[stage], lane);
+        ++k;
       }
+      __syncwarp();
+      d0 = d1;
+      d1 = d2;
+    }
+    if (!ok) {
+      // watchdog abort: metadata copies still in flight must land before the CTA leaves
+      for (uint32_t q = m; q < m + 2; ++q) {
+        const int iq = blockIdx.x + (int)q * G;
+        if (iq < P.n_items) mbar_wait(&metab[q & 1], (q >> 1) & 1u);
+      }
+    }
+    // END marker: consumers drain every issued stage, then stop
+    const uint32_t stage = k % kStages, use = k / kStages;
+    if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
+    uint8_t *st = stages + (size_t)stage * kTmaBufBytes;
+    if (lane == 0) {
+      reinterpret_cast<DevItem *>(st)->op = OP_END;
+      mbar_arrive(&full[stage]);
     }
   } else {
     // ------------------------------- consumer warps ------------------------------------------
     const uint32_t tid = threadIdx.x - 32, T = blockDim.x - 32;
-    uint32_t k = 0;
-    for (int it = blockIdx.x; it < P.n_items; it += gridDim.x) {
-      const DevItem item = P.items[it];
-      const DevGroup &G = P.groups[item.group];
-      const int op = G.op;
-      if (op == OP_WAIT) {
-        // forward completion: the halo is complete when the launch ends
-        if (tid == 0 && !wait_group_sources(P, G, 200000 + item.group)) s_abort = 1;
-        continue;
-      }
-      if (!is_data_op(op)) continue;
+    const int cw = warp - 1;
+    for (uint32_t k = 0;; ++k) {
       const uint32_t stage = k % kStages, use = k / kStages;
-      const unsigned nw = (unsigned)n_cons_warps;
-      if (P.use_ready && G.ready_rank >= 0) {
-        // the destination GPU's buffers must be free for this call before we write them
-        if (tid == 0 &&
-            !wait_geq(P.flags[G.exec_rank] + kReadyBase + G.ready_rank, P.seq, P,
-                      1000 + item.group))
-          s_abort = 1;
-        if (!consumer_barrier(&s_bar_count, &s_bar_gen, nw, &s_abort, lane)) return;
-      }
-      if (!mbar_wait(&full[stage], use & 1u, &s_abort)) return;
-      const uint8_t *buf = bufs + (size_t)stage * kStageBytes;
-      if (op == OP_COPY)
-        store_copy(P, G, item, buf, tid, T);
+      mbar_wait(&full[stage], use & 1u);
+      const uint8_t *st = stages + (size_t)stage * kTmaBufBytes;
+      const DevItem I = *reinterpret_cast<const DevItem *>(st);
+      if (I.op == OP_END) break;
+      if (I.op == OP_COPY)
+        store_copy(P, I, st, tid, T);
       else
-        store_fold(P, G, item, buf, tid, T);
-      if (item.flags & kItemSignal) {
-        __threadfence_system();  // this thread's stores are visible system-wide ...
-        // ... for every consumer thread ...
-        if (!consumer_barrier(&s_bar_count, &s_bar_gen, nw, &s_abort, lane)) return;
-        release_rows(P.flags[G.dst_rank] + G.sig_ctr, (uint64_t)(item.row_end - item.row_begin),
-                     tid == 0);  // ... before the receiver can observe the count (done flag)
+        store_fold(P, I, st, tid, T);
+      if (I.flags & kItemSignal) {
+        // this warp's stores are visible system-wide before its share of the rows is counted;
+        // the receiver sees the item's full count only after every warp published (done flag)
+        __threadfence_system();
+        __syncwarp();
+        const int64_t lo = (int64_t)I.rows * cw / n_cons_warps;
+        const int64_t hi = (int64_t)I.rows * (cw + 1) / n_cons_warps;
+        if (lane == 0 && hi > lo) red_release_sys_add(P.flags[I.dst_rank] + I.sig_ctr, hi - lo);
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // this warp is done reading the stage
-      ++k;
     }
   }
 }

@@ -34,20 +34,20 @@ void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim
       std::memcpy(d, s, sizeof(float) * dim);
     } else {
       const int64_t t0 = low.term_ptr[g.term_ptr + i], t1 = low.term_ptr[g.term_ptr + i + 1];
+      auto operand = [&](uint32_t term) -> const float * {
+        if (g.term_mode == kTermRankHgrad)
+          return row_ptr(B, K_HGRAD, (int)(term >> 28), term & kTermRowMask);
+        return row_ptr(B, (term & kTermSlot) ? K_SLOT : K_HGRAD, g.exec_rank, term & ~kTermSlot);
+      };
       for (int c = 0; c < dim; ++c) {
         int64_t t = t0;
         float acc;
-        if (g.fold_init) {
+        if (g.fold_init)
           acc = d[c];
-        } else {
-          const uint32_t term = low.terms[t++];
-          const int kind = (term & kTermSlot) ? K_SLOT : K_HGRAD;
-          acc = row_ptr(B, kind, g.exec_rank, term & ~kTermSlot)[c];
-        }
+        else
+          acc = operand(low.terms[t++])[c];
         for (; t < t1; ++t) {
-          const uint32_t term = low.terms[t];
-          const int kind = (term & kTermSlot) ? K_SLOT : K_HGRAD;
-          volatile float v = row_ptr(B, kind, g.exec_rank, term & ~kTermSlot)[c];
+          volatile float v = operand(low.terms[t])[c];
           acc = acc + v;  // one IEEE fp32 add per term, in list order
         }
         d[c] = acc;
@@ -58,9 +58,10 @@ void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim
 
 }  // namespace
 
-void hostsim_run(const Lowered &low, int dir, const std::vector<int64_t> &row_off,
-                 const std::vector<int64_t> &halo_off, int64_t pitch, int dim, const float *emb,
-                 float *halo, const float *halo_grad, float *emb_grad) {
+void hostsim_run(const Lowered &low, const std::vector<int32_t> &gids,
+                 const std::vector<int64_t> &row_off, const std::vector<int64_t> &halo_off,
+                 int64_t pitch, int dim, const float *emb, float *halo, const float *halo_grad,
+                 float *emb_grad) {
   const int m = low.m;
   std::vector<std::vector<float>> relay(m), slot(m);
   HostBufs B;
@@ -76,11 +77,10 @@ void hostsim_run(const Lowered &low, int dir, const std::vector<int64_t> &row_of
     B.base[K_RELAY][r] = relay[r].data();
     B.base[K_SLOT][r] = slot[r].data();
   }
-  const size_t g0 = dir == DIR_FWD ? 0 : (size_t)low.n_fwd_groups;
-  for (size_t gi = g0; gi < low.groups.size(); ++gi) {
+  for (int32_t gi : gids) {  // the program's groups, in stage order
     const DevGroup &g = low.groups[gi];
-    if (g.dir != dir || g.op == OP_READY || g.op == OP_WAIT) continue;
-    run_group(low, g, B, dim);  // groups are stored in stage order
+    if (g.op == OP_READY || g.op == OP_WAIT) continue;
+    run_group(low, g, B, dim);
   }
 }
 

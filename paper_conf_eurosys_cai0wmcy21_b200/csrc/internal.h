@@ -30,7 +30,8 @@ enum Op : int32_t {
   OP_COPY = 0,   // dst[dst_row(i)] = src[src_row(i)]
   OP_FOLD = 1,   // dst[dst_row(i)] = fold(init ? dst : -, terms(i)) in order, fp32 adds
   OP_READY = 2,  // write ready[exec_rank] = seq into every peer's flag region
-  OP_WAIT = 3    // wait on the group's wait list (forward completion)
+  OP_WAIT = 3,   // wait on the group's wait list (forward completion)
+  OP_END = 4     // (device only) end-of-stream marker from the producer warp to the consumers
 };
 
 enum Dir : int32_t { DIR_FWD = 0, DIR_BWD = 1 };
@@ -44,8 +45,14 @@ constexpr int64_t kFlagWords = kReadyBase + kMaxRanks;
 constexpr int64_t kFlagBytes = 8192;  // region reserved (>= kFlagWords * 8)
 static_assert(kFlagWords * 8 <= kFlagBytes, "flag region");
 
-// term encoding for OP_FOLD: bit 31 set => SLOT(exec) row, else HGRAD(exec) row
+// term encodings for OP_FOLD
+//   kTermLocal:     bit 31 set => SLOT(exec) row, else HGRAD(exec) row
+//   kTermRankHgrad: bits 31..28 = rank r, bits 27..0 = row of HGRAD(r)  (loopback direct reduce:
+//                   every virtual rank's halo gradients live on the same device)
 constexpr uint32_t kTermSlot = 0x80000000u;
+constexpr int32_t kTermLocal = 0;
+constexpr int32_t kTermRankHgrad = 1;
+constexpr uint32_t kTermRowMask = 0x0FFFFFFFu;
 
 struct DevGroup {
   int32_t op;
@@ -60,6 +67,8 @@ struct DevGroup {
   int32_t ready_rank;  // wait ready[ready_rank] >= seq before writing (-1: none)
   int32_t wait_off;    // waits[wait_off .. wait_off + wait_n) on exec_rank's counters
   int32_t wait_n;
+  int32_t term_mode;   // OP_FOLD terms: kTermLocal (SLOT/HGRAD of exec) or kTermRankHgrad
+  int32_t pad2;
   int64_t n_rows;
   int64_t src_idx;     // offset into idx pool, or -1 => rows src_base + i
   int64_t src_base;
@@ -68,13 +77,26 @@ struct DevGroup {
   int64_t term_ptr;    // OP_FOLD: offset into term_ptr pool (n_rows + 1 entries)
 };
 
-struct DevItem {
-  int32_t group;
-  int32_t row_begin;
-  int32_t row_end;
-  int32_t flags;       // bit 0: signal the group's counter after the rows
+// One work item = a row range of one group, self-contained (64 B, one descriptor load): the
+// executor never dereferences the group table on the hot path.
+struct alignas(16) DevItem {
+  uint8_t op, dir, exec_rank, dst_rank;
+  uint8_t src_kind, dst_kind, fold_init, term_mode;
+  int8_t ready_rank;   // wait ready[ready_rank] >= seq before writing (-1: none)
+  uint8_t flags;       // kItemSignal: add `rows` to the receiver's counter sig_ctr afterwards
+  int16_t wait_n;      // waits[wait_off .. +wait_n) on exec_rank's counters (source readiness)
+  int32_t rows;
+  int32_t sig_ctr;
+  int32_t wait_off;
+  int64_t src;         // >= 0: first source row (rows are consecutive); < 0: ~(idx pool offset)
+  int64_t dst;         // same encoding for the destination rows
+  int64_t tp;          // OP_FOLD: term_ptr pool index of the first row (rows + 1 entries)
+  int64_t t0;          // OP_FOLD: term_ptr[tp] (index of the first term)
+  int32_t nterms;      // OP_FOLD: terms of the item
+  int32_t group;       // originating group (diagnostics / watchdog codes)
 };
-constexpr int32_t kItemSignal = 1;
+static_assert(sizeof(DevItem) == 64, "DevItem is one 64-B descriptor");
+constexpr uint8_t kItemSignal = 1;
 
 struct DevWait {
   int32_t ctr;         // counter index on the executing rank
@@ -114,7 +136,17 @@ struct ExecParams {
   int32_t pad1;
 };
 
-constexpr int kTmaBufBytes = 48 * 1024;  // per stage; 4 stages -> 192 KB dynamic shared memory per CTA
+// Bulk-copy executor (executor_tma.cu) shared-memory geometry and the item limits it implies:
+//   stage  = [0,64) item header | [64,128) info | [128,2176) term_ptr window (FOLD) |
+//            [2176,4096) destination-row window | [4096, 48K) gathered operand rows
+//   meta   = producer-private: [0,2K) source-row / term_ptr window | [2K,4K) destination rows |
+//            [4K,12K) terms window
+constexpr int kTmaBufBytes = 48 * 1024;  // per stage; 4 stages -> 192 KB dynamic shared memory
+constexpr int kStageHdrBytes = 4096;
+constexpr int kTmaOperandBytes = kTmaBufBytes - kStageHdrBytes;
+constexpr int kMaxItemRows = 464;        // (1920 B dst window) / 4 B - alignment slack
+constexpr int kMaxFoldRows = 240;        // (2048 B term_ptr window) / 8 B - slack
+constexpr int kMaxItemTerms = 2040;      // (8 KB terms window) / 4 B - slack
 
 // fast unsigned division by a runtime constant d >= 1, exact for x < 2^31
 struct FastDiv {

@@ -351,6 +351,37 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     g.wait_n = (int32_t)L.waits.size() - g.wait_off;
     L.groups.push_back(g);
   }
+  // ---- loopback direct reduce (single-stage plans only) ----
+  // When every virtual rank lives on one device the owner can read its requesters' halo-gradient
+  // rows in place: emb_grad[loc u] = ((emb_grad[loc u] + G_c1[pos]) + G_c2[pos]) + ..., c
+  // ascending — the same fold, terms and order as push + RED, without the slot round trip.
+  L.direct_begin = (int)L.groups.size();
+  if (K <= 1) {
+    for (int s = 0; s < m; ++s) {
+      std::vector<std::pair<int64_t, int64_t>> rows;  // (loc, u)
+      for (int64_t vi = 0; vi < NV; ++vi) {
+        const int64_t u = plan.order[vi];
+        if (part[u] == s) rows.push_back({loc[u], u});
+      }
+      if (rows.empty()) continue;
+      std::sort(rows.begin(), rows.end());
+      DevGroup g = base_group(OP_FOLD, DIR_BWD, s, s, 1);
+      g.dst_kind = K_EGRAD;
+      g.fold_init = 1;
+      g.term_mode = kTermRankHgrad;
+      g.term_ptr = (int64_t)L.term_ptr.size();
+      L.term_ptr.push_back((int64_t)L.terms.size());
+      std::vector<int64_t> dst, src;
+      for (auto &r : rows) {
+        dst.push_back(r.first);
+        for (int64_t q = rel.d_ptr[r.second]; q < rel.d_ptr[r.second + 1]; ++q)
+          L.terms.push_back(((uint32_t)rel.d_gpu[q] << 28) | ((uint32_t)rel.d_pos[q] & kTermRowMask));
+        L.term_ptr.push_back((int64_t)L.terms.size());
+      }
+      flush_group(L.groups, g, src, dst);
+    }
+  }
+  L.direct_end = (int)L.groups.size();
   L.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
 }
 
@@ -361,7 +392,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
   // of the bulk-copy executor): a COPY row costs one row, a FOLD row (1 + #terms) rows.
   items->clear();
   const int64_t row16 = (row_bytes + 15) / 16 * 16;
-  const int64_t cap = std::max<int64_t>(row16, std::min<int64_t>(item_bytes, kTmaBufBytes));
+  const int64_t cap = std::max<int64_t>(row16, std::min<int64_t>(item_bytes, kTmaOperandBytes));
   size_t i = 0;
   std::vector<std::vector<int32_t>> bounds;  // per group of the stage: chunk start rows + end
   while (i < gids.size()) {
@@ -380,7 +411,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       std::vector<int32_t> &b = bounds[q - i];
       b.push_back(0);
       if (g.op == OP_COPY) {
-        const int64_t rpi = std::max<int64_t>(1, cap / row16);
+        const int64_t rpi = std::min<int64_t>(kMaxItemRows, std::max<int64_t>(1, cap / row16));
         for (int64_t r = rpi; r < g.n_rows; r += rpi) b.push_back((int32_t)r);
         b.push_back((int32_t)g.n_rows);
       } else if (g.op == OP_FOLD) {
@@ -389,7 +420,8 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
           const int64_t slots = low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r] +
                                 (g.fold_init ? 1 : 0);
           const int64_t cost = slots * row16;
-          if (acc > 0 && acc + cost > cap) {
+          const int64_t nt = low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + b.back()];
+          if (acc > 0 && (acc + cost > cap || r - b.back() >= kMaxFoldRows || nt > kMaxItemTerms)) {
             b.push_back((int32_t)r);
             acc = 0;
           }
@@ -407,11 +439,32 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         const DevGroup &g = low.groups[gids[q]];
         const std::vector<int32_t> &b = bounds[q - i];
         if (c + 1 >= b.size()) continue;
+        const bool data = g.op == OP_COPY || g.op == OP_FOLD;
+        const int64_t rb = b[c];
         DevItem it;
+        std::memset(&it, 0, sizeof(it));
+        it.op = (uint8_t)g.op;
+        it.dir = (uint8_t)g.dir;
+        it.exec_rank = (uint8_t)g.exec_rank;
+        it.dst_rank = (uint8_t)g.dst_rank;
+        it.src_kind = (uint8_t)g.src_kind;
+        it.dst_kind = (uint8_t)g.dst_kind;
+        it.fold_init = (uint8_t)g.fold_init;
+        it.term_mode = (uint8_t)g.term_mode;
+        it.ready_rank = (int8_t)g.ready_rank;
+        it.wait_n = (int16_t)g.wait_n;
+        it.wait_off = g.wait_off;
+        it.sig_ctr = g.sig_ctr;
         it.group = gids[q];
-        it.row_begin = b[c];
-        it.row_end = b[c + 1];
-        bool sig = g.sig_ctr >= 0 && (g.op == OP_COPY || g.op == OP_FOLD);
+        it.rows = data ? b[c + 1] - b[c] : 0;
+        it.src = g.src_idx >= 0 ? ~(g.src_idx + rb) : g.src_base + rb;
+        it.dst = g.dst_idx >= 0 ? ~(g.dst_idx + rb) : g.dst_base + rb;
+        if (g.op == OP_FOLD) {
+          it.tp = g.term_ptr + rb;
+          it.t0 = low.term_ptr[it.tp];
+          it.nterms = (int32_t)(low.term_ptr[it.tp + it.rows] - it.t0);
+        }
+        bool sig = data && g.sig_ctr >= 0;
         if (sig && !signal_all)
           sig = needed_ctr[(size_t)g.dst_rank * kFlagWords + g.sig_ctr] != 0;
         it.flags = sig ? kItemSignal : 0;

@@ -59,8 +59,9 @@ struct HostGroup {
 struct Lowered {
   int m = 0;
   int n_stages = 0;                      // forward stages K
-  std::vector<DevGroup> groups;          // forward groups, then backward groups
+  std::vector<DevGroup> groups;          // forward, backward, READY/WAIT, then direct-reduce
   int n_fwd_groups = 0;
+  int direct_begin = 0, direct_end = 0;  // loopback direct-reduce backward groups (direct plans)
   std::vector<int32_t> idx;              // row index pool
   std::vector<int64_t> term_ptr;         // fold row pointers
   std::vector<uint32_t> terms;           // fold terms

@@ -30,9 +30,11 @@ def test_library_exports_every_header_symbol(built):
     assert declared == set(D.SYMBOLS)
 
 
-def _ctx(g, dims, topo=None, seed=0, device=-1):
+def _ctx(g, dims, topo=None, seed=0, device=-1, options=None):
     D = _D()
     c = D.loopback(g.m, g.part, dims, device=device)
+    for k, v in (options or {}).items():
+        c.set_option(k, v)
     c.build_plan(g.req_ptr, g.req_ids, seed=seed, topology=topo)
     return c
 
@@ -89,11 +91,11 @@ def test_unreachable_gpu_is_eplan():
     assert e.value.status == 6
 
 
-def _check_lowering(g, dims, topo, seed):
+def _check_lowering(g, dims, topo, seed, options=None):
     m = g.m
     R = [g.R(d) for d in range(m)]
     loc, _ = halo.local_rows(g.part, m)
-    c = _ctx(g, dims, topo, seed)
+    c = _ctx(g, dims, topo, seed, options=options)
     info = c.plan_info()
     E = c.plan_export()
     owner, Dd = spst.relation_from_lists(R, g.part)
@@ -132,10 +134,11 @@ def _check_lowering(g, dims, topo, seed):
     return info
 
 
-@pytest.mark.parametrize("m", [2, 3, 8])
-def test_uniform_plan_and_lowering(m):
+@pytest.mark.parametrize("m,direct", [(2, 1), (3, 1), (8, 1), (3, 0), (8, 0)])
+def test_uniform_plan_and_lowering(m, direct):
+    """direct=1: loopback in-place reduce program; direct=0: push to slots + owner reduce."""
     g = synth.make_graph(1500, 12000, m, graph_seed=m, part_seed=50 + m)
-    info = _check_lowering(g, [16, 5], None, seed=3)
+    info = _check_lowering(g, [16, 5], None, seed=3, options={"direct_reduce": direct})
     assert info["n_stages"] == 1 and info["n_relay_rows"] == 0
 
 
