@@ -35,8 +35,10 @@ constexpr int kTabTp = 128;          // stage: term_ptr window (FOLD)
 constexpr int kTabDst = 2176;        // stage: destination-row window
 constexpr int kMetaDst = 2048;       // meta: destination rows (FOLD init operand)
 constexpr int kMetaTerms = 4096;     // meta: terms window
-constexpr size_t kMetaOff = 128;
-constexpr size_t kStageOff = kMetaOff + 2 * (size_t)kMetaBytes;
+constexpr int kDescSlots = 4;        // producer descriptor ring
+constexpr size_t kMetaOff = 128;     // after the mbarriers (4 full, 4 empty, 2 meta, 4 desc)
+constexpr size_t kDescOff = kMetaOff + 2 * (size_t)kMetaBytes;
+constexpr size_t kStageOff = kDescOff + kDescSlots * 64;
 constexpr size_t kSmemBytes = kStageOff + (size_t)kStages * kTmaBufBytes;
 static_assert(kSmemBytes <= 227 * 1024, "shared memory budget");
 
@@ -291,7 +293,9 @@ __global__ void __launch_bounds__(512, 1)
   uint64_t *full = reinterpret_cast<uint64_t *>(dsmem);
   uint64_t *empty = full + kStages;
   uint64_t *metab = empty + kStages;
+  uint64_t *descb = metab + 2;
   uint8_t *metas = dsmem + kMetaOff;
+  DevItem *descs = reinterpret_cast<DevItem *>(dsmem + kDescOff);
   uint8_t *stages = dsmem + kStageOff;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
@@ -302,30 +306,44 @@ __global__ void __launch_bounds__(512, 1)
     }
     mbar_init(&metab[0], 1);
     mbar_init(&metab[1], 1);
+    for (int s = 0; s < kDescSlots; ++s) mbar_init(&descb[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
 
   if (warp == 0) {
     // ------------------------------- producer warp -------------------------------------------
-    const int G = gridDim.x;
+    // item q of this CTA is P.items[blockIdx.x + q * gridDim.x]; its descriptor is bulk-copied
+    // into ring slot q % 4 two items ahead, its index windows into meta buffer q % 2 one ahead
+    const uint32_t G = gridDim.x;
+    const uint32_t nmine =
+        blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
+    auto request_desc = [&](uint32_t q) {  // lane 0
+      const uint32_t s = q % kDescSlots;
+      fence_proxy_async_smem();
+      mbar_expect_tx(&descb[s], (uint32_t)sizeof(DevItem));
+      bulk_g2s(descs + s, P.items + blockIdx.x + q * G, (uint32_t)sizeof(DevItem), &descb[s]);
+    };
+    auto desc_ready = [&](uint32_t q) -> const DevItem & {
+      mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
+      return descs[q % kDescSlots];
+    };
     uint32_t k = 0;  // data items issued (stage sequence)
-    uint32_t m = 0;  // items whose metadata was issued (meta buffer sequence)
+    uint32_t m = 0;  // this CTA's item sequence
     bool ok = true;
-    int it = blockIdx.x;
-    DevItem d0, d1;
-    if (it < P.n_items) {
-      d0 = load_item(P.items, it);
-      if (lane == 0) issue_meta(P, d0, metas, &metab[0]);
+    if (lane == 0)
+      for (uint32_t q = 0; q < 2 && q < nmine; ++q) request_desc(q);
+    if (nmine > 0) {
+      const DevItem &I0 = desc_ready(0);
+      if (lane == 0) issue_meta(P, I0, metas, &metab[0]);
     }
-    if (it + G < P.n_items) d1 = load_item(P.items, it + G);
-    for (; it < P.n_items; it += G, ++m) {
-      // metadata of the next item and the descriptor of the one after
-      if (it + G < P.n_items && lane == 0)
-        issue_meta(P, d1, metas + ((m + 1) & 1) * kMetaBytes, &metab[(m + 1) & 1]);
-      DevItem d2;
-      if (it + 2 * G < P.n_items) d2 = load_item(P.items, it + 2 * G);
-      const DevItem &I = d0;
+    for (; m < nmine; ++m) {
+      if (lane == 0 && m + 2 < nmine) request_desc(m + 2);
+      if (m + 1 < nmine) {
+        const DevItem &In = desc_ready(m + 1);
+        if (lane == 0) issue_meta(P, In, metas + ((m + 1) & 1) * kMetaBytes, &metab[(m + 1) & 1]);
+      }
+      const DevItem &I = desc_ready(m);
       if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer
         if (lane == 0)
@@ -357,15 +375,12 @@ __global__ void __launch_bounds__(512, 1)
         ++k;
       }
       __syncwarp();
-      d0 = d1;
-      d1 = d2;
     }
     if (!ok) {
-      // watchdog abort: metadata copies still in flight must land before the CTA leaves
-      for (uint32_t q = m; q < m + 2; ++q) {
-        const int iq = blockIdx.x + (int)q * G;
-        if (iq < P.n_items) mbar_wait(&metab[q & 1], (q >> 1) & 1u);
-      }
+      // watchdog abort: descriptor / metadata copies still in flight land before the CTA leaves
+      for (uint32_t q = m; q < m + 3 && q < nmine; ++q)
+        mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
+      for (uint32_t q = m; q < m + 2 && q < nmine; ++q) mbar_wait(&metab[q & 1], (q >> 1) & 1u);
     }
     // END marker: consumers drain every issued stage, then stop
     const uint32_t stage = k % kStages, use = k / kStages;
