@@ -33,6 +33,7 @@ inline int64_t pitch_of(int dim) { return (dim + 3) / 4 * 4; }
 struct Program {
   // one launch: items for one (layer, direction, executing rank or -1 = fused loopback)
   std::vector<DevItem> items;
+  std::vector<DevRun> runs;
   size_t dev_off = 0;  // offset (in items) into the device item pool
 };
 
@@ -73,6 +74,10 @@ struct dgcl_ctx {
   int64_t *d_term_ptr = nullptr;
   uint32_t *d_terms = nullptr;
   DevItem *d_items = nullptr;
+  DevRun *d_runs = nullptr;
+  int64_t run_bytes = 0;
+  bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
+  bool bulk_store_peer = false;   // TMA stores into peer memory over NVLink (not yet validated)
   std::vector<Program> progs;  // index prog_index(layer, dir, r)
   std::vector<int32_t> host_gids[2];  // group order of the host interpreter per direction
   bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
@@ -282,7 +287,8 @@ void build_programs(dgcl_ctx *c) {
       for (int r = 0; r < c->n_prog_ranks; ++r) {
         Program &P = c->progs[c->prog_index(l, dir, r)];
         const std::vector<uint8_t> need = needed_counters(L, gids[r]);
-        build_items(L, gids[r], (int64_t)c->dims[l] * 4, c->item_bytes, !fused, need, &P.items);
+        build_items(L, gids[r], (int64_t)c->dims[l] * 4, c->item_bytes, !fused, need, &P.items,
+                    &P.runs);
       }
     }
   }
@@ -355,6 +361,8 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   P.err = c->err_dev;
   P.row16 = (P.row_bytes + 15) / 16 * 16;
   P.tma_buf = kTmaBufBytes;
+  P.runs = c->d_runs;
+  P.bulk_store = (c->loopback ? c->bulk_store_local : c->bulk_store_peer) ? 1 : 0;
   // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage
   P.use_tma = (v16 && c->use_tma && c->tma_ctas > 0 &&
                c->max_fold_slots * P.row16 <= kTmaOperandBytes) ? 1 : 0;
@@ -514,11 +522,19 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   if ((s = upload(c, &c->d_term_ptr, c->low.term_ptr)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_terms, c->low.terms)) != DGCL_OK) return s;
   std::vector<DevItem> all;
+  std::vector<DevRun> all_runs;
   for (Program &p : c->progs) {
     p.dev_off = all.size();
-    all.insert(all.end(), p.items.begin(), p.items.end());
+    const int64_t run_base = (int64_t)all_runs.size();
+    for (DevItem it : p.items) {
+      if (it.op == OP_COPY) it.tp += run_base;  // program-relative -> pool index
+      all.push_back(it);
+    }
+    all_runs.insert(all_runs.end(), p.runs.begin(), p.runs.end());
   }
   if ((s = upload(c, &c->d_items, all)) != DGCL_OK) return s;
+  if ((s = upload(c, &c->d_runs, all_runs)) != DGCL_OK) return s;
+  c->run_bytes = (int64_t)(all_runs.size() * sizeof(DevRun));
   // watchdog word in mapped host memory
   CUDA_TRY(c, cudaHostAlloc((void **)&c->err_host, 64, cudaHostAllocMapped));
   std::memset(c->err_host, 0, 64);
@@ -799,6 +815,14 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     c->use_tma = value != 0;
     return DGCL_OK;
   }
+  if (k == "bulk_store") {  // TMA stores for local (loopback) destinations
+    c->bulk_store_local = value != 0;
+    return DGCL_OK;
+  }
+  if (k == "bulk_store_peer") {  // TMA stores into peer memory (multi-GPU)
+    c->bulk_store_peer = value != 0;
+    return DGCL_OK;
+  }
   if (k == "direct_reduce") {
     c->direct_reduce = value != 0;
     if (c->planned) build_programs(c);
@@ -861,6 +885,7 @@ dgcl_status dgcl_destroy(dgcl_ctx *c) {
     cudaFree(c->d_term_ptr);
     cudaFree(c->d_terms);
     cudaFree(c->d_items);
+    cudaFree(c->d_runs);
     if (c->stage_a) cudaFree(c->stage_a);
     if (c->stage_b) cudaFree(c->stage_b);
     if (c->err_host) cudaFreeHost(c->err_host);

@@ -78,6 +78,20 @@ __device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t 
       "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+__device__ __forceinline__ void bulk_s2g(void *gdst, const void *ssrc, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst),
+               "r"(smem_u32(ssrc)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() {
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() {
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
 // generic-proxy accesses (acquired flags, smem reads) before async-proxy bulk copies
 __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -119,9 +133,9 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
                                            uint64_t *bar) {
   uint32_t tx = 0;
   Win ws = {0, 0, 0}, wd = {0, 0, 0}, wt = {0, 0, 0};
-  if (I.op == OP_COPY && I.src < 0) {
-    ws = window(~I.src, I.rows, 4);
-    tx += ws.bytes;
+  if (I.op == OP_COPY) {
+    wt = {I.tp, (uint32_t)I.nterms * (uint32_t)sizeof(DevRun), 0};  // the item's row runs
+    tx += wt.bytes;
   } else if (I.op == OP_FOLD) {
     ws = window(I.tp, I.rows + 1, 8);
     wt = window(I.t0, I.nterms, 4);
@@ -137,7 +151,10 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
     bulk_g2s(meta, I.op == OP_FOLD ? (const void *)(P.term_ptr + ws.a) : (const void *)(P.idx + ws.a),
              ws.bytes, bar);
   if (wd.bytes) bulk_g2s(meta + kMetaDst, P.idx + wd.a, wd.bytes, bar);
-  if (wt.bytes) bulk_g2s(meta + kMetaTerms, P.terms + wt.a, wt.bytes, bar);
+  if (wt.bytes)
+    bulk_g2s(meta + kMetaTerms,
+             I.op == OP_COPY ? (const void *)(P.runs + wt.a) : (const void *)(P.terms + wt.a),
+             wt.bytes, bar);
 }
 
 // operand bytes of a data item (must equal the sum of the row gathers issued)
@@ -171,13 +188,23 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
   }
   uint8_t *ops = st + kStageHdrBytes;
   if (I.op == OP_COPY) {
+    // one bulk copy per run of consecutive source rows when rows are packed (pitch == row16)
     const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
     const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
-    const int32_t *sidx = reinterpret_cast<const int32_t *>(meta);
-    const int32_t skew = I.src < 0 ? (int32_t)(~I.src - window(~I.src, I.rows, 4).a) : 0;
-    for (int r = lane; r < I.rows; r += 32) {
-      const int64_t srow = I.src >= 0 ? I.src + r : (int64_t)sidx[skew + r];
-      bulk_g2s(ops + (size_t)r * r16, sbase + srow * spitch, r16, full);
+    const DevRun *runs = reinterpret_cast<const DevRun *>(meta + kMetaTerms);
+    if (spitch == (int64_t)r16) {
+      for (int q = lane; q < I.nterms; q += 32) {
+        const DevRun R = runs[q];
+        bulk_g2s(ops + (size_t)R.pos * r16, sbase + (int64_t)R.src * spitch,
+                 (uint32_t)R.len * r16, full);
+      }
+    } else {
+      for (int q = lane; q < I.nterms; q += 32) {
+        const DevRun R = runs[q];
+        for (int j = 0; j < R.len; ++j)
+          bulk_g2s(ops + (size_t)(R.pos + j) * r16, sbase + (int64_t)(R.src + j) * spitch, r16,
+                   full);
+      }
     }
   } else {
     const int64_t *tpm = reinterpret_cast<const int64_t *>(meta);
@@ -400,10 +427,29 @@ __global__ void __launch_bounds__(512, 1)
       const uint8_t *st = stages + (size_t)stage * kTmaBufBytes;
       const DevItem I = *reinterpret_cast<const DevItem *>(st);
       if (I.op == OP_END) break;
-      if (I.op == OP_COPY)
+      const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
+      const bool bulk =
+          I.op == OP_COPY && P.bulk_store && I.dst >= 0 && DB.pitch == (int64_t)P.row16;
+      if (bulk) {
+        // consecutive packed destination rows: this warp's share is one bulk (TMA) store
+        const int64_t lo = (int64_t)I.rows * cw / n_cons_warps;
+        const int64_t hi = (int64_t)I.rows * (cw + 1) / n_cons_warps;
+        if (lane == 0 && hi > lo) {
+          bulk_s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
+                   (uint32_t)((hi - lo) * P.row16));
+          bulk_commit();
+          if (I.flags & kItemSignal) {
+            bulk_wait_all();              // writes performed ...
+            fence_proxy_async_global();   // ... and ordered before the generic release below
+          } else {
+            bulk_wait_read();             // the stage may be reused
+          }
+        }
+      } else if (I.op == OP_COPY) {
         store_copy(P, I, st, tid, T);
-      else
+      } else {
         store_fold(P, I, st, tid, T);
+      }
       if (I.flags & kItemSignal) {
         // this warp's stores are visible system-wide before its share of the rows is counted;
         // the receiver sees the item's full count only after every warp published (done flag)
@@ -416,6 +462,7 @@ __global__ void __launch_bounds__(512, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // this warp is done reading the stage
     }
+    if (lane == 0) bulk_wait_all();  // bulk stores complete before the CTA retires
   }
 }
 

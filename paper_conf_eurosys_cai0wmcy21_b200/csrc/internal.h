@@ -91,8 +91,9 @@ struct alignas(16) DevItem {
   int64_t src;         // >= 0: first source row (rows are consecutive); < 0: ~(idx pool offset)
   int64_t dst;         // same encoding for the destination rows
   int64_t tp;          // OP_FOLD: term_ptr pool index of the first row (rows + 1 entries)
+                       // OP_COPY: index of the item's first DevRun in the run pool
   int64_t t0;          // OP_FOLD: term_ptr[tp] (index of the first term)
-  int32_t nterms;      // OP_FOLD: terms of the item
+  int32_t nterms;      // OP_FOLD: terms of the item; OP_COPY: runs of the item
   int32_t group;       // originating group (diagnostics / watchdog codes)
 };
 static_assert(sizeof(DevItem) == 64, "DevItem is one 64-B descriptor");
@@ -132,8 +133,16 @@ struct ExecParams {
   int *err;            // host-mapped error word (0 = ok)
   int32_t use_tma;     // 1: bulk-copy (TMA) gather into shared memory, then store from smem
   int32_t row16;       // row bytes rounded up to 16 (bulk-copy size per row)
-  int32_t tma_buf;     // bytes per shared-memory stage buffer (two stages)
-  int32_t pad1;
+  int32_t tma_buf;     // bytes per shared-memory stage buffer
+  int32_t bulk_store;  // 1: contiguous COPY destinations are written with bulk (TMA) stores
+  const struct DevRun *runs;  // COPY items: maximal runs of consecutive (source, destination) rows
+};
+
+// A run of `len` rows whose source rows src.. and destination rows dst.. are both consecutive;
+// `pos` is the first row's index inside its item.  One bulk copy moves a run when the pitches
+// equal the 16-B-rounded row.
+struct DevRun {
+  int32_t src, dst, len, pos;
 };
 
 // Bulk-copy executor (executor_tma.cu) shared-memory geometry and the item limits it implies:

@@ -387,7 +387,8 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
 
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
                  int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
-                 std::vector<DevItem> *items) {
+                 std::vector<DevItem> *items, std::vector<DevRun> *runs) {
+  runs->clear();
   // An item is a row range whose gathered operands fit `item_bytes` (and one shared-memory stage
   // of the bulk-copy executor): a COPY row costs one row, a FOLD row (1 + #terms) rows.
   items->clear();
@@ -463,6 +464,23 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
           it.tp = g.term_ptr + rb;
           it.t0 = low.term_ptr[it.tp];
           it.nterms = (int32_t)(low.term_ptr[it.tp + it.rows] - it.t0);
+        } else if (g.op == OP_COPY) {
+          // maximal runs of consecutive source and destination rows (one bulk copy each)
+          it.tp = (int64_t)runs->size();
+          auto srow = [&](int64_t i) {
+            return g.src_idx >= 0 ? (int64_t)low.idx[g.src_idx + i] : g.src_base + i;
+          };
+          auto drow = [&](int64_t i) {
+            return g.dst_idx >= 0 ? (int64_t)low.idx[g.dst_idx + i] : g.dst_base + i;
+          };
+          for (int64_t i = rb; i < rb + it.rows;) {
+            int64_t j = i + 1;
+            while (j < rb + it.rows && srow(j) == srow(j - 1) + 1 && drow(j) == drow(j - 1) + 1)
+              ++j;
+            runs->push_back({(int32_t)srow(i), (int32_t)drow(i), (int32_t)(j - i), (int32_t)(i - rb)});
+            i = j;
+          }
+          it.nterms = (int32_t)((int64_t)runs->size() - it.tp);
         }
         bool sig = data && g.sig_ctr >= 0;
         if (sig && !signal_all)

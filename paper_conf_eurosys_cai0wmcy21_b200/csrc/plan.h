@@ -88,9 +88,10 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
 // Work items for one launch: the groups `gids` (already in stage order) cut into row ranges of
 // about item_bytes bytes and interleaved across groups within a stage.
 // completion_rank >= 0 appends nothing (the WAIT group is passed in gids by the caller).
+// COPY items also get their row runs appended to `runs` (item.tp = first run, program-relative).
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
                  int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
-                 std::vector<DevItem> *items);
+                 std::vector<DevItem> *items, std::vector<DevRun> *runs);
 
 // largest number of operand rows one FOLD row gathers (1 + #terms); bounds the bulk-copy stage
 int64_t max_fold_slots(const Lowered &low);

@@ -142,13 +142,16 @@ def test_tiny_config_bit_exact():
     _check_case(Case(g, cfg.dims))
 
 
-@pytest.mark.parametrize("m,tma,direct", [(3, 1, 1), (4, 1, 1), (8, 1, 1), (4, 0, 1), (8, 0, 1),
-                                          (8, 1, 0), (3, 0, 0)])
-def test_uniform_loopback_fused(m, tma, direct):
+@pytest.mark.parametrize("m,tma,direct,bulk", [(3, 1, 1, 1), (4, 1, 1, 1), (8, 1, 1, 1),
+                                               (8, 1, 1, 0), (4, 0, 1, 1), (8, 0, 1, 1),
+                                               (8, 1, 0, 1), (3, 0, 0, 1), (4, 1, 0, 0)])
+def test_uniform_loopback_fused(m, tma, direct, bulk):
     """tma=1: bulk-copy (cp.async.bulk) gather executor; tma=0: the register (LDG) executor.
-    direct=1: loopback in-place reduce; direct=0: push to slots + owner reduce (multi-GPU form)."""
+    direct=1: loopback in-place reduce; direct=0: push to slots + owner reduce (multi-GPU form).
+    bulk=1: packed contiguous destinations written with bulk (TMA) stores; 0: 16-B st.global."""
     g = synth.make_graph(6000, 60000, m, graph_seed=m, part_seed=7 * m)
-    _check_case(Case(g, [64, 5, 602], options={"tma": tma, "direct_reduce": direct}))
+    _check_case(Case(g, [64, 5, 602], options={"tma": tma, "direct_reduce": direct,
+                                               "bulk_store": bulk}))
 
 
 @pytest.mark.parametrize("m", [2, 8])
