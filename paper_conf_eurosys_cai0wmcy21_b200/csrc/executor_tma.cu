@@ -217,25 +217,28 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     const BufRef SL = P.buf[K_SLOT][I.exec_rank];
     const BufRef HG = P.buf[K_HGRAD][I.exec_rank];
     const int init = I.fold_init;
-    for (int r = lane; r < I.rows; r += 32) {
+    // row by row; the row's operands (init row, then terms) are gathered by lanes 0, 1, ... in
+    // parallel (at most 1 + 16 operands per row)
+    for (int r = 0; r < I.rows; ++r) {
       const int64_t ta = tpm[tps + r], tb = tpm[tps + r + 1];
-      uint32_t slot = (uint32_t)(ta - I.t0) + (init ? r : 0);
-      if (init) {
-        const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)dm[ds + r];
-        bulk_g2s(ops + (size_t)(slot++) * r16, D.ptr + drow * D.pitch, r16, full);
-      }
-      for (int64_t t = ta; t < tb; ++t) {
-        const uint32_t term = tm[ts + (t - I.t0)];
-        const BufRef *B;
-        uint32_t row;
-        if (I.term_mode == kTermRankHgrad) {
-          B = &P.buf[K_HGRAD][term >> 28];
-          row = term & kTermRowMask;
+      const uint32_t slot0 = (uint32_t)(ta - I.t0) + (init ? r : 0);
+      const int cnt = (int)(tb - ta) + (init ? 1 : 0);
+      for (int j = lane; j < cnt; j += 32) {
+        const char *src;
+        if (init && j == 0) {
+          const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)dm[ds + r];
+          src = D.ptr + drow * D.pitch;
         } else {
-          B = (term & kTermSlot) ? &SL : &HG;
-          row = term & ~kTermSlot;
+          const uint32_t term = tm[ts + (ta - I.t0) + j - (init ? 1 : 0)];
+          if (I.term_mode == kTermRankHgrad) {
+            const BufRef &B = P.buf[K_HGRAD][term >> 28];
+            src = B.ptr + (int64_t)(term & kTermRowMask) * B.pitch;
+          } else {
+            const BufRef &B = (term & kTermSlot) ? SL : HG;
+            src = B.ptr + (int64_t)(term & ~kTermSlot) * B.pitch;
+          }
         }
-        bulk_g2s(ops + (size_t)(slot++) * r16, B->ptr + (int64_t)row * B->pitch, r16, full);
+        bulk_g2s(ops + (size_t)(slot0 + j) * r16, src, r16, full);
       }
     }
   }
