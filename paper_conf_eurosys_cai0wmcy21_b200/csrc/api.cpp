@@ -365,7 +365,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   P.bulk_store = (c->loopback ? c->bulk_store_local : c->bulk_store_peer) ? 1 : 0;
   // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage
   P.use_tma = (v16 && c->use_tma && c->tma_ctas > 0 &&
-               c->max_fold_slots * P.row16 <= kTmaOperandBytes) ? 1 : 0;
+               P.row16 <= kTmaOperandBytes) ? 1 : 0;
   const int grid_all = P.use_tma ? c->n_sm * c->tma_ctas : c->grid;
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
   P.use_ready = (!fused && m > 1) ? 1 : 0;

@@ -136,15 +136,8 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
   if (I.op == OP_COPY) {
     wt = {I.tp, (uint32_t)I.nterms * (uint32_t)sizeof(DevRun), 0};  // the item's row runs
     tx += wt.bytes;
-  } else if (I.op == OP_FOLD) {
-    ws = window(I.tp, I.rows + 1, 8);
-    wt = window(I.t0, I.nterms, 4);
-    tx += ws.bytes + wt.bytes;
-    if (I.fold_init && I.dst < 0) {
-      wd = window(~I.dst, I.rows, 4);
-      tx += wd.bytes;
-    }
   }
+  // OP_FOLD: the consumers gather the operands themselves; nothing for the producer to prefetch
   fence_proxy_async_smem();
   mbar_expect_tx(bar, tx);
   if (ws.bytes)
@@ -157,11 +150,10 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
              wt.bytes, bar);
 }
 
-// operand bytes of a data item (must equal the sum of the row gathers issued)
+// bytes bulk-copied into the operand area of a stage (gathered rows, or a FOLD's terms window)
 __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const DevItem &I) {
-  const uint32_t slots =
-      I.op == OP_COPY ? (uint32_t)I.rows : (uint32_t)I.nterms + (I.fold_init ? I.rows : 0);
-  return slots * (uint32_t)P.row16;
+  if (I.op == OP_COPY) return (uint32_t)I.rows * (uint32_t)P.row16;
+  return window(I.t0, I.nterms, 4).bytes;
 }
 
 // producer warp: header, consumer tables and row gathers of data item I into `st`
@@ -206,41 +198,11 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
                    full);
       }
     }
-  } else {
-    const int64_t *tpm = reinterpret_cast<const int64_t *>(meta);
-    const int32_t tps = (int32_t)(I.tp - window(I.tp, I.rows + 1, 8).a);
-    const uint32_t *tm = reinterpret_cast<const uint32_t *>(meta + kMetaTerms);
-    const int32_t ts = (int32_t)(I.t0 - window(I.t0, I.nterms, 4).a);
-    const int32_t *dm = reinterpret_cast<const int32_t *>(meta + kMetaDst);
-    const int32_t ds = I.dst < 0 ? (int32_t)(~I.dst - window(~I.dst, I.rows, 4).a) : 0;
-    const BufRef D = P.buf[I.dst_kind][I.dst_rank];
-    const BufRef SL = P.buf[K_SLOT][I.exec_rank];
-    const BufRef HG = P.buf[K_HGRAD][I.exec_rank];
-    const int init = I.fold_init;
-    // row by row; the row's operands (init row, then terms) are gathered by lanes 0, 1, ... in
-    // parallel (at most 1 + 16 operands per row)
-    for (int r = 0; r < I.rows; ++r) {
-      const int64_t ta = tpm[tps + r], tb = tpm[tps + r + 1];
-      const uint32_t slot0 = (uint32_t)(ta - I.t0) + (init ? r : 0);
-      const int cnt = (int)(tb - ta) + (init ? 1 : 0);
-      for (int j = lane; j < cnt; j += 32) {
-        const char *src;
-        if (init && j == 0) {
-          const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)dm[ds + r];
-          src = D.ptr + drow * D.pitch;
-        } else {
-          const uint32_t term = tm[ts + (ta - I.t0) + j - (init ? 1 : 0)];
-          if (I.term_mode == kTermRankHgrad) {
-            const BufRef &B = P.buf[K_HGRAD][term >> 28];
-            src = B.ptr + (int64_t)(term & kTermRowMask) * B.pitch;
-          } else {
-            const BufRef &B = (term & kTermSlot) ? SL : HG;
-            src = B.ptr + (int64_t)(term & ~kTermSlot) * B.pitch;
-          }
-        }
-        bulk_g2s(ops + (size_t)(slot0 + j) * r16, src, r16, full);
-      }
-    }
+  } else if (lane == 0) {
+    // OP_FOLD: only the terms window is staged (into the operand area); the consumers gather
+    // the operand rows themselves, many loads in flight per warp
+    const Win wt = window(I.t0, I.nterms, 4);
+    if (wt.bytes) bulk_g2s(ops, P.terms + wt.a, wt.bytes, full);
   }
 }
 
@@ -292,24 +254,56 @@ __device__ __forceinline__ void store_fold(const ExecParams &P, const DevItem &I
   const int32_t *info = reinterpret_cast<const int32_t *>(st + kHdrInfo);
   const int64_t *tp = reinterpret_cast<const int64_t *>(st + kTabTp) + info[0];
   const int32_t *tab = reinterpret_cast<const int32_t *>(st + kTabDst) + info[1];
+  const uint32_t *tm = reinterpret_cast<const uint32_t *>(st + kStageHdrBytes) +
+                       window(I.t0, I.nterms, 4).skew;  // the item's terms, staged by the producer
   const int init = I.fold_init;
+  const int mode = I.term_mode;
+  const int exec = I.exec_rank;
   const uint32_t nch = (uint32_t)P.n_chunks;
-  const uint32_t r16 = (uint32_t)P.row16;
   const uint32_t total = (uint32_t)I.rows * nch;
   const int tail = P.row_bytes - (int)(nch - 1) * 16;
-  const uint8_t *ops = st + kStageHdrBytes;
+  // operand j of the current row at chunk col: halo-gradient rows are read-only inputs (nc),
+  // slots were written during the launch (cg)
+  auto operand = [&](uint32_t term, uint32_t col, int nb) -> int4 {
+    const bool slot = mode == kTermLocal && (term & kTermSlot) != 0;
+    const BufRef &B = mode == kTermRankHgrad ? P.buf[K_HGRAD][term >> 28]
+                      : slot                 ? P.buf[K_SLOT][exec]
+                                             : P.buf[K_HGRAD][exec];
+    const uint32_t row = mode == kTermRankHgrad ? (term & kTermRowMask) : (term & ~kTermSlot);
+    const char *p = B.ptr + (int64_t)row * B.pitch + (int64_t)col * 16;
+    if (nb == 16) return slot ? ld_cg_v4(p) : ld_nc_v4(p);
+    return slot ? ld_part<false>(p, nb) : ld_part<true>(p, nb);
+  };
+  constexpr int kBatch = 8;
   for (uint32_t e = tid; e < total; e += T) {
     const uint32_t r = fdiv(e, P);
     const uint32_t col = e - r * nch;
+    const int nb = col + 1 == nch ? tail : 16;
     const int64_t ta = tp[r], tb = tp[r + 1];
-    const uint32_t base = (uint32_t)(ta - I.t0) + (init ? r : 0);
-    const uint32_t cnt = (uint32_t)(tb - ta) + (init ? 1 : 0);
-    const uint8_t *p = ops + (size_t)base * r16 + col * 16;
-    float4 acc = as_f4(lds_v4(p));
-    for (uint32_t j = 1; j < cnt; ++j) add4(acc, lds_v4(p + (size_t)j * r16));
+    const uint32_t *rt = tm + (ta - I.t0);
+    const int cnt = (int)(tb - ta);
     const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
     char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
-    const int nb = col + 1 == nch ? tail : 16;
+    float4 acc;
+    int j = 0;
+    if (init) {
+      acc = as_f4(nb == 16 ? ld_cg_v4(dp) : ld_part<false>(dp, nb));
+    } else {
+      acc = as_f4(operand(rt[0], col, nb));
+      j = 1;
+    }
+    while (j < cnt) {
+      // up to kBatch independent loads in flight, then the adds in list order
+      int4 v[kBatch];
+      const int n = cnt - j < kBatch ? cnt - j : kBatch;
+#pragma unroll
+      for (int q = 0; q < kBatch; ++q)
+        if (q < n) v[q] = operand(rt[j + q], col, nb);
+#pragma unroll
+      for (int q = 0; q < kBatch; ++q)
+        if (q < n) add4(acc, v[q]);
+      j += n;
+    }
     if (nb == 16)
       st_v4(dp, as_i4(acc));
     else

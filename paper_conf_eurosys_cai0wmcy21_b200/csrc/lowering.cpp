@@ -420,9 +420,12 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         for (int64_t r = 0; r < g.n_rows; ++r) {
           const int64_t slots = low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r] +
                                 (g.fold_init ? 1 : 0);
+          // FOLD operands are gathered by the consumers straight from memory (not staged): the
+          // item is bounded by 4x the gathered bytes of a COPY item and by its tables
           const int64_t cost = slots * row16;
           const int64_t nt = low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + b.back()];
-          if (acc > 0 && (acc + cost > cap || r - b.back() >= kMaxFoldRows || nt > kMaxItemTerms)) {
+          if (acc > 0 &&
+              (acc + cost > 4 * cap || r - b.back() >= kMaxFoldRows || nt > kMaxItemTerms)) {
             b.push_back((int32_t)r);
             acc = 0;
           }
