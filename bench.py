@@ -33,7 +33,6 @@ sys.path.insert(0, ROOT)
 
 METRIC = "per-layer embedding-exchange ms and NVLink GB/s/GPU at 1/2/4/8 B200 vs 900 GB/s"
 UNIT = "GB/s"
-NVLINK_PEER_GBS = 770.0  # measured peer copy per direction (B200_PROFILING.md); 900 nominal
 
 
 def log(*a):
@@ -366,143 +365,6 @@ def run_ours_single(args, w):
     return out
 
 
-def run_ours_multi(args, w, rank, world, local_rank):
-    """One process per GPU; the exchange runs over NVLink peer memory (CUDA IPC)."""
-    import torch
-    import torch.distributed as dist
-    import paper_conf_eurosys_cai0wmcy21_b200 as D
-    c = w.cfg
-    g = w.g
-    dev = 0 if args.share_gpu else local_rank
-    torch.cuda.set_device(dev)
-    topo = None
-    if c.topology != "uniform_nvswitch":
-        import synth
-        topo = synth.topology.by_name(c.topology, world)
-    # the partition of this run: the config's graph partitioned over `world` GPUs
-    import synth
-    part = synth.partition(c.n, world, c.part_seed)
-    # required lists for this world size (rank 0 computes, all ranks receive)
-    src_dst = None
-    ctx = D.init(part, list(c.dims), rank, world, dev)
-    lists = w.lists
-    ptr = np.zeros(world + 1, np.int64)
-    ptr[1:] = np.cumsum([len(x) for x in lists])
-    ids = np.concatenate(lists)
-    ctx.build_plan(ptr, ids, seed=0, topology=topo)
-    ctx.register_workspace()
-    blobs = [None] * world
-    dist.all_gather_object(blobs, ctx.ipc_export())
-    ctx.ipc_import(blobs)
-    dist.barrier()
-    info = ctx.plan_info()
-    order = np.nonzero(part == rank)[0]
-    n_local = order.shape[0]
-    my_R = lists[rank]
-    emb, hg, eg = {}, {}, {}
-    for l in w.fwd_layers:
-        p = ctx.pitch(l)
-        emb[l] = torch.from_numpy(synth.fill_values(n_local, c.dims[l], p, keys=order,
-                                                    seed=c.emb_seed,
-                                                    stream=synth.values.STREAM_EMB + l)).cuda()
-    for l in w.bwd_layers:
-        p = ctx.pitch(l)
-        hg[l] = torch.from_numpy(synth.fill_values(len(my_R), c.dims[l], p, seed=c.grad_seed,
-                                                   stream=synth.values.STREAM_HGRAD + l)).cuda()
-        eg[l] = torch.from_numpy(synth.fill_values(n_local, c.dims[l], p, keys=order,
-                                                   seed=c.grad_seed,
-                                                   stream=synth.values.STREAM_EGRAD + l)).cuda()
-    stream = torch.cuda.current_stream()
-    names = ["fwd%d_d%d" % (l, c.dims[l]) for l in w.fwd_layers] + \
-            ["bwd%d_d%d" % (l, c.dims[l]) for l in w.bwd_layers]
-
-    def step(evs=None):
-        i = 0
-        for l in w.fwd_layers:
-            if evs is not None:
-                evs[i][0].record(stream)
-            ctx.forward(l, emb[l], stream=stream)
-            if evs is not None:
-                evs[i][1].record(stream)
-            i += 1
-        for l in w.bwd_layers:
-            if evs is not None:
-                evs[i][0].record(stream)
-            ctx.backward(l, hg[l], eg[l], stream=stream)
-            if evs is not None:
-                evs[i][1].record(stream)
-            i += 1
-
-    clk = ClockSampler(dev) if rank == 0 else None
-    if clk:
-        clk.start()
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize()
-    ctx.check()
-    K = args.steps
-    evs = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)]
-            for _ in names] for _ in range(K)]
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    l0 = ctx.launch_count()
-    dist.barrier()
-    torch.cuda.synchronize()
-    tw0 = time.time()
-    e0.record(stream)
-    for k in range(K):
-        step(evs[k])
-    e1.record(stream)
-    torch.cuda.synchronize()
-    dist.barrier()
-    tw1 = time.time()
-    ctx.check()
-    launches = ctx.launch_count() - l0
-    t = torch.tensor([e0.elapsed_time(e1)] + [statistics.mean(
-        evs[k][i][0].elapsed_time(evs[k][i][1]) for k in range(K)) for i in range(len(names))],
-        dtype=torch.float64)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    lt = torch.tensor([float(launches)], dtype=torch.float64)
-    dist.all_reduce(lt)
-    if clk:
-        clk.stop()
-    if rank != 0:
-        ctx.destroy()
-        return None
-    ms_step = float(t[0]) / K
-    per_op = {n: float(t[1 + i]) for i, n in enumerate(names)}
-    payload = w.S * 4 * (sum(c.dims[l] for l in w.fwd_layers) + sum(c.dims[l] for l in w.bwd_layers))
-    value = payload / (ms_step * 1e-3) / 1e9
-    counts = ctx.plan_counts()
-    out_rows = counts.sum(axis=(0, 2))
-    in_rows = counts.sum(axis=(0, 1))
-    dom = names[0]
-    maxport = int(max(out_rows.max(), in_rows.max()))
-    alg = maxport * c.dims[w.fwd_layers[0]] * 4
-    achieved = alg / (per_op[dom] * 1e-3) / 1e9
-    out = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K,
-        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
-        "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "impl": "ours",
-        "config": {"workload": "%s-shaped R-MAT, %d-way partition over %d B200 (NVLink 5)" %
-                               (c.name, world, world), "config": c.name, "dims": list(c.dims),
-                   "world": world, "parallelism": "graph-partition x%d" % world,
-                   "l2": "inputs larger than L2 (no flush needed)"},
-        "ms_per_layer": per_op,
-        "gbs_per_gpu": value / world,
-        "roofline": {"bound": "nvlink", "kernel": "executor_kernel (%s)" % dom,
-                     "achieved": achieved, "peak": NVLINK_PEER_GBS, "unit": "GB/s",
-                     "frac": achieved / NVLINK_PEER_GBS, "traffic": None,
-                     "nominal_peak": 900.0,
-                     "algorithmic_bytes_per_launch": alg},
-        "cpu_baseline": None, "e2e": None, "gpu_launches": int(lt[0]),
-        "clocks": clk.summary(tw0, tw1) if clk else None,
-        "plan": info,
-    }
-    ctx.destroy()
-    return out
-
-
 def run_reference(args, w):
     """The reference arm of this tier: the CPU oracle as it stands, timed per step on a bounded
     sample of the same workload (one destination/owner rank per step)."""
@@ -564,30 +426,11 @@ def main():
         print(json.dumps(out), flush=True)
         return
 
-    import torch.distributed as dist
-    dist.init_process_group("gloo" if args.share_gpu else "nccl")
-    import synth
-    cfg = synth.get_config(args.config)
-    # rank 0 builds the graph and the required lists for this world size; broadcast to all
-    objs = [None]
-    if rank == 0:
-        w = Workload(args.config)
-        src, dst = synth.rmat_edges(cfg.n, cfg.e, cfg.graph_seed)
-        part = synth.partition(cfg.n, world, cfg.part_seed)
-        ptr, ids = synth.required_lists(src, dst, part, world)
-        w.lists = [ids[ptr[d]:ptr[d + 1]] for d in range(world)]
-        w.S = int(ptr[-1])
-        w.g = None
-        objs = [w]
-    if dist.get_backend() == "nccl":
-        import torch
-        torch.cuda.set_device(local_rank)
-    dist.broadcast_object_list(objs, src=0)
-    w = objs[0]
-    w.g = type("G", (), {})()
-    out = run_ours_multi(args, w, rank, world, local_rank)
+    from bench_multi import run_multi
+    out = run_multi(args, METRIC, UNIT, rank, world, local_rank, ClockSampler)
     if rank == 0:
         print(json.dumps(out), flush=True)
+    import torch.distributed as dist
     dist.barrier()
     dist.destroy_process_group()
 

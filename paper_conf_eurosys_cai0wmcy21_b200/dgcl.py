@@ -245,6 +245,20 @@ def init(part, dims, rank, world, device):
     return Context(h, world, rank, part, dims, False, device)
 
 
+def build_plan_distributed(ctx, my_required, topology=None, seed=0, group=None):
+    """buildCommInfo over a process group: all-gather every rank's required list (its halo row
+    order), then every rank runs the identical deterministic plan (no master)."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    lists = [None] * world
+    dist.all_gather_object(lists, np.asarray(my_required, dtype=np.int64), group=group)
+    ptr = np.zeros(world + 1, np.int64)
+    ptr[1:] = np.cumsum([len(x) for x in lists])
+    ids = np.concatenate(lists) if ptr[-1] else np.zeros(0, np.int64)
+    ctx.build_plan(ptr, ids, seed=seed, topology=topology)
+    return ptr, ids
+
+
 def setup_distributed(part, dims, my_required, topology=None, seed=0, group=None, device=None):
     """Collective setup over a torch.distributed process group (any backend).
 
@@ -259,12 +273,7 @@ def setup_distributed(part, dims, my_required, topology=None, seed=0, group=None
     if device is None:
         device = torch.cuda.current_device()
     ctx = init(part, dims, rank, world, device)
-    lists = [None] * world
-    dist.all_gather_object(lists, np.asarray(my_required, dtype=np.int64), group=group)
-    ptr = np.zeros(world + 1, np.int64)
-    ptr[1:] = np.cumsum([len(x) for x in lists])
-    ids = np.concatenate(lists) if ptr[-1] else np.zeros(0, np.int64)
-    ctx.build_plan(ptr, ids, seed=seed, topology=topology)
+    build_plan_distributed(ctx, my_required, topology=topology, seed=seed, group=group)
     ctx.register_workspace()
     blobs = [None] * world
     dist.all_gather_object(blobs, ctx.ipc_export(), group=group)
