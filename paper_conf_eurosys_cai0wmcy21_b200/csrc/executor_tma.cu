@@ -103,6 +103,37 @@ __device__ __forceinline__ int4 lds_v4(const uint8_t *p) {
   return *reinterpret_cast<const int4 *>(p);
 }
 
+// Barrier over the consumer warps only (the producer never joins): lane 0 of each warp arrives,
+// the last one advances the generation.
+__device__ __forceinline__ void consumer_barrier(unsigned *count, volatile unsigned *gen,
+                                                 unsigned nwarps, int lane) {
+  __syncwarp();
+  if (lane == 0) {
+    const unsigned g = *gen;
+    __threadfence_block();
+    if (atomicAdd(count, 1u) == nwarps - 1) {
+      *count = 0;
+      __threadfence_block();
+      atomicAdd((unsigned *)gen, 1u);
+    } else {
+      while (*gen == g) {
+      }
+    }
+    __threadfence_block();
+  }
+  __syncwarp();
+}
+
+// non-blocking: are all counter waits of I already satisfied?
+__device__ __forceinline__ bool waits_ready(const ExecParams &P, const DevItem &I) {
+  for (int w = 0; w < I.wait_n; ++w) {
+    const DevWait W = P.waits[I.wait_off + w];
+    if (ld_acquire_sys(P.flags[I.exec_rank] + W.ctr) < P.epoch[I.dir] * (uint64_t)W.amount)
+      return false;
+  }
+  return true;
+}
+
 __device__ __forceinline__ DevItem load_item(const DevItem *items, int i) {
   DevItem d;
   const int4 *s = reinterpret_cast<const int4 *>(items + i);
@@ -133,7 +164,7 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
                                            uint64_t *bar) {
   uint32_t tx = 0;
   Win ws = {0, 0, 0}, wd = {0, 0, 0}, wt = {0, 0, 0};
-  if (I.op == OP_COPY) {
+  if (I.op == OP_COPY && !(I.flags & kItemDirect)) {
     wt = {I.tp, (uint32_t)I.nterms * (uint32_t)sizeof(DevRun), 0};  // the item's row runs
     tx += wt.bytes;
   }
@@ -152,7 +183,10 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
 
 // bytes bulk-copied into the operand area of a stage (gathered rows, or a FOLD's terms window)
 __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const DevItem &I) {
-  if (I.op == OP_COPY) return (uint32_t)I.rows * (uint32_t)P.row16;
+  if (I.op == OP_COPY) {
+    if (!(I.flags & kItemDirect)) return (uint32_t)I.rows * (uint32_t)P.row16;
+    return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;  // source-row window only
+  }
   return window(I.t0, I.nterms, 4).bytes;
 }
 
@@ -179,7 +213,13 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     if (wdst.bytes) bulk_g2s(st + kTabDst, P.idx + wdst.a, wdst.bytes, full);
   }
   uint8_t *ops = st + kStageHdrBytes;
-  if (I.op == OP_COPY) {
+  if (I.op == OP_COPY && (I.flags & kItemDirect)) {
+    // short runs: stage only the source-row window; the consumers gather the rows
+    if (lane == 0 && I.src < 0) {
+      const Win ws = window(~I.src, I.rows, 4);
+      bulk_g2s(ops, P.idx + ws.a, ws.bytes, full);
+    }
+  } else if (I.op == OP_COPY) {
     // one bulk copy per run of consecutive source rows when rows are packed (pitch == row16)
     const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
     const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
@@ -241,6 +281,50 @@ __device__ __forceinline__ void store_copy(const ExecParams &P, const DevItem &I
           const uint32_t col = e - r * nch;
           st_v4(dbase + (int64_t)tab[r] * dpitch + col * 16, lds_v4(ops + r * r16 + col * 16));
         }
+      }
+    }
+  }
+}
+
+// consumers: COPY item with short runs — gather each row chunk straight from memory (8 loads in
+// flight per thread) and store it; whole 16-B chunks (library-owned destination rows)
+__device__ __forceinline__ void store_copy_direct(const ExecParams &P, const DevItem &I,
+                                                  const uint8_t *st, uint32_t tid, uint32_t T) {
+  constexpr int kU = 8;
+  const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
+  const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
+  char *dbase = P.buf[I.dst_kind][I.dst_rank].ptr;
+  const int64_t dpitch = P.buf[I.dst_kind][I.dst_rank].pitch;
+  const int32_t *sidx = I.src < 0 ? reinterpret_cast<const int32_t *>(st + kStageHdrBytes) +
+                                        window(~I.src, I.rows, 4).skew
+                                  : nullptr;
+  const int32_t *didx = I.dst < 0 ? reinterpret_cast<const int32_t *>(st + kTabDst) +
+                                        reinterpret_cast<const int32_t *>(st + kHdrInfo)[1]
+                                  : nullptr;
+  const bool nc = readonly_kind(I.src_kind);
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  for (uint32_t e0 = tid; e0 < total; e0 += T * kU) {
+    int4 v[kU];
+#pragma unroll
+    for (int j = 0; j < kU; ++j) {
+      const uint32_t e = e0 + j * T;
+      if (e < total) {
+        const uint32_t r = fdiv(e, P);
+        const uint32_t col = e - r * nch;
+        const int64_t srow = sidx ? (int64_t)sidx[r] : I.src + r;
+        const char *sp = sbase + srow * spitch + (int64_t)col * 16;
+        v[j] = nc ? ld_nc_v4(sp) : ld_cg_v4(sp);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < kU; ++j) {
+      const uint32_t e = e0 + j * T;
+      if (e < total) {
+        const uint32_t r = fdiv(e, P);
+        const uint32_t col = e - r * nch;
+        const int64_t drow = didx ? (int64_t)didx[r] : I.dst + r;
+        st_v4(dbase + drow * dpitch + (int64_t)col * 16, v[j]);
       }
     }
   }
@@ -321,9 +405,17 @@ __global__ void __launch_bounds__(512, 1)
   uint8_t *metas = dsmem + kMetaOff;
   DevItem *descs = reinterpret_cast<DevItem *>(dsmem + kDescOff);
   uint8_t *stages = dsmem + kStageOff;
+  __shared__ uint32_t s_pend[kMaxRanks * kMaxRanks];  // rows stored, per (source, receiver)
+  __shared__ int s_pend_base;                          // their counter family
+  __shared__ unsigned s_bar_count;
+  __shared__ volatile unsigned s_bar_gen;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
+  for (int i = threadIdx.x; i < kMaxRanks * kMaxRanks; i += blockDim.x) s_pend[i] = 0;
   if (threadIdx.x == 0) {
+    s_pend_base = 0;
+    s_bar_count = 0;
+    s_bar_gen = 0;
     for (int s = 0; s < kStages; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], n_cons_warps);
@@ -352,9 +444,21 @@ __global__ void __launch_bounds__(512, 1)
       mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
       return descs[q % kDescSlots];
     };
-    uint32_t k = 0;  // data items issued (stage sequence)
+    uint32_t k = 0;  // stages issued (data items and markers)
     uint32_t m = 0;  // this CTA's item sequence
     bool ok = true;
+    bool pend = false;  // signalling items issued since the last FLUSH
+    int pend_key = -1;  // their counter family: ctr_index(dir, stage, 0)
+    auto emit_marker = [&](uint8_t op) {  // header-only stage: FLUSH or END
+      const uint32_t stage = k % kStages, use = k / kStages;
+      if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
+      if (lane == 0) {
+        reinterpret_cast<DevItem *>(stages + (size_t)stage * kTmaBufBytes)->op = op;
+        mbar_arrive(&full[stage]);
+      }
+      __syncwarp();
+      ++k;
+    };
     if (lane == 0)
       for (uint32_t q = 0; q < 2 && q < nmine; ++q) request_desc(q);
     if (nmine > 0) {
@@ -375,11 +479,32 @@ __global__ void __launch_bounds__(512, 1)
             if (s != I.exec_rank) st_release_sys(P.flags[s] + kReadyBase + I.exec_rank, P.seq);
       } else if (I.op == OP_WAIT) {
         // forward completion: the launch ends only once every incoming row landed
+        if (pend) {
+          emit_marker(OP_FLUSH);
+          pend = false;
+        }
         int w = 1;
         if (lane == 0) w = wait_item_sources(P, I, 200000 + I.group) ? 1 : 0;
         ok = __shfl_sync(0xffffffffu, w, 0) != 0;
         if (!ok) break;
       } else if (I.op == OP_COPY || I.op == OP_FOLD) {
+        // Done counts are published in batches (FLUSH markers): before this producer could
+        // block on a wait, and whenever the counter family (direction, stage) changes.
+        const bool sig = (I.flags & kItemSignal) != 0;
+        const int key = sig ? I.sig_ctr - I.exec_rank : -1;
+        if (pend) {
+          int ready = 1;
+          if (lane == 0) {
+            ready = waits_ready(P, I) ? 1 : 0;
+            if (ready && P.use_ready && I.ready_rank >= 0)
+              ready = ld_acquire_sys(P.flags[I.exec_rank] + kReadyBase + I.ready_rank) >= P.seq;
+          }
+          ready = __shfl_sync(0xffffffffu, ready, 0);
+          if (!ready || (sig && key != pend_key)) {
+            emit_marker(OP_FLUSH);
+            pend = false;
+          }
+        }
         int w = 1;
         if (lane == 0) {
           // sources final (stage chaining) and the destination's buffers free (ready word)
@@ -397,6 +522,10 @@ __global__ void __launch_bounds__(512, 1)
         issue_item(P, I, stages + (size_t)stage * kTmaBufBytes, metas + (m & 1) * kMetaBytes,
                    &full[stage], lane);
         ++k;
+        if (sig) {
+          pend = true;
+          pend_key = key;
+        }
       }
       __syncwarp();
     }
@@ -406,14 +535,8 @@ __global__ void __launch_bounds__(512, 1)
         mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
       for (uint32_t q = m; q < m + 2 && q < nmine; ++q) mbar_wait(&metab[q & 1], (q >> 1) & 1u);
     }
-    // END marker: consumers drain every issued stage, then stop
-    const uint32_t stage = k % kStages, use = k / kStages;
-    if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
-    uint8_t *st = stages + (size_t)stage * kTmaBufBytes;
-    if (lane == 0) {
-      reinterpret_cast<DevItem *>(st)->op = OP_END;
-      mbar_arrive(&full[stage]);
-    }
+    // END marker: consumers drain every issued stage, publish pending counts, then stop
+    emit_marker(OP_END);
   } else {
     // ------------------------------- consumer warps ------------------------------------------
     const uint32_t tid = threadIdx.x - 32, T = blockDim.x - 32;
@@ -423,10 +546,32 @@ __global__ void __launch_bounds__(512, 1)
       mbar_wait(&full[stage], use & 1u);
       const uint8_t *st = stages + (size_t)stage * kTmaBufBytes;
       const DevItem I = *reinterpret_cast<const DevItem *>(st);
-      if (I.op == OP_END) break;
+      if (I.op == OP_END || I.op == OP_FLUSH) {
+        // publish the rows stored since the last flush: every thread's stores (and this warp's
+        // bulk stores) are visible system-wide before one release-add per (source, receiver)
+        if (lane == 0) {
+          bulk_wait_all();
+          fence_proxy_async_global();
+        }
+        __threadfence_system();
+        consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
+        if (tid < (uint32_t)(kMaxRanks * kMaxRanks)) {
+          const uint32_t amt = s_pend[tid];
+          if (amt) {
+            const int ex = (int)(tid / kMaxRanks), dst = (int)(tid % kMaxRanks);
+            red_release_sys_add(P.flags[dst] + s_pend_base + ex, amt);
+            s_pend[tid] = 0;
+          }
+        }
+        consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
+        if (I.op == OP_END) break;
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[stage]);
+        continue;
+      }
       const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
-      const bool bulk =
-          I.op == OP_COPY && P.bulk_store && I.dst >= 0 && DB.pitch == (int64_t)P.row16;
+      const bool bulk = I.op == OP_COPY && !(I.flags & kItemDirect) && P.bulk_store &&
+                        I.dst >= 0 && DB.pitch == (int64_t)P.row16;
       if (bulk) {
         // consecutive packed destination rows: this warp's share is one bulk (TMA) store
         const int64_t lo = (int64_t)I.rows * cw / n_cons_warps;
@@ -435,26 +580,20 @@ __global__ void __launch_bounds__(512, 1)
           bulk_s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
                    (uint32_t)((hi - lo) * P.row16));
           bulk_commit();
-          if (I.flags & kItemSignal) {
-            bulk_wait_all();              // writes performed ...
-            fence_proxy_async_global();   // ... and ordered before the generic release below
-          } else {
-            bulk_wait_read();             // the stage may be reused
-          }
+          bulk_wait_read();  // the stage may be reused once the bulk store has read it
         }
       } else if (I.op == OP_COPY) {
-        store_copy(P, I, st, tid, T);
+        if (I.flags & kItemDirect)
+          store_copy_direct(P, I, st, tid, T);
+        else
+          store_copy(P, I, st, tid, T);
       } else {
         store_fold(P, I, st, tid, T);
       }
-      if (I.flags & kItemSignal) {
-        // this warp's stores are visible system-wide before its share of the rows is counted;
-        // the receiver sees the item's full count only after every warp published (done flag)
-        __threadfence_system();
-        __syncwarp();
-        const int64_t lo = (int64_t)I.rows * cw / n_cons_warps;
-        const int64_t hi = (int64_t)I.rows * (cw + 1) / n_cons_warps;
-        if (lane == 0 && hi > lo) red_release_sys_add(P.flags[I.dst_rank] + I.sig_ctr, hi - lo);
+      if ((I.flags & kItemSignal) && tid == 0) {
+        // counted now, published by the next FLUSH / END marker (done flags)
+        atomicAdd(&s_pend[I.exec_rank * kMaxRanks + I.dst_rank], (uint32_t)I.rows);
+        s_pend_base = I.sig_ctr - I.exec_rank;
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // this warp is done reading the stage

@@ -31,7 +31,8 @@ enum Op : int32_t {
   OP_FOLD = 1,   // dst[dst_row(i)] = fold(init ? dst : -, terms(i)) in order, fp32 adds
   OP_READY = 2,  // write ready[exec_rank] = seq into every peer's flag region
   OP_WAIT = 3,   // wait on the group's wait list (forward completion)
-  OP_END = 4     // (device only) end-of-stream marker from the producer warp to the consumers
+  OP_END = 4,    // (device only) end-of-stream marker from the producer warp to the consumers
+  OP_FLUSH = 5   // (device only) publish the done counts accumulated since the last flush
 };
 
 enum Dir : int32_t { DIR_FWD = 0, DIR_BWD = 1 };
@@ -98,6 +99,7 @@ struct alignas(16) DevItem {
 };
 static_assert(sizeof(DevItem) == 64, "DevItem is one 64-B descriptor");
 constexpr uint8_t kItemSignal = 1;
+constexpr uint8_t kItemDirect = 2;  // COPY: consumers gather rows themselves (short row runs)
 
 struct DevWait {
   int32_t ctr;         // counter index on the executing rank

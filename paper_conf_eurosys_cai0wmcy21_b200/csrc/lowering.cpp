@@ -489,6 +489,9 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         if (sig && !signal_all)
           sig = needed_ctr[(size_t)g.dst_rank * kFlagWords + g.sig_ctr] != 0;
         it.flags = sig ? kItemSignal : 0;
+        // short runs (< 4 rows on average): one bulk copy per run costs more than gathering the
+        // rows with plain loads, so the consumers gather them directly
+        if (g.op == OP_COPY && (int64_t)it.nterms * 4 > (int64_t)it.rows) it.flags |= kItemDirect;
         items->push_back(it);
       }
     }
