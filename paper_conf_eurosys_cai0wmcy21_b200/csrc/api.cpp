@@ -81,6 +81,7 @@ struct dgcl_ctx {
   std::vector<Program> progs;  // index prog_index(layer, dir, r)
   std::vector<int32_t> host_gids[2];  // group order of the host interpreter per direction
   bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
+  int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   int n_prog_ranks = 1;        // programs per (layer, dir)
 
   uint64_t seq = 0, epoch[2] = {0, 0};
@@ -288,7 +289,7 @@ void build_programs(dgcl_ctx *c) {
         Program &P = c->progs[c->prog_index(l, dir, r)];
         const std::vector<uint8_t> need = needed_counters(L, gids[r]);
         build_items(L, gids[r], (int64_t)c->dims[l] * 4, c->item_bytes, !fused, need, &P.items,
-                    &P.runs);
+                    &P.runs, c->direct_copy_rows);
       }
     }
   }
@@ -813,6 +814,12 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "tma") {
     c->use_tma = value != 0;
+    return DGCL_OK;
+  }
+  if (k == "direct_copy_rows") {
+    if (value < 0) return fail(c, DGCL_EINVAL, "direct_copy_rows must be >= 0");
+    c->direct_copy_rows = value;
+    if (c->planned) build_programs(c);
     return DGCL_OK;
   }
   if (k == "bulk_store") {  // TMA stores for local (loopback) destinations

@@ -290,7 +290,7 @@ __device__ __forceinline__ void store_copy(const ExecParams &P, const DevItem &I
 // flight per thread) and store it; whole 16-B chunks (library-owned destination rows)
 __device__ __forceinline__ void store_copy_direct(const ExecParams &P, const DevItem &I,
                                                   const uint8_t *st, uint32_t tid, uint32_t T) {
-  constexpr int kU = 8;
+  constexpr int kU = 4;
   const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
   const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
   char *dbase = P.buf[I.dst_kind][I.dst_rank].ptr;
@@ -358,40 +358,63 @@ __device__ __forceinline__ void store_fold(const ExecParams &P, const DevItem &I
     if (nb == 16) return slot ? ld_cg_v4(p) : ld_nc_v4(p);
     return slot ? ld_part<false>(p, nb) : ld_part<true>(p, nb);
   };
-  constexpr int kBatch = 8;
-  for (uint32_t e = tid; e < total; e += T) {
-    const uint32_t r = fdiv(e, P);
-    const uint32_t col = e - r * nch;
-    const int nb = col + 1 == nch ? tail : 16;
-    const int64_t ta = tp[r], tb = tp[r + 1];
-    const uint32_t *rt = tm + (ta - I.t0);
-    const int cnt = (int)(tb - ta);
+  // kE independent output chunks per thread; every round issues one operand load per chunk (kE
+  // loads in flight) and then adds them, so each chunk's terms are still added in list order
+  constexpr int kE = 8;
+  const int j0 = init ? 0 : 1;  // first term still to add after the starting value
+  auto dst_of = [&](uint32_t r, uint32_t col) -> char * {
     const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
-    char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
-    float4 acc;
-    int j = 0;
-    if (init) {
-      acc = as_f4(nb == 16 ? ld_cg_v4(dp) : ld_part<false>(dp, nb));
-    } else {
-      acc = as_f4(operand(rt[0], col, nb));
-      j = 1;
-    }
-    while (j < cnt) {
-      // up to kBatch independent loads in flight, then the adds in list order
-      int4 v[kBatch];
-      const int n = cnt - j < kBatch ? cnt - j : kBatch;
+    return D.ptr + drow * D.pitch + (int64_t)col * 16;
+  };
+  for (uint32_t e0 = tid; e0 < total; e0 += T * kE) {
+    float4 acc[kE];
+    uint32_t rc[kE];  // (row << 16) | chunk, 0xffffffff when past the end
+    int cnt[kE];
+    int rounds = 0;
 #pragma unroll
-      for (int q = 0; q < kBatch; ++q)
-        if (q < n) v[q] = operand(rt[j + q], col, nb);
-#pragma unroll
-      for (int q = 0; q < kBatch; ++q)
-        if (q < n) add4(acc, v[q]);
-      j += n;
+    for (int q = 0; q < kE; ++q) {
+      const uint32_t e = e0 + q * T;
+      cnt[q] = 0;
+      rc[q] = 0xffffffffu;
+      if (e < total) {
+        const uint32_t r = fdiv(e, P);
+        const uint32_t col = e - r * nch;
+        rc[q] = (r << 16) | col;
+        const int nb = col + 1 == nch ? tail : 16;
+        cnt[q] = (int)(tp[r + 1] - tp[r]);
+        if (init) {
+          char *dp = dst_of(r, col);
+          acc[q] = as_f4(nb == 16 ? ld_cg_v4(dp) : ld_part<false>(dp, nb));
+        } else {
+          acc[q] = as_f4(operand(tm[tp[r] - I.t0], col, nb));
+        }
+        rounds = max(rounds, cnt[q] - j0);
+      }
     }
-    if (nb == 16)
-      st_v4(dp, as_i4(acc));
-    else
-      st_part(dp, as_i4(acc), nb);
+    for (int t = 0; t < rounds; ++t) {
+      int4 v[kE];
+#pragma unroll
+      for (int q = 0; q < kE; ++q) {
+        if (j0 + t < cnt[q]) {
+          const uint32_t r = rc[q] >> 16, col = rc[q] & 0xffffu;
+          v[q] = operand(tm[tp[r] - I.t0 + j0 + t], col, col + 1 == nch ? tail : 16);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < kE; ++q)
+        if (j0 + t < cnt[q]) add4(acc[q], v[q]);
+    }
+#pragma unroll
+    for (int q = 0; q < kE; ++q) {
+      if (rc[q] == 0xffffffffu) continue;
+      const uint32_t r = rc[q] >> 16, col = rc[q] & 0xffffu;
+      const int nb = col + 1 == nch ? tail : 16;
+      char *dp = dst_of(r, col);
+      if (nb == 16)
+        st_v4(dp, as_i4(acc[q]));
+      else
+        st_part(dp, as_i4(acc[q]), nb);
+    }
   }
 }
 

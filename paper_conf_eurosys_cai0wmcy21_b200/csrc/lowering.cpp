@@ -387,7 +387,8 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
 
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
                  int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
-                 std::vector<DevItem> *items, std::vector<DevRun> *runs) {
+                 std::vector<DevItem> *items, std::vector<DevRun> *runs,
+                 int64_t direct_copy_rows) {
   runs->clear();
   // An item is a row range whose gathered operands fit `item_bytes` (and one shared-memory stage
   // of the bulk-copy executor): a COPY row costs one row, a FOLD row (1 + #terms) rows.
@@ -489,9 +490,12 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         if (sig && !signal_all)
           sig = needed_ctr[(size_t)g.dst_rank * kFlagWords + g.sig_ctr] != 0;
         it.flags = sig ? kItemSignal : 0;
-        // short runs (< 4 rows on average): one bulk copy per run costs more than gathering the
-        // rows with plain loads, so the consumers gather them directly
-        if (g.op == OP_COPY && (int64_t)it.nterms * 4 > (int64_t)it.rows) it.flags |= kItemDirect;
+        // optional: items whose runs average fewer than `direct_copy_rows` rows are gathered by
+        // the consumers with plain loads instead of one bulk copy per run (0 = never; measured
+        // slower than per-row bulk copies on the BASELINE graphs)
+        if (g.op == OP_COPY && direct_copy_rows > 0 &&
+            (int64_t)it.nterms * direct_copy_rows > (int64_t)it.rows)
+          it.flags |= kItemDirect;
         items->push_back(it);
       }
     }

@@ -91,7 +91,8 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
 // COPY items also get their row runs appended to `runs` (item.tp = first run, program-relative).
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
                  int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
-                 std::vector<DevItem> *items, std::vector<DevRun> *runs);
+                 std::vector<DevItem> *items, std::vector<DevRun> *runs,
+                 int64_t direct_copy_rows = 0);
 
 // largest number of operand rows one FOLD row gathers (1 + #terms); bounds the bulk-copy stage
 int64_t max_fold_slots(const Lowered &low);
