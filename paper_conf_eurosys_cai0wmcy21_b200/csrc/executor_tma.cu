@@ -332,7 +332,7 @@ __device__ __forceinline__ void store_copy_direct(const ExecParams &P, const Dev
 
 // consumers: fold a gathered FOLD item (operands in list order) and store it; the row's last
 // chunk is stored partially (the destination may be the caller's emb_grad)
-__device__ __forceinline__ void store_fold(const ExecParams &P, const DevItem &I, const uint8_t *st,
+__device__ __forceinline__ void store_fold_multi(const ExecParams &P, const DevItem &I, const uint8_t *st,
                                            uint32_t tid, uint32_t T) {
   const BufRef D = P.buf[I.dst_kind][I.dst_rank];
   const int32_t *info = reinterpret_cast<const int32_t *>(st + kHdrInfo);
@@ -360,7 +360,7 @@ __device__ __forceinline__ void store_fold(const ExecParams &P, const DevItem &I
   };
   // kE independent output chunks per thread; every round issues one operand load per chunk (kE
   // loads in flight) and then adds them, so each chunk's terms are still added in list order
-  constexpr int kE = 8;
+  constexpr int kE = 6;
   const int j0 = init ? 0 : 1;  // first term still to add after the starting value
   auto dst_of = [&](uint32_t r, uint32_t col) -> char * {
     const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
@@ -415,6 +415,68 @@ __device__ __forceinline__ void store_fold(const ExecParams &P, const DevItem &I
       else
         st_part(dp, as_i4(acc[q]), nb);
     }
+  }
+}
+
+// consumers: FOLD item with many terms per row — one output chunk at a time, its terms loaded in
+// batches of 8 independent loads, then added in list order
+__device__ __forceinline__ void store_fold_rows(const ExecParams &P, const DevItem &I,
+                                             const uint8_t *st, uint32_t tid, uint32_t T) {
+  const BufRef D = P.buf[I.dst_kind][I.dst_rank];
+  const int32_t *info = reinterpret_cast<const int32_t *>(st + kHdrInfo);
+  const int64_t *tp = reinterpret_cast<const int64_t *>(st + kTabTp) + info[0];
+  const int32_t *tab = reinterpret_cast<const int32_t *>(st + kTabDst) + info[1];
+  const uint32_t *tm = reinterpret_cast<const uint32_t *>(st + kStageHdrBytes) +
+                       window(I.t0, I.nterms, 4).skew;
+  const int init = I.fold_init;
+  const int mode = I.term_mode;
+  const int exec = I.exec_rank;
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  const int tail = P.row_bytes - (int)(nch - 1) * 16;
+  auto operand = [&](uint32_t term, uint32_t col, int nb) -> int4 {
+    const bool slot = mode == kTermLocal && (term & kTermSlot) != 0;
+    const BufRef &B = mode == kTermRankHgrad ? P.buf[K_HGRAD][term >> 28]
+                      : slot                 ? P.buf[K_SLOT][exec]
+                                             : P.buf[K_HGRAD][exec];
+    const uint32_t row = mode == kTermRankHgrad ? (term & kTermRowMask) : (term & ~kTermSlot);
+    const char *p = B.ptr + (int64_t)row * B.pitch + (int64_t)col * 16;
+    if (nb == 16) return slot ? ld_cg_v4(p) : ld_nc_v4(p);
+    return slot ? ld_part<false>(p, nb) : ld_part<true>(p, nb);
+  };
+  constexpr int kBatch = 8;
+  for (uint32_t e = tid; e < total; e += T) {
+    const uint32_t r = fdiv(e, P);
+    const uint32_t col = e - r * nch;
+    const int nb = col + 1 == nch ? tail : 16;
+    const int64_t ta = tp[r], tb = tp[r + 1];
+    const uint32_t *rt = tm + (ta - I.t0);
+    const int cnt = (int)(tb - ta);
+    const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
+    char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
+    float4 acc;
+    int j = 0;
+    if (init) {
+      acc = as_f4(nb == 16 ? ld_cg_v4(dp) : ld_part<false>(dp, nb));
+    } else {
+      acc = as_f4(operand(rt[0], col, nb));
+      j = 1;
+    }
+    while (j < cnt) {
+      int4 v[kBatch];
+      const int n = cnt - j < kBatch ? cnt - j : kBatch;
+#pragma unroll
+      for (int q = 0; q < kBatch; ++q)
+        if (q < n) v[q] = operand(rt[j + q], col, nb);
+#pragma unroll
+      for (int q = 0; q < kBatch; ++q)
+        if (q < n) add4(acc, v[q]);
+      j += n;
+    }
+    if (nb == 16)
+      st_v4(dp, as_i4(acc));
+    else
+      st_part(dp, as_i4(acc), nb);
   }
 }
 
@@ -611,7 +673,11 @@ __global__ void __launch_bounds__(512, 1)
         else
           store_copy(P, I, st, tid, T);
       } else {
-        store_fold(P, I, st, tid, T);
+        // many terms per row: batch a row's terms; few: batch across output chunks
+        if (I.nterms >= 4 * I.rows)
+          store_fold_rows(P, I, st, tid, T);
+        else
+          store_fold_multi(P, I, st, tid, T);
       }
       if ((I.flags & kItemSignal) && tid == 0) {
         // counted now, published by the next FLUSH / END marker (done flags)
