@@ -35,6 +35,7 @@ struct Program {
   std::vector<DevItem> items;
   std::vector<DevRun> runs;
   size_t dev_off = 0;  // offset (in items) into the device item pool
+  int op_mask = 0;     // kMaskCopy / kMaskFold / kMaskDirect items present
 };
 
 }  // namespace
@@ -290,6 +291,11 @@ void build_programs(dgcl_ctx *c) {
         const std::vector<uint8_t> need = needed_counters(L, gids[r]);
         build_items(L, gids[r], (int64_t)c->dims[l] * 4, c->item_bytes, !fused, need, &P.items,
                     &P.runs, c->direct_copy_rows);
+        P.op_mask = 0;
+        for (const DevItem &it : P.items) {
+          if (it.op == OP_FOLD) P.op_mask |= kMaskFold;
+          if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
+        }
       }
     }
   }
@@ -375,6 +381,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     const Program &pg = c->progs[c->prog_index(layer, dir, fused ? 0 : (c->loopback ? r : r))];
     if (pg.items.empty()) return DGCL_OK;
     P.items = c->d_items + pg.dev_off;
+    P.op_mask = pg.op_mask;
     P.n_items = (int32_t)pg.items.size();
     const int grid = std::min<int64_t>(grid_all, (int64_t)pg.items.size());
     int e = launch_executor(P, grid, c->threads, stream);
@@ -392,6 +399,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     if (!pg.items.empty() && r != c->debug_skip_rank) {
       ExecParams Pr = P;
       Pr.items = c->d_items + pg.dev_off;
+      Pr.op_mask = pg.op_mask;
       Pr.n_items = (int32_t)pg.items.size();
       int e = launch_executor(Pr, std::min<int64_t>(grid_r, (int64_t)pg.items.size()),
                               c->threads, c->rank_streams[r]);

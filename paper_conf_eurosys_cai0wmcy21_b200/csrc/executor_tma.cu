@@ -480,6 +480,7 @@ __device__ __forceinline__ void store_fold_rows(const ExecParams &P, const DevIt
   }
 }
 
+template <int kMask>
 __global__ void __launch_bounds__(512, 1)
     executor_tma_kernel(const __grid_constant__ ExecParams P) {
   extern __shared__ __align__(128) uint8_t dsmem[];
@@ -654,25 +655,26 @@ __global__ void __launch_bounds__(512, 1)
         if (lane == 0) mbar_arrive(&empty[stage]);
         continue;
       }
-      const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
-      const bool bulk = I.op == OP_COPY && !(I.flags & kItemDirect) && P.bulk_store &&
-                        I.dst >= 0 && DB.pitch == (int64_t)P.row16;
-      if (bulk) {
-        // consecutive packed destination rows: this warp's share is one bulk (TMA) store
-        const int64_t lo = (int64_t)I.rows * cw / n_cons_warps;
-        const int64_t hi = (int64_t)I.rows * (cw + 1) / n_cons_warps;
-        if (lane == 0 && hi > lo) {
-          bulk_s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
-                   (uint32_t)((hi - lo) * P.row16));
-          bulk_commit();
-          bulk_wait_read();  // the stage may be reused once the bulk store has read it
-        }
-      } else if (I.op == OP_COPY) {
-        if (I.flags & kItemDirect)
-          store_copy_direct(P, I, st, tid, T);
-        else
+      // kMask: the item kinds this instance was compiled for (the host picks the instance from
+      // the launch's items, so e.g. a forward launch carries no fold code / registers)
+      if ((kMask & kMaskCopy) && I.op == OP_COPY && !(I.flags & kItemDirect)) {
+        const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
+        if (P.bulk_store && I.dst >= 0 && DB.pitch == (int64_t)P.row16) {
+          // consecutive packed destination rows: this warp's share is one bulk (TMA) store
+          const int64_t lo = (int64_t)I.rows * cw / n_cons_warps;
+          const int64_t hi = (int64_t)I.rows * (cw + 1) / n_cons_warps;
+          if (lane == 0 && hi > lo) {
+            bulk_s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
+                     (uint32_t)((hi - lo) * P.row16));
+            bulk_commit();
+            bulk_wait_read();  // the stage may be reused once the bulk store has read it
+          }
+        } else {
           store_copy(P, I, st, tid, T);
-      } else {
+        }
+      } else if ((kMask & kMaskDirect) && I.op == OP_COPY) {
+        store_copy_direct(P, I, st, tid, T);
+      } else if ((kMask & kMaskFold) && I.op == OP_FOLD) {
         // many terms per row: batch a row's terms; few: batch across output chunks
         if (I.nterms >= 4 * I.rows)
           store_fold_rows(P, I, st, tid, T);
@@ -693,26 +695,43 @@ __global__ void __launch_bounds__(512, 1)
 
 }  // namespace
 
-int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream) {
+namespace {
+
+template <int kMask>
+int launch_mask(const ExecParams &p, int grid, int block, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel,
+    cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kMask>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)kSmemBytes);
     if (e != cudaSuccess) return (int)e;
     attr = true;
   }
-  executor_tma_kernel<<<grid, block, kSmemBytes, (cudaStream_t)stream>>>(p);
+  executor_tma_kernel<kMask><<<grid, block, kSmemBytes, s>>>(p);
   return (int)cudaGetLastError();
 }
 
+constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect;
+
+}  // namespace
+
+int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  switch (p.op_mask) {
+    case kMaskCopy: return launch_mask<kMaskCopy>(p, grid, block, s);
+    case kMaskFold: return launch_mask<kMaskFold>(p, grid, block, s);
+    case kMaskCopy | kMaskFold: return launch_mask<kMaskCopy | kMaskFold>(p, grid, block, s);
+    default: return launch_mask<kAll>(p, grid, block, s);
+  }
+}
+
 int tma_executor_occupancy(int block, int *ctas_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel,
+  cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kAll>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)kSmemBytes);
   if (e != cudaSuccess) return (int)e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, executor_tma_kernel, block,
-                                                    kSmemBytes);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, executor_tma_kernel<kAll>,
+                                                    block, kSmemBytes);
   return (int)e;
 }
 

@@ -138,7 +138,10 @@ struct ExecParams {
   int32_t tma_buf;     // bytes per shared-memory stage buffer
   int32_t bulk_store;  // 1: contiguous COPY destinations are written with bulk (TMA) stores
   const struct DevRun *runs;  // COPY items: maximal runs of consecutive (source, destination) rows
+  int32_t op_mask;     // kinds of data items in this launch (kMaskCopy | kMaskFold | kMaskDirect):
+  int32_t pad3;        // selects a kernel instance that carries only the code it needs
 };
+constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4;
 
 // A run of `len` rows whose source rows src.. and destination rows dst.. are both consecutive;
 // `pos` is the first row's index inside its item.  One bulk copy moves a run when the pitches
