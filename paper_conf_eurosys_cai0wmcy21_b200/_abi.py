@@ -6,7 +6,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libdgcl.so")
+# DGCL_LIBRARY: load another in-tree build (A/B performance comparisons); default the package's.
+LIB_PATH = os.environ.get("DGCL_LIBRARY") or os.path.join(_HERE, "libdgcl.so")
 
 STATUS = {0: "DGCL_OK", 1: "DGCL_EINVAL", 2: "DGCL_ESTATE", 3: "DGCL_ECUDA", 4: "DGCL_ENOMEM",
           5: "DGCL_ETIMEOUT", 6: "DGCL_EPLAN"}

@@ -28,18 +28,28 @@ using namespace dev;
 
 namespace {
 
-constexpr int kStages = 4;
-constexpr int kMetaBytes = 12 * 1024;
+constexpr int kStages = kTmaStages;
+#ifndef DGCL_STORE_SPLIT
+#define DGCL_STORE_SPLIT 15  // every consumer warp stores its share (measured best, Reddit)
+#endif
+constexpr int kStoreSplit = DGCL_STORE_SPLIT;  // bulk stores per COPY item (<= consumer warps)
+constexpr int kMetaBytes = 8 * 1024;  // one item's row runs (<= kMaxItemRows x 16 B)
+constexpr int kMetaSlots = 4;         // run windows prefetched kMetaAhead items ahead
+constexpr int kMetaAhead = 3;
+constexpr int kDescAhead = 6;         // descriptors prefetched further ahead (ring of kDescSlots)
+static_assert(kMaxItemRows * 16 <= kMetaBytes, "meta slot holds an item's runs");
 constexpr int kHdrInfo = 64;         // stage: int32 info words after the 64-B item header
 constexpr int kTabTp = 128;          // stage: term_ptr window (FOLD)
 constexpr int kTabDst = 2176;        // stage: destination-row window
-constexpr int kMetaDst = 2048;       // meta: destination rows (FOLD init operand)
-constexpr int kMetaTerms = 4096;     // meta: terms window
-constexpr int kDescSlots = 4;        // producer descriptor ring
-constexpr size_t kMetaOff = 128;     // after the mbarriers (4 full, 4 empty, 2 meta, 4 desc)
-constexpr size_t kDescOff = kMetaOff + 2 * (size_t)kMetaBytes;
+constexpr int kDescSlots = 8;        // producer descriptor ring
+static_assert(kDescAhead > kMetaAhead && kDescAhead < kDescSlots && kMetaAhead < kMetaSlots,
+              "prefetch distances");
+constexpr size_t kMetaOff = 256;     // after the mbarriers (full, empty, meta, desc)
+static_assert((2 * kTmaStages + kMetaSlots + kDescSlots) * 8 <= 256, "mbarrier region");
+constexpr size_t kDescOff = kMetaOff + kMetaSlots * (size_t)kMetaBytes;
 constexpr size_t kStageOff = kDescOff + kDescSlots * 64;
-constexpr size_t kSmemBytes = kStageOff + (size_t)kStages * kTmaBufBytes;
+constexpr size_t kPendOff = kStageOff + (size_t)kStages * kTmaBufBytes;  // 1 KB counts + 3 words
+constexpr size_t kSmemBytes = kPendOff + 1152;
 static_assert(kSmemBytes <= 227 * 1024, "shared memory budget");
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -162,23 +172,14 @@ __device__ __forceinline__ Win window(int64_t off, int64_t n, int sz) {
 // producer lane 0: bulk-copy the metadata the producer needs to issue item I's gathers
 __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I, uint8_t *meta,
                                            uint64_t *bar) {
-  uint32_t tx = 0;
-  Win ws = {0, 0, 0}, wd = {0, 0, 0}, wt = {0, 0, 0};
-  if (I.op == OP_COPY && !(I.flags & kItemDirect)) {
-    wt = {I.tp, (uint32_t)I.nterms * (uint32_t)sizeof(DevRun), 0};  // the item's row runs
-    tx += wt.bytes;
-  }
-  // OP_FOLD: the consumers gather the operands themselves; nothing for the producer to prefetch
+  // COPY (bulk path): the item's row runs.  FOLD and direct COPY items need nothing here (the
+  // consumers gather their operands); the barrier phase then completes on the arrive alone.
+  const uint32_t tx = (I.op == OP_COPY && !(I.flags & kItemDirect))
+                          ? (uint32_t)I.nterms * (uint32_t)sizeof(DevRun)
+                          : 0u;
   fence_proxy_async_smem();
   mbar_expect_tx(bar, tx);
-  if (ws.bytes)
-    bulk_g2s(meta, I.op == OP_FOLD ? (const void *)(P.term_ptr + ws.a) : (const void *)(P.idx + ws.a),
-             ws.bytes, bar);
-  if (wd.bytes) bulk_g2s(meta + kMetaDst, P.idx + wd.a, wd.bytes, bar);
-  if (wt.bytes)
-    bulk_g2s(meta + kMetaTerms,
-             I.op == OP_COPY ? (const void *)(P.runs + wt.a) : (const void *)(P.terms + wt.a),
-             wt.bytes, bar);
+  if (tx) bulk_g2s(meta, P.runs + I.tp, tx, bar);
 }
 
 // bytes bulk-copied into the operand area of a stage (gathered rows, or a FOLD's terms window)
@@ -223,7 +224,7 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     // one bulk copy per run of consecutive source rows when rows are packed (pitch == row16)
     const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
     const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
-    const DevRun *runs = reinterpret_cast<const DevRun *>(meta + kMetaTerms);
+    const DevRun *runs = reinterpret_cast<const DevRun *>(meta);
     if (spitch == (int64_t)r16) {
       for (int q = lane; q < I.nterms; q += 32) {
         const DevRun R = runs[q];
@@ -487,14 +488,16 @@ __global__ void __launch_bounds__(512, 1)
   uint64_t *full = reinterpret_cast<uint64_t *>(dsmem);
   uint64_t *empty = full + kStages;
   uint64_t *metab = empty + kStages;
-  uint64_t *descb = metab + 2;
+  uint64_t *descb = metab + kMetaSlots;
   uint8_t *metas = dsmem + kMetaOff;
   DevItem *descs = reinterpret_cast<DevItem *>(dsmem + kDescOff);
   uint8_t *stages = dsmem + kStageOff;
-  __shared__ uint32_t s_pend[kMaxRanks * kMaxRanks];  // rows stored, per (source, receiver)
-  __shared__ int s_pend_base;                          // their counter family
-  __shared__ unsigned s_bar_count;
-  __shared__ volatile unsigned s_bar_gen;
+  // rows stored since the last flush per (source, receiver), their counter family, and the
+  // consumer barrier words: carved from the dynamic region (no static shared memory)
+  uint32_t *s_pend = reinterpret_cast<uint32_t *>(dsmem + kPendOff);
+  int &s_pend_base = *reinterpret_cast<int *>(dsmem + kPendOff + 1024);
+  unsigned &s_bar_count = *reinterpret_cast<unsigned *>(dsmem + kPendOff + 1028);
+  volatile unsigned &s_bar_gen = *reinterpret_cast<volatile unsigned *>(dsmem + kPendOff + 1032);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
   for (int i = threadIdx.x; i < kMaxRanks * kMaxRanks; i += blockDim.x) s_pend[i] = 0;
@@ -506,8 +509,7 @@ __global__ void __launch_bounds__(512, 1)
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], n_cons_warps);
     }
-    mbar_init(&metab[0], 1);
-    mbar_init(&metab[1], 1);
+    for (int s = 0; s < kMetaSlots; ++s) mbar_init(&metab[s], 1);
     for (int s = 0; s < kDescSlots; ++s) mbar_init(&descb[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -516,7 +518,8 @@ __global__ void __launch_bounds__(512, 1)
   if (warp == 0) {
     // ------------------------------- producer warp -------------------------------------------
     // item q of this CTA is P.items[blockIdx.x + q * gridDim.x]; its descriptor is bulk-copied
-    // into ring slot q % 4 two items ahead, its index windows into meta buffer q % 2 one ahead
+    // into ring slot q % kDescSlots kDescAhead items ahead, its row runs into meta slot
+    // q % kMetaSlots kMetaAhead items ahead, so their latency never stalls the issue loop
     const uint32_t G = gridDim.x;
     const uint32_t nmine =
         blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
@@ -545,17 +548,19 @@ __global__ void __launch_bounds__(512, 1)
       __syncwarp();
       ++k;
     };
+    auto meta_of = [&](uint32_t q) { return metas + (size_t)(q % kMetaSlots) * kMetaBytes; };
     if (lane == 0)
-      for (uint32_t q = 0; q < 2 && q < nmine; ++q) request_desc(q);
-    if (nmine > 0) {
-      const DevItem &I0 = desc_ready(0);
-      if (lane == 0) issue_meta(P, I0, metas, &metab[0]);
+      for (uint32_t q = 0; q < (uint32_t)kDescAhead && q < nmine; ++q) request_desc(q);
+    for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nmine; ++q) {
+      const DevItem &Iq = desc_ready(q);
+      if (lane == 0) issue_meta(P, Iq, meta_of(q), &metab[q % kMetaSlots]);
     }
     for (; m < nmine; ++m) {
-      if (lane == 0 && m + 2 < nmine) request_desc(m + 2);
-      if (m + 1 < nmine) {
-        const DevItem &In = desc_ready(m + 1);
-        if (lane == 0) issue_meta(P, In, metas + ((m + 1) & 1) * kMetaBytes, &metab[(m + 1) & 1]);
+      if (lane == 0 && m + kDescAhead < nmine) request_desc(m + kDescAhead);
+      if (m + kMetaAhead < nmine) {
+        const uint32_t q = m + kMetaAhead;
+        const DevItem &In = desc_ready(q);
+        if (lane == 0) issue_meta(P, In, meta_of(q), &metab[q % kMetaSlots]);
       }
       const DevItem &I = desc_ready(m);
       if (I.op == OP_READY) {
@@ -578,7 +583,11 @@ __global__ void __launch_bounds__(512, 1)
         // block on a wait, and whenever the counter family (direction, stage) changes.
         const bool sig = (I.flags & kItemSignal) != 0;
         const int key = sig ? I.sig_ctr - I.exec_rank : -1;
+#ifdef DGCL_EXPERIMENT_NO_FLUSH
+        if (false) {
+#else
         if (pend) {
+#endif
           int ready = 1;
           if (lane == 0) {
             ready = waits_ready(P, I) ? 1 : 0;
@@ -602,11 +611,10 @@ __global__ void __launch_bounds__(512, 1)
         ok = __shfl_sync(0xffffffffu, w, 0) != 0;
         if (!ok) break;
         if (I.wait_n > 0) fence_proxy_async_global();  // acquired peers' rows -> bulk reads
-        mbar_wait(&metab[m & 1], (m >> 1) & 1u);
+        mbar_wait(&metab[m % kMetaSlots], (m / kMetaSlots) & 1u);
         const uint32_t stage = k % kStages, use = k / kStages;
         if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
-        issue_item(P, I, stages + (size_t)stage * kTmaBufBytes, metas + (m & 1) * kMetaBytes,
-                   &full[stage], lane);
+        issue_item(P, I, stages + (size_t)stage * kTmaBufBytes, meta_of(m), &full[stage], lane);
         ++k;
         if (sig) {
           pend = true;
@@ -617,9 +625,10 @@ __global__ void __launch_bounds__(512, 1)
     }
     if (!ok) {
       // watchdog abort: descriptor / metadata copies still in flight land before the CTA leaves
-      for (uint32_t q = m; q < m + 3 && q < nmine; ++q)
+      for (uint32_t q = m; q <= m + kDescAhead && q < nmine; ++q)
         mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
-      for (uint32_t q = m; q < m + 2 && q < nmine; ++q) mbar_wait(&metab[q & 1], (q >> 1) & 1u);
+      for (uint32_t q = m; q <= m + kMetaAhead && q < nmine; ++q)
+        mbar_wait(&metab[q % kMetaSlots], (q / kMetaSlots) & 1u);
     }
     // END marker: consumers drain every issued stage, publish pending counts, then stop
     emit_marker(OP_END);
@@ -660,14 +669,20 @@ __global__ void __launch_bounds__(512, 1)
       if ((kMask & kMaskCopy) && I.op == OP_COPY && !(I.flags & kItemDirect)) {
         const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
         if (P.bulk_store && I.dst >= 0 && DB.pitch == (int64_t)P.row16) {
-          // consecutive packed destination rows: this warp's share is one bulk (TMA) store
-          const int64_t lo = (int64_t)I.rows * cw / n_cons_warps;
-          const int64_t hi = (int64_t)I.rows * (cw + 1) / n_cons_warps;
-          if (lane == 0 && hi > lo) {
-            bulk_s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
-                     (uint32_t)((hi - lo) * P.row16));
-            bulk_commit();
-            bulk_wait_read();  // the stage may be reused once the bulk store has read it
+          // consecutive packed destination rows: kStoreSplit bulk (TMA) stores move the item,
+          // issued by consumer warps (k * kStoreSplit + j) % n_cons_warps, so the stores of
+          // several stages overlap while the other warps move on
+          const int first = (int)((k * (uint32_t)kStoreSplit) % (uint32_t)n_cons_warps);
+          const int j = (cw - first + n_cons_warps) % n_cons_warps;
+          if (j < kStoreSplit && lane == 0) {
+            const int64_t lo = (int64_t)I.rows * j / kStoreSplit;
+            const int64_t hi = (int64_t)I.rows * (j + 1) / kStoreSplit;
+            if (hi > lo) {
+              bulk_s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
+                       (uint32_t)((hi - lo) * P.row16));
+              bulk_commit();
+              bulk_wait_read();  // the stage may be reused once the bulk store has read it
+            }
           }
         } else {
           store_copy(P, I, st, tid, T);
