@@ -672,11 +672,12 @@ __global__ void __launch_bounds__(512, 1)
           // consecutive packed destination rows: kStoreSplit bulk (TMA) stores move the item,
           // issued by consumer warps (k * kStoreSplit + j) % n_cons_warps, so the stores of
           // several stages overlap while the other warps move on
-          const int first = (int)((k * (uint32_t)kStoreSplit) % (uint32_t)n_cons_warps);
+          const int split = kStoreSplit < n_cons_warps ? kStoreSplit : n_cons_warps;
+          const int first = (int)((k * (uint32_t)split) % (uint32_t)n_cons_warps);
           const int j = (cw - first + n_cons_warps) % n_cons_warps;
-          if (j < kStoreSplit && lane == 0) {
-            const int64_t lo = (int64_t)I.rows * j / kStoreSplit;
-            const int64_t hi = (int64_t)I.rows * (j + 1) / kStoreSplit;
+          if (j < split && lane == 0) {
+            const int64_t lo = (int64_t)I.rows * j / split;
+            const int64_t hi = (int64_t)I.rows * (j + 1) / split;
             if (hi > lo) {
               bulk_s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
                        (uint32_t)((hi - lo) * P.row16));
