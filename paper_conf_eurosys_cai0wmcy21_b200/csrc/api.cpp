@@ -83,6 +83,7 @@ struct dgcl_ctx {
   std::vector<int32_t> host_gids[2];  // group order of the host interpreter per direction
   bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
+  bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   int n_prog_ranks = 1;        // programs per (layer, dir)
 
   uint64_t seq = 0, epoch[2] = {0, 0};
@@ -323,6 +324,42 @@ dgcl_status check_dead(dgcl_ctx *c) {
 
 inline bool al16(const void *p) { return ((uintptr_t)p & 15) == 0; }
 
+// 2-D tensor map over `rows` packed rows of row_bytes (<= 1 KB) starting at `base`: box = one row,
+// for cp.async.bulk.tensor ... tile::gather4.  The driver entry point is resolved through the
+// runtime (no libcuda link).  Returns false if the map cannot be built (the launch then uses
+// per-run bulk copies).
+bool encode_rows_tmap(dgcl_ctx *c, unsigned char *out, const void *base, int64_t rows,
+                      int row_bytes) {
+  typedef CUresult (*Encode)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                             const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                             const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                             CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+  static Encode fn = nullptr;
+  if (!fn) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) !=
+            cudaSuccess ||
+        !p || q != cudaDriverEntryPointSuccess)
+      return false;
+    fn = (Encode)p;
+  }
+  (void)c;
+  const cuuint64_t dims[2] = {(cuuint64_t)(row_bytes / 4), (cuuint64_t)rows};
+  const cuuint64_t strides[1] = {(cuuint64_t)row_bytes};
+  const cuuint32_t box[2] = {(cuuint32_t)(row_bytes / 4), 1};
+  const cuuint32_t estr[2] = {1, 1};
+  CUtensorMap map;
+  const CUresult r = fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void *>(base), dims,
+                        strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                        CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return false;
+  static_assert(sizeof(CUtensorMap) == 128, "tensor map size");
+  std::memcpy(out, &map, sizeof(map));
+  return true;
+}
+
 dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_pitch,
                    float *out, int64_t out_pitch, cudaStream_t stream) {
   const int m = c->world;
@@ -373,6 +410,17 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage
   P.use_tma = (v16 && c->use_tma && c->tma_ctas > 0 &&
                P.row16 <= kTmaOperandBytes) ? 1 : 0;
+  // forward launches over packed embedding rows of <= 1 KB: a 2-D tensor map for the TMA row
+  // gather (gather4) used by items whose source rows come in short runs
+  if (P.use_tma && dir == DIR_FWD && c->use_gather4 && in_pitch * 4 == P.row16 &&
+      P.row16 <= kGather4MaxRowBytes) {
+    const int64_t rows = c->loopback ? c->n : c->n_local[c->rank];
+    if (rows > 0 && rows < INT32_MAX && encode_rows_tmap(c, P.tmap_emb, in, rows, P.row16)) {
+      P.use_gather4 = 1;
+      for (int r = 0; r < m; ++r)
+        P.tmap_row_off[r] = c->loopback ? (int32_t)c->row_off[r] : 0;
+    }
+  }
   const int grid_all = P.use_tma ? c->n_sm * c->tma_ctas : c->grid;
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
   P.use_ready = (!fused && m > 1) ? 1 : 0;
@@ -828,6 +876,10 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (value < 0) return fail(c, DGCL_EINVAL, "direct_copy_rows must be >= 0");
     c->direct_copy_rows = value;
     if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "gather4") {  // TMA gather4 (four rows per instruction) for short-run row gathers
+    c->use_gather4 = value != 0;
     return DGCL_OK;
   }
   if (k == "bulk_store") {  // TMA stores for local (loopback) destinations

@@ -169,15 +169,36 @@ __device__ __forceinline__ Win window(int64_t off, int64_t n, int sz) {
   return w;
 }
 
+// COPY item gathered four rows per TMA instruction (tile::gather4 through the launch's tensor map)
+__device__ __forceinline__ bool uses_gather4(const ExecParams &P, const DevItem &I) {
+  return P.use_gather4 && (I.flags & kItemGather4) && I.op == OP_COPY && I.src < 0;
+}
+
+__device__ __forceinline__ void tma_gather4(void *sdst, const void *tmap, int32_t col, int32_t r0,
+                                            int32_t r1, int32_t r2, int32_t r3, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(sdst)),
+      "l"(tmap), "r"(col), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(bar))
+      : "memory");
+}
+
 // producer lane 0: bulk-copy the metadata the producer needs to issue item I's gathers
 __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I, uint8_t *meta,
                                            uint64_t *bar) {
-  // COPY (bulk path): the item's row runs.  FOLD and direct COPY items need nothing here (the
-  // consumers gather their operands); the barrier phase then completes on the arrive alone.
+  // COPY (bulk path): the item's row runs, or its source rows for a gather4 item.  FOLD and
+  // direct COPY items need nothing here (the consumers gather their operands); the barrier phase
+  // then completes on the arrive alone.
+  fence_proxy_async_smem();
+  if (uses_gather4(P, I)) {
+    const Win ws = window(~I.src, I.rows, 4);
+    mbar_expect_tx(bar, ws.bytes);
+    bulk_g2s(meta, P.idx + ws.a, ws.bytes, bar);
+    return;
+  }
   const uint32_t tx = (I.op == OP_COPY && !(I.flags & kItemDirect))
                           ? (uint32_t)I.nterms * (uint32_t)sizeof(DevRun)
                           : 0u;
-  fence_proxy_async_smem();
   mbar_expect_tx(bar, tx);
   if (tx) bulk_g2s(meta, P.runs + I.tp, tx, bar);
 }
@@ -185,6 +206,7 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
 // bytes bulk-copied into the operand area of a stage (gathered rows, or a FOLD's terms window)
 __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const DevItem &I) {
   if (I.op == OP_COPY) {
+    if (uses_gather4(P, I)) return (uint32_t)((I.rows + 3) / 4 * 4) * (uint32_t)P.row16;
     if (!(I.flags & kItemDirect)) return (uint32_t)I.rows * (uint32_t)P.row16;
     return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;  // source-row window only
   }
@@ -219,6 +241,19 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     if (lane == 0 && I.src < 0) {
       const Win ws = window(~I.src, I.rows, 4);
       bulk_g2s(ops, P.idx + ws.a, ws.bytes, full);
+    }
+  } else if (uses_gather4(P, I)) {
+    // four rows per instruction (the last group repeats the item's last row; the stage holds
+    // the padding rows, the consumers never store them)
+    const int32_t *sidx = reinterpret_cast<const int32_t *>(meta) +
+                          (int32_t)(~I.src - window(~I.src, I.rows, 4).a);
+    const int32_t base = P.tmap_row_off[I.exec_rank];
+    const int ng = (I.rows + 3) / 4;
+    for (int g = lane; g < ng; g += 32) {
+      const int r = 4 * g, last = I.rows - 1;
+      tma_gather4(ops + (size_t)r * r16, P.tmap_emb, 0, base + sidx[r],
+                  base + sidx[min(r + 1, last)], base + sidx[min(r + 2, last)],
+                  base + sidx[min(r + 3, last)], full);
     }
   } else if (I.op == OP_COPY) {
     // one bulk copy per run of consecutive source rows when rows are packed (pitch == row16)

@@ -100,6 +100,8 @@ struct alignas(16) DevItem {
 static_assert(sizeof(DevItem) == 64, "DevItem is one 64-B descriptor");
 constexpr uint8_t kItemSignal = 1;
 constexpr uint8_t kItemDirect = 2;  // COPY: consumers gather rows themselves (short row runs)
+constexpr uint8_t kItemGather4 = 4; // COPY from embeddings with short runs: TMA gather4 of rows
+constexpr int kGather4MaxRowBytes = 1024;  // one tensor box (<= 256 fp32) per row
 
 struct DevWait {
   int32_t ctr;         // counter index on the executing rank
@@ -112,7 +114,12 @@ struct BufRef {
   int64_t pitch;       // bytes
 };
 
-struct ExecParams {
+struct alignas(64) ExecParams {
+  // 2-D tensor map (CUtensorMap, 128 B) over the embedding rows of this launch, for the
+  // row-gather TMA (cp.async.bulk.tensor ... tile::gather4: four arbitrary rows per instruction)
+  alignas(64) unsigned char tmap_emb[128];
+  int32_t use_gather4;              // tmap_emb valid for this launch
+  int32_t tmap_row_off[kMaxRanks];  // first tensor row of each rank's embeddings
   BufRef buf[K_NKINDS][kMaxRanks];
   uint64_t *flags[kMaxRanks];  // flag region of every rank (peer-mapped in multi-GPU mode)
   const DevGroup *groups;

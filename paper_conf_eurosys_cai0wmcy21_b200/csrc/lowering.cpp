@@ -413,7 +413,9 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       std::vector<int32_t> &b = bounds[q - i];
       b.push_back(0);
       if (g.op == OP_COPY) {
-        const int64_t rpi = std::min<int64_t>(kMaxItemRows, std::max<int64_t>(1, cap / row16));
+        // rows per item; a multiple of 4 when gather4 may apply (its groups are padded to 4 rows)
+        int64_t rpi = std::min<int64_t>(kMaxItemRows, std::max<int64_t>(1, cap / row16));
+        if (row16 <= kGather4MaxRowBytes && rpi >= 4) rpi = rpi / 4 * 4;
         for (int64_t r = rpi; r < g.n_rows; r += rpi) b.push_back((int32_t)r);
         b.push_back((int32_t)g.n_rows);
       } else if (g.op == OP_FOLD) {
@@ -496,6 +498,14 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         if (g.op == OP_COPY && direct_copy_rows > 0 &&
             (int64_t)it.nterms * direct_copy_rows > (int64_t)it.rows)
           it.flags |= kItemDirect;
+        // rows from the embeddings with short runs (< 4 rows on average) and rows that fit one
+        // tensor box: gather four rows per TMA instruction instead of one bulk copy per run
+        // (used only when the launch provides the tensor map, see ExecParams::use_gather4)
+        // (a 4-row group must start 128-B aligned in shared memory: row16 % 32 == 0)
+        else if (g.op == OP_COPY && g.src_kind == K_EMB && g.src_idx >= 0 &&
+                 row16 <= kGather4MaxRowBytes && row16 % 32 == 0 &&
+                 (int64_t)it.nterms * 4 > (int64_t)it.rows)
+          it.flags |= kItemGather4;
         items->push_back(it);
       }
     }

@@ -142,16 +142,22 @@ def test_tiny_config_bit_exact():
     _check_case(Case(g, cfg.dims))
 
 
-@pytest.mark.parametrize("m,tma,direct,bulk", [(3, 1, 1, 1), (4, 1, 1, 1), (8, 1, 1, 1),
-                                               (8, 1, 1, 0), (4, 0, 1, 1), (8, 0, 1, 1),
-                                               (8, 1, 0, 1), (3, 0, 0, 1), (4, 1, 0, 0)])
-def test_uniform_loopback_fused(m, tma, direct, bulk):
-    """tma=1: bulk-copy (cp.async.bulk) gather executor; tma=0: the register (LDG) executor.
-    direct=1: loopback in-place reduce; direct=0: push to slots + owner reduce (multi-GPU form).
-    bulk=1: packed contiguous destinations written with bulk (TMA) stores; 0: 16-B st.global."""
+@pytest.mark.parametrize("m,opts", [
+    (3, {}), (4, {}), (8, {}),
+    (8, {"bulk_store": 0}),
+    (4, {"tma": 0}), (8, {"tma": 0}),
+    (8, {"direct_reduce": 0}), (3, {"tma": 0, "direct_reduce": 0}),
+    (4, {"direct_reduce": 0, "bulk_store": 0}),
+    (8, {"gather4": 0}),
+    (4, {"direct_copy_rows": 4}),
+])
+def test_uniform_loopback_fused(m, opts):
+    """Executor variants: tma (bulk-copy executor vs the register LDG executor), direct_reduce
+    (loopback in-place reduce vs push to slots + owner reduce, the multi-GPU form), bulk_store
+    (TMA stores vs 16-B st.global), gather4 (TMA row gather of 4 rows per instruction vs one bulk
+    copy per run), direct_copy_rows (consumer-side gathers for short runs)."""
     g = synth.make_graph(6000, 60000, m, graph_seed=m, part_seed=7 * m)
-    _check_case(Case(g, [64, 5, 602], options={"tma": tma, "direct_reduce": direct,
-                                               "bulk_store": bulk}))
+    _check_case(Case(g, [64, 5, 602, 32], options=opts))
 
 
 @pytest.mark.parametrize("m", [2, 8])
