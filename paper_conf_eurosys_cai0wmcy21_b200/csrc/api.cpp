@@ -36,6 +36,7 @@ struct Program {
   std::vector<DevRun> runs;
   size_t dev_off = 0;  // offset (in items) into the device item pool
   int op_mask = 0;     // kMaskCopy / kMaskFold / kMaskDirect items present
+  bool fold_wide = false;  // FOLD rows average >= 4 terms
 };
 
 }  // namespace
@@ -293,10 +294,16 @@ void build_programs(dgcl_ctx *c) {
         build_items(L, gids[r], (int64_t)c->dims[l] * 4, c->item_bytes, !fused, need, &P.items,
                     &P.runs, c->direct_copy_rows);
         P.op_mask = 0;
+        int64_t fold_rows = 0, fold_terms = 0;
         for (const DevItem &it : P.items) {
-          if (it.op == OP_FOLD) P.op_mask |= kMaskFold;
+          if (it.op == OP_FOLD) {
+            P.op_mask |= kMaskFold;
+            fold_rows += it.rows;
+            fold_terms += it.nterms;
+          }
           if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
         }
+        P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
       }
     }
   }
@@ -430,6 +437,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     if (pg.items.empty()) return DGCL_OK;
     P.items = c->d_items + pg.dev_off;
     P.op_mask = pg.op_mask;
+    P.fold_wide = pg.fold_wide ? 1 : 0;
     P.n_items = (int32_t)pg.items.size();
     const int grid = std::min<int64_t>(grid_all, (int64_t)pg.items.size());
     int e = launch_executor(P, grid, c->threads, stream);
@@ -448,6 +456,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
       ExecParams Pr = P;
       Pr.items = c->d_items + pg.dev_off;
       Pr.op_mask = pg.op_mask;
+      Pr.fold_wide = pg.fold_wide ? 1 : 0;
       Pr.n_items = (int32_t)pg.items.size();
       int e = launch_executor(Pr, std::min<int64_t>(grid_r, (int64_t)pg.items.size()),
                               c->threads, c->rank_streams[r]);

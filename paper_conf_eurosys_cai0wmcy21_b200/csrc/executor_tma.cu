@@ -368,6 +368,7 @@ __device__ __forceinline__ void store_copy_direct(const ExecParams &P, const Dev
 
 // consumers: fold a gathered FOLD item (operands in list order) and store it; the row's last
 // chunk is stored partially (the destination may be the caller's emb_grad)
+template <int kE>
 __device__ __forceinline__ void store_fold_multi(const ExecParams &P, const DevItem &I, const uint8_t *st,
                                            uint32_t tid, uint32_t T) {
   const BufRef D = P.buf[I.dst_kind][I.dst_rank];
@@ -396,7 +397,6 @@ __device__ __forceinline__ void store_fold_multi(const ExecParams &P, const DevI
   };
   // kE independent output chunks per thread; every round issues one operand load per chunk (kE
   // loads in flight) and then adds them, so each chunk's terms are still added in list order
-  constexpr int kE = 6;
   const int j0 = init ? 0 : 1;  // first term still to add after the starting value
   auto dst_of = [&](uint32_t r, uint32_t col) -> char * {
     const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
@@ -456,6 +456,7 @@ __device__ __forceinline__ void store_fold_multi(const ExecParams &P, const DevI
 
 // consumers: FOLD item with many terms per row — one output chunk at a time, its terms loaded in
 // batches of 8 independent loads, then added in list order
+template <int kBatch>
 __device__ __forceinline__ void store_fold_rows(const ExecParams &P, const DevItem &I,
                                              const uint8_t *st, uint32_t tid, uint32_t T) {
   const BufRef D = P.buf[I.dst_kind][I.dst_rank];
@@ -480,7 +481,6 @@ __device__ __forceinline__ void store_fold_rows(const ExecParams &P, const DevIt
     if (nb == 16) return slot ? ld_cg_v4(p) : ld_nc_v4(p);
     return slot ? ld_part<false>(p, nb) : ld_part<true>(p, nb);
   };
-  constexpr int kBatch = 8;
   for (uint32_t e = tid; e < total; e += T) {
     const uint32_t r = fdiv(e, P);
     const uint32_t col = e - r * nch;
@@ -516,8 +516,8 @@ __device__ __forceinline__ void store_fold_rows(const ExecParams &P, const DevIt
   }
 }
 
-template <int kMask>
-__global__ void __launch_bounds__(512, 1)
+template <int kMask, int kMaxThreads = 512>
+__global__ void __launch_bounds__(kMaxThreads, 1)
     executor_tma_kernel(const __grid_constant__ ExecParams P) {
   extern __shared__ __align__(128) uint8_t dsmem[];
   uint64_t *full = reinterpret_cast<uint64_t *>(dsmem);
@@ -728,9 +728,9 @@ __global__ void __launch_bounds__(512, 1)
       } else if ((kMask & kMaskFold) && I.op == OP_FOLD) {
         // many terms per row: batch a row's terms; few: batch across output chunks
         if (I.nterms >= 4 * I.rows)
-          store_fold_rows(P, I, st, tid, T);
+          store_fold_rows<(kMaxThreads > 512 ? 4 : 8)>(P, I, st, tid, T);
         else
-          store_fold_multi(P, I, st, tid, T);
+          store_fold_multi<(kMaxThreads > 512 ? 3 : 6)>(P, I, st, tid, T);
       }
       if ((I.flags & kItemSignal) && tid == 0) {
         // counted now, published by the next FLUSH / END marker (done flags)
@@ -748,17 +748,17 @@ __global__ void __launch_bounds__(512, 1)
 
 namespace {
 
-template <int kMask>
+template <int kMask, int kThreads = 512>
 int launch_mask(const ExecParams &p, int grid, int block, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kMask>,
+    cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kMask, kThreads>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)kSmemBytes);
     if (e != cudaSuccess) return (int)e;
     attr = true;
   }
-  executor_tma_kernel<kMask><<<grid, block, kSmemBytes, s>>>(p);
+  executor_tma_kernel<kMask, kThreads><<<grid, block, kSmemBytes, s>>>(p);
   return (int)cudaGetLastError();
 }
 
@@ -770,7 +770,13 @@ int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream) 
   cudaStream_t s = (cudaStream_t)stream;
   switch (p.op_mask) {
     case kMaskCopy: return launch_mask<kMaskCopy>(p, grid, block, s);
-    case kMaskFold: return launch_mask<kMaskFold>(p, grid, block, s);
+    case kMaskFold:
+      // fold-only launches are latency-bound gathers by the consumer warps: with the default
+      // CTA size, run 1024 threads (31 consumer warps, <= 64 registers) for twice the loads in
+      // flight per SM
+      // (only when rows carry many terms: few-term rows want the wider per-thread batching)
+      if (block == 512 && p.fold_wide) return launch_mask<kMaskFold, 1024>(p, grid, 1024, s);
+      return launch_mask<kMaskFold>(p, grid, block, s);
     case kMaskCopy | kMaskFold: return launch_mask<kMaskCopy | kMaskFold>(p, grid, block, s);
     default: return launch_mask<kAll>(p, grid, block, s);
   }

@@ -146,7 +146,8 @@ struct alignas(64) ExecParams {
   int32_t bulk_store;  // 1: contiguous COPY destinations are written with bulk (TMA) stores
   const struct DevRun *runs;  // COPY items: maximal runs of consecutive (source, destination) rows
   int32_t op_mask;     // kinds of data items in this launch (kMaskCopy | kMaskFold | kMaskDirect):
-  int32_t pad3;        // selects a kernel instance that carries only the code it needs
+                       // selects a kernel instance that carries only the code it needs
+  int32_t fold_wide;   // FOLD rows average >= 4 terms (selects the 1024-thread fold instance)
 };
 constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4;
 
