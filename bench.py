@@ -197,6 +197,42 @@ def oracle_sample(w, emb, hg, eg, budget_s=15.0, ranks=None):
 
 
 # ---------------------------------------------------------------------------------------------
+def torch_gather_baseline(w, emb, hg, eg, stream, reps=5):
+    """The same loopback exchange with stock PyTorch ops on the same GPU (context for the
+    executor's numbers, not our kernels): forward = one torch.index_select of every halo row;
+    backward = torch.index_add_ of the halo gradients into the owner rows (atomic scatter-add,
+    order not fixed — the Table 9 'atomic' alternative)."""
+    import torch
+    g = w.g
+    inv = np.empty(g.n, np.int64)
+    inv[w.order] = np.arange(g.n)
+    src = torch.from_numpy(inv[g.req_ids]).cuda()
+    out = {}
+
+    def timed(fn):
+        fn()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(reps):
+            fn()
+        b.record(stream)
+        torch.cuda.synchronize()
+        return a.elapsed_time(b) / reps
+
+    for l in w.fwd_layers:
+        buf = torch.empty(w.S, emb[l].shape[1], dtype=torch.float32, device="cuda")
+        out["fwd%d_d%d" % (l, w.cfg.dims[l])] = timed(
+            lambda: torch.index_select(emb[l], 0, src, out=buf))
+        del buf
+    for l in w.bwd_layers:
+        e2 = eg[l].clone()
+        out["bwd%d_d%d" % (l, w.cfg.dims[l])] = timed(lambda: e2.index_add_(0, src, hg[l]))
+        del e2
+    return {"ms_per_layer": out, "ops": "torch.index_select (forward), torch.index_add_ "
+            "(backward, atomic)", "note": "stock PyTorch on the same B200, same layouts"}
+
+
 def run_ours_single(args, w):
     import torch
     import paper_conf_eurosys_cai0wmcy21_b200 as D
@@ -334,6 +370,7 @@ def run_ours_single(args, w):
                 "per_kernel": kernels}
 
     value = w.step_payload_bytes() / (ms_step * 1e-3) / 1e9
+    torch_base = None if args.no_torch_baseline else torch_gather_baseline(w, emb, hg, eg, stream)
     cpu = None
     if not args.no_cpu_baseline:
         gbs, secs, used, thr = oracle_sample(w, emb_h, hg_h, eg_h, budget_s=args.cpu_budget)
@@ -360,6 +397,7 @@ def run_ours_single(args, w):
         "gpu_launches": int(launches),
         "clocks": clocks,
         "plan": dict(info, planner_wall_s=plan_s, graph_gen_s=w.gen_s),
+        "torch_gather_baseline": torch_base,
     }
     ctx.destroy()
     return out
@@ -402,6 +440,7 @@ def main():
     ap.add_argument("--config", default="reddit")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-torch-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--item-bytes", type=int, default=0)
     ap.add_argument("--share-gpu", action="store_true", help=argparse.SUPPRESS)
