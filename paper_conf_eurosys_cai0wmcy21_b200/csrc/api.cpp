@@ -90,7 +90,6 @@ struct dgcl_ctx {
   uint64_t seq = 0, epoch[2] = {0, 0};
   int *err_host = nullptr, *err_dev = nullptr;
   int threads = 512, ctas_per_sm = 0, grid = 0, n_sm = 0, tma_ctas = 0, use_tma = 1;
-  int64_t max_fold_slots = 1;
   int64_t item_bytes = kTmaBufBytes, timeout_ms = 20000;
   std::vector<cudaStream_t> rank_streams;
   std::vector<cudaEvent_t> rank_events;
@@ -543,7 +542,6 @@ dgcl_status dgcl_build_plan(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *
     for (int d = 0; d < c->world; ++d)  // direct-reduce terms hold 28-bit halo rows
       if (c->rel.n_halo[d] > (int64_t)kTermRowMask) c->direct_reduce = false;
     build_programs(c);
-    c->max_fold_slots = max_fold_slots(c->low);
   } catch (const std::bad_alloc &) {
     return fail(c, DGCL_ENOMEM, "host allocation failed while planning");
   }

@@ -3,22 +3,21 @@
 // Same semantics as executor.cu (items / counters, see internal.h), different data movement.
 // PAPER.md §6.1-6.2: the sender packs rows by its send table and writes them into
 // the receiver's buffer.  Here the "pack" is a gather of whole rows into shared memory by the
-// Tensor Memory Accelerator (one cp.async.bulk per row), and the "send" is a coalesced 16-B store
-// stream from shared memory to the destination rows (a peer's halo over NVLink 5, or local HBM).
+// Tensor Memory Accelerator (one cp.async.bulk per run of consecutive rows, or tile::gather4 for
+// four scattered rows), and the "send" is a bulk (TMA) store or a coalesced 16-B store stream from
+// shared memory to the destination rows (a peer's halo over NVLink 5, or local HBM).
 //
-// Per CTA (one per SM, 512 threads, 4 x 48 KB stages + 2 x 12 KB metadata buffers):
-//   warp 0 (producer) walks the CTA's items in order with a metadata pipeline — item descriptor
-//     two items ahead (registers), the next item's index windows (source rows, term pointers,
-//     terms) one item ahead (bulk copies into a metadata buffer) — so no dependent global load is
-//     on its critical path.  Per data item it resolves the source waits (stage chaining) and the
-//     destination's ready word, waits for a free stage, writes the item header, arms the stage's
-//     "full" mbarrier with the byte count and issues the row gathers (lane l: rows l, l+32, ...)
-//     plus the consumers' row-table windows;
-//   warps 1-15 (consumers) take stages in order: store (COPY) or fold-and-store (FOLD) from shared
-//     memory, publish (per warp: fence.sys, then red.release.sys of the warp's share of the rows
-//     on the receiver's counter — the shares sum to the item's rows, so no CTA barrier is needed)
-//     and release the stage.  An END header stops them (also used to unwind after a watchdog).
-// Up to 4 x 44 KB of gathers are in flight per SM, hiding HBM / NVLink latency without registers.
+// Per CTA (one per SM, 512 threads, 3 x 64 KB stages, descriptor ring, 4 x 8 KB run windows):
+//   warp 0 (producer) walks the CTA's items in order with a metadata pipeline — descriptors
+//     bulk-copied 6 items ahead, row runs / source rows 3 items ahead — so no dependent global
+//     load is on its critical path.  Per data item it resolves the source waits (stage chaining)
+//     and the destination's ready word, claims a stage, writes the item header, arms the stage's
+//     "full" mbarrier with the byte count and issues the row gathers plus the consumers' tables;
+//     before it could block on a wait it inserts a FLUSH marker so pending done counts go out;
+//   warps 1-15 (consumers) take stages in order: store (COPY) or fold-and-store (FOLD), count the
+//     item's rows in shared memory (published at FLUSH / END: fence.sys, then one
+//     red.release.sys per (source, receiver)) and release the stage.  An END header stops them.
+// Up to 3 x 60 KB of gathers are in flight per SM, hiding HBM / NVLink latency without registers.
 
 #include "device_common.cuh"
 
@@ -142,15 +141,6 @@ __device__ __forceinline__ bool waits_ready(const ExecParams &P, const DevItem &
       return false;
   }
   return true;
-}
-
-__device__ __forceinline__ DevItem load_item(const DevItem *items, int i) {
-  DevItem d;
-  const int4 *s = reinterpret_cast<const int4 *>(items + i);
-  int4 *o = reinterpret_cast<int4 *>(&d);
-#pragma unroll
-  for (int q = 0; q < 4; ++q) o[q] = __ldg(s + q);
-  return d;
 }
 
 // 16-B aligned window [a, e) of `n` elements of size `sz` starting at element `off`
@@ -618,11 +608,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         // block on a wait, and whenever the counter family (direction, stage) changes.
         const bool sig = (I.flags & kItemSignal) != 0;
         const int key = sig ? I.sig_ctr - I.exec_rank : -1;
-#ifdef DGCL_EXPERIMENT_NO_FLUSH
-        if (false) {
-#else
         if (pend) {
-#endif
           int ready = 1;
           if (lane == 0) {
             ready = waits_ready(P, I) ? 1 : 0;

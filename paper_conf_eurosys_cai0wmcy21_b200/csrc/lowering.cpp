@@ -513,15 +513,4 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
   }
 }
 
-int64_t max_fold_slots(const Lowered &low) {
-  int64_t mx = 1;
-  for (const DevGroup &g : low.groups) {
-    if (g.op != OP_FOLD) continue;
-    for (int64_t r = 0; r < g.n_rows; ++r)
-      mx = std::max<int64_t>(mx, low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r] +
-                                     (g.fold_init ? 1 : 0));
-  }
-  return mx;
-}
-
 }  // namespace dgcl

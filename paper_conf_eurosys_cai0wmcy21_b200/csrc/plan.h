@@ -52,10 +52,6 @@ std::string spst_plan(const Topology &topo, const int32_t *part, const Relation 
 
 // ---- lowering ----------------------------------------------------------------------------
 
-struct HostGroup {
-  DevGroup g;        // descriptor (offsets relative to the pools below)
-};
-
 struct Lowered {
   int m = 0;
   int n_stages = 0;                      // forward stages K
@@ -85,16 +81,14 @@ struct Lowered {
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
                 const std::vector<int64_t> &loc, Lowered *out);
 
-// Work items for one launch: the groups `gids` (already in stage order) cut into row ranges of
-// about item_bytes bytes and interleaved across groups within a stage.
-// completion_rank >= 0 appends nothing (the WAIT group is passed in gids by the caller).
-// COPY items also get their row runs appended to `runs` (item.tp = first run, program-relative).
+// Work items for one launch: the groups `gids` (already in stage order, READY / WAIT groups
+// included by the caller) cut into row ranges of about item_bytes gathered bytes and interleaved
+// across the groups of a stage.  COPY items also get their row runs appended to `runs`
+// (item.tp = first run, program-relative); items of short runs are flagged for gather4 (or for
+// consumer gathers when direct_copy_rows > 0).
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
                  int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
                  std::vector<DevItem> *items, std::vector<DevRun> *runs,
                  int64_t direct_copy_rows = 0);
-
-// largest number of operand rows one FOLD row gathers (1 + #terms); bounds the bulk-copy stage
-int64_t max_fold_slots(const Lowered &low);
 
 }  // namespace dgcl
