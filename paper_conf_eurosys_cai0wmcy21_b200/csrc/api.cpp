@@ -312,8 +312,11 @@ template <typename T>
 dgcl_status upload(dgcl_ctx *c, T **dptr, const std::vector<T> &v) {
   if (*dptr) cudaFree(*dptr);
   *dptr = nullptr;
-  const size_t bytes = std::max<size_t>(sizeof(T), v.size() * sizeof(T));
+  // + 64 zeroed bytes: the executor bulk-copies 16-B aligned windows of these pools, whose last
+  // window may extend up to 15 bytes past the final element
+  const size_t bytes = v.size() * sizeof(T) + 64;
   CUDA_TRY(c, cudaMalloc((void **)dptr, bytes));
+  CUDA_TRY(c, cudaMemset(*dptr, 0, bytes));
   if (!v.empty()) CUDA_TRY(c, cudaMemcpy(*dptr, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice));
   return DGCL_OK;
 }

@@ -333,3 +333,34 @@ def _sampled_full(name, dims_override=None, n_samples=3000):
                                   "google8_dgx1"])
 def test_full_size_sampled(name):
     _sampled_full(name)
+
+
+def test_single_rank_is_noop():
+    """world = 1: nothing to exchange — forward leaves the (empty) halo alone, backward leaves
+    emb_grad unchanged, and no executor launch happens."""
+    D = _D()
+    torch = _torch()
+    part = np.zeros(100, np.int32)
+    ctx = D.loopback(1, part, [8], device=0)
+    ctx.build_plan([0, 0], [])
+    ctx.register_workspace()
+    emb = torch.randn(100, 8, device="cuda")
+    ctx.forward(0, emb)
+    eg = torch.randn(100, 8, device="cuda")
+    before = eg.clone()
+    ctx.backward(0, torch.zeros(1, 8, device="cuda"), eg)
+    torch.cuda.synchronize()
+    assert torch.equal(eg, before) and ctx.launch_count() == 0
+
+
+def test_sixteen_virtual_ranks():
+    g = synth.make_graph(8000, 60000, 16, graph_seed=71, part_seed=72)
+    _check_case(Case(g, [24]))
+
+
+@pytest.mark.parametrize("dims", [[4000], [20000]])
+def test_wide_rows(dims):
+    """4000 floats: a few rows per bulk-copy stage; 20000 floats (80 KB rows): wider than a
+    stage, so the register executor runs the launch."""
+    g = synth.make_graph(600, 3000, 3, graph_seed=81, part_seed=82)
+    _check_case(Case(g, dims))
