@@ -246,6 +246,9 @@ def run_ours_single(args, w):
     ctx = D.loopback(c.m, g.part, list(c.dims), device=0)
     if args.item_bytes:
         ctx.set_option("item_bytes", args.item_bytes)
+    for kv in args.opt:  # executor options (dgcl_set_option), for A/B runs
+        k, v = kv.split("=")
+        ctx.set_option(k, int(v))
     t = time.time()
     ctx.build_plan(g.req_ptr, g.req_ids, seed=0, topology=topo)
     plan_s = time.time() - t
@@ -443,6 +446,8 @@ def main():
     ap.add_argument("--no-torch-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--item-bytes", type=int, default=0)
+    ap.add_argument("--opt", action="append", default=[], metavar="KEY=VALUE",
+                    help="executor option (dgcl_set_option) before planning, e.g. stage_fold=0")
     ap.add_argument("--share-gpu", action="store_true", help=argparse.SUPPRESS)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)

@@ -192,6 +192,19 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    aligned; 0: the register (LDG/STG) executor
  *   "ctas_per_sm"    executor CTAs per SM (default: occupancy, max 4)
  *   "threads"        executor CTA size (128..512, multiple of 32; default 512)
+ *   "gather4"        1 (default): TMA tile::gather4 (four rows per instruction) for short-run
+ *                    embedding gathers with rows <= 1 KB
+ *   "stage_fold"     1 (default): backward folds bulk-copy all their operand rows into shared
+ *                    memory (segments of consecutive rows) before adding them; 0: consumers
+ *                    gather the operands with plain loads
+ *   "direct_reduce"  1 (default): fused loopback with a single-stage plan folds the requesters'
+ *                    halo gradients in place (no slot round trip); 0: push + owner reduce
+ *   "direct_copy_rows" COPY items whose runs average fewer rows are gathered by the consumer
+ *                    warps with plain loads (default 0 = never)
+ *   "bulk_store", "bulk_store_peer"  TMA stores for packed contiguous destinations in local HBM
+ *                    (default 1) / peer memory (default 0)
+ * Options other than "timeout_ms" and "debug_skip_rank" must be set before
+ * dgcl_register_workspace (ESTATE otherwise).
  *   "debug_skip_rank" fault injection for DGCL_LOOPBACK_PER_RANK contexts: never launch that
  *                    virtual rank's program, so its peers' flag waits hit the watchdog (any time;
  *                    -1 = off)

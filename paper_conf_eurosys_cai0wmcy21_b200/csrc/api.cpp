@@ -34,9 +34,11 @@ struct Program {
   // one launch: items for one (layer, direction, executing rank or -1 = fused loopback)
   std::vector<DevItem> items;
   std::vector<DevRun> runs;
+  std::vector<uint32_t> sterms;  // staged FOLD items: operand row of every term
   size_t dev_off = 0;  // offset (in items) into the device item pool
-  int op_mask = 0;     // kMaskCopy / kMaskFold / kMaskDirect items present
+  int op_mask = 0;     // kMaskCopy / kMaskFold / kMaskDirect / kMaskStaged items present
   bool fold_wide = false;  // FOLD rows average >= 4 terms
+  int geo = 0;             // bulk-copy launch geometry: 0 = kGeoWide, 1 = kGeoDual
 };
 
 }  // namespace
@@ -77,6 +79,7 @@ struct dgcl_ctx {
   uint32_t *d_terms = nullptr;
   DevItem *d_items = nullptr;
   DevRun *d_runs = nullptr;
+  uint32_t *d_sterms = nullptr;
   int64_t run_bytes = 0;
   bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
   bool bulk_store_peer = false;   // TMA stores into peer memory over NVLink (not yet validated)
@@ -85,11 +88,16 @@ struct dgcl_ctx {
   bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
+  bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
+  bool hostsim_items = false;         // debug host interpreter: run the work items, not groups
+  int geometry = 0;                   // bulk-copy geometry: 0 auto per program, 1 WIDE, 2 DUAL
+  bool threads_set = false, ctas_set = false;  // user overrides of the CTA shape
+  int tma_ctas_geo[2][2] = {{0, 0}, {0, 0}};   // [geo][1024-thread fold instance] CTAs per SM
   int n_prog_ranks = 1;        // programs per (layer, dir)
 
   uint64_t seq = 0, epoch[2] = {0, 0};
   int *err_host = nullptr, *err_dev = nullptr;
-  int threads = 512, ctas_per_sm = 0, grid = 0, n_sm = 0, tma_ctas = 0, use_tma = 1;
+  int threads = 512, ctas_per_sm = 0, grid = 0, n_sm = 0, use_tma = 1;
   int64_t item_bytes = kTmaBufBytes, timeout_ms = 20000;
   std::vector<cudaStream_t> rank_streams;
   std::vector<cudaEvent_t> rank_events;
@@ -290,19 +298,43 @@ void build_programs(dgcl_ctx *c) {
       for (int r = 0; r < c->n_prog_ranks; ++r) {
         Program &P = c->progs[c->prog_index(l, dir, r)];
         const std::vector<uint8_t> need = needed_counters(L, gids[r]);
-        build_items(L, gids[r], (int64_t)c->dims[l] * 4, c->item_bytes, !fused, need, &P.items,
-                    &P.runs, c->direct_copy_rows);
-        P.op_mask = 0;
-        int64_t fold_rows = 0, fold_terms = 0;
-        for (const DevItem &it : P.items) {
-          if (it.op == OP_FOLD) {
-            P.op_mask |= kMaskFold;
-            fold_rows += it.rows;
-            fold_terms += it.nterms;
+        const int64_t row_bytes = (int64_t)c->dims[l] * 4, row16 = (row_bytes + 15) / 16 * 16;
+        auto build = [&](int geo) {
+          P.geo = geo;
+          build_items(L, gids[r], row_bytes,
+                      item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes), !fused, need,
+                      &P.items, &P.runs, c->direct_copy_rows,
+                      c->stage_fold ? &P.sterms : nullptr);
+          P.op_mask = 0;
+          int64_t fold_rows = 0, fold_terms = 0;
+          for (const DevItem &it : P.items) {
+            if (it.op == OP_FOLD && (it.flags & kItemStaged)) {
+              P.op_mask |= kMaskStaged;
+            } else if (it.op == OP_FOLD) {
+              P.op_mask |= kMaskFold;
+              fold_rows += it.rows;
+              fold_terms += it.nterms;
+            }
+            if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
           }
-          if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
+          P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
+        };
+        if (c->geometry) {
+          build(c->geometry - 1);
+          continue;
         }
-        P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
+        // auto: DUAL (two producer warps per SM) unless the launch is bulk-copy friendly —
+        // copies only, >= 8 KB per bulk operation (long runs of rows) — or carries unstaged folds
+        // (consumer gathers, which want the 1024-thread instance); see TmaGeometry
+        build(1);
+        int64_t ops = 0, bytes = 0;
+        for (const DevItem &it : P.items) {
+          if (it.op != OP_COPY) continue;
+          bytes += (int64_t)it.rows * row16;
+          ops += (it.flags & kItemGather4) ? (it.rows + 3) / 4 : it.nterms;
+        }
+        const bool copy_only = (P.op_mask & ~kMaskCopy) == 0;
+        if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & kMaskFold)) build(0);
       }
     }
   }
@@ -413,12 +445,12 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   P.timeout_ns = (uint64_t)c->timeout_ms * 1000000ull;
   P.err = c->err_dev;
   P.row16 = (P.row_bytes + 15) / 16 * 16;
-  P.tma_buf = kTmaBufBytes;
   P.runs = c->d_runs;
+  P.sterms = c->d_sterms;
   P.bulk_store = (c->loopback ? c->bulk_store_local : c->bulk_store_peer) ? 1 : 0;
-  // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage
-  P.use_tma = (v16 && c->use_tma && c->tma_ctas > 0 &&
-               P.row16 <= kTmaOperandBytes) ? 1 : 0;
+  // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage (checked
+  // again per program against its geometry in launch_program)
+  P.use_tma = (v16 && c->use_tma && P.row16 <= kTmaOperandBytes) ? 1 : 0;
   // forward launches over packed embedding rows of <= 1 KB: a 2-D tensor map for the TMA row
   // gather (gather4) used by items whose source rows come in short runs
   if (P.use_tma && dir == DIR_FWD && c->use_gather4 && in_pitch * 4 == P.row16 &&
@@ -430,19 +462,38 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
         P.tmap_row_off[r] = c->loopback ? (int32_t)c->row_off[r] : 0;
     }
   }
-  const int grid_all = P.use_tma ? c->n_sm * c->tma_ctas : c->grid;
+  // one program's launch: its items, kernel instance, CTA shape and bulk-copy geometry
+  auto launch_program = [&](const Program &pg, int grid_div, cudaStream_t st) -> int {
+    ExecParams Pp = P;
+    Pp.items = c->d_items + pg.dev_off;
+    Pp.op_mask = pg.op_mask;
+    Pp.fold_wide = pg.fold_wide ? 1 : 0;
+    Pp.n_items = (int32_t)pg.items.size();
+    const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
+    const bool wide_fold = pg.geo == 0 && pg.op_mask == kMaskFold && pg.fold_wide &&
+                           !c->threads_set;
+    int block = c->threads, grid_all = c->grid;
+    if (Pp.use_tma && Pp.row16 <= G.stage_bytes - kStageHdrBytes &&
+        c->tma_ctas_geo[pg.geo][wide_fold ? 1 : 0] > 0) {
+      block = wide_fold ? 1024 : (c->threads_set ? c->threads : G.threads);
+      grid_all = c->n_sm * c->tma_ctas_geo[pg.geo][wide_fold ? 1 : 0];
+      Pp.tma_stages = G.stages;
+      Pp.tma_buf = G.stage_bytes;
+      Pp.meta_bytes = G.meta_bytes;
+    } else {
+      Pp.use_tma = 0;
+      Pp.use_gather4 = 0;
+    }
+    const int grid = (int)std::min<int64_t>(std::max(1, grid_all / grid_div), Pp.n_items);
+    return launch_executor(Pp, grid, block, st);
+  };
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
   P.use_ready = (!fused && m > 1) ? 1 : 0;
   if (fused || !c->loopback) {
     const int r = fused ? 0 : c->rank;
     const Program &pg = c->progs[c->prog_index(layer, dir, fused ? 0 : (c->loopback ? r : r))];
     if (pg.items.empty()) return DGCL_OK;
-    P.items = c->d_items + pg.dev_off;
-    P.op_mask = pg.op_mask;
-    P.fold_wide = pg.fold_wide ? 1 : 0;
-    P.n_items = (int32_t)pg.items.size();
-    const int grid = std::min<int64_t>(grid_all, (int64_t)pg.items.size());
-    int e = launch_executor(P, grid, c->threads, stream);
+    int e = launch_program(pg, 1, stream);
     if (e != 0) return fail(c, DGCL_ECUDA, "executor launch failed: %s",
                             cudaGetErrorString((cudaError_t)e));
     c->launches++;
@@ -450,18 +501,11 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   }
   // loopback, one launch per virtual rank on its own stream (full flag protocol)
   CUDA_TRY(c, cudaEventRecord(c->fork_event, stream));
-  const int grid_r = std::max(1, grid_all / m);
   for (int r = 0; r < m; ++r) {
     const Program &pg = c->progs[c->prog_index(layer, dir, r)];
     CUDA_TRY(c, cudaStreamWaitEvent(c->rank_streams[r], c->fork_event, 0));
     if (!pg.items.empty() && r != c->debug_skip_rank) {
-      ExecParams Pr = P;
-      Pr.items = c->d_items + pg.dev_off;
-      Pr.op_mask = pg.op_mask;
-      Pr.fold_wide = pg.fold_wide ? 1 : 0;
-      Pr.n_items = (int32_t)pg.items.size();
-      int e = launch_executor(Pr, std::min<int64_t>(grid_r, (int64_t)pg.items.size()),
-                              c->threads, c->rank_streams[r]);
+      int e = launch_program(pg, m, c->rank_streams[r]);
       if (e != 0) return fail(c, DGCL_ECUDA, "executor launch failed: %s",
                               cudaGetErrorString((cudaError_t)e));
       c->launches++;
@@ -590,18 +634,27 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   if ((s = upload(c, &c->d_terms, c->low.terms)) != DGCL_OK) return s;
   std::vector<DevItem> all;
   std::vector<DevRun> all_runs;
+  std::vector<uint32_t> all_sterms;
   for (Program &p : c->progs) {
     p.dev_off = all.size();
     const int64_t run_base = (int64_t)all_runs.size();
+    const int64_t sterm_base = (int64_t)all_sterms.size();
     for (DevItem it : p.items) {
-      if (it.op == OP_COPY) it.tp += run_base;  // program-relative -> pool index
+      // program-relative -> pool indices
+      if (it.op == OP_COPY) it.tp += run_base;
+      if (it.op == OP_FOLD && (it.flags & kItemStaged)) {
+        it.src += run_base;  // low bits: first segment
+        it.t0 += sterm_base;
+      }
       all.push_back(it);
     }
     all_runs.insert(all_runs.end(), p.runs.begin(), p.runs.end());
+    all_sterms.insert(all_sterms.end(), p.sterms.begin(), p.sterms.end());
   }
   if ((s = upload(c, &c->d_items, all)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_runs, all_runs)) != DGCL_OK) return s;
-  c->run_bytes = (int64_t)(all_runs.size() * sizeof(DevRun));
+  if ((s = upload(c, &c->d_sterms, all_sterms)) != DGCL_OK) return s;
+  c->run_bytes = (int64_t)(all_runs.size() * sizeof(DevRun) + all_sterms.size() * 4);
   // watchdog word in mapped host memory
   CUDA_TRY(c, cudaHostAlloc((void **)&c->err_host, 64, cudaHostAllocMapped));
   std::memset(c->err_host, 0, 64);
@@ -609,8 +662,21 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   // launch geometry: persistent grid of co-resident CTAs
   CUDA_TRY(c, cudaDeviceGetAttribute(&c->n_sm, cudaDevAttrMultiProcessorCount, c->device));
   int occ = 0;
-  int e = executor_occupancy(c->threads, &occ, &c->tma_ctas);
+  int e = executor_occupancy(c->threads, &occ);
   if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");
+  // bulk-copy executor: co-resident CTAs per SM for each geometry at its CTA size
+  for (int geo = 0; geo < 2; ++geo) {
+    const TmaGeometry &G = geo ? kGeoDual : kGeoWide;
+    for (int wide_fold = 0; wide_fold < 2; ++wide_fold) {
+      const int block = wide_fold ? 1024 : (c->threads_set ? c->threads : G.threads);
+      int n = 0;
+      e = executor_tma_occupancy(block, tma_smem_bytes(G), &n);
+      if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");
+      n = std::min(n, G.ctas_per_sm);
+      if (c->ctas_set) n = std::min(n, c->ctas_per_sm);
+      c->tma_ctas_geo[geo][wide_fold] = n;
+    }
+  }
   if (c->ctas_per_sm <= 0) c->ctas_per_sm = std::min(occ, 4);
   c->ctas_per_sm = std::max(1, std::min(c->ctas_per_sm, occ));
   c->grid = c->n_sm * c->ctas_per_sm;
@@ -866,6 +932,17 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     c->timeout_ms = value;
     return DGCL_OK;
   }
+  if (k == "geometry") {  // bulk-copy launch geometry: 0 auto, 1 WIDE, 2 DUAL (TmaGeometry)
+    if (value < 0 || value > 2) return fail(c, DGCL_EINVAL, "geometry must be 0, 1 or 2");
+    if (c->registered) return fail(c, DGCL_ESTATE, "geometry must be set before registration");
+    c->geometry = (int)value;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "hostsim_items") {  // verification aid: the host interpreter runs the work items
+    c->hostsim_items = value != 0;
+    return DGCL_OK;
+  }
   if (k == "debug_skip_rank") {
     if (value < -1 || value >= c->world) return fail(c, DGCL_EINVAL, "debug_skip_rank");
     c->debug_skip_rank = (int)value;
@@ -900,6 +977,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     c->bulk_store_peer = value != 0;
     return DGCL_OK;
   }
+  if (k == "stage_fold") {  // bulk-copy FOLD operand rows into the stage (bulk-copy executor)
+    c->stage_fold = value != 0;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
   if (k == "direct_reduce") {
     c->direct_reduce = value != 0;
     if (c->planned) build_programs(c);
@@ -908,11 +990,13 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   if (k == "ctas_per_sm") {
     if (value < 1 || value > 32) return fail(c, DGCL_EINVAL, "ctas_per_sm out of range");
     c->ctas_per_sm = (int)value;
+    c->ctas_set = true;
     return DGCL_OK;
   }
   if (k == "threads") {
     if (value < 128 || value > 512 || value % 32) return fail(c, DGCL_EINVAL, "threads");
     c->threads = (int)value;
+    c->threads_set = true;
     return DGCL_OK;
   }
   return fail(c, DGCL_EINVAL, "unknown option %s", key);
@@ -963,6 +1047,7 @@ dgcl_status dgcl_destroy(dgcl_ctx *c) {
     cudaFree(c->d_terms);
     cudaFree(c->d_items);
     cudaFree(c->d_runs);
+    cudaFree(c->d_sterms);
     if (c->stage_a) cudaFree(c->stage_a);
     if (c->stage_b) cudaFree(c->stage_b);
     if (c->err_host) cudaFreeHost(c->err_host);
@@ -980,6 +1065,13 @@ dgcl_status dgcl_debug_hostsim_forward(dgcl_ctx *c, int32_t layer, const float *
   if (!c || !emb || !halo) return DGCL_EINVAL;
   if (!c->planned || !c->loopback) return fail(c, DGCL_ESTATE, "needs a planned loopback context");
   if (layer < 0 || layer >= c->n_layers) return DGCL_EINVAL;
+  if (c->hostsim_items && c->lb_flags == DGCL_LOOPBACK_FUSED) {
+    const Program &P = c->progs[c->prog_index(layer, DIR_FWD, 0)];
+    if (!hostsim_run_items(c->low, P.items, P.runs, P.sterms, c->row_off, c->halo_off,
+                           c->pitch[layer], c->dims[layer], emb, halo, nullptr, nullptr))
+      return fail(c, DGCL_EPLAN, "malformed work item");
+    return DGCL_OK;
+  }
   hostsim_run(c->low, c->host_gids[DIR_FWD], c->row_off, c->halo_off, c->pitch[layer],
               c->dims[layer], emb, halo, nullptr, nullptr);
   return DGCL_OK;
@@ -990,6 +1082,13 @@ dgcl_status dgcl_debug_hostsim_backward(dgcl_ctx *c, int32_t layer, const float 
   if (!c || !halo_grad || !emb_grad) return DGCL_EINVAL;
   if (!c->planned || !c->loopback) return fail(c, DGCL_ESTATE, "needs a planned loopback context");
   if (layer < 0 || layer >= c->n_layers) return DGCL_EINVAL;
+  if (c->hostsim_items && c->lb_flags == DGCL_LOOPBACK_FUSED) {
+    const Program &P = c->progs[c->prog_index(layer, DIR_BWD, 0)];
+    if (!hostsim_run_items(c->low, P.items, P.runs, P.sterms, c->row_off, c->halo_off,
+                           c->pitch[layer], c->dims[layer], nullptr, nullptr, halo_grad, emb_grad))
+      return fail(c, DGCL_EPLAN, "malformed work item");
+    return DGCL_OK;
+  }
   hostsim_run(c->low, c->host_gids[DIR_BWD], c->row_off, c->halo_off, c->pitch[layer],
               c->dims[layer], nullptr, nullptr, halo_grad, emb_grad);
   return DGCL_OK;

@@ -216,7 +216,7 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
 
 // executor_tma.cu
 int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream);
-int tma_executor_occupancy(int block, int *ctas_per_sm);
+int tma_executor_occupancy(int block, size_t smem_bytes, int *ctas_per_sm);
 
 int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   if (grid <= 0) return 0;
@@ -229,10 +229,12 @@ int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   return (int)cudaGetLastError();
 }
 
-int executor_occupancy(int block, int *ctas_per_sm, int *tma_ctas_per_sm) {
+int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm) {
+  return tma_executor_occupancy(block, smem_bytes, ctas_per_sm);
+}
+
+int executor_occupancy(int block, int *ctas_per_sm) {
   int a = 0, b = 0;
-  int e = tma_executor_occupancy(block, tma_ctas_per_sm);
-  if (e != 0) return e;
   cudaError_t ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, executor_kernel<true>, block, 0);
   if (ce != cudaSuccess) return (int)ce;
   ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, executor_kernel<false>, block, 0);

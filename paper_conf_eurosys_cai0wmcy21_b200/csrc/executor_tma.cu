@@ -27,29 +27,30 @@ using namespace dev;
 
 namespace {
 
-constexpr int kStages = kTmaStages;
 #ifndef DGCL_STORE_SPLIT
 #define DGCL_STORE_SPLIT 15  // every consumer warp stores its share (measured best, Reddit)
 #endif
 constexpr int kStoreSplit = DGCL_STORE_SPLIT;  // bulk stores per COPY item (<= consumer warps)
-constexpr int kMetaBytes = 8 * 1024;  // one item's row runs (<= kMaxItemRows x 16 B)
 constexpr int kMetaSlots = 4;         // run windows prefetched kMetaAhead items ahead
 constexpr int kMetaAhead = 3;
 constexpr int kDescAhead = 6;         // descriptors prefetched further ahead (ring of kDescSlots)
-static_assert(kMaxItemRows * 16 <= kMetaBytes, "meta slot holds an item's runs");
 constexpr int kHdrInfo = 64;         // stage: int32 info words after the 64-B item header
 constexpr int kTabTp = 128;          // stage: term_ptr window (FOLD)
 constexpr int kTabDst = 2176;        // stage: destination-row window
 constexpr int kDescSlots = 8;        // producer descriptor ring
 static_assert(kDescAhead > kMetaAhead && kDescAhead < kDescSlots && kMetaAhead < kMetaSlots,
               "prefetch distances");
+// shared-memory carve-up (internal.h, tma_smem_bytes): offsets depend on the launch geometry
 constexpr size_t kMetaOff = 256;     // after the mbarriers (full, empty, meta, desc)
-static_assert((2 * kTmaStages + kMetaSlots + kDescSlots) * 8 <= 256, "mbarrier region");
-constexpr size_t kDescOff = kMetaOff + kMetaSlots * (size_t)kMetaBytes;
-constexpr size_t kStageOff = kDescOff + kDescSlots * 64;
-constexpr size_t kPendOff = kStageOff + (size_t)kStages * kTmaBufBytes;  // 1 KB counts + 3 words
-constexpr size_t kSmemBytes = kPendOff + 1152;
-static_assert(kSmemBytes <= 227 * 1024, "shared memory budget");
+static_assert((2 * kMaxTmaStages + kMetaSlots + kDescSlots) * 8 <= 256, "mbarrier region");
+static_assert(kMetaSlots * 8 * 64 <= 4 * 8 * 1024 && kDescSlots == 8, "layout of tma_smem_bytes");
+constexpr size_t kSmemMax = tma_smem_bytes(kGeoWide);
+
+// k-th stage use of a ring of ns (2 or 3) stages: slot and use count without a division
+__device__ __forceinline__ void ring_pos(uint32_t k, uint32_t ns, uint32_t &slot, uint32_t &use) {
+  use = ns == 2 ? (k >> 1) : (__umulhi(k, 0xAAAAAAABu) >> 1);
+  slot = k - use * ns;
+}
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -173,6 +174,18 @@ __device__ __forceinline__ void tma_gather4(void *sdst, const void *tmap, int32_
       : "memory");
 }
 
+// staged FOLD item: operand rows bulk-copied into the stage (destination rows first when the
+// fold starts from them, then one row per term), followed by the staged-term window
+__device__ __forceinline__ bool is_staged(const DevItem &I) {
+  return I.op == OP_FOLD && (I.flags & kItemStaged);
+}
+__device__ __forceinline__ uint32_t staged_rows(const DevItem &I) {
+  return (I.fold_init ? (uint32_t)I.rows : 0u) + (uint32_t)I.nterms;
+}
+__device__ __forceinline__ uint32_t n_segments(const DevItem &I) {
+  return (uint32_t)(I.src >> kSegShift);
+}
+
 // producer lane 0: bulk-copy the metadata the producer needs to issue item I's gathers
 __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I, uint8_t *meta,
                                            uint64_t *bar) {
@@ -184,6 +197,12 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
     const Win ws = window(~I.src, I.rows, 4);
     mbar_expect_tx(bar, ws.bytes);
     bulk_g2s(meta, P.idx + ws.a, ws.bytes, bar);
+    return;
+  }
+  if (is_staged(I)) {  // the item's segments
+    const uint32_t tx = n_segments(I) * (uint32_t)sizeof(DevRun);
+    mbar_expect_tx(bar, tx);
+    bulk_g2s(meta, P.runs + (I.src & ((1ll << kSegShift) - 1)), tx, bar);
     return;
   }
   const uint32_t tx = (I.op == OP_COPY && !(I.flags & kItemDirect))
@@ -200,6 +219,7 @@ __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const Dev
     if (!(I.flags & kItemDirect)) return (uint32_t)I.rows * (uint32_t)P.row16;
     return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;  // source-row window only
   }
+  if (is_staged(I)) return staged_rows(I) * (uint32_t)P.row16 + window(I.t0, I.nterms, 4).bytes;
   return window(I.t0, I.nterms, 4).bytes;
 }
 
@@ -263,6 +283,26 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
           bulk_g2s(ops + (size_t)(R.pos + j) * r16, sbase + (int64_t)(R.src + j) * spitch, r16,
                    full);
       }
+    }
+  } else if (is_staged(I)) {
+    // staged FOLD: one bulk copy per segment of consecutive operand rows, then the staged terms
+    const DevRun *segs = reinterpret_cast<const DevRun *>(meta);
+    const int ns = (int)n_segments(I);
+    for (int q = lane; q < ns; q += 32) {
+      const DevRun R = segs[q];
+      const BufRef B = P.buf[R.dst >> 8][R.dst & 255];
+      if (B.pitch == (int64_t)r16) {
+        bulk_g2s(ops + (size_t)R.pos * r16, B.ptr + (int64_t)R.src * B.pitch,
+                 (uint32_t)R.len * r16, full);
+      } else {
+        for (int j = 0; j < R.len; ++j)
+          bulk_g2s(ops + (size_t)(R.pos + j) * r16, B.ptr + (int64_t)(R.src + j) * B.pitch, r16,
+                   full);
+      }
+    }
+    if (lane == 0) {
+      const Win wt = window(I.t0, I.nterms, 4);
+      if (wt.bytes) bulk_g2s(ops + (size_t)staged_rows(I) * r16, P.sterms + wt.a, wt.bytes, full);
     }
   } else if (lane == 0) {
     // OP_FOLD: only the terms window is staged (into the operand area); the consumers gather
@@ -444,6 +484,54 @@ __device__ __forceinline__ void store_fold_multi(const ExecParams &P, const DevI
   }
 }
 
+// consumers: staged FOLD item — every operand row is in the stage; add each output chunk's terms
+// in list order (init row first when the fold starts from the destination) and store it
+__device__ __forceinline__ void store_fold_staged(const ExecParams &P, const DevItem &I,
+                                                  const uint8_t *st, uint32_t tid, uint32_t T) {
+  const BufRef D = P.buf[I.dst_kind][I.dst_rank];
+  const int32_t *info = reinterpret_cast<const int32_t *>(st + kHdrInfo);
+  const int64_t *tp = reinterpret_cast<const int64_t *>(st + kTabTp) + info[0];
+  const int32_t *tab = reinterpret_cast<const int32_t *>(st + kTabDst) + info[1];
+  const uint32_t r16 = (uint32_t)P.row16;
+  const uint8_t *ops = st + kStageHdrBytes;
+  const uint32_t *stt = reinterpret_cast<const uint32_t *>(ops + (size_t)staged_rows(I) * r16) +
+                        window(I.t0, I.nterms, 4).skew;
+  const int init = I.fold_init;
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  const int tail = P.row_bytes - (int)(nch - 1) * 16;
+  const int64_t tbase = tp[0];
+  for (uint32_t e = tid; e < total; e += T) {
+    const uint32_t r = fdiv(e, P);
+    const uint32_t col = e - r * nch;
+    const uint8_t *oc = ops + col * 16;
+    int j = (int)(tp[r] - tbase);
+    const int je = (int)(tp[r + 1] - tbase);
+    float4 acc;
+    if (init) {
+      acc = as_f4(lds_v4(oc + r * r16));
+    } else {
+      acc = as_f4(lds_v4(oc + stt[j] * r16));
+      ++j;
+    }
+    for (; j + 4 <= je; j += 4) {
+      const int4 v0 = lds_v4(oc + stt[j] * r16), v1 = lds_v4(oc + stt[j + 1] * r16);
+      const int4 v2 = lds_v4(oc + stt[j + 2] * r16), v3 = lds_v4(oc + stt[j + 3] * r16);
+      add4(acc, v0);
+      add4(acc, v1);
+      add4(acc, v2);
+      add4(acc, v3);
+    }
+    for (; j < je; ++j) add4(acc, lds_v4(oc + stt[j] * r16));
+    const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
+    char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
+    if (col + 1 < nch || tail == 16)
+      st_v4(dp, as_i4(acc));
+    else
+      st_part(dp, as_i4(acc), tail);
+  }
+}
+
 // consumers: FOLD item with many terms per row — one output chunk at a time, its terms loaded in
 // batches of 8 independent loads, then added in list order
 template <int kBatch>
@@ -510,9 +598,14 @@ template <int kMask, int kMaxThreads = 512>
 __global__ void __launch_bounds__(kMaxThreads, 1)
     executor_tma_kernel(const __grid_constant__ ExecParams P) {
   extern __shared__ __align__(128) uint8_t dsmem[];
+  const uint32_t NS = (uint32_t)P.tma_stages;
+  const size_t stage_bytes = (size_t)P.tma_buf, meta_bytes = (size_t)P.meta_bytes;
+  const size_t kDescOff = kMetaOff + kMetaSlots * meta_bytes;
+  const size_t kStageOff = kDescOff + kDescSlots * 64;
+  const size_t kPendOff = kStageOff + NS * stage_bytes;  // 1 KB counts + 3 words
   uint64_t *full = reinterpret_cast<uint64_t *>(dsmem);
-  uint64_t *empty = full + kStages;
-  uint64_t *metab = empty + kStages;
+  uint64_t *empty = full + kMaxTmaStages;
+  uint64_t *metab = empty + kMaxTmaStages;
   uint64_t *descb = metab + kMetaSlots;
   uint8_t *metas = dsmem + kMetaOff;
   DevItem *descs = reinterpret_cast<DevItem *>(dsmem + kDescOff);
@@ -530,7 +623,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     s_pend_base = 0;
     s_bar_count = 0;
     s_bar_gen = 0;
-    for (int s = 0; s < kStages; ++s) {
+    for (int s = 0; s < (int)NS; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], n_cons_warps);
     }
@@ -564,16 +657,17 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     bool pend = false;  // signalling items issued since the last FLUSH
     int pend_key = -1;  // their counter family: ctr_index(dir, stage, 0)
     auto emit_marker = [&](uint8_t op) {  // header-only stage: FLUSH or END
-      const uint32_t stage = k % kStages, use = k / kStages;
+      uint32_t stage, use;
+      ring_pos(k, NS, stage, use);
       if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
       if (lane == 0) {
-        reinterpret_cast<DevItem *>(stages + (size_t)stage * kTmaBufBytes)->op = op;
+        reinterpret_cast<DevItem *>(stages + (size_t)stage * stage_bytes)->op = op;
         mbar_arrive(&full[stage]);
       }
       __syncwarp();
       ++k;
     };
-    auto meta_of = [&](uint32_t q) { return metas + (size_t)(q % kMetaSlots) * kMetaBytes; };
+    auto meta_of = [&](uint32_t q) { return metas + (size_t)(q % kMetaSlots) * meta_bytes; };
     if (lane == 0)
       for (uint32_t q = 0; q < (uint32_t)kDescAhead && q < nmine; ++q) request_desc(q);
     for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nmine; ++q) {
@@ -633,9 +727,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         if (!ok) break;
         if (I.wait_n > 0) fence_proxy_async_global();  // acquired peers' rows -> bulk reads
         mbar_wait(&metab[m % kMetaSlots], (m / kMetaSlots) & 1u);
-        const uint32_t stage = k % kStages, use = k / kStages;
+        uint32_t stage, use;
+        ring_pos(k, NS, stage, use);
         if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
-        issue_item(P, I, stages + (size_t)stage * kTmaBufBytes, meta_of(m), &full[stage], lane);
+        issue_item(P, I, stages + (size_t)stage * stage_bytes, meta_of(m), &full[stage], lane);
         ++k;
         if (sig) {
           pend = true;
@@ -658,9 +753,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     const uint32_t tid = threadIdx.x - 32, T = blockDim.x - 32;
     const int cw = warp - 1;
     for (uint32_t k = 0;; ++k) {
-      const uint32_t stage = k % kStages, use = k / kStages;
+      uint32_t stage, use;
+      ring_pos(k, NS, stage, use);
       mbar_wait(&full[stage], use & 1u);
-      const uint8_t *st = stages + (size_t)stage * kTmaBufBytes;
+      const uint8_t *st = stages + (size_t)stage * stage_bytes;
       const DevItem I = *reinterpret_cast<const DevItem *>(st);
       if (I.op == OP_END || I.op == OP_FLUSH) {
         // publish the rows stored since the last flush: every thread's stores (and this warp's
@@ -711,6 +807,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         }
       } else if ((kMask & kMaskDirect) && I.op == OP_COPY) {
         store_copy_direct(P, I, st, tid, T);
+      } else if ((kMask & kMaskStaged) && is_staged(I)) {
+        store_fold_staged(P, I, st, tid, T);
       } else if ((kMask & kMaskFold) && I.op == OP_FOLD) {
         // many terms per row: batch a row's terms; few: batch across output chunks
         if (I.nterms >= 4 * I.rows)
@@ -740,15 +838,16 @@ int launch_mask(const ExecParams &p, int grid, int block, cudaStream_t s) {
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kMask, kThreads>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)kSmemBytes);
+                                         (int)kSmemMax);
     if (e != cudaSuccess) return (int)e;
     attr = true;
   }
-  executor_tma_kernel<kMask, kThreads><<<grid, block, kSmemBytes, s>>>(p);
+  const TmaGeometry g = {p.tma_stages, p.tma_buf, p.meta_bytes, block, 0, 0};
+  executor_tma_kernel<kMask, kThreads><<<grid, block, tma_smem_bytes(g), s>>>(p);
   return (int)cudaGetLastError();
 }
 
-constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect;
+constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged;
 
 }  // namespace
 
@@ -757,24 +856,36 @@ int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream) 
   switch (p.op_mask) {
     case kMaskCopy: return launch_mask<kMaskCopy>(p, grid, block, s);
     case kMaskFold:
-      // fold-only launches are latency-bound gathers by the consumer warps: with the default
-      // CTA size, run 1024 threads (31 consumer warps, <= 64 registers) for twice the loads in
-      // flight per SM
-      // (only when rows carry many terms: few-term rows want the wider per-thread batching)
-      if (block == 512 && p.fold_wide) return launch_mask<kMaskFold, 1024>(p, grid, 1024, s);
+      // fold-only launches of unstaged folds are latency-bound gathers by the consumer warps:
+      // the host may run them with 1024 threads (31 consumer warps, <= 64 registers) for twice
+      // the loads in flight per SM (rows with many terms, WIDE geometry)
+      if (block == 1024) return launch_mask<kMaskFold, 1024>(p, grid, 1024, s);
       return launch_mask<kMaskFold>(p, grid, block, s);
     case kMaskCopy | kMaskFold: return launch_mask<kMaskCopy | kMaskFold>(p, grid, block, s);
+    // staged folds (backward reduce / partial-sum pushes with every operand row bulk-copied)
+    case kMaskStaged: return launch_mask<kMaskStaged>(p, grid, block, s);
+    case kMaskCopy | kMaskStaged: return launch_mask<kMaskCopy | kMaskStaged>(p, grid, block, s);
     default: return launch_mask<kAll>(p, grid, block, s);
   }
 }
 
-int tma_executor_occupancy(int block, int *ctas_per_sm) {
+// co-resident CTAs per SM of the worst-case instance at this geometry (the persistent grid must
+// be fully resident: CTAs wait on flags other CTAs set)
+int tma_executor_occupancy(int block, size_t smem_bytes, int *ctas_per_sm) {
   cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kAll>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)kSmemBytes);
+                                       (int)kSmemMax);
   if (e != cudaSuccess) return (int)e;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, executor_tma_kernel<kAll>,
-                                                    block, kSmemBytes);
+                                                    block, smem_bytes);
+  if (e != cudaSuccess || block != 1024) return (int)e;
+  int c2 = 0;
+  e = cudaFuncSetAttribute(executor_tma_kernel<kMaskFold, 1024>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemMax);
+  if (e == cudaSuccess)
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c2, executor_tma_kernel<kMaskFold, 1024>,
+                                                      1024, smem_bytes);
+  *ctas_per_sm = c2;
   return (int)e;
 }
 

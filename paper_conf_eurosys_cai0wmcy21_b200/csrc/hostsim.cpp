@@ -5,6 +5,7 @@
 // the CPU test-suite check planning + lowering against the oracle without a GPU.  It is NOT a
 // fallback: dgcl_dispatch_* never reaches it (see dgcl.h, "verification aids").
 
+#include <cmath>
 #include <cstring>
 #include <vector>
 
@@ -56,27 +57,115 @@ void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim
   }
 }
 
+// one work item the way the bulk-copy executor moves it: COPY items by their row runs, staged
+// FOLD items through an emulated shared-memory stage (segments copied in, terms read back by
+// their staged rows), other FOLD items term by term
+// returns false if the item is malformed (shape checks the device executor relies on)
+bool run_item(const Lowered &low, const DevItem &it, const std::vector<DevRun> &runs,
+              const std::vector<uint32_t> &sterms, const HostBufs &B, int dim) {
+  if (it.op != OP_COPY && it.op != OP_FOLD) return it.rows == 0;
+  if (it.rows <= 0 || it.rows > (it.op == OP_COPY ? kMaxItemRows : kMaxFoldRows)) return false;
+  auto drow = [&](int64_t r) { return it.dst >= 0 ? it.dst + r : (int64_t)low.idx[~it.dst + r]; };
+  if (it.op == OP_COPY) {
+    int64_t covered = 0;
+    for (int32_t q = 0; q < it.nterms; ++q) {
+      const DevRun &R = runs[it.tp + q];
+      if (R.pos != covered || R.len < 1) return false;
+      covered += R.len;
+      for (int32_t j = 0; j < R.len; ++j)
+        std::memcpy(row_ptr(B, it.dst_kind, it.dst_rank, R.dst + j),
+                    row_ptr(B, it.src_kind, it.exec_rank, R.src + j), sizeof(float) * dim);
+    }
+    return covered == it.rows;
+  }
+  const int64_t *tp = low.term_ptr.data() + it.tp;
+  if (it.flags & kItemStaged) {
+    const int64_t nseg = it.src >> kSegShift, seg0 = it.src & ((1ll << kSegShift) - 1);
+    const int64_t nst = (it.fold_init ? it.rows : 0) + it.nterms;
+    if (nst > kMaxItemRows || nseg < 1 || nseg > nst) return false;
+    std::vector<float> stage((size_t)nst * B.pitch, std::nanf(""));
+    std::vector<uint8_t> hit(nst, 0);
+    for (int64_t q = 0; q < nseg; ++q) {
+      const DevRun &R = runs[seg0 + q];
+      if (R.pos < 0 || R.len < 1 || R.pos + R.len > nst) return false;
+      for (int32_t j = 0; j < R.len; ++j) {
+        if (hit[R.pos + j]) return false;
+        hit[R.pos + j] = 1;
+      }
+      for (int32_t j = 0; j < R.len; ++j)
+        std::memcpy(&stage[(size_t)(R.pos + j) * B.pitch],
+                    row_ptr(B, R.dst >> 8, R.dst & 255, R.src + j), sizeof(float) * dim);
+    }
+    for (int64_t r = 0; r < it.rows; ++r) {
+      float *d = row_ptr(B, it.dst_kind, it.dst_rank, drow(r));
+      for (int c = 0; c < dim; ++c) {
+        int64_t j = tp[r] - tp[0];
+        const int64_t je = tp[r + 1] - tp[0];
+        float acc = it.fold_init ? stage[(size_t)r * B.pitch + c]
+                                 : stage[(size_t)sterms[it.t0 + j++] * B.pitch + c];
+        for (; j < je; ++j) {
+          volatile float v = stage[(size_t)sterms[it.t0 + j] * B.pitch + c];
+          acc = acc + v;
+        }
+        d[c] = acc;
+      }
+    }
+    for (uint8_t h : hit)
+      if (!h) return false;  // every staged row is filled by exactly one segment
+    return true;
+  }
+  DevGroup g = low.groups[it.group];
+  g.n_rows = it.rows;
+  g.term_ptr = it.tp;
+  g.dst_idx = it.dst < 0 ? ~it.dst : -1;
+  g.dst_base = it.dst;
+  run_group(low, g, B, dim);
+  return true;
+}
+
+void setup_bufs(const Lowered &low, const std::vector<int64_t> &row_off,
+                const std::vector<int64_t> &halo_off, int64_t pitch, const float *emb, float *halo,
+                const float *halo_grad, float *emb_grad, std::vector<std::vector<float>> &relay,
+                std::vector<std::vector<float>> &slot, HostBufs *B) {
+  const int m = low.m;
+  relay.assign(m, {});
+  slot.assign(m, {});
+  std::memset(B, 0, sizeof(*B));
+  B->pitch = pitch;
+  for (int r = 0; r < m; ++r) {
+    relay[r].assign((size_t)low.n_relay[r] * pitch, 0.f);
+    slot[r].assign((size_t)low.n_slot[r] * pitch, 0.f);
+    B->base[K_EMB][r] = const_cast<float *>(emb) + (emb ? row_off[r] * pitch : 0);
+    B->base[K_EGRAD][r] = emb_grad + (emb_grad ? row_off[r] * pitch : 0);
+    B->base[K_HALO][r] = halo + (halo ? halo_off[r] * pitch : 0);
+    B->base[K_HGRAD][r] = const_cast<float *>(halo_grad) + (halo_grad ? halo_off[r] * pitch : 0);
+    B->base[K_RELAY][r] = relay[r].data();
+    B->base[K_SLOT][r] = slot[r].data();
+  }
+}
+
 }  // namespace
+
+bool hostsim_run_items(const Lowered &low, const std::vector<DevItem> &items,
+                       const std::vector<DevRun> &runs, const std::vector<uint32_t> &sterms,
+                       const std::vector<int64_t> &row_off, const std::vector<int64_t> &halo_off,
+                       int64_t pitch, int dim, const float *emb, float *halo,
+                       const float *halo_grad, float *emb_grad) {
+  std::vector<std::vector<float>> relay, slot;
+  HostBufs B;
+  setup_bufs(low, row_off, halo_off, pitch, emb, halo, halo_grad, emb_grad, relay, slot, &B);
+  for (const DevItem &it : items)  // stage order
+    if (!run_item(low, it, runs, sterms, B, dim)) return false;
+  return true;
+}
 
 void hostsim_run(const Lowered &low, const std::vector<int32_t> &gids,
                  const std::vector<int64_t> &row_off, const std::vector<int64_t> &halo_off,
                  int64_t pitch, int dim, const float *emb, float *halo, const float *halo_grad,
                  float *emb_grad) {
-  const int m = low.m;
-  std::vector<std::vector<float>> relay(m), slot(m);
+  std::vector<std::vector<float>> relay, slot;
   HostBufs B;
-  std::memset(&B, 0, sizeof(B));
-  B.pitch = pitch;
-  for (int r = 0; r < m; ++r) {
-    relay[r].assign((size_t)low.n_relay[r] * pitch, 0.f);
-    slot[r].assign((size_t)low.n_slot[r] * pitch, 0.f);
-    B.base[K_EMB][r] = const_cast<float *>(emb) + (emb ? row_off[r] * pitch : 0);
-    B.base[K_EGRAD][r] = emb_grad + (emb_grad ? row_off[r] * pitch : 0);
-    B.base[K_HALO][r] = halo + (halo ? halo_off[r] * pitch : 0);
-    B.base[K_HGRAD][r] = const_cast<float *>(halo_grad) + (halo_grad ? halo_off[r] * pitch : 0);
-    B.base[K_RELAY][r] = relay[r].data();
-    B.base[K_SLOT][r] = slot[r].data();
-  }
+  setup_bufs(low, row_off, halo_off, pitch, emb, halo, halo_grad, emb_grad, relay, slot, &B);
   for (int32_t gi : gids) {  // the program's groups, in stage order
     const DevGroup &g = low.groups[gi];
     if (g.op == OP_READY || g.op == OP_WAIT) continue;

@@ -8,6 +8,7 @@
 // "ready" word, so no flag is ever reset and no host round-trip happens between stages.
 #pragma once
 
+#include <cstddef>
 #include <cstdint>
 
 namespace dgcl {
@@ -101,6 +102,11 @@ static_assert(sizeof(DevItem) == 64, "DevItem is one 64-B descriptor");
 constexpr uint8_t kItemSignal = 1;
 constexpr uint8_t kItemDirect = 2;  // COPY: consumers gather rows themselves (short row runs)
 constexpr uint8_t kItemGather4 = 4; // COPY from embeddings with short runs: TMA gather4 of rows
+// FOLD whose operand rows are all bulk-copied into the stage (bulk-copy executor only; the
+// register executor ignores the flag): src = (segments << 40) | first segment in the run pool,
+// t0 = first staged term (shared-memory row of each term, per-program pool `sterms`)
+constexpr uint8_t kItemStaged = 8;
+constexpr int kSegShift = 40;
 constexpr int kGather4MaxRowBytes = 1024;  // one tensor box (<= 256 fp32) per row
 
 struct DevWait {
@@ -142,38 +148,57 @@ struct alignas(64) ExecParams {
   int *err;            // host-mapped error word (0 = ok)
   int32_t use_tma;     // 1: bulk-copy (TMA) gather into shared memory, then store from smem
   int32_t row16;       // row bytes rounded up to 16 (bulk-copy size per row)
-  int32_t tma_buf;     // bytes per shared-memory stage buffer
+  int32_t tma_buf;     // bytes per shared-memory stage buffer (launch geometry, TmaGeometry)
+  int32_t tma_stages;  // stage buffers per CTA (<= kMaxTmaStages)
+  int32_t meta_bytes;  // bytes per producer metadata slot
   int32_t bulk_store;  // 1: contiguous COPY destinations are written with bulk (TMA) stores
   const struct DevRun *runs;  // COPY items: maximal runs of consecutive (source, destination) rows
-  int32_t op_mask;     // kinds of data items in this launch (kMaskCopy | kMaskFold | kMaskDirect):
+  int32_t op_mask;     // kinds of data items in this launch (kMaskCopy | kMaskFold | kMaskDirect |
+                       // kMaskStaged):
                        // selects a kernel instance that carries only the code it needs
   int32_t fold_wide;   // FOLD rows average >= 4 terms (selects the 1024-thread fold instance)
+  const uint32_t *sterms;  // staged FOLD items: operand row (in the stage) of every term
 };
-constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4;
+constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8;
 
 // A run of `len` rows whose source rows src.. and destination rows dst.. are both consecutive;
 // `pos` is the first row's index inside its item.  One bulk copy moves a run when the pitches
-// equal the 16-B-rounded row.
+// equal the 16-B-rounded row.  For a staged FOLD item the run is a SEGMENT: `len` consecutive
+// rows src.. of buffer (kind = dst >> 8, rank = dst & 255) copied to operand rows pos.. .
 struct DevRun {
   int32_t src, dst, len, pos;
 };
 
-// Bulk-copy executor (executor_tma.cu) shared-memory geometry and the item limits it implies:
-//   stage  = [0,64) item header | [64,128) info | [128,2176) term_ptr window (FOLD) |
-//            [2176,4096) destination-row window | [4096, 48K) gathered operand rows
-//   meta   = producer-private: [0,2K) source-row / term_ptr window | [2K,4K) destination rows |
-//            [4K,12K) terms window
-// 3 x 64 KB measured best on the Reddit-shaped loopback (vs 4 x 48 KB and 2 x 96 KB; the
-// producer's per-item cost favours large items, the store/load overlap favours >= 3 stages)
-#ifndef DGCL_TMA_STAGES
-#define DGCL_TMA_STAGES 3
-#define DGCL_TMA_STAGE_KB 64
-#endif
-constexpr int kTmaStages = DGCL_TMA_STAGES;
-constexpr int kTmaBufBytes = DGCL_TMA_STAGE_KB * 1024;  // per stage (3 x 64 KB = 192 KB)
+// Bulk-copy executor (executor_tma.cu) shared-memory geometry and the item limits it implies.
+// Dynamic shared memory of a CTA:
+//   [0,256) mbarriers | meta slots (4 x meta_bytes, producer-private row runs / segments) |
+//   descriptor ring (8 x 64 B) | stages (stages x stage_bytes) | 1152 B done counts + barrier
+// and one stage = [0,64) item header | [64,128) info | [128,2176) term_ptr window (FOLD) |
+//   [2176,4096) destination-row window | [4096, stage_bytes) operand rows + staged terms.
+// Two geometries, chosen per launch (per program) by the host:
+//   WIDE: 1 CTA per SM, 3 x 64 KB stages — large items; best for long row runs of big rows
+//         (write-dominated forward of Reddit-shaped rows: 0.94 vs 0.75 of HBM peak)
+//   DUAL: 2 CTAs per SM, 2 x 47 KB stages — two producer warps per SM; best when the producer's
+//         per-item work dominates (short runs, staged folds: backward 0.70 -> 0.95-1.0 of peak)
+// (measured on the Reddit / Web-Google / Com-Orkut loopbacks)
+struct TmaGeometry {
+  int32_t stages, stage_bytes, meta_bytes, threads, ctas_per_sm, max_item_rows;
+};
+constexpr TmaGeometry kGeoWide = {3, 64 * 1024, 8 * 1024, 256, 1, 464};
+constexpr TmaGeometry kGeoDual = {2, 47 * 1024, 4 * 1024, 256, 2, 240};
+constexpr int kMaxTmaStages = 3;
 constexpr int kStageHdrBytes = 4096;
+constexpr int kTmaBufBytes = kGeoWide.stage_bytes;          // largest stage
 constexpr int kTmaOperandBytes = kTmaBufBytes - kStageHdrBytes;
-constexpr int kMaxItemRows = 464;        // (1920 B dst window) / 4 B - alignment slack
+constexpr size_t tma_smem_bytes(const TmaGeometry &g) {
+  return 256 + 4 * (size_t)g.meta_bytes + 8 * 64 + (size_t)g.stages * g.stage_bytes + 1152;
+}
+static_assert(tma_smem_bytes(kGeoWide) <= 227 * 1024, "WIDE: one CTA per SM");
+static_assert(tma_smem_bytes(kGeoDual) <= 113 * 1024, "DUAL: two CTAs per SM");
+static_assert(kGeoWide.max_item_rows * 16 <= kGeoWide.meta_bytes &&
+                  kGeoDual.max_item_rows * 16 <= kGeoDual.meta_bytes,
+              "a meta slot holds an item's 16-B runs");
+constexpr int kMaxItemRows = 464;        // <= (1920 B dst window) / 4 B - slack
 constexpr int kMaxFoldRows = 240;        // (2048 B term_ptr window) / 8 B - slack
 constexpr int kMaxItemTerms = 2040;      // (8 KB terms window) / 4 B - slack
 
@@ -197,6 +222,7 @@ inline uint32_t fastdiv_host(uint32_t x, FastDiv f) {
 
 // launch wrapper implemented in executor.cu; returns a cudaError_t value
 int launch_executor(const ExecParams &p, int grid, int block, void *stream);
-int executor_occupancy(int block, int *ctas_per_sm, int *tma_ctas_per_sm);
+int executor_occupancy(int block, int *ctas_per_sm);                          // register path
+int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm);  // bulk-copy path
 
 }  // namespace dgcl

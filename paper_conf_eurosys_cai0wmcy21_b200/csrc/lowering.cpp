@@ -385,18 +385,103 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   L.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
 }
 
+namespace {
+
+// Staged FOLD item (bulk-copy executor): operand rows [0, rows) of the stage are the
+// destination rows the fold starts from (fold_init), then every term's source row, sorted by
+// (buffer kind, rank, row) so that consecutive rows form one segment = one bulk copy.  With the
+// harness's halo order (owner, id) an owner's requesters' rows are consecutive, so a loopback
+// reduce item needs one segment per requesting rank.  The terms keep their order; sterms only
+// says where each one's row sits in the stage.
+constexpr int64_t kMinSegmentRows = 4;  // staged FOLD groups: average operand rows per segment
+
+void stage_fold_item(const Lowered &low, const DevGroup &g, DevItem *it, std::vector<DevRun> *runs,
+                     std::vector<uint32_t> *sterms) {
+  struct Ref {
+    int32_t key;  // (kind << 8) | rank
+    int32_t row;
+    int64_t t;    // term index (or -1 - r for the destination row r)
+  };
+  std::vector<Ref> refs;
+  auto drow = [&](int64_t r) {
+    return g.dst_idx >= 0 ? (int64_t)low.idx[g.dst_idx + r] : g.dst_base + r;
+  };
+  const int64_t rb = it->tp - g.term_ptr;
+  const int64_t seg0 = (int64_t)runs->size();
+  if (g.fold_init) {
+    for (int64_t r = 0; r < it->rows;) {  // destination rows: operand rows 0 .. rows-1
+      int64_t e = r + 1;
+      while (e < it->rows && drow(rb + e) == drow(rb + e - 1) + 1) ++e;
+      runs->push_back({(int32_t)drow(rb + r), (g.dst_kind << 8) | g.dst_rank, (int32_t)(e - r),
+                       (int32_t)r});
+      r = e;
+    }
+  }
+  for (int64_t t = it->t0; t < it->t0 + it->nterms; ++t) {
+    const uint32_t x = low.terms[t];
+    Ref f;
+    if (g.term_mode == kTermRankHgrad) {
+      f.key = (K_HGRAD << 8) | (int32_t)(x >> 28);
+      f.row = (int32_t)(x & kTermRowMask);
+    } else if (x & kTermSlot) {
+      f.key = (K_SLOT << 8) | g.exec_rank;
+      f.row = (int32_t)(x & ~kTermSlot);
+    } else {
+      f.key = (K_HGRAD << 8) | g.exec_rank;
+      f.row = (int32_t)x;
+    }
+    f.t = t;
+    refs.push_back(f);
+  }
+  std::sort(refs.begin(), refs.end(), [](const Ref &a, const Ref &b) {
+    return a.key != b.key ? a.key < b.key : a.row < b.row;
+  });
+  const int64_t base = g.fold_init ? it->rows : 0;
+  const int64_t st0 = (int64_t)sterms->size();
+  sterms->resize(st0 + it->nterms);
+  for (size_t a = 0; a < refs.size();) {
+    size_t e = a + 1;
+    while (e < refs.size() && refs[e].key == refs[a].key && refs[e].row == refs[e - 1].row + 1) ++e;
+    runs->push_back({refs[a].row, refs[a].key, (int32_t)(e - a), (int32_t)(base + (int64_t)a)});
+    a = e;
+  }
+  for (size_t a = 0; a < refs.size(); ++a)
+    (*sterms)[st0 + (refs[a].t - it->t0)] = (uint32_t)(base + (int64_t)a);
+  it->flags |= kItemStaged;
+  it->src = ((int64_t)((int64_t)runs->size() - seg0) << kSegShift) | seg0;
+  it->t0 = st0;
+}
+
+}  // namespace
+
+ItemLimits item_limits(const TmaGeometry &g, int64_t item_bytes) {
+  ItemLimits l;
+  l.operand_bytes = std::min<int64_t>(item_bytes, g.stage_bytes - kStageHdrBytes);
+  l.max_rows = std::min<int64_t>(kMaxItemRows, g.max_item_rows);
+  return l;
+}
+
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
-                 int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
+                 const ItemLimits &lim, bool signal_all, const std::vector<uint8_t> &needed_ctr,
                  std::vector<DevItem> *items, std::vector<DevRun> *runs,
-                 int64_t direct_copy_rows) {
+                 int64_t direct_copy_rows, std::vector<uint32_t> *sterms) {
   runs->clear();
+  if (sterms) sterms->clear();
   // An item is a row range whose gathered operands fit `item_bytes` (and one shared-memory stage
   // of the bulk-copy executor): a COPY row costs one row, a FOLD row (1 + #terms) rows.
   items->clear();
   const int64_t row16 = (row_bytes + 15) / 16 * 16;
-  const int64_t cap = std::max<int64_t>(row16, std::min<int64_t>(item_bytes, kTmaOperandBytes));
+  const int64_t cap = std::max<int64_t>(row16, lim.operand_bytes);
   size_t i = 0;
   std::vector<std::vector<int32_t>> bounds;  // per group of the stage: chunk start rows + end
+  std::vector<uint8_t> staged;               // per group of the stage: FOLD items are staged
+  // staged FOLD item: operand rows (destination rows of the fold start + one per term) and the
+  // staged-term window share one stage; segments (<= one per operand row) fill one meta slot
+  const int64_t stage_rows_cap = std::min<int64_t>(lim.max_rows, lim.operand_bytes / row16);
+  auto staged_fits = [&](int64_t srows, int64_t nt) {
+    return srows <= stage_rows_cap &&
+           srows * row16 + (nt * 4 + 15) / 16 * 16 + 16 <= lim.operand_bytes;
+  };
   while (i < gids.size()) {
     // one stage (READY / WAIT are their own runs)
     const DevGroup &g0 = low.groups[gids[i]];
@@ -407,18 +492,66 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       ++j;
     if (j == i) j = i + 1;
     bounds.assign(j - i, std::vector<int32_t>());
+    staged.assign(j - i, 0);
     size_t max_chunks = 0;
     for (size_t q = i; q < j; ++q) {
       const DevGroup &g = low.groups[gids[q]];
       std::vector<int32_t> &b = bounds[q - i];
       b.push_back(0);
+      if (g.op == OP_FOLD && sterms) {
+        // staged: every row must fit a stage on its own
+        bool ok = true;
+        for (int64_t r = 0; r < g.n_rows && ok; ++r) {
+          const int64_t nt = low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r];
+          ok = staged_fits(nt + (g.fold_init ? 1 : 0), nt);
+        }
+        staged[q - i] = ok ? 1 : 0;
+      }
       if (g.op == OP_COPY) {
         // rows per item; a multiple of 4 when gather4 may apply (its groups are padded to 4 rows)
-        int64_t rpi = std::min<int64_t>(kMaxItemRows, std::max<int64_t>(1, cap / row16));
+        int64_t rpi = std::min<int64_t>(lim.max_rows, std::max<int64_t>(1, cap / row16));
         if (row16 <= kGather4MaxRowBytes && rpi >= 4) rpi = rpi / 4 * 4;
         for (int64_t r = rpi; r < g.n_rows; r += rpi) b.push_back((int32_t)r);
         b.push_back((int32_t)g.n_rows);
-      } else if (g.op == OP_FOLD) {
+      } else if (g.op == OP_FOLD && staged[q - i]) {
+        int64_t srows = 0, nt = 0;
+        for (int64_t r = 0; r < g.n_rows; ++r) {
+          const int64_t c = low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r];
+          const int64_t add = c + (g.fold_init ? 1 : 0);
+          if (r > b.back() && (!staged_fits(srows + add, nt + c) || r - b.back() >= kMaxFoldRows ||
+                               nt + c > kMaxItemTerms)) {
+            b.push_back((int32_t)r);
+            srows = nt = 0;
+          }
+          srows += add;
+          nt += c;
+        }
+        b.push_back((int32_t)g.n_rows);
+        // staging pays when segments are long (one bulk copy each); operand rows scattered in
+        // short runs (e.g. relay slots) are better gathered by the consumers' plain loads
+        int64_t nseg = 0, nst = 0;
+        std::vector<DevRun> trial_runs;
+        std::vector<uint32_t> trial_st;
+        for (size_t c = 0; c + 1 < b.size(); ++c) {
+          DevItem t;
+          std::memset(&t, 0, sizeof(t));
+          t.rows = b[c + 1] - b[c];
+          t.tp = g.term_ptr + b[c];
+          t.t0 = low.term_ptr[t.tp];
+          t.nterms = (int32_t)(low.term_ptr[t.tp + t.rows] - t.t0);
+          t.dst = g.dst_idx >= 0 ? ~(g.dst_idx + b[c]) : g.dst_base + b[c];
+          trial_runs.clear();
+          trial_st.clear();
+          stage_fold_item(low, g, &t, &trial_runs, &trial_st);
+          nseg += (int64_t)trial_runs.size();
+          nst += t.nterms + (g.fold_init ? t.rows : 0);
+        }
+        if (nst < kMinSegmentRows * nseg) {
+          staged[q - i] = 0;
+          b.assign(1, 0);
+        }
+      }
+      if (g.op == OP_FOLD && !staged[q - i]) {
         int64_t acc = 0;
         for (int64_t r = 0; r < g.n_rows; ++r) {
           const int64_t slots = low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r] +
@@ -435,7 +568,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
           acc += cost;
         }
         b.push_back((int32_t)g.n_rows);
-      } else {
+      } else if (g.op != OP_FOLD && g.op != OP_COPY) {
         b.push_back(0);  // READY / WAIT: one empty item
       }
       max_chunks = std::max(max_chunks, b.size() - 1);
@@ -470,6 +603,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
           it.tp = g.term_ptr + rb;
           it.t0 = low.term_ptr[it.tp];
           it.nterms = (int32_t)(low.term_ptr[it.tp + it.rows] - it.t0);
+          if (staged[q - i]) stage_fold_item(low, g, &it, runs, sterms);
         } else if (g.op == OP_COPY) {
           // maximal runs of consecutive source and destination rows (one bulk copy each)
           it.tp = (int64_t)runs->size();
@@ -491,7 +625,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         bool sig = data && g.sig_ctr >= 0;
         if (sig && !signal_all)
           sig = needed_ctr[(size_t)g.dst_rank * kFlagWords + g.sig_ctr] != 0;
-        it.flags = sig ? kItemSignal : 0;
+        it.flags |= sig ? kItemSignal : 0;
         // optional: items whose runs average fewer than `direct_copy_rows` rows are gathered by
         // the consumers with plain loads instead of one bulk copy per run (0 = never; measured
         // slower than per-row bulk copies on the BASELINE graphs)

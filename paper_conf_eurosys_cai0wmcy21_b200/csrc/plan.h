@@ -85,10 +85,20 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
 // included by the caller) cut into row ranges of about item_bytes gathered bytes and interleaved
 // across the groups of a stage.  COPY items also get their row runs appended to `runs`
 // (item.tp = first run, program-relative); items of short runs are flagged for gather4 (or for
-// consumer gathers when direct_copy_rows > 0).
+// consumer gathers when direct_copy_rows > 0).  With `sterms`, FOLD groups whose rows fit are
+// cut into STAGED items: every operand row (the destination rows a fold starts from, then each
+// term's source row) is bulk-copied into the stage as segments of consecutive rows (appended to
+// `runs`), and `sterms` receives each term's operand row (item.t0 = first, program-relative).
+// The item limits follow the launch geometry (internal.h, TmaGeometry): operand bytes of one
+// stage and rows per item (one meta slot of runs).
+struct ItemLimits {
+  int64_t operand_bytes;  // gathered bytes of one item (<= stage_bytes - kStageHdrBytes)
+  int64_t max_rows;       // rows (COPY) / operand rows (staged FOLD) of one item
+};
+ItemLimits item_limits(const TmaGeometry &g, int64_t item_bytes);
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
-                 int64_t item_bytes, bool signal_all, const std::vector<uint8_t> &needed_ctr,
+                 const ItemLimits &lim, bool signal_all, const std::vector<uint8_t> &needed_ctr,
                  std::vector<DevItem> *items, std::vector<DevRun> *runs,
-                 int64_t direct_copy_rows = 0);
+                 int64_t direct_copy_rows = 0, std::vector<uint32_t> *sterms = nullptr);
 
 }  // namespace dgcl

@@ -142,6 +142,33 @@ def test_uniform_plan_and_lowering(m, direct):
     assert info["n_stages"] == 1 and info["n_relay_rows"] == 0
 
 
+@pytest.mark.parametrize("m,opts", [(2, {}), (8, {}), (8, {"stage_fold": 0}),
+                                    (4, {"direct_reduce": 0}),
+                                    (8, {"direct_reduce": 0, "item_bytes": 2048}),
+                                    (3, {"gather4": 0, "stage_fold": 0}),
+                                    (8, {"geometry": 1}), (8, {"geometry": 2}),
+                                    (4, {"geometry": 2, "direct_reduce": 0})])
+def test_work_items_host(m, opts):
+    """The fused program's WORK ITEMS (not the groups) moved the way the bulk-copy executor moves
+    them — COPY row runs, staged FOLD segments read back through the staged-term table — on the
+    host, against the oracle: checks build_items (item cuts, runs, segments, staged rows)."""
+    g = synth.make_graph(1500, 14000, m, graph_seed=20 + m, part_seed=60 + m)
+    _check_lowering(g, [16, 5, 602], None, seed=3, options=dict(opts, hostsim_items=1))
+
+
+@pytest.mark.parametrize("name,sf", [("dgx1_like", 1), ("ring", 1), ("ring", 0)])
+def test_work_items_host_relay(name, sf):
+    g = synth.make_graph(500, 2500, 8, graph_seed=9, part_seed=19)
+    _check_lowering(g, [12, 3], synth.topology.by_name(name), seed=5,
+                    options={"hostsim_items": 1, "stage_fold": sf})
+
+
+def test_work_items_host_shuffled():
+    g = synth.make_graph(800, 6000, 4, graph_seed=2, part_seed=3)
+    g.req_ids = synth.graph.shuffle_lists(g.req_ptr, g.req_ids, 77)
+    _check_lowering(g, [8, 64], None, seed=1, options={"hostsim_items": 1})
+
+
 @pytest.mark.parametrize("name", ["dgx1_like", "ring"])
 def test_relay_plan_and_lowering(name):
     g = synth.make_graph(500, 2500, 8, graph_seed=9, part_seed=19)

@@ -150,12 +150,17 @@ def test_tiny_config_bit_exact():
     (4, {"direct_reduce": 0, "bulk_store": 0}),
     (8, {"gather4": 0}),
     (4, {"direct_copy_rows": 4}),
+    (8, {"stage_fold": 0}), (4, {"stage_fold": 0, "direct_reduce": 0}),
+    (8, {"direct_reduce": 0, "item_bytes": 4096}),
+    (8, {"geometry": 1}), (8, {"geometry": 2}), (4, {"geometry": 2, "direct_reduce": 0}),
+    (3, {"geometry": 1, "stage_fold": 0}),
 ])
 def test_uniform_loopback_fused(m, opts):
     """Executor variants: tma (bulk-copy executor vs the register LDG executor), direct_reduce
     (loopback in-place reduce vs push to slots + owner reduce, the multi-GPU form), bulk_store
     (TMA stores vs 16-B st.global), gather4 (TMA row gather of 4 rows per instruction vs one bulk
-    copy per run), direct_copy_rows (consumer-side gathers for short runs)."""
+    copy per run), direct_copy_rows (consumer-side gathers for short runs), stage_fold (backward
+    folds with every operand row bulk-copied into shared memory vs consumer gathers)."""
     g = synth.make_graph(6000, 60000, m, graph_seed=m, part_seed=7 * m)
     _check_case(Case(g, [64, 5, 602, 32], options=opts))
 
@@ -171,13 +176,18 @@ def test_per_rank_flag_protocol(m):
         _check_case(c)
 
 
-@pytest.mark.parametrize("name,flags,tma", [("dgx1_like", 0, 1), ("ring", 0, 1),
-                                            ("dgx1_like", 1, 1), ("ring", 1, 1),
-                                            ("ring", 0, 0), ("dgx1_like", 1, 0)])
-def test_relay_plans(name, flags, tma):
+@pytest.mark.parametrize("name,flags,tma,sf", [("dgx1_like", 0, 1, 1), ("ring", 0, 1, 1),
+                                               ("dgx1_like", 1, 1, 1), ("ring", 1, 1, 1),
+                                               ("ring", 0, 0, 1), ("dgx1_like", 1, 0, 1),
+                                               ("ring", 1, 1, 0), ("dgx1_like", 0, 1, 0),
+                                               ("ring", 0, 1, 2), ("dgx1_like", 1, 1, 3)])
+def test_relay_plans(name, flags, tma, sf):
+    """sf: stage_fold 0/1; 2, 3 = stage_fold with the DUAL / WIDE geometry forced."""
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
-    c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags,
-             options={"tma": tma})
+    opts = {"tma": tma, "stage_fold": min(sf, 1)}
+    if sf >= 2:
+        opts["geometry"] = 2 if sf == 2 else 1
+    c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags, options=opts)
     assert c.ctx.plan_info()["n_stages"] >= 2
     _check_case(c)
 
