@@ -92,6 +92,7 @@ struct dgcl_ctx {
   bool hostsim_items = false;         // debug host interpreter: run the work items, not groups
   int geometry = 0;                   // bulk-copy geometry: 0 auto per program, 1 WIDE, 2 DUAL
   bool threads_set = false, ctas_set = false;  // user overrides of the CTA shape
+  int sm_count = 148;  // SMs of the device (B200 until queried), for cutting small stages
   int tma_ctas_geo[2][2] = {{0, 0}, {0, 0}};   // [geo][1024-thread fold instance] CTAs per SM
   int n_prog_ranks = 1;        // programs per (layer, dir)
 
@@ -177,6 +178,8 @@ dgcl_status init_common(int32_t rank, int32_t world, int32_t dev, int64_t n, con
   c->topo = Topology::uniform_nvswitch(world);
   if (dev >= 0) {
     cudaError_t e = cudaSetDevice(dev);
+    if (e == cudaSuccess)
+      e = cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, dev);
     if (e != cudaSuccess) {
       delete c;
       return DGCL_ECUDA;
@@ -302,7 +305,9 @@ void build_programs(dgcl_ctx *c) {
         auto build = [&](int geo) {
           P.geo = geo;
           build_items(L, gids[r], row_bytes,
-                      item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes), !fused, need,
+                      item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
+                                  (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm),
+                      !fused, need,
                       &P.items, &P.runs, c->direct_copy_rows,
                       c->stage_fold ? &P.sterms : nullptr);
           P.op_mask = 0;

@@ -169,6 +169,11 @@ template <bool V16>
 __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant__ ExecParams P) {
   __shared__ int s_abort;
   __shared__ DevItem s_item;
+  // per executing rank: the wait list last found satisfied (monotonic counters, fixed targets)
+  __shared__ int32_t s_wait_ok[kMaxRanks];
+  __shared__ uint32_t s_ready_ok;
+  if (threadIdx.x < kMaxRanks) s_wait_ok[threadIdx.x] = -1;
+  if (threadIdx.x == 0) s_ready_ok = 0;
   for (int it = blockIdx.x; it < P.n_items; it += gridDim.x) {
     if (threadIdx.x < 4)
       reinterpret_cast<int4 *>(&s_item)[threadIdx.x] =
@@ -182,10 +187,15 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
         for (int s = 0; s < P.world; ++s)
           if (s != I.exec_rank) st_release_sys(P.flags[s] + kReadyBase + I.exec_rank, P.seq);
       }
-      if (P.use_ready && I.ready_rank >= 0)
+      if (P.use_ready && I.ready_rank >= 0 && !((s_ready_ok >> I.ready_rank) & 1u)) {
         ok = wait_geq(P.flags[I.exec_rank] + kReadyBase + I.ready_rank, P.seq, P,
                       1000 + I.group);
-      if (ok) ok = wait_item_sources(P, I, 100000 + I.group);
+        if (ok) s_ready_ok |= 1u << I.ready_rank;
+      }
+      if (ok && I.wait_n > 0 && s_wait_ok[I.exec_rank] != I.wait_off) {
+        ok = wait_item_sources(P, I, 100000 + I.group);
+        if (ok) s_wait_ok[I.exec_rank] = I.wait_off;
+      }
       s_abort = ok ? 0 : 1;
     }
     __syncthreads();

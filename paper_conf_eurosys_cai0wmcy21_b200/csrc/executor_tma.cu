@@ -186,13 +186,13 @@ __device__ __forceinline__ uint32_t n_segments(const DevItem &I) {
   return (uint32_t)(I.src >> kSegShift);
 }
 
-// producer lane 0: bulk-copy the metadata the producer needs to issue item I's gathers
+// producer lane 0: bulk-copy the metadata the producer needs to issue item I's gathers (the
+// caller has fenced generic accesses to the slot against the async proxy)
 __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I, uint8_t *meta,
                                            uint64_t *bar) {
   // COPY (bulk path): the item's row runs, or its source rows for a gather4 item.  FOLD and
   // direct COPY items need nothing here (the consumers gather their operands); the barrier phase
   // then completes on the arrive alone.
-  fence_proxy_async_smem();
   if (uses_gather4(P, I)) {
     const Win ws = window(~I.src, I.rows, 4);
     mbar_expect_tx(bar, ws.bytes);
@@ -223,15 +223,18 @@ __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const Dev
   return window(I.t0, I.nterms, 4).bytes;
 }
 
-// producer warp: header, consumer tables and row gathers of data item I into `st`
-__device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I, uint8_t *st,
-                                           const uint8_t *meta, uint64_t *full, int lane) {
+// producer warp: header, consumer tables and row gathers of data item I (in registers; Ism = its
+// descriptor in shared memory, copied as the stage header) into `st`.  The caller waited for the
+// stage to be free and fenced the consumers' generic reads of it against the async proxy.
+__device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I,
+                                           const DevItem *Ism, uint8_t *st, const uint8_t *meta,
+                                           uint64_t *full, int lane) {
   const uint32_t r16 = (uint32_t)P.row16;
   // consumer tables: term_ptr window (FOLD) and destination rows (when not consecutive)
   Win wtp = {0, 0, 0}, wdst = {0, 0, 0};
   if (I.op == OP_FOLD) wtp = window(I.tp, I.rows + 1, 8);
   if (I.dst < 0) wdst = window(~I.dst, I.rows, 4);
-  if (lane < 4) reinterpret_cast<int4 *>(st)[lane] = reinterpret_cast<const int4 *>(&I)[lane];
+  if (lane < 4) reinterpret_cast<int4 *>(st)[lane] = reinterpret_cast<const int4 *>(Ism)[lane];
   if (lane == 4) {
     int32_t *info = reinterpret_cast<int32_t *>(st + kHdrInfo);
     info[0] = wtp.skew;
@@ -240,7 +243,6 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
   __syncwarp();  // header and info written before lane 0's arrive publishes the stage
   if (lane == 0) mbar_expect_tx(full, operand_bytes(P, I) + wtp.bytes + wdst.bytes);
   __syncwarp();
-  fence_proxy_async_smem();
   if (lane == 0) {
     if (wtp.bytes) bulk_g2s(st + kTabTp, P.term_ptr + wtp.a, wtp.bytes, full);
     if (wdst.bytes) bulk_g2s(st + kTabDst, P.idx + wdst.a, wdst.bytes, full);
@@ -616,6 +618,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   int &s_pend_base = *reinterpret_cast<int *>(dsmem + kPendOff + 1024);
   unsigned &s_bar_count = *reinterpret_cast<unsigned *>(dsmem + kPendOff + 1028);
   volatile unsigned &s_bar_gen = *reinterpret_cast<volatile unsigned *>(dsmem + kPendOff + 1032);
+  // producer-private: per executing rank, the wait list last found satisfied (counters are
+  // monotonic and their targets fixed for the launch, so it stays satisfied: later items of the
+  // same (direction, stage, rank) skip the flag reads)
+  int32_t *s_wait_ok = reinterpret_cast<int32_t *>(dsmem + kPendOff + 1040);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
   for (int i = threadIdx.x; i < kMaxRanks * kMaxRanks; i += blockDim.x) s_pend[i] = 0;
@@ -623,6 +629,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     s_pend_base = 0;
     s_bar_count = 0;
     s_bar_gen = 0;
+    for (int r = 0; r < kMaxRanks; ++r) s_wait_ok[r] = -1;
     for (int s = 0; s < (int)NS; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], n_cons_warps);
@@ -641,9 +648,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     const uint32_t G = gridDim.x;
     const uint32_t nmine =
         blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
-    auto request_desc = [&](uint32_t q) {  // lane 0
+    auto request_desc = [&](uint32_t q) {  // lane 0, after a proxy fence
       const uint32_t s = q % kDescSlots;
-      fence_proxy_async_smem();
       mbar_expect_tx(&descb[s], (uint32_t)sizeof(DevItem));
       bulk_g2s(descs + s, P.items + blockIdx.x + q * G, (uint32_t)sizeof(DevItem), &descb[s]);
     };
@@ -654,6 +660,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     uint32_t k = 0;  // stages issued (data items and markers)
     uint32_t m = 0;  // this CTA's item sequence
     bool ok = true;
+    uint32_t ready_ok = 0;  // lane 0: destinations whose ready word reached seq (bit per rank)
+    auto known_sources = [&](const DevItem &I) {
+      return I.wait_n == 0 || s_wait_ok[I.exec_rank] == I.wait_off;
+    };
     bool pend = false;  // signalling items issued since the last FLUSH
     int pend_key = -1;  // their counter family: ctr_index(dir, stage, 0)
     auto emit_marker = [&](uint8_t op) {  // header-only stage: FLUSH or END
@@ -668,20 +678,20 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       ++k;
     };
     auto meta_of = [&](uint32_t q) { return metas + (size_t)(q % kMetaSlots) * meta_bytes; };
+    // One proxy fence per item: generic reads of the descriptor ring, the meta slots and (by the
+    // consumers, ordered by the empty barrier) the stage come before every bulk copy into them.
+    // Prefetches are issued after the item, so the item's fence covers them too.
+    fence_proxy_async_smem();
     if (lane == 0)
       for (uint32_t q = 0; q < (uint32_t)kDescAhead && q < nmine; ++q) request_desc(q);
     for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nmine; ++q) {
-      const DevItem &Iq = desc_ready(q);
+      const DevItem Iq = desc_ready(q);
       if (lane == 0) issue_meta(P, Iq, meta_of(q), &metab[q % kMetaSlots]);
     }
     for (; m < nmine; ++m) {
-      if (lane == 0 && m + kDescAhead < nmine) request_desc(m + kDescAhead);
-      if (m + kMetaAhead < nmine) {
-        const uint32_t q = m + kMetaAhead;
-        const DevItem &In = desc_ready(q);
-        if (lane == 0) issue_meta(P, In, meta_of(q), &metab[q % kMetaSlots]);
-      }
-      const DevItem &I = desc_ready(m);
+      const DevItem I = desc_ready(m);  // registers: no shared-memory reload per field
+      const DevItem *Ism = &descs[m % kDescSlots];
+      bool fenced = false;
       if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer
         if (lane == 0)
@@ -694,7 +704,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           pend = false;
         }
         int w = 1;
-        if (lane == 0) w = wait_item_sources(P, I, 200000 + I.group) ? 1 : 0;
+        if (lane == 0 && !known_sources(I)) w = wait_item_sources(P, I, 200000 + I.group) ? 1 : 0;
         ok = __shfl_sync(0xffffffffu, w, 0) != 0;
         if (!ok) break;
       } else if (I.op == OP_COPY || I.op == OP_FOLD) {
@@ -705,8 +715,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         if (pend) {
           int ready = 1;
           if (lane == 0) {
-            ready = waits_ready(P, I) ? 1 : 0;
-            if (ready && P.use_ready && I.ready_rank >= 0)
+            ready = known_sources(I) || waits_ready(P, I) ? 1 : 0;
+            if (ready && P.use_ready && I.ready_rank >= 0 && !((ready_ok >> I.ready_rank) & 1u))
               ready = ld_acquire_sys(P.flags[I.exec_rank] + kReadyBase + I.ready_rank) >= P.seq;
           }
           ready = __shfl_sync(0xffffffffu, ready, 0);
@@ -718,10 +728,15 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         int w = 1;
         if (lane == 0) {
           // sources final (stage chaining) and the destination's buffers free (ready word)
-          w = wait_item_sources(P, I, 100000 + I.group) ? 1 : 0;
-          if (w && P.use_ready && I.ready_rank >= 0)
+          if (!known_sources(I)) {
+            w = wait_item_sources(P, I, 100000 + I.group) ? 1 : 0;
+            if (w) s_wait_ok[I.exec_rank] = I.wait_off;
+          }
+          if (w && P.use_ready && I.ready_rank >= 0 && !((ready_ok >> I.ready_rank) & 1u)) {
             w = wait_geq(P.flags[I.exec_rank] + kReadyBase + I.ready_rank, P.seq, P,
                          1000 + I.group) ? 1 : 0;
+            if (w) ready_ok |= 1u << I.ready_rank;
+          }
         }
         ok = __shfl_sync(0xffffffffu, w, 0) != 0;
         if (!ok) break;
@@ -730,7 +745,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         uint32_t stage, use;
         ring_pos(k, NS, stage, use);
         if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
-        issue_item(P, I, stages + (size_t)stage * stage_bytes, meta_of(m), &full[stage], lane);
+        fence_proxy_async_smem();
+        fenced = true;
+        issue_item(P, I, Ism, stages + (size_t)stage * stage_bytes, meta_of(m), &full[stage],
+                   lane);
         ++k;
         if (sig) {
           pend = true;
@@ -738,12 +756,22 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         }
       }
       __syncwarp();
+      // prefetch: descriptor kDescAhead items ahead, row runs / segments kMetaAhead items ahead
+      if (!fenced && (m + kMetaAhead < nmine)) fence_proxy_async_smem();
+      if (lane == 0 && m + kDescAhead < nmine) request_desc(m + kDescAhead);
+      if (m + kMetaAhead < nmine) {
+        const uint32_t q = m + kMetaAhead;
+        const DevItem In = desc_ready(q);
+        if (lane == 0) issue_meta(P, In, meta_of(q), &metab[q % kMetaSlots]);
+      }
     }
     if (!ok) {
       // watchdog abort: descriptor / metadata copies still in flight land before the CTA leaves
-      for (uint32_t q = m; q <= m + kDescAhead && q < nmine; ++q)
+      // (item m aborted before its own prefetches: requested so far are descriptors < m +
+      // kDescAhead and metadata < m + kMetaAhead)
+      for (uint32_t q = m; q < m + kDescAhead && q < nmine; ++q)
         mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
-      for (uint32_t q = m; q <= m + kMetaAhead && q < nmine; ++q)
+      for (uint32_t q = m; q < m + kMetaAhead && q < nmine; ++q)
         mbar_wait(&metab[q % kMetaSlots], (q / kMetaSlots) & 1u);
     }
     // END marker: consumers drain every issued stage, publish pending counts, then stop

@@ -454,8 +454,9 @@ void stage_fold_item(const Lowered &low, const DevGroup &g, DevItem *it, std::ve
 
 }  // namespace
 
-ItemLimits item_limits(const TmaGeometry &g, int64_t item_bytes) {
+ItemLimits item_limits(const TmaGeometry &g, int64_t item_bytes, int64_t min_items) {
   ItemLimits l;
+  l.min_items = min_items;
   l.operand_bytes = std::min<int64_t>(item_bytes, g.stage_bytes - kStageHdrBytes);
   l.max_rows = std::min<int64_t>(kMaxItemRows, g.max_item_rows);
   return l;
@@ -494,6 +495,14 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     bounds.assign(j - i, std::vector<int32_t>());
     staged.assign(j - i, 0);
     size_t max_chunks = 0;
+    // small stages: cut COPY items finer so that every co-resident CTA gets work (latency-bound
+    // launches, e.g. the tiny config or the last relay stage), down to 4 rows per item
+    int64_t copy_rows = 0;
+    for (size_t q = i; q < j; ++q)
+      if (low.groups[gids[q]].op == OP_COPY) copy_rows += low.groups[gids[q]].n_rows;
+    int64_t spread_rpi = lim.max_rows;
+    if (lim.min_items > 0 && copy_rows < lim.min_items * lim.max_rows)
+      spread_rpi = std::max<int64_t>(4, (copy_rows + lim.min_items - 1) / lim.min_items);
     for (size_t q = i; q < j; ++q) {
       const DevGroup &g = low.groups[gids[q]];
       std::vector<int32_t> &b = bounds[q - i];
@@ -509,7 +518,8 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       }
       if (g.op == OP_COPY) {
         // rows per item; a multiple of 4 when gather4 may apply (its groups are padded to 4 rows)
-        int64_t rpi = std::min<int64_t>(lim.max_rows, std::max<int64_t>(1, cap / row16));
+        int64_t rpi = std::min<int64_t>(std::min(lim.max_rows, spread_rpi),
+                                        std::max<int64_t>(1, cap / row16));
         if (row16 <= kGather4MaxRowBytes && rpi >= 4) rpi = rpi / 4 * 4;
         for (int64_t r = rpi; r < g.n_rows; r += rpi) b.push_back((int32_t)r);
         b.push_back((int32_t)g.n_rows);

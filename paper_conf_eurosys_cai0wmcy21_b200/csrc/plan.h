@@ -94,8 +94,9 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
 struct ItemLimits {
   int64_t operand_bytes;  // gathered bytes of one item (<= stage_bytes - kStageHdrBytes)
   int64_t max_rows;       // rows (COPY) / operand rows (staged FOLD) of one item
+  int64_t min_items;      // COPY items per stage to aim for (co-resident CTAs; 0 = no spreading)
 };
-ItemLimits item_limits(const TmaGeometry &g, int64_t item_bytes);
+ItemLimits item_limits(const TmaGeometry &g, int64_t item_bytes, int64_t min_items = 0);
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,
                  const ItemLimits &lim, bool signal_all, const std::vector<uint8_t> &needed_ctr,
                  std::vector<DevItem> *items, std::vector<DevRun> *runs,

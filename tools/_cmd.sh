@@ -7,6 +7,9 @@ run() { # cfg opts...
   timeout 600 python bench.py --config $C --steps 10 --warmup 3 --e2e-steps 0 --no-cpu-baseline --no-torch-baseline "$@" 2>/dev/null | python3 -c "
 import json,sys; d=json.loads(sys.stdin.read()); print('$C $*', round(d['ms_per_step'],3), {k: (round(v['ms'],3), round(v['frac'],3)) for k,v in d['roofline']['per_kernel'].items()})"
 }
-for C in reddit google8 orkut google8_dgx1 reddit_dgx1 google8_ring google2 tiny; do
+for C in google8_dgx1 reddit_dgx1 google8_ring; do
   for G in 0 1 2; do run $C --opt geometry=$G; done
+  run $C --opt stage_fold=0
 done
+run reddit
+run tiny

@@ -59,10 +59,19 @@ def main(tag, names, config="reddit"):
         ki, vi = hdr.index("Kernel Name"), hdr.index("Metric Value")
         ks = [(r[ki], float(r[vi].replace(",", ""))) for r in rows[h + 1:] if len(r) > vi]
         tot = sum(v for _, v in ks)
-        lines += ["", "Launch list (`--metrics gpu__time_duration.sum`): %d launches, all "
-                  "`executor_tma_kernel` = %.1f %% of GPU time; per step the three launches "
-                  "repeat fwd602 / fwd256 / bwd256." % (len(ks), 100.0 * sum(
-                      v for k, v in ks if "executor" in k) / max(tot, 1))]
+        by = {}
+        for k, v in ks:
+            short = k.split("(")[0][-60:]
+            n, t = by.get(short, (0, 0.0))
+            by[short] = (n + 1, t + v)
+        lines += ["", "Launch list (`--metrics gpu__time_duration.sum`, whole process: input "
+                  "generation, warm-up and timed steps): %d launches; executor launches = %.1f %% "
+                  "of all GPU time (the other kernels are input fills and copies outside the "
+                  "timed region; inside it only executor launches run, three per step)." % (
+                      len(ks), 100.0 * sum(v for k, v in ks if "executor" in k) / max(tot, 1)),
+                  "", "| kernel | launches | total us |", "|---|---|---|"]
+        for short, (n, t) in sorted(by.items(), key=lambda x: -x[1][1]):
+            lines.append("| `%s` | %d | %.1f |" % (short, n, t / 1e3))
         with open(os.path.join(ROOT, "profiles", "%s_launches.csv" % tag), "w") as f:
             f.write("kernel,gpu__time_duration_ns\n")
             for k, v in ks:
