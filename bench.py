@@ -352,6 +352,17 @@ def run_ours_single(args, w):
     # read-modify-writes every owner row that has requesters.
     peaks, src = measured_peaks()
     nv = info["n_vertices_planned"]
+    # relay plans (several stages) must move more than the direct minimum: every tree edge writes
+    # a row and every forwarding GPU re-reads the row it forwards; the backward pushes one
+    # partial-sum row per tree edge into a slot that the parent reads back.  Reported next to
+    # the direct minimum as plan_algorithmic_bytes / plan_frac.
+    plan_rows = None
+    if info["n_stages"] > 1:
+        E = ctx.plan_export()                       # (u, parent, child, stage)
+        owner = g.part[E[:, 0]]
+        fwd_pairs = np.unique(E[E[:, 1] != owner][:, [0, 1]], axis=0).shape[0]
+        ne = int(info["n_tree_edges"])
+        plan_rows = {"fwd": nv + fwd_pairs + ne, "bwd": w.S + 2 * ne + 2 * nv}
     kernels = {}
     for i, n in enumerate(names):
         l = (w.fwd_layers + w.bwd_layers)[i]
@@ -364,6 +375,10 @@ def run_ours_single(args, w):
         kernels[n] = {"ms": per_op[n], "algorithmic_bytes": int(alg), "achieved_gbs": ach,
                       "frac": ach / peaks["hbm_gbs"],
                       "traffic": profiled_traffic("%s/%s" % (c.name, n))}
+        if plan_rows is not None:
+            pb = plan_rows["fwd" if n.startswith("fwd") else "bwd"] * row
+            kernels[n]["plan_algorithmic_bytes"] = int(pb)
+            kernels[n]["plan_frac"] = pb / (per_op[n] * 1e-3) / 1e9 / peaks["hbm_gbs"]
     dom = max(names, key=lambda n: per_op[n])
     roofline = {"bound": "hbm", "kernel": "executor_tma_kernel (%s)" % dom,
                 "achieved": kernels[dom]["achieved_gbs"], "peak": peaks["hbm_gbs"],

@@ -14,9 +14,12 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <map>
 #include <new>
 #include <string>
 #include <vector>
+
+#include <map>
 
 #include "dgcl.h"
 #include "hostsim.h"
@@ -93,7 +96,7 @@ struct dgcl_ctx {
   int geometry = 0;                   // bulk-copy geometry: 0 auto per program, 1 WIDE, 2 DUAL
   bool threads_set = false, ctas_set = false;  // user overrides of the CTA shape
   int sm_count = 148;  // SMs of the device (B200 until queried), for cutting small stages
-  int tma_ctas_geo[2][2] = {{0, 0}, {0, 0}};   // [geo][1024-thread fold instance] CTAs per SM
+  std::map<std::pair<int, int>, int> tma_ctas;  // (geo, block) -> co-resident CTAs per SM
   int n_prog_ranks = 1;        // programs per (layer, dir)
 
   uint64_t seq = 0, epoch[2] = {0, 0};
@@ -330,16 +333,21 @@ void build_programs(dgcl_ctx *c) {
         }
         // auto: DUAL (two producer warps per SM) unless the launch is bulk-copy friendly —
         // copies only, >= 8 KB per bulk operation (long runs of rows) — or carries unstaged folds
-        // (consumer gathers, which want the 1024-thread instance); see TmaGeometry
+        // (consumer gathers, which want more consumer warps), or chains stages on flags (relay
+        // plans: DUAL's forward time was bimodal, 0.83 / 2.1 ms, on the Web-Google dgx1_like
+        // plan, WIDE a steady 0.9-1.1 ms); see TmaGeometry
         build(1);
         int64_t ops = 0, bytes = 0;
+        bool waits = false;
         for (const DevItem &it : P.items) {
+          waits = waits || (it.wait_n > 0 && (it.op == OP_COPY || it.op == OP_FOLD));
           if (it.op != OP_COPY) continue;
           bytes += (int64_t)it.rows * row16;
           ops += (it.flags & kItemGather4) ? (it.rows + 3) / 4 : it.nterms;
         }
         const bool copy_only = (P.op_mask & ~kMaskCopy) == 0;
-        if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & kMaskFold)) build(0);
+        if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & kMaskFold) || waits)
+          build(0);
       }
     }
   }
@@ -356,6 +364,17 @@ dgcl_status upload(dgcl_ctx *c, T **dptr, const std::vector<T> &v) {
   CUDA_TRY(c, cudaMemset(*dptr, 0, bytes));
   if (!v.empty()) CUDA_TRY(c, cudaMemcpy(*dptr, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice));
   return DGCL_OK;
+}
+
+// CTA size of a program's bulk-copy launch: the geometry's, except that unstaged folds
+// (consumer-side gathers, latency-bound) get more consumer warps — 1024 threads for fold-only
+// launches with many terms per row, 512 otherwise — and the user's "threads" option wins
+int tma_block(const dgcl_ctx *c, const Program &pg) {
+  if (c->threads_set) return c->threads;
+  const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
+  if (pg.geo == 0 && (pg.op_mask & kMaskFold))
+    return pg.op_mask == kMaskFold && pg.fold_wide ? 1024 : 512;
+  return G.threads;
 }
 
 dgcl_status check_dead(dgcl_ctx *c) {
@@ -475,13 +494,13 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     Pp.fold_wide = pg.fold_wide ? 1 : 0;
     Pp.n_items = (int32_t)pg.items.size();
     const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
-    const bool wide_fold = pg.geo == 0 && pg.op_mask == kMaskFold && pg.fold_wide &&
-                           !c->threads_set;
+    const int tblock = tma_block(c, pg);
+    const auto occ = c->tma_ctas.find({pg.geo, tblock});
+    const int tctas = occ == c->tma_ctas.end() ? 0 : occ->second;
     int block = c->threads, grid_all = c->grid;
-    if (Pp.use_tma && Pp.row16 <= G.stage_bytes - kStageHdrBytes &&
-        c->tma_ctas_geo[pg.geo][wide_fold ? 1 : 0] > 0) {
-      block = wide_fold ? 1024 : (c->threads_set ? c->threads : G.threads);
-      grid_all = c->n_sm * c->tma_ctas_geo[pg.geo][wide_fold ? 1 : 0];
+    if (Pp.use_tma && Pp.row16 <= G.stage_bytes - kStageHdrBytes && tctas > 0) {
+      block = tblock;
+      grid_all = c->n_sm * tctas;
       Pp.tma_stages = G.stages;
       Pp.tma_buf = G.stage_bytes;
       Pp.meta_bytes = G.meta_bytes;
@@ -669,18 +688,17 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   int occ = 0;
   int e = executor_occupancy(c->threads, &occ);
   if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");
-  // bulk-copy executor: co-resident CTAs per SM for each geometry at its CTA size
-  for (int geo = 0; geo < 2; ++geo) {
-    const TmaGeometry &G = geo ? kGeoDual : kGeoWide;
-    for (int wide_fold = 0; wide_fold < 2; ++wide_fold) {
-      const int block = wide_fold ? 1024 : (c->threads_set ? c->threads : G.threads);
-      int n = 0;
-      e = executor_tma_occupancy(block, tma_smem_bytes(G), &n);
-      if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");
-      n = std::min(n, G.ctas_per_sm);
-      if (c->ctas_set) n = std::min(n, c->ctas_per_sm);
-      c->tma_ctas_geo[geo][wide_fold] = n;
-    }
+  // bulk-copy executor: co-resident CTAs per SM for every (geometry, CTA size) a program uses
+  for (const Program &pg : c->progs) {
+    const int block = tma_block(c, pg);
+    if (c->tma_ctas.count({pg.geo, block})) continue;
+    const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
+    int n = 0;
+    e = executor_tma_occupancy(block, tma_smem_bytes(G), &n);
+    if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");
+    n = std::min(n, G.ctas_per_sm);
+    if (c->ctas_set) n = std::min(n, c->ctas_per_sm);
+    c->tma_ctas[{pg.geo, block}] = n;
   }
   if (c->ctas_per_sm <= 0) c->ctas_per_sm = std::min(occ, 4);
   c->ctas_per_sm = std::max(1, std::min(c->ctas_per_sm, occ));

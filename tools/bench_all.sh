@@ -17,6 +17,7 @@ for line in open('gpurun_out/bench_all.jsonl'):
     print(d['config']['config'], 'ms/step %.3f' % d['ms_per_step'], 'GB/s %.0f' % d['value'],
           {k: round(v, 3) for k, v in d['ms_per_layer'].items()},
           {k: round(v['frac'], 3) for k, v in r['per_kernel'].items()},
+          {k: round(v['plan_frac'], 3) for k, v in r['per_kernel'].items() if 'plan_frac' in v},
           'stages', d['plan']['n_stages'], 'plan_s %.2f' % d['plan']['planner_seconds'],
           'gen_s %.1f' % d['plan']['graph_gen_s'])
 PY
