@@ -110,6 +110,21 @@ dgcl_status dgcl_set_topology(dgcl_ctx *ctx, const dgcl_topology *topo);
 dgcl_status dgcl_build_plan(dgcl_ctx *ctx, const int64_t *req_ptr, const int64_t *req_ids,
                             uint64_t seed);
 
+/* Build the plan from saved trees instead of running SPST (checkpoint/resume of the planning
+ * step: the plan is made once before training, and SPST costs seconds to minutes at
+ * scale, Table 8).  The trees are the tuples dgcl_plan_export returns — edge e =
+ * (u[e], parent[e], child[e], stage[e]), all host arrays of n_edges entries, the edges of one
+ * vertex contiguous and in root-to-leaf order (a parent is u's owner or an earlier child).  The
+ * same relation checks as dgcl_build_plan, then the plan invariants of the oracle:
+ * every vertex some GPU requests has exactly one tree, rooted at its owner, reaching every
+ * requester over existing links, stage = tree depth <= world-1, no leaf that did not request
+ * it; t(S) is recomputed (dgcl_plan_info).  Errors: as dgcl_build_plan; EPLAN for an invalid
+ * tree (dgcl_last_error says which edge / vertex); EINVAL for NULL arrays with n_edges > 0. */
+dgcl_status dgcl_build_plan_from_trees(dgcl_ctx *ctx, const int64_t *req_ptr,
+                                       const int64_t *req_ids, int64_t n_edges, const int64_t *u,
+                                       const int32_t *parent, const int32_t *child,
+                                       const int32_t *stage);
+
 /* Device workspace.  The caller allocates ONE device buffer of at least *bytes bytes, 256-B
  * aligned (PyTorch does), keeps it alive until dgcl_destroy, and registers it.  The library carves
  * out halos (one per layer), relay staging, backward gradient slots and flag words, zeroes the flag

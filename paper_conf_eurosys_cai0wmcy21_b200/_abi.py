@@ -18,6 +18,7 @@ IPC_BLOB_BYTES = 256
 # every symbol include/dgcl.h declares (tests check the library exports all of them)
 SYMBOLS = [
     "dgcl_init", "dgcl_init_loopback", "dgcl_set_topology", "dgcl_build_plan",
+    "dgcl_build_plan_from_trees",
     "dgcl_workspace_bytes", "dgcl_register_workspace", "dgcl_halo_view", "dgcl_rank_rows",
     "dgcl_ipc_export", "dgcl_ipc_import", "dgcl_dispatch_forward", "dgcl_dispatch_backward",
     "dgcl_forward_host", "dgcl_backward_host", "dgcl_plan_info", "dgcl_plan_counts",
@@ -67,6 +68,7 @@ def lib():
             "dgcl_init_loopback": [I32, I32, I64, P, I32, P, I32, pp],
             "dgcl_set_topology": [P, ctypes.POINTER(Topology)],
             "dgcl_build_plan": [P, P, P, U64],
+            "dgcl_build_plan_from_trees": [P, P, P, I64, P, P, P, P],
             "dgcl_workspace_bytes": [P, ctypes.POINTER(SZ)],
             "dgcl_register_workspace": [P, P, SZ],
             "dgcl_halo_view": [P, I32, ctypes.POINTER(SZ), ctypes.POINTER(I64), ctypes.POINTER(I64)],

@@ -593,17 +593,26 @@ dgcl_status dgcl_set_topology(dgcl_ctx *c, const dgcl_topology *t) {
   return DGCL_OK;
 }
 
-dgcl_status dgcl_build_plan(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *req_ids,
-                            uint64_t seed) {
+}  // extern "C"
+
+namespace {
+
+// build_plan / build_plan_from_trees: the relation, then a plan from SPST (trees == nullptr) or
+// from the caller's saved trees, then lowering, workspace layout and the launch programs
+dgcl_status plan_common(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *req_ids,
+                        uint64_t seed, int64_t n_edges, const int64_t *tu, const int32_t *tp,
+                        const int32_t *tc, const int32_t *ts, bool trees) {
   if (!c || !req_ptr) return DGCL_EINVAL;
   if (c->planned) return fail(c, DGCL_ESTATE, "plan already built");
   if (req_ptr[c->world] > 0 && !req_ids) return DGCL_EINVAL;
+  if (trees && (n_edges < 0 || (n_edges > 0 && (!tu || !tp || !tc || !ts)))) return DGCL_EINVAL;
   try {
     std::string e = build_relation(c->n, c->world, c->part.data(), req_ptr, req_ids, &c->rel);
     if (!e.empty()) return fail(c, DGCL_EINVAL, "%s", e.c_str());
     for (int d = 0; d < c->world; ++d)
       if (req_ptr[d + 1] - req_ptr[d] > INT32_MAX) return fail(c, DGCL_EINVAL, "halo too large");
-    e = spst_plan(c->topo, c->part.data(), c->rel, seed, &c->plan);
+    e = trees ? import_plan(c->topo, c->part.data(), c->rel, n_edges, tu, tp, tc, ts, &c->plan)
+              : spst_plan(c->topo, c->part.data(), c->rel, seed, &c->plan);
     if (!e.empty()) return fail(c, DGCL_EPLAN, "%s", e.c_str());
     if (c->plan.n_stages >= kMaxStages) return fail(c, DGCL_EPLAN, "too many stages");
     lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low);
@@ -618,6 +627,22 @@ dgcl_status dgcl_build_plan(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *
   }
   c->planned = true;
   return DGCL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+dgcl_status dgcl_build_plan(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *req_ids,
+                            uint64_t seed) {
+  return plan_common(c, req_ptr, req_ids, seed, 0, nullptr, nullptr, nullptr, nullptr, false);
+}
+
+dgcl_status dgcl_build_plan_from_trees(dgcl_ctx *c, const int64_t *req_ptr,
+                                       const int64_t *req_ids, int64_t n_edges, const int64_t *u,
+                                       const int32_t *parent, const int32_t *child,
+                                       const int32_t *stage) {
+  return plan_common(c, req_ptr, req_ids, 0, n_edges, u, parent, child, stage, true);
 }
 
 dgcl_status dgcl_workspace_bytes(dgcl_ctx *c, size_t *bytes) {

@@ -50,6 +50,12 @@ std::string build_relation(int64_t n, int m, const int32_t *part, const int64_t 
 std::string spst_plan(const Topology &topo, const int32_t *part, const Relation &rel,
                       uint64_t seed, Plan *out);
 
+// A saved plan (trees, as dgcl_plan_export gives them) instead of SPST; the plan invariants are
+// checked and t(S) recomputed.  Returns "" or an error message (EPLAN).
+std::string import_plan(const Topology &topo, const int32_t *part, const Relation &rel,
+                        int64_t n_edges, const int64_t *u, const int32_t *parent,
+                        const int32_t *child, const int32_t *stage, Plan *out);
+
 // ---- lowering ----------------------------------------------------------------------------
 
 struct Lowered {

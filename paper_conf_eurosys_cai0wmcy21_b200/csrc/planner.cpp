@@ -13,6 +13,7 @@
 // demand for the relaxed edges only (the optimisation the paper mentions at P:1384-1392): because
 // S is fixed during one Dijkstra, C(k, e) = max(t^k, max_{h in e} (c_h^k + 1) w_h) - t^k exactly.
 
+#include <algorithm>
 #include <chrono>
 #include <cstring>
 #include <string>
@@ -223,6 +224,82 @@ std::string spst_plan(const Topology &topo, const int32_t *part, const Relation 
   P.cost = 0;
   for (int k = 1; k < m; ++k) P.cost += tk[k];
   P.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+  return "";
+}
+
+// A plan given as trees (e.g. saved from dgcl_plan_export of an earlier run: planning happens
+// once before training, and costs seconds to minutes at scale, Table 8):
+// edges grouped per vertex, each group in root-to-leaf order (a parent is the owner or an
+// earlier child).  Checks the §8(c) plan invariants and recomputes t(S) with the §5.1 rules.
+std::string import_plan(const Topology &topo, const int32_t *part, const Relation &rel,
+                        int64_t n_edges, const int64_t *u, const int32_t *parent,
+                        const int32_t *child, const int32_t *stage, Plan *out) {
+  Plan &P = *out;
+  P = Plan();
+  const int m = topo.m;
+  P.m = m;
+  const int H = (int)topo.w.size();
+  std::vector<int64_t> load((size_t)kMaxStages * H, 0);
+  std::vector<int64_t> tk(kMaxStages, 0);
+  std::vector<uint8_t> seen(rel.n, 0);
+  int64_t planned = 0;
+  for (int64_t v = 0; v < rel.n; ++v) planned += rel.d_ptr[v + 1] > rel.d_ptr[v] ? 1 : 0;
+  P.e_ptr.push_back(0);
+  int max_stage = 0;
+  for (int64_t e = 0; e < n_edges;) {
+    const int64_t v = u[e];
+    if (v < 0 || v >= rel.n) return "edge " + std::to_string(e) + ": vertex out of range";
+    if (seen[v]) return "vertex " + std::to_string(v) + ": its edges are not contiguous";
+    seen[v] = 1;
+    if (rel.d_ptr[v + 1] == rel.d_ptr[v])
+      return "vertex " + std::to_string(v) + ": no GPU requests it";
+    const int root = part[v];
+    int depth[kMaxRanks], nchild[kMaxRanks];
+    for (int x = 0; x < m; ++x) depth[x] = -1, nchild[x] = 0;
+    depth[root] = 0;
+    int64_t f = e;
+    for (; f < n_edges && u[f] == v; ++f) {
+      const int p = parent[f], c = child[f], k = stage[f];
+      if (p < 0 || p >= m || c < 0 || c >= m) return "edge " + std::to_string(f) + ": GPU id";
+      if (depth[p] < 0) return "edge " + std::to_string(f) + ": parent not yet in the tree";
+      if (depth[c] >= 0) return "edge " + std::to_string(f) + ": node already in the tree";
+      if (k != depth[p] + 1 || k > m - 1 || k >= kMaxStages)
+        return "edge " + std::to_string(f) + ": stage is not the tree depth";
+      if (!topo.has(p, c)) return "edge " + std::to_string(f) + ": no such link";
+      depth[c] = k;
+      nchild[p]++;
+      max_stage = std::max(max_stage, k);
+      P.e_parent.push_back(p);
+      P.e_child.push_back(c);
+      P.e_stage.push_back(k);
+      int64_t *ld = &load[(size_t)k * H];
+      for (int32_t q = topo.link_ptr[p * m + c]; q < topo.link_ptr[p * m + c + 1]; ++q) {
+        const int h = topo.link_hops[q];
+        ld[h] += 1;
+        tk[k] = std::max(tk[k], ld[h] * topo.w[h]);
+      }
+    }
+    uint32_t req = 0;
+    for (int64_t q = rel.d_ptr[v]; q < rel.d_ptr[v + 1]; ++q) {
+      req |= 1u << rel.d_gpu[q];
+      if (depth[rel.d_gpu[q]] < 0)
+        return "vertex " + std::to_string(v) + ": GPU " + std::to_string(rel.d_gpu[q]) +
+               " requests it but is not in its tree";
+    }
+    for (int x = 0; x < m; ++x)  // a relay that forwards nothing would only waste a row
+      if (x != root && depth[x] >= 0 && !(req >> x & 1) && nchild[x] == 0)
+        return "vertex " + std::to_string(v) + ": GPU " + std::to_string(x) +
+               " is a leaf that did not request it";
+    P.order.push_back(v);
+    P.e_ptr.push_back((int64_t)P.e_parent.size());
+    e = f;
+  }
+  if ((int64_t)P.order.size() != planned)
+    return "plan covers " + std::to_string(P.order.size()) + " of " + std::to_string(planned) +
+           " requested vertices";
+  P.n_stages = max_stage;
+  P.cost = 0;
+  for (int k = 1; k < kMaxStages; ++k) P.cost += tk[k];
   return "";
 }
 

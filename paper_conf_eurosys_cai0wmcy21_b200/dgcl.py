@@ -78,15 +78,29 @@ class Context:
                           hops.ctypes.data if hops.size else None)
         check(lib().dgcl_set_topology(self.handle, ctypes.byref(t)), self.handle)
 
-    def build_plan(self, req_ptr, req_ids, seed=0, topology=None):
-        """buildCommInfo: plan from ALL ranks' required lists (CSR)."""
+    def build_plan(self, req_ptr, req_ids, seed=0, topology=None, trees=None):
+        """buildCommInfo: plan from ALL ranks' required lists (CSR).
+
+        trees: a saved plan, [E x 4] (u, parent, child, stage) as plan_export() returns it (e.g.
+        np.save'd by an earlier run): used instead of running SPST, after the plan invariants are
+        checked (checkpoint/resume of the planning step)."""
         if topology is not None:
             self.set_topology(topology)
         req_ptr = _np(req_ptr, np.int64)
         req_ids = _np(req_ids, np.int64)
-        check(lib().dgcl_build_plan(self.handle, req_ptr.ctypes.data,
-                                    req_ids.ctypes.data if req_ids.size else None,
-                                    ctypes.c_uint64(seed)), self.handle)
+        ids = req_ids.ctypes.data if req_ids.size else None
+        if trees is None:
+            check(lib().dgcl_build_plan(self.handle, req_ptr.ctypes.data, ids,
+                                        ctypes.c_uint64(seed)), self.handle)
+        else:
+            E = np.asarray(trees)
+            u = np.ascontiguousarray(E[:, 0], np.int64)
+            pc = [np.ascontiguousarray(E[:, i], np.int32) for i in (1, 2, 3)]
+            n = len(u)
+            ptr = lambda a: a.ctypes.data if n else None
+            check(lib().dgcl_build_plan_from_trees(self.handle, req_ptr.ctypes.data, ids, n,
+                                                   ptr(u), ptr(pc[0]), ptr(pc[1]), ptr(pc[2])),
+                  self.handle)
         nl = np.zeros(self.world, np.int64)
         nh = np.zeros(self.world, np.int64)
         check(lib().dgcl_rank_rows(self.handle, nl.ctypes.data, nh.ctypes.data), self.handle)

@@ -182,6 +182,70 @@ def test_shuffled_halo_order():
     _check_lowering(g, [8], None, seed=1)
 
 
+@pytest.mark.parametrize("topo_name", [None, "dgx1_like", "ring"])
+def test_plan_save_and_resume(topo_name):
+    """Checkpoint/resume of the planning step: plan_export -> build_plan(trees=...) in a fresh
+    context gives the same plan, cost and lowered program (host interpreter vs the oracle)."""
+    g = synth.make_graph(700, 5000, 8, graph_seed=31, part_seed=32)
+    topo = synth.topology.by_name(topo_name) if topo_name else None
+    a = _ctx(g, [12, 5], topo, seed=4)
+    E = a.plan_export()
+    D = _D()
+    b = D.loopback(g.m, g.part, [12, 5], device=-1)
+    b.build_plan(g.req_ptr, g.req_ids, topology=topo, trees=E)
+    assert np.array_equal(b.plan_export(), E)
+    ia, ib = a.plan_info(), b.plan_info()
+    for k in ("n_stages", "n_tree_edges", "n_relay_rows", "model_cost_ticks", "n_fwd_groups",
+              "n_bwd_groups"):
+        assert ia[k] == ib[k], k
+    # the resumed plan through the lowering, on the host, against the oracle
+    m = g.m
+    R = [g.R(d) for d in range(m)]
+    loc, _ = halo.local_rows(g.part, m)
+    pitch = b.halo_view(0)[2]
+    emb = synth.fill_values(g.n, 12, pitch, keys=np.argsort(g.part, kind="stable"), seed=3)
+    H = np.zeros((int(g.req_ptr[-1]), pitch), np.float32)
+    b.debug_hostsim_forward(0, emb, H)
+    Ho = halo.forward([emb[b.row_off[d]:b.row_off[d + 1], :12] for d in range(m)], R, g.part, loc)
+    for d in range(m):
+        assert np.array_equal(H[g.req_ptr[d]:g.req_ptr[d + 1], :12], Ho[d])
+
+
+def test_saved_plan_is_validated():
+    """Invalid trees are rejected with EPLAN (each §8(c) tree invariant broken once)."""
+    D = _D()
+    g = synth.make_graph(300, 2000, 4, graph_seed=41, part_seed=42)
+    topo = synth.fig6()
+    E = _ctx(g, [4], topo, seed=1).plan_export()
+    assert (E[:, 3] > 1).any()          # the Fig. 6 model relays
+
+    def rejected(E2):
+        c = D.loopback(g.m, g.part, [4], device=-1)
+        with pytest.raises(D.DGCLError) as e:
+            c.build_plan(g.req_ptr, g.req_ids, topology=topo, trees=E2)
+        assert e.value.status == 6, e.value     # DGCL_EPLAN
+
+    deep = int(np.nonzero(E[:, 3] > 1)[0][0])
+    bad = E.copy(); bad[deep, 3] += 1; rejected(bad)               # stage != tree depth
+    bad = E.copy(); bad[0, 1] = bad[0, 2]; rejected(bad)           # parent not in the tree
+    first = E[E[:, 0] == E[0, 0]]
+    rejected(E[len(first):])                                       # a requested vertex missing
+    bad = np.concatenate([E[len(first):], first, first[:1]])
+    rejected(bad)                                                  # a vertex's edges split
+    # an extra leaf on a GPU that did not request the vertex
+    for v in np.unique(E[:, 0]):
+        rows = E[E[:, 0] == v]
+        nodes = set(rows[:, 1]) | set(rows[:, 2])
+        free = [x for x in range(4) if x not in nodes]
+        if free:
+            k = int(np.nonzero(E[:, 0] == v)[0][-1])
+            extra = np.array([[v, g.part[v], free[0], 1]], E.dtype)
+            rejected(np.concatenate([E[:k + 1], extra, E[k + 1:]]))
+            break
+    else:
+        pytest.fail("no vertex with a GPU outside its tree")
+
+
 def test_fig6_plan_from_library():
     """The Fig. 6 worked example through the C planner (T_a = d1-d2-d3-d4)."""
     D = _D()
