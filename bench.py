@@ -327,6 +327,10 @@ def run_ours_single(args, w):
             sum(a.numel() * 4 for a in hg_p.values()) + sum(a.numel() * 4 for a in eg_p.values())
         d2h = sum(a.numel() * 4 for a in halo_p.values()) + sum(a.numel() * 4 for a in eg_p.values())
 
+        # pipelined host calls: each call's input copy overlaps the previous call's output copy
+        # (host_async); the step ends when the stream is synchronized (the timed events below)
+        ctx.set_option("host_async", 1)
+
         def e2e_step():
             for l in w.fwd_layers:
                 ctx.forward_host(l, emb_p[l], halo_p[l], stream=stream)

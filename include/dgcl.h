@@ -178,7 +178,11 @@ dgcl_status dgcl_dispatch_backward(dgcl_ctx *ctx, int32_t layer, const float *ha
                                    void *stream);
 
 /* End-to-end variants with HOST buffers (pinned or pageable): copy the input rows host->device
- * into library-owned staging, dispatch, copy the result device->host, synchronize `stream`.
+ * into library-owned staging (one buffer per layer and input), dispatch on `stream`, copy the
+ * result device->host, then synchronize `stream`.  The two copies run on library-owned copy
+ * streams, ordered against `stream` by events, so with option "host_async" = 1 (no synchronize;
+ * the host result is complete once `stream` is synchronized, and the host buffers must stay
+ * valid until then) the input copy of the next call overlaps the output copy of this one.
  * forward:  host_emb [rows x pitch] -> host_halo [halo rows x pitch] (pitch = the halo view pitch)
  * backward: host_halo_grad [halo rows x pitch] and host_emb_grad in/out [rows x pitch].
  * Errors: as the device variants, plus ENOMEM for staging. */
@@ -216,9 +220,13 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    halo gradients in place (no slot round trip); 0: push + owner reduce
  *   "direct_copy_rows" COPY items whose runs average fewer rows are gathered by the consumer
  *                    warps with plain loads (default 0 = never)
+ *   "host_async"     0 (default) / 1: dgcl_forward_host / dgcl_backward_host return before the
+ *                    device->host copy completes (any time)
+ *   "geometry"       bulk-copy launch geometry: 0 (default) auto per launch, 1 WIDE (1 CTA per
+ *                    SM, 3 x 64 KB stages), 2 DUAL (2 CTAs per SM, 2 x 47 KB stages)
  *   "bulk_store", "bulk_store_peer"  TMA stores for packed contiguous destinations in local HBM
  *                    (default 1) / peer memory (default 0)
- * Options other than "timeout_ms" and "debug_skip_rank" must be set before
+ * Options other than "timeout_ms", "debug_skip_rank" and "host_async" must be set before
  * dgcl_register_workspace (ESTATE otherwise).
  *   "debug_skip_rank" fault injection for DGCL_LOOPBACK_PER_RANK contexts: never launch that
  *                    virtual rank's program, so its peers' flag waits hit the watchdog (any time;

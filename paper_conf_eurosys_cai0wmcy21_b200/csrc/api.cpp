@@ -106,8 +106,17 @@ struct dgcl_ctx {
   std::vector<cudaStream_t> rank_streams;
   std::vector<cudaEvent_t> rank_events;
   cudaEvent_t fork_event = nullptr;
-  void *stage_a = nullptr, *stage_b = nullptr;
-  size_t stage_a_bytes = 0, stage_b_bytes = 0;
+  // host-buffer entry points: device staging per (buffer, layer), each with the event of its
+  // last device-side use, and two copy streams so that the host->device copy of one call runs
+  // while the device->host copy of the previous one is in flight (PCIe is full duplex)
+  struct Stage {
+    void *ptr = nullptr;
+    size_t bytes = 0;
+    cudaEvent_t free = nullptr;  // recorded after the last kernel / copy that reads it
+  };
+  std::map<int, Stage> stages;  // key: kind * 4096 + layer (kind 0 emb, 1 halo grad, 2 emb grad)
+  cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;
+  bool host_async = false;  // host calls return before the device->host copy completes
   uint64_t launches = 0;
   int debug_skip_rank = -1;  // fault injection (per-rank loopback): never launch this rank
   bool dead = false;
@@ -860,15 +869,62 @@ dgcl_status dgcl_dispatch_backward(dgcl_ctx *c, int32_t layer, const float *halo
   return launch(c, layer, DIR_BWD, halo_grad, hg_pitch, emb_grad, eg_pitch, (cudaStream_t)stream);
 }
 
-static dgcl_status ensure_stage(dgcl_ctx *c, void **p, size_t *cap, size_t bytes) {
-  if (*cap >= bytes) return DGCL_OK;
-  if (*p) cudaFree(*p);
-  *p = nullptr;
-  *cap = 0;
-  if (cudaMalloc(p, std::max<size_t>(bytes, 256)) != cudaSuccess)
-    return fail(c, DGCL_ENOMEM, "staging allocation of %zu bytes failed", bytes);
-  *cap = bytes;
+static dgcl_status get_stage(dgcl_ctx *c, int kind, int layer, size_t bytes,
+                             dgcl_ctx::Stage **out) {
+  dgcl_ctx::Stage &S = c->stages[kind * 4096 + layer];
+  if (!S.free) CUDA_TRY(c, cudaEventCreateWithFlags(&S.free, cudaEventDisableTiming));
+  if (S.bytes < bytes) {
+    // the old buffer may still be in use by queued work: wait for it before freeing
+    if (S.ptr) {
+      CUDA_TRY(c, cudaEventSynchronize(S.free));
+      cudaFree(S.ptr);
+    }
+    S.ptr = nullptr;
+    S.bytes = 0;
+    if (cudaMalloc(&S.ptr, std::max<size_t>(bytes, 256)) != cudaSuccess)
+      return fail(c, DGCL_ENOMEM, "staging allocation of %zu bytes failed", bytes);
+    S.bytes = bytes;
+  }
+  if (!c->h2d_stream) {
+    CUDA_TRY(c, cudaStreamCreateWithFlags(&c->h2d_stream, cudaStreamNonBlocking));
+    CUDA_TRY(c, cudaStreamCreateWithFlags(&c->d2h_stream, cudaStreamNonBlocking));
+  }
+  *out = &S;
   return DGCL_OK;
+}
+
+// `to` waits for the work queued so far on `from`
+static dgcl_status stream_after(dgcl_ctx *c, cudaStream_t to, cudaStream_t from) {
+  cudaEvent_t e;
+  CUDA_TRY(c, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  CUDA_TRY(c, cudaEventRecord(e, from));
+  CUDA_TRY(c, cudaStreamWaitEvent(to, e, 0));
+  cudaEventDestroy(e);  // released once the recorded work completes
+  return DGCL_OK;
+}
+
+// host -> staging on the copy stream, after the staging buffer's last reader; `st` waits for it
+static dgcl_status stage_in(dgcl_ctx *c, dgcl_ctx::Stage *S, const void *host, size_t bytes,
+                            cudaStream_t st) {
+  if (!bytes) return DGCL_OK;
+  CUDA_TRY(c, cudaStreamWaitEvent(c->h2d_stream, S->free, 0));
+  CUDA_TRY(c, cudaMemcpyAsync(S->ptr, host, bytes, cudaMemcpyHostToDevice, c->h2d_stream));
+  return stream_after(c, st, c->h2d_stream);
+}
+
+// device -> host on the second copy stream once `st`'s work is done; `st` then waits for the copy
+// (so synchronizing the caller's stream means the host result is there), `src_free` is recorded
+// after it, and in synchronous mode the call waits
+static dgcl_status stage_out(dgcl_ctx *c, void *host, const void *dev, size_t bytes,
+                             cudaStream_t st, cudaEvent_t src_free) {
+  dgcl_status s = stream_after(c, c->d2h_stream, st);
+  if (s != DGCL_OK) return s;
+  if (bytes)
+    CUDA_TRY(c, cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, c->d2h_stream));
+  if (src_free) CUDA_TRY(c, cudaEventRecord(src_free, c->d2h_stream));
+  if ((s = stream_after(c, st, c->d2h_stream)) != DGCL_OK) return s;
+  if (!c->host_async) CUDA_TRY(c, cudaStreamSynchronize(st));
+  return check_dead(c);
 }
 
 dgcl_status dgcl_forward_host(dgcl_ctx *c, int32_t layer, const float *host_emb, float *host_halo,
@@ -879,16 +935,15 @@ dgcl_status dgcl_forward_host(dgcl_ctx *c, int32_t layer, const float *host_emb,
   const int64_t rows = c->loopback ? c->n : c->n_local[c->rank];
   const int64_t hrows = c->loopback ? c->halo_off[c->world] : c->rel.n_halo[c->rank];
   cudaStream_t st = (cudaStream_t)stream;
-  if ((s = ensure_stage(c, &c->stage_a, &c->stage_a_bytes, rows * p * 4)) != DGCL_OK) return s;
-  if (rows > 0)
-    CUDA_TRY(c, cudaMemcpyAsync(c->stage_a, host_emb, rows * p * 4, cudaMemcpyHostToDevice, st));
-  if ((s = dgcl_dispatch_forward(c, layer, (const float *)c->stage_a, p, nullptr, stream)) != DGCL_OK)
+  dgcl_ctx::Stage *E;
+  if ((s = get_stage(c, 0, layer, rows * p * 4, &E)) != DGCL_OK) return s;
+  if ((s = stage_in(c, E, host_emb, rows * p * 4, st)) != DGCL_OK) return s;
+  if ((s = dgcl_dispatch_forward(c, layer, (const float *)E->ptr, p, nullptr, stream)) != DGCL_OK)
     return s;
+  CUDA_TRY(c, cudaEventRecord(E->free, st));
   const char *view = c->base[c->loopback ? 0 : c->rank] + c->off_halo[layer][c->loopback ? 0 : c->rank];
-  if (hrows > 0)
-    CUDA_TRY(c, cudaMemcpyAsync(host_halo, view, hrows * p * 4, cudaMemcpyDeviceToHost, st));
-  CUDA_TRY(c, cudaStreamSynchronize(st));
-  return check_dead(c);
+  // (the next call writing this halo is queued on `st` after this copy: stage_out makes `st` wait)
+  return stage_out(c, host_halo, view, hrows * p * 4, st, nullptr);
 }
 
 dgcl_status dgcl_backward_host(dgcl_ctx *c, int32_t layer, const float *host_halo_grad,
@@ -899,19 +954,16 @@ dgcl_status dgcl_backward_host(dgcl_ctx *c, int32_t layer, const float *host_hal
   const int64_t rows = c->loopback ? c->n : c->n_local[c->rank];
   const int64_t hrows = c->loopback ? c->halo_off[c->world] : c->rel.n_halo[c->rank];
   cudaStream_t st = (cudaStream_t)stream;
-  if ((s = ensure_stage(c, &c->stage_a, &c->stage_a_bytes, rows * p * 4)) != DGCL_OK) return s;
-  if ((s = ensure_stage(c, &c->stage_b, &c->stage_b_bytes, hrows * p * 4)) != DGCL_OK) return s;
-  if (hrows > 0)
-    CUDA_TRY(c, cudaMemcpyAsync(c->stage_b, host_halo_grad, hrows * p * 4, cudaMemcpyHostToDevice, st));
-  if (rows > 0)
-    CUDA_TRY(c, cudaMemcpyAsync(c->stage_a, host_emb_grad, rows * p * 4, cudaMemcpyHostToDevice, st));
-  if ((s = dgcl_dispatch_backward(c, layer, (const float *)c->stage_b, p, (float *)c->stage_a, p,
+  dgcl_ctx::Stage *G, *E;
+  if ((s = get_stage(c, 1, layer, hrows * p * 4, &G)) != DGCL_OK) return s;
+  if ((s = get_stage(c, 2, layer, rows * p * 4, &E)) != DGCL_OK) return s;
+  if ((s = stage_in(c, G, host_halo_grad, hrows * p * 4, st)) != DGCL_OK) return s;
+  if ((s = stage_in(c, E, host_emb_grad, rows * p * 4, st)) != DGCL_OK) return s;
+  if ((s = dgcl_dispatch_backward(c, layer, (const float *)G->ptr, p, (float *)E->ptr, p,
                                   stream)) != DGCL_OK)
     return s;
-  if (rows > 0)
-    CUDA_TRY(c, cudaMemcpyAsync(host_emb_grad, c->stage_a, rows * p * 4, cudaMemcpyDeviceToHost, st));
-  CUDA_TRY(c, cudaStreamSynchronize(st));
-  return check_dead(c);
+  CUDA_TRY(c, cudaEventRecord(G->free, st));
+  return stage_out(c, host_emb_grad, E->ptr, rows * p * 4, st, E->free);
 }
 
 dgcl_status dgcl_plan_info(dgcl_ctx *c, dgcl_plan_stats *info) {
@@ -985,6 +1037,10 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->registered) return fail(c, DGCL_ESTATE, "geometry must be set before registration");
     c->geometry = (int)value;
     if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "host_async") {  // host-buffer calls return once queued (see dgcl_forward_host)
+    c->host_async = value != 0;
     return DGCL_OK;
   }
   if (k == "hostsim_items") {  // verification aid: the host interpreter runs the work items
@@ -1096,8 +1152,12 @@ dgcl_status dgcl_destroy(dgcl_ctx *c) {
     cudaFree(c->d_items);
     cudaFree(c->d_runs);
     cudaFree(c->d_sterms);
-    if (c->stage_a) cudaFree(c->stage_a);
-    if (c->stage_b) cudaFree(c->stage_b);
+    for (auto &kv : c->stages) {
+      if (kv.second.ptr) cudaFree(kv.second.ptr);
+      if (kv.second.free) cudaEventDestroy(kv.second.free);
+    }
+    if (c->h2d_stream) cudaStreamDestroy(c->h2d_stream);
+    if (c->d2h_stream) cudaStreamDestroy(c->d2h_stream);
     if (c->err_host) cudaFreeHost(c->err_host);
     for (cudaStream_t s : c->rank_streams)
       if (s) cudaStreamDestroy(s);
