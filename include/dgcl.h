@@ -220,6 +220,8 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    halo gradients in place (no slot round trip); 0: push + owner reduce
  *   "direct_copy_rows" COPY items whose runs average fewer rows are gathered by the consumer
  *                    warps with plain loads (default 0 = never)
+ *   "small_launch_bytes" launches moving fewer bytes (rows x row size) run the register
+ *                    executor instead of the bulk-copy pipeline (latency; default 4 MiB, 0 = never)
  *   "host_async"     0 (default) / 1: dgcl_forward_host / dgcl_backward_host return before the
  *                    device->host copy completes (any time)
  *   "geometry"       bulk-copy launch geometry: 0 (default) auto per launch, 1 WIDE (1 CTA per

@@ -42,6 +42,7 @@ struct Program {
   int op_mask = 0;     // kMaskCopy / kMaskFold / kMaskDirect / kMaskStaged items present
   bool fold_wide = false;  // FOLD rows average >= 4 terms
   int geo = 0;             // bulk-copy launch geometry: 0 = kGeoWide, 1 = kGeoDual
+  int64_t bytes = 0;       // operand rows moved (rows x 16-B-rounded row, + fold terms)
 };
 
 }  // namespace
@@ -117,6 +118,7 @@ struct dgcl_ctx {
   std::map<int, Stage> stages;  // key: kind * 4096 + layer (kind 0 emb, 1 halo grad, 2 emb grad)
   cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;
   bool host_async = false;  // host calls return before the device->host copy completes
+  int64_t small_launch_bytes = 4 << 20;  // launches moving less use the register executor
   uint64_t launches = 0;
   int debug_skip_rank = -1;  // fault injection (per-rank loopback): never launch this rank
   bool dead = false;
@@ -335,6 +337,10 @@ void build_programs(dgcl_ctx *c) {
             if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
           }
           P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
+          P.bytes = 0;
+          for (const DevItem &it : P.items)
+            if (it.op == OP_COPY || it.op == OP_FOLD)
+              P.bytes += (int64_t)(it.rows + (it.op == OP_FOLD ? it.nterms : 0)) * row16;
         };
         if (c->geometry) {
           build(c->geometry - 1);
@@ -507,7 +513,10 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     const auto occ = c->tma_ctas.find({pg.geo, tblock});
     const int tctas = occ == c->tma_ctas.end() ? 0 : occ->second;
     int block = c->threads, grid_all = c->grid;
-    if (Pp.use_tma && Pp.row16 <= G.stage_bytes - kStageHdrBytes && tctas > 0) {
+    // latency-bound launches (a few MB) skip the bulk-copy pipeline: the register executor's
+    // single round trip per item is shorter (tiny config: 10 vs 14-19 us per launch)
+    const bool small = pg.bytes < c->small_launch_bytes;
+    if (Pp.use_tma && !small && Pp.row16 <= G.stage_bytes - kStageHdrBytes && tctas > 0) {
       block = tblock;
       grid_all = c->n_sm * tctas;
       Pp.tma_stages = G.stages;
@@ -1037,6 +1046,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->registered) return fail(c, DGCL_ESTATE, "geometry must be set before registration");
     c->geometry = (int)value;
     if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "small_launch_bytes") {  // below: register executor (latency), 0 = always bulk-copy
+    if (value < 0) return fail(c, DGCL_EINVAL, "small_launch_bytes must be >= 0");
+    c->small_launch_bytes = value;
     return DGCL_OK;
   }
   if (k == "host_async") {  // host-buffer calls return once queued (see dgcl_forward_host)

@@ -273,12 +273,14 @@ def build_plan_distributed(ctx, my_required, topology=None, seed=0, group=None):
     return ptr, ids
 
 
-def setup_distributed(part, dims, my_required, topology=None, seed=0, group=None, device=None):
+def setup_distributed(part, dims, my_required, topology=None, seed=0, group=None, device=None,
+                      options=None):
     """Collective setup over a torch.distributed process group (any backend).
 
     my_required: this rank's required vertex ids R_me (its halo row order).  The lists of all ranks
     are all-gathered so every rank runs the identical deterministic plan (no master on
     the data path); workspaces are allocated with torch, IPC blobs all-gathered and imported.
+    options: {key: value} for dgcl_set_option before planning (the same on every rank).
     """
     import torch
     import torch.distributed as dist
@@ -287,6 +289,8 @@ def setup_distributed(part, dims, my_required, topology=None, seed=0, group=None
     if device is None:
         device = torch.cuda.current_device()
     ctx = init(part, dims, rank, world, device)
+    for k, v in (options or {}).items():
+        ctx.set_option(k, v)
     build_plan_distributed(ctx, my_required, topology=topology, seed=seed, group=group)
     ctx.register_workspace()
     blobs = [None] * world

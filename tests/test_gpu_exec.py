@@ -40,7 +40,9 @@ class Case:
         D = _D()
         self.g, self.m, self.dims = g, g.m, list(dims)
         self.ctx = D.loopback(g.m, g.part, dims, device=0, flags=flags)
-        for k, v in (options or {}).items():
+        # test graphs are small: force the bulk-copy executor unless a case asks otherwise (the
+        # default hands launches under small_launch_bytes to the register executor)
+        for k, v in dict({"small_launch_bytes": 0}, **(options or {})).items():
             self.ctx.set_option(k, v)
         self.ctx.build_plan(g.req_ptr, g.req_ids, seed=seed, topology=topo)
         self.ctx.register_workspace()
@@ -135,11 +137,14 @@ def _check_case(c, layers=None, bwd=True):
         assert _eq(out, out2)
 
 
-def test_tiny_config_bit_exact():
-    """configs[0]: 10k vertices, 100k edges, random 2-way, dim 16, one layer fwd + bwd."""
+@pytest.mark.parametrize("small", [0, 4 << 20])
+def test_tiny_config_bit_exact(small):
+    """configs[0]: 10k vertices, 100k edges, random 2-way, dim 16, one layer fwd + bwd — through
+    the bulk-copy executor (small=0) and through the default latency choice (register executor
+    below 4 MiB per launch)."""
     cfg = synth.get_config("tiny")
     g = synth.make_graph(cfg.n, cfg.e, cfg.m, cfg.graph_seed, cfg.part_seed)
-    _check_case(Case(g, cfg.dims))
+    _check_case(Case(g, cfg.dims, options={"small_launch_bytes": small}))
 
 
 @pytest.mark.parametrize("m,opts", [

@@ -38,7 +38,8 @@ def _worker(rank, world, port, q, n, e, dims, topo_name):
         dist.init_process_group("gloo", rank=rank, world_size=world)
         g = synth.make_graph(n, e, world, graph_seed=77, part_seed=78)
         topo = synth.topology.by_name(topo_name, world) if topo_name else None
-        ctx = D.setup_distributed(g.part, dims, g.R(rank), topology=topo, seed=5, device=0)
+        ctx = D.setup_distributed(g.part, dims, g.R(rank), topology=topo, seed=5, device=0,
+                                  options={"small_launch_bytes": 0})  # the bulk-copy path
         ctx.set_option("timeout_ms", 120000)
         mine = np.nonzero(g.part == rank)[0]           # my global ids, loc order
         ok = True
