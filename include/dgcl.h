@@ -220,6 +220,7 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    halo gradients in place (no slot round trip); 0: push + owner reduce
  *   "direct_copy_rows" COPY items whose runs average fewer rows are gathered by the consumer
  *                    warps with plain loads (default 0 = never)
+ *   "trace"          1: record per-item timelines of every launch (dgcl_trace_read); default 0
  *   "small_launch_bytes" launches moving fewer bytes (rows x row size) run the register
  *                    executor instead of the bulk-copy pipeline (latency; default 4 MiB, 0 = never)
  *   "host_async"     0 (default) / 1: dgcl_forward_host / dgcl_backward_host return before the
@@ -235,6 +236,19 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    -1 = off)
  * EINVAL for an unknown key or bad value. */
 dgcl_status dgcl_set_option(dgcl_ctx *ctx, const char *key, int64_t value);
+
+/* Per-item timeline of the LAST launch of program (layer, dir = 0 forward / 1 backward, rank =
+ * the virtual rank for per-rank loopback contexts, ignored otherwise), recorded when option
+ * "trace" was set before dgcl_register_workspace (ESTATE otherwise).  One record per work item
+ * in launch order: %globaltimer ns when the executor reached it, when its source waits (stage
+ * chaining, ready words) were satisfied, and when its rows were stored; the SM that ran it.
+ * recs == NULL: *n = number of records.  Synchronizes the device. */
+typedef struct dgcl_trace_rec {
+  uint64_t t_start, t_ready, t_done;
+  uint32_t sm, tag;  /* op | dir << 4 | exec rank << 8 | dst rank << 16 | stage << 24 */
+} dgcl_trace_rec;
+dgcl_status dgcl_trace_read(dgcl_ctx *ctx, int32_t layer, int32_t dir, int32_t rank,
+                            dgcl_trace_rec *recs, int64_t *n);
 
 /* Number of executor kernel launches issued so far by this context. */
 dgcl_status dgcl_launch_count(dgcl_ctx *ctx, uint64_t *count);

@@ -43,6 +43,7 @@ struct Program {
   bool fold_wide = false;  // FOLD rows average >= 4 terms
   int geo = 0;             // bulk-copy launch geometry: 0 = kGeoWide, 1 = kGeoDual
   int64_t bytes = 0;       // operand rows moved (rows x 16-B-rounded row, + fold terms)
+  TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
 };
 
 }  // namespace
@@ -119,6 +120,7 @@ struct dgcl_ctx {
   cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;
   bool host_async = false;  // host calls return before the device->host copy completes
   int64_t small_launch_bytes = 4 << 20;  // launches moving less use the register executor
+  bool trace = false;                    // per-item timelines (dgcl_trace_read)
   uint64_t launches = 0;
   int debug_skip_rank = -1;  // fault injection (per-rank loopback): never launch this rank
   bool dead = false;
@@ -508,6 +510,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     Pp.op_mask = pg.op_mask;
     Pp.fold_wide = pg.fold_wide ? 1 : 0;
     Pp.n_items = (int32_t)pg.items.size();
+    Pp.trace = pg.d_trace;
     const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
     const int tblock = tma_block(c, pg);
     const auto occ = c->tma_ctas.find({pg.geo, tblock});
@@ -722,6 +725,12 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   if ((s = upload(c, &c->d_runs, all_runs)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_sterms, all_sterms)) != DGCL_OK) return s;
   c->run_bytes = (int64_t)(all_runs.size() * sizeof(DevRun) + all_sterms.size() * 4);
+  if (c->trace)
+    for (Program &p : c->progs)
+      if (!p.items.empty()) {
+        CUDA_TRY(c, cudaMalloc((void **)&p.d_trace, p.items.size() * sizeof(TraceRec)));
+        CUDA_TRY(c, cudaMemset(p.d_trace, 0, p.items.size() * sizeof(TraceRec)));
+      }
   // watchdog word in mapped host memory
   CUDA_TRY(c, cudaHostAlloc((void **)&c->err_host, 64, cudaHostAllocMapped));
   std::memset(c->err_host, 0, 64);
@@ -1048,6 +1057,10 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }
+  if (k == "trace") {  // per-item timelines of every launch (dgcl_trace_read)
+    c->trace = value != 0;
+    return DGCL_OK;
+  }
   if (k == "small_launch_bytes") {  // below: register executor (latency), 0 = always bulk-copy
     if (value < 0) return fail(c, DGCL_EINVAL, "small_launch_bytes must be >= 0");
     c->small_launch_bytes = value;
@@ -1120,6 +1133,31 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   return fail(c, DGCL_EINVAL, "unknown option %s", key);
 }
 
+dgcl_status dgcl_trace_read(dgcl_ctx *c, int32_t layer, int32_t dir, int32_t rank,
+                            dgcl_trace_rec *recs, int64_t *n) {
+  if (!c || !n) return DGCL_EINVAL;
+  if (!c->registered || !c->trace) return fail(c, DGCL_ESTATE, "tracing is off (option \"trace\")");
+  if (layer < 0 || layer >= c->n_layers || dir < 0 || dir > 1) return DGCL_EINVAL;
+  const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
+  if (fused) rank = 0;
+  else if (!c->loopback) rank = c->rank;
+  if (rank < 0 || rank >= c->n_prog_ranks) return DGCL_EINVAL;
+  const Program &pg = c->progs[c->prog_index(layer, dir, rank)];
+  const int64_t cnt = (int64_t)pg.items.size();
+  if (!recs) {
+    *n = cnt;
+    return DGCL_OK;
+  }
+  if (*n < cnt) return fail(c, DGCL_EINVAL, "trace buffer holds %lld < %lld records",
+                            (long long)*n, (long long)cnt);
+  static_assert(sizeof(dgcl_trace_rec) == sizeof(TraceRec), "trace record layout");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  CUDA_TRY(c, cudaDeviceSynchronize());
+  if (cnt) CUDA_TRY(c, cudaMemcpy(recs, pg.d_trace, cnt * sizeof(TraceRec), cudaMemcpyDeviceToHost));
+  *n = cnt;
+  return DGCL_OK;
+}
+
 dgcl_status dgcl_launch_count(dgcl_ctx *c, uint64_t *count) {
   if (!c || !count) return DGCL_EINVAL;
   *count = c->launches;
@@ -1166,6 +1204,8 @@ dgcl_status dgcl_destroy(dgcl_ctx *c) {
     cudaFree(c->d_items);
     cudaFree(c->d_runs);
     cudaFree(c->d_sterms);
+    for (Program &p : c->progs)
+      if (p.d_trace) cudaFree(p.d_trace);
     for (auto &kv : c->stages) {
       if (kv.second.ptr) cudaFree(kv.second.ptr);
       if (kv.second.free) cudaEventDestroy(kv.second.free);

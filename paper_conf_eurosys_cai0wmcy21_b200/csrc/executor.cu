@@ -182,6 +182,13 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
     const DevItem I = s_item;
     if (threadIdx.x == 0) {
       bool ok = true;
+      if (P.trace) {
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        P.trace[it].t_start = globaltimer();
+        P.trace[it].sm = smid;
+        P.trace[it].tag = trace_tag(I, P.groups[I.group].stage);
+      }
       if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer
         for (int s = 0; s < P.world; ++s)
@@ -197,6 +204,7 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
         if (ok) s_wait_ok[I.exec_rank] = I.wait_off;
       }
       s_abort = ok ? 0 : 1;
+      if (P.trace) P.trace[it].t_ready = globaltimer();
     }
     __syncthreads();
     if (s_abort) return;  // the watchdog fired; the error word is set, leave the launch
@@ -211,6 +219,10 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
       }
     } else if (I.op == OP_FOLD) {
       fold_rows<V16>(P, I);
+    }
+    if (P.trace) {
+      __syncthreads();
+      if (threadIdx.x == 0) P.trace[it].t_done = globaltimer();
     }
     if (I.flags & kItemSignal) {
       __threadfence_system();  // this thread's row stores are visible system-wide ...

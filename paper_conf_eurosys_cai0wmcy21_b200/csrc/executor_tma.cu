@@ -228,7 +228,7 @@ __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const Dev
 // stage to be free and fenced the consumers' generic reads of it against the async proxy.
 __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I,
                                            const DevItem *Ism, uint8_t *st, const uint8_t *meta,
-                                           uint64_t *full, int lane) {
+                                           uint64_t *full, int lane, uint32_t item_index) {
   const uint32_t r16 = (uint32_t)P.row16;
   // consumer tables: term_ptr window (FOLD) and destination rows (when not consecutive)
   Win wtp = {0, 0, 0}, wdst = {0, 0, 0};
@@ -239,6 +239,7 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     int32_t *info = reinterpret_cast<int32_t *>(st + kHdrInfo);
     info[0] = wtp.skew;
     info[1] = wdst.skew;
+    info[2] = (int32_t)item_index;  // (trace records)
   }
   __syncwarp();  // header and info written before lane 0's arrive publishes the stage
   if (lane == 0) mbar_expect_tx(full, operand_bytes(P, I) + wtp.bytes + wdst.bytes);
@@ -692,6 +693,14 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       const DevItem I = desc_ready(m);  // registers: no shared-memory reload per field
       const DevItem *Ism = &descs[m % kDescSlots];
       bool fenced = false;
+      const uint32_t gidx = blockIdx.x + m * G;  // the item's index in the launch
+      if (P.trace && lane == 0) {
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        P.trace[gidx].t_start = globaltimer();
+        P.trace[gidx].sm = smid;
+        P.trace[gidx].tag = trace_tag(I, P.groups[I.group].stage);
+      }
       if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer
         if (lane == 0)
@@ -745,10 +754,11 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         uint32_t stage, use;
         ring_pos(k, NS, stage, use);
         if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
+        if (P.trace && lane == 0) P.trace[gidx].t_ready = globaltimer();
         fence_proxy_async_smem();
         fenced = true;
         issue_item(P, I, Ism, stages + (size_t)stage * stage_bytes, meta_of(m), &full[stage],
-                   lane);
+                   lane, gidx);
         ++k;
         if (sig) {
           pend = true;
@@ -844,6 +854,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         else
           store_fold_multi<(kMaxThreads > 512 ? 3 : 6)>(P, I, st, tid, T);
       }
+      if (P.trace && tid == 0)  // this warp's share of the item is stored
+        P.trace[reinterpret_cast<const int32_t *>(st + kHdrInfo)[2]].t_done = globaltimer();
       if ((I.flags & kItemSignal) && tid == 0) {
         // counted now, published by the next FLUSH / END marker (done flags)
         atomicAdd(&s_pend[I.exec_rank * kMaxRanks + I.dst_rank], (uint32_t)I.rows);

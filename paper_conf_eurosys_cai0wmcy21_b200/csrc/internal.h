@@ -158,7 +158,25 @@ struct alignas(64) ExecParams {
                        // selects a kernel instance that carries only the code it needs
   int32_t fold_wide;   // FOLD rows average >= 4 terms (selects the 1024-thread fold instance)
   const uint32_t *sterms;  // staged FOLD items: operand row (in the stage) of every term
+  struct TraceRec *trace;  // option "trace": one record per item of this launch, or nullptr
 };
+
+// Per-item timeline (%globaltimer ns), written when tracing is on: the executor reached the item,
+// its source waits were satisfied (stage chaining), its rows were stored; and what it was.
+struct TraceRec {
+  uint64_t t_start, t_ready, t_done;
+  uint32_t sm, tag;  /* op | dir << 4 | exec rank << 8 | dst rank << 16 | stage << 24 */
+};
+static_assert(sizeof(TraceRec) == 32, "trace record");
+#ifdef __CUDACC__
+#define DGCL_HD __host__ __device__
+#else
+#define DGCL_HD
+#endif
+DGCL_HD inline uint32_t trace_tag(const DevItem &I, int stage) {
+  return (uint32_t)I.op | (uint32_t)I.dir << 4 | (uint32_t)I.exec_rank << 8 |
+         (uint32_t)I.dst_rank << 16 | (uint32_t)stage << 24;
+}
 constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8;
 
 // A run of `len` rows whose source rows src.. and destination rows dst.. are both consecutive;

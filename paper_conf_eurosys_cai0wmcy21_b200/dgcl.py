@@ -184,6 +184,26 @@ class Context:
                                        _host_ptr(host_emb_grad), _stream_ptr(stream)), self.handle)
 
     # ---- introspection ----------------------------------------------------------------------
+    TRACE_DTYPE = np.dtype([("t_start", "<u8"), ("t_ready", "<u8"), ("t_done", "<u8"),
+                            ("sm", "<u4"), ("tag", "<u4")])
+
+    def trace(self, layer, direction=0, rank=0):
+        """Per-item timeline of the last launch (option "trace"): a structured array with
+        t_start / t_ready / t_done (%globaltimer ns), sm, and op, dir, exec, dst, stage decoded
+        from the tag."""
+        n = ctypes.c_int64(0)
+        check(lib().dgcl_trace_read(self.handle, layer, direction, rank, None, ctypes.byref(n)),
+              self.handle)
+        rec = np.zeros(n.value, self.TRACE_DTYPE)
+        check(lib().dgcl_trace_read(self.handle, layer, direction, rank,
+                                    rec.ctypes.data if n.value else None, ctypes.byref(n)),
+              self.handle)
+        out = {k: rec[k] for k in rec.dtype.names}
+        t = rec["tag"]
+        out.update(op=t & 15, dir=(t >> 4) & 15, exec=(t >> 8) & 255, dst=(t >> 16) & 255,
+                   stage=t >> 24)
+        return out
+
     def plan_info(self):
         s = _abi.PlanStats()
         check(lib().dgcl_plan_info(self.handle, ctypes.byref(s)), self.handle)

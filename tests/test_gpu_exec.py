@@ -197,6 +197,33 @@ def test_relay_plans(name, flags, tma, sf):
     _check_case(c)
 
 
+@pytest.mark.parametrize("tma,flags", [(1, 0), (0, 0), (1, 1)])
+def test_trace_stage_causality(tma, flags):
+    """Option "trace": per-item timelines of a relay plan's forward.  Stage chaining on device
+    flags means no stage-k item of GPU r passes its waits before every stage-(k-1) item into r
+    has stored its rows; every item is traced once, in order start <= ready <= done."""
+    D = _D()
+    g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
+    c = Case(g, [40], topo=synth.topology.by_name("dgx1_like"), seed=9, flags=flags,
+             options={"tma": tma, "trace": 1})
+    K = c.ctx.plan_info()["n_stages"]
+    assert K >= 2
+    _check_case(c, bwd=False)
+    ranks = range(c.m) if flags == D.LOOPBACK_PER_RANK else [0]
+    T = [c.ctx.trace(0, 0, r) for r in ranks]
+    T = {k: np.concatenate([t[k] for t in T]) for k in T[0]}
+    data = T["op"] <= 1
+    assert data.sum() > 0 and np.all(T["t_start"][data] > 0)
+    assert np.all(T["t_start"][data] <= T["t_ready"][data])
+    assert np.all(T["t_ready"][data] <= T["t_done"][data])
+    for r in range(c.m):
+        for k in range(2, K + 1):
+            after = data & (T["exec"] == r) & (T["stage"] == k)
+            before = data & (T["dst"] == r) & (T["stage"] == k - 1)
+            if after.any() and before.any():
+                assert T["t_ready"][after].min() >= T["t_done"][before].max(), (r, k)
+
+
 def test_unaligned_pitch_scalar_path():
     g = synth.make_graph(3000, 20000, 4, graph_seed=2, part_seed=2)
     _check_case(Case(g, [5], emb_pitch=5))   # 20-B rows: not 16-B aligned -> 4-B path
