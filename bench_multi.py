@@ -113,9 +113,46 @@ def run_multi(args, metric, unit, rank, world, local_rank, ClockSampler):
     tw1 = time.time()
     ctx.check()
     launches = ctx.launch_count() - l0
+
+    # ---- e2e through the host-buffer C-ABI calls: every step copies this rank's inputs from
+    # pinned host memory and its halos / gradients back (inside the timed region) ----
+    e2e_ms, h2d, d2h = 0.0, 0, 0
+    if args.e2e_steps > 0:
+        pin = lambda t: t.cpu().pin_memory()
+        emb_p = {l: pin(a) for l, a in emb.items()}
+        hg_p = {l: pin(a) for l, a in hg.items()}
+        eg_p = {l: pin(a) for l, a in eg.items()}
+        halo_p = {l: torch.empty(n_halo, ctx.pitch(l), dtype=torch.float32).pin_memory()
+                  for l in fwd_layers}
+        h2d = sum(a.numel() * 4 for d_ in (emb_p, hg_p, eg_p) for a in d_.values())
+        d2h = sum(a.numel() * 4 for d_ in (halo_p, eg_p) for a in d_.values())
+        ctx.set_option("host_async", 1)
+
+        def e2e_step():
+            for l in fwd_layers:
+                ctx.forward_host(l, emb_p[l], halo_p[l], stream=stream)
+            for l in bwd_layers:
+                ctx.backward_host(l, hg_p[l], eg_p[l], stream=stream)
+
+        e2e_step()
+        torch.cuda.synchronize()
+        dist.barrier()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        a1.record(stream)
+        torch.cuda.synchronize()
+        dist.barrier()
+        ctx.check()
+        e2e_ms = a0.elapsed_time(a1) / args.e2e_steps
     t = torch.tensor([e0.elapsed_time(e1)] + [statistics.mean(
-        evs[k][i][0].elapsed_time(evs[k][i][1]) for k in range(K)) for i in range(len(names))],
-        dtype=torch.float64)
+        evs[k][i][0].elapsed_time(evs[k][i][1]) for k in range(K)) for i in range(len(names))] +
+        [e2e_ms], dtype=torch.float64)
+    hb = torch.tensor([float(h2d), float(d2h)], dtype=torch.float64)
+    if not share:
+        hb = hb.cuda()
+    dist.all_reduce(hb)
     if not share:
         t = t.cuda()
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -146,6 +183,13 @@ def run_multi(args, metric, unit, rank, world, local_rank, ClockSampler):
         kernels[n] = {"ms": per_op[n], "algorithmic_bytes_max_port": alg, "achieved_gbs": ach,
                       "frac": ach / NVLINK_PEER_GBS}
     dom = max(names, key=lambda n: per_op[n])
+    e2e = None
+    if args.e2e_steps > 0:
+        e2e_ms = float(t[1 + len(names)])
+        hb = hb.cpu()
+        e2e = {"value": payload / (e2e_ms * 1e-3) / 1e9, "unit": unit, "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": int(hb[0]), "d2h_bytes_per_step": int(hb[1]),
+               "note": "all ranks' host copies, max over ranks of the step time"}
     clocks = clk.summary(tw0, tw1) if clk else None
     if clocks and clocks["samples"] == 0:
         clocks = clk.summary()
@@ -168,6 +212,6 @@ def run_multi(args, metric, unit, rank, world, local_rank, ClockSampler):
                      "nominal_peak": 900.0,
                      "algorithmic_bytes_per_launch": kernels[dom]["algorithmic_bytes_max_port"],
                      "per_kernel": kernels},
-        "cpu_baseline": None, "e2e": None, "gpu_launches": int(lt[0]),
+        "cpu_baseline": None, "e2e": e2e, "gpu_launches": int(lt[0]),
         "clocks": clocks, "plan": dict(info, graph_gen_s=gen_s),
     }
