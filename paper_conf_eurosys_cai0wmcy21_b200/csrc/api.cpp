@@ -43,6 +43,7 @@ struct Program {
   bool fold_wide = false;  // FOLD rows average >= 4 terms
   int geo = 0;             // bulk-copy launch geometry: 0 = kGeoWide, 1 = kGeoDual
   int64_t bytes = 0;       // operand rows moved (rows x 16-B-rounded row, + fold terms)
+  int g4_kinds = 0;        // source kinds of its gather4 items (tensor maps the launch needs)
   TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
 };
 
@@ -225,11 +226,15 @@ void compute_layout(dgcl_ctx *c) {
         c->off_halo[l][r] = off + (size_t)c->halo_off[r] * c->pitch[l] * 4;
       off = align_up(off + (size_t)c->halo_off[m] * c->pitch[l] * 4);
     }
-    for (int l = 0; l < c->n_layers; ++l)
+    // relay staging: every layer's rows of all ranks contiguous too (one tensor map per layer)
+    for (int l = 0; l < c->n_layers; ++l) {
+      size_t rows = 0;
       for (int r = 0; r < m; ++r) {
-        c->off_relay[l][r] = off;
-        off = align_up(off + (size_t)L.n_relay[r] * c->pitch[l] * 4);
+        c->off_relay[l][r] = off + rows * c->pitch[l] * 4;
+        rows += (size_t)L.n_relay[r];
       }
+      off = align_up(off + rows * c->pitch[l] * 4);
+    }
     for (int r = 0; r < m; ++r) {
       c->off_slot[r] = off;
       off = align_up(off + (size_t)L.n_slot[r] * c->max_pitch * 4);
@@ -339,6 +344,9 @@ void build_programs(dgcl_ctx *c) {
             if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
           }
           P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
+          P.g4_kinds = 0;
+          for (const DevItem &it : P.items)
+            if (it.op == OP_COPY && (it.flags & kItemGather4)) P.g4_kinds |= 1 << it.src_kind;
           P.bytes = 0;
           for (const DevItem &it : P.items)
             if (it.op == OP_COPY || it.op == OP_FOLD)
@@ -492,17 +500,36 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage (checked
   // again per program against its geometry in launch_program)
   P.use_tma = (v16 && c->use_tma && P.row16 <= kTmaOperandBytes) ? 1 : 0;
-  // forward launches over packed embedding rows of <= 1 KB: a 2-D tensor map for the TMA row
-  // gather (gather4) used by items whose source rows come in short runs
-  if (P.use_tma && dir == DIR_FWD && c->use_gather4 && in_pitch * 4 == P.row16 &&
-      P.row16 <= kGather4MaxRowBytes) {
-    const int64_t rows = c->loopback ? c->n : c->n_local[c->rank];
-    if (rows > 0 && rows < INT32_MAX && encode_rows_tmap(c, P.tmap_emb, in, rows, P.row16)) {
-      P.use_gather4 = 1;
+  // TMA row gather (gather4) for items whose source rows come in short runs: one 2-D tensor
+  // map per source kind over the packed rows this process reads — the caller's embeddings
+  // (forward) or halo gradients (backward), and the workspace's halo / relay staging of this
+  // layer (relay forwarding).  In loopback every kind's rows of all ranks are one array (the
+  // caller's buffer, the buffer-major workspace); a rank's first row is its tensor row offset.
+  // Encoded per launch for the kinds its program uses (Program::g4_kinds).
+  auto encode_g4 = [&](ExecParams &Q, int kinds) {
+    Q.gather4_mask = 0;
+    if (!Q.use_tma || !c->use_gather4 || Q.row16 > kGather4MaxRowBytes || Q.row16 % 32) return;
+    const int me = c->loopback ? 0 : c->rank;
+    for (int k = 0; k < kG4Kinds; ++k) {
+      if (!((kinds >> k) & 1)) continue;
+      const BufRef &B0 = Q.buf[k][me];
+      if (!B0.ptr || B0.pitch != Q.row16) continue;
+      int64_t rows = 0;
+      if (k == in_kind)
+        rows = c->loopback ? (dir == DIR_FWD ? c->n : c->halo_off[m])
+                           : (dir == DIR_FWD ? c->n_local[c->rank] : c->rel.n_halo[c->rank]);
+      else if (k == K_HALO)
+        rows = c->loopback ? c->halo_off[m] : c->rel.n_halo[c->rank];
+      else if (k == K_RELAY)
+        for (int r = 0; r < m; ++r)
+          rows += (c->loopback || r == c->rank) ? c->low.n_relay[r] : 0;
+      if (rows <= 0 || rows >= INT32_MAX || !encode_rows_tmap(c, Q.tmap[k], B0.ptr, rows, Q.row16))
+        continue;
+      Q.gather4_mask |= 1 << k;
       for (int r = 0; r < m; ++r)
-        P.tmap_row_off[r] = c->loopback ? (int32_t)c->row_off[r] : 0;
+        Q.tmap_row_off[k][r] = c->loopback ? (int32_t)((Q.buf[k][r].ptr - B0.ptr) / Q.row16) : 0;
     }
-  }
+  };
   // one program's launch: its items, kernel instance, CTA shape and bulk-copy geometry
   auto launch_program = [&](const Program &pg, int grid_div, cudaStream_t st) -> int {
     ExecParams Pp = P;
@@ -527,8 +554,8 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
       Pp.meta_bytes = G.meta_bytes;
     } else {
       Pp.use_tma = 0;
-      Pp.use_gather4 = 0;
     }
+    encode_g4(Pp, pg.g4_kinds);
     const int grid = (int)std::min<int64_t>(std::max(1, grid_all / grid_div), Pp.n_items);
     return launch_executor(Pp, grid, block, st);
   };

@@ -162,7 +162,8 @@ __device__ __forceinline__ Win window(int64_t off, int64_t n, int sz) {
 
 // COPY item gathered four rows per TMA instruction (tile::gather4 through the launch's tensor map)
 __device__ __forceinline__ bool uses_gather4(const ExecParams &P, const DevItem &I) {
-  return P.use_gather4 && (I.flags & kItemGather4) && I.op == OP_COPY && I.src < 0;
+  return (I.flags & kItemGather4) && I.op == OP_COPY && I.src < 0 && I.src_kind < kG4Kinds &&
+         ((P.gather4_mask >> I.src_kind) & 1);
 }
 
 __device__ __forceinline__ void tma_gather4(void *sdst, const void *tmap, int32_t col, int32_t r0,
@@ -260,11 +261,12 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     // the padding rows, the consumers never store them)
     const int32_t *sidx = reinterpret_cast<const int32_t *>(meta) +
                           (int32_t)(~I.src - window(~I.src, I.rows, 4).a);
-    const int32_t base = P.tmap_row_off[I.exec_rank];
+    const int32_t base = P.tmap_row_off[I.src_kind][I.exec_rank];
+    const void *tmap = P.tmap[I.src_kind];
     const int ng = (I.rows + 3) / 4;
     for (int g = lane; g < ng; g += 32) {
       const int r = 4 * g, last = I.rows - 1;
-      tma_gather4(ops + (size_t)r * r16, P.tmap_emb, 0, base + sidx[r],
+      tma_gather4(ops + (size_t)r * r16, tmap, 0, base + sidx[r],
                   base + sidx[min(r + 1, last)], base + sidx[min(r + 2, last)],
                   base + sidx[min(r + 3, last)], full);
     }

@@ -27,6 +27,10 @@ enum Kind : int32_t {
   K_NKINDS = 6
 };
 
+// source kinds a COPY item may gather with tile::gather4 (tensor map per kind, ExecParams::tmap)
+constexpr int kG4Kinds = 4;
+static_assert(K_EMB == 0 && K_HALO == 1 && K_RELAY == 2 && K_HGRAD == 3, "gather4 kinds");
+
 enum Op : int32_t {
   OP_COPY = 0,   // dst[dst_row(i)] = src[src_row(i)]
   OP_FOLD = 1,   // dst[dst_row(i)] = fold(init ? dst : -, terms(i)) in order, fp32 adds
@@ -101,7 +105,7 @@ struct alignas(16) DevItem {
 static_assert(sizeof(DevItem) == 64, "DevItem is one 64-B descriptor");
 constexpr uint8_t kItemSignal = 1;
 constexpr uint8_t kItemDirect = 2;  // COPY: consumers gather rows themselves (short row runs)
-constexpr uint8_t kItemGather4 = 4; // COPY from embeddings with short runs: TMA gather4 of rows
+constexpr uint8_t kItemGather4 = 4; // COPY with short source runs (kind < kG4Kinds): TMA gather4
 // FOLD whose operand rows are all bulk-copied into the stage (bulk-copy executor only; the
 // register executor ignores the flag): src = (segments << 40) | first segment in the run pool,
 // t0 = first staged term (shared-memory row of each term, per-program pool `sterms`)
@@ -121,11 +125,12 @@ struct BufRef {
 };
 
 struct alignas(64) ExecParams {
-  // 2-D tensor map (CUtensorMap, 128 B) over the embedding rows of this launch, for the
+  // 2-D tensor maps (CUtensorMap, 128 B) over the packed rows of the source buffers of this
+  // launch — embeddings, halos, relay staging, halo gradients (index = buffer kind) — for the
   // row-gather TMA (cp.async.bulk.tensor ... tile::gather4: four arbitrary rows per instruction)
-  alignas(64) unsigned char tmap_emb[128];
-  int32_t use_gather4;              // tmap_emb valid for this launch
-  int32_t tmap_row_off[kMaxRanks];  // first tensor row of each rank's embeddings
+  alignas(64) unsigned char tmap[kG4Kinds][128];
+  int32_t gather4_mask;                       // bit k: tmap[k] valid for this launch
+  int32_t tmap_row_off[kG4Kinds][kMaxRanks];  // first tensor row of each rank's rows of kind k
   BufRef buf[K_NKINDS][kMaxRanks];
   uint64_t *flags[kMaxRanks];  // flag region of every rank (peer-mapped in multi-GPU mode)
   const DevGroup *groups;

@@ -642,11 +642,12 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         if (g.op == OP_COPY && direct_copy_rows > 0 &&
             (int64_t)it.nterms * direct_copy_rows > (int64_t)it.rows)
           it.flags |= kItemDirect;
-        // rows from the embeddings with short runs (< 4 rows on average) and rows that fit one
-        // tensor box: gather four rows per TMA instruction instead of one bulk copy per run
-        // (used only when the launch provides the tensor map, see ExecParams::use_gather4)
+        // source rows in short runs (< 4 rows on average) of embeddings, halos (relay
+        // forwarding), relay staging or halo gradients, rows that fit one tensor box: gather four
+        // rows per TMA instruction instead of one bulk copy per run (used only when the launch
+        // provides the kind's tensor map, see ExecParams::gather4_mask)
         // (a 4-row group must start 128-B aligned in shared memory: row16 % 32 == 0)
-        else if (g.op == OP_COPY && g.src_kind == K_EMB && g.src_idx >= 0 &&
+        else if (g.op == OP_COPY && g.src_kind < kG4Kinds && g.src_idx >= 0 &&
                  row16 <= kGather4MaxRowBytes && row16 % 32 == 0 &&
                  (int64_t)it.nterms * 4 > (int64_t)it.rows)
           it.flags |= kItemGather4;
