@@ -212,10 +212,15 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "ctas_per_sm"    executor CTAs per SM (default: occupancy, max 4)
  *   "threads"        executor CTA size (128..512, multiple of 32; default 512)
  *   "gather4"        1 (default): TMA tile::gather4 (four rows per instruction) for short-run
- *                    embedding gathers with rows <= 1 KB
+ *                    row gathers (embeddings, halos, relay staging, halo gradients), rows <= 1 KB
  *   "stage_fold"     1 (default): backward folds bulk-copy all their operand rows into shared
  *                    memory (segments of consecutive rows) before adding them; 0: consumers
  *                    gather the operands with plain loads
+ *   "atomic_backward" 0 (default) / 1: ABLATION ONLY (the paper's "Atomic" baseline, Table 9
+ *                    P:2531-2537): a fused loopback with a single-stage plan runs the backward as
+ *                    requesters adding their halo-gradient rows into the owners' rows with atomic
+ *                    reductions (TMA bulk reduce-add).  The sum is the same but its order is not
+ *                    fixed, so results may differ from the fixed-order fold in the last bits
  *   "direct_reduce"  1 (default): fused loopback with a single-stage plan folds the requesters'
  *                    halo gradients in place (no slot round trip); 0: push + owner reduce
  *   "direct_copy_rows" COPY items whose runs average fewer rows are gathered by the consumer

@@ -92,6 +92,7 @@ struct dgcl_ctx {
   std::vector<Program> progs;  // index prog_index(layer, dir, r)
   std::vector<int32_t> host_gids[2];  // group order of the host interpreter per direction
   bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
+  bool atomic_backward = false;       // ablation: loopback backward with atomic adds
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
@@ -290,7 +291,7 @@ void build_programs(dgcl_ctx *c) {
       for (int gi = 0; gi < ng; ++gi) {
         const DevGroup &g = L.groups[gi];
         if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
-        if (gi >= L.direct_begin && gi < L.direct_end) continue;
+        if (gi >= L.direct_begin && gi < L.atomic_end) continue;
         if (!fused && g.exec_rank != r) continue;
         gids[r].push_back(gi);
       }
@@ -300,21 +301,27 @@ void build_programs(dgcl_ctx *c) {
       }
     }
     // fused loopback, single-stage plan: the owner folds its requesters' halo gradients in place
-    const bool direct = fused && dir == DIR_BWD && c->direct_reduce && L.n_stages <= 1 &&
-                        L.direct_end > L.direct_begin;
-    if (direct) {
+    // (ablation, option "atomic_backward": requesters add their rows into the owners' rows with
+    // atomic reductions instead)
+    const bool atomic = fused && dir == DIR_BWD && c->atomic_backward && L.n_stages <= 1 &&
+                        L.atomic_end > L.direct_end;
+    const bool direct = !atomic && fused && dir == DIR_BWD && c->direct_reduce &&
+                        L.n_stages <= 1 && L.direct_end > L.direct_begin;
+    if (direct || atomic) {
       gids[0].clear();
-      for (int gi = L.direct_begin; gi < L.direct_end; ++gi) gids[0].push_back(gi);
+      for (int gi = atomic ? L.direct_end : L.direct_begin; gi < (atomic ? L.atomic_end : L.direct_end);
+           ++gi)
+        gids[0].push_back(gi);
     }
     // the host interpreter runs the fused-order program of this direction
     c->host_gids[dir].clear();
-    if (direct) {
+    if (direct || atomic) {
       c->host_gids[dir] = gids[0];
     } else {
       for (int gi = 0; gi < ng; ++gi) {
         const DevGroup &g = L.groups[gi];
         if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
-        if (gi >= L.direct_begin && gi < L.direct_end) continue;
+        if (gi >= L.direct_begin && gi < L.atomic_end) continue;
         c->host_gids[dir].push_back(gi);
       }
     }
@@ -1137,6 +1144,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "stage_fold") {  // bulk-copy FOLD operand rows into the stage (bulk-copy executor)
     c->stage_fold = value != 0;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "atomic_backward") {  // ablation: loopback single-stage backward with atomic adds
+    c->atomic_backward = value != 0;
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }

@@ -73,6 +73,23 @@ __device__ __forceinline__ void copy_rows_v16(const ExecParams &P, const DevItem
   }
 }
 
+// ---- OP_COPY with atomic adds (ablation, option "atomic_backward"): one fp32 atomic per word --
+__device__ __forceinline__ void copy_rows_atomic(const ExecParams &P, const DevItem &I) {
+  const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
+  const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
+  char *dbase = P.buf[I.dst_kind][I.dst_rank].ptr;
+  const int64_t dpitch = P.buf[I.dst_kind][I.dst_rank].pitch;
+  const int32_t *sidx = idx_of(P, I.src), *didx = idx_of(P, I.dst);
+  const uint32_t dim = (uint32_t)P.row_bytes / 4;
+  const uint32_t total = (uint32_t)I.rows * dim;
+  for (uint32_t e = threadIdx.x; e < total; e += blockDim.x) {
+    const uint32_t r = e / dim, w = e - r * dim;
+    const float v = *reinterpret_cast<const float *>(sbase + row_of(sidx, I.src, r) * spitch +
+                                                     (int64_t)w * 4);
+    atomicAdd(reinterpret_cast<float *>(dbase + row_of(didx, I.dst, r) * dpitch) + w, v);
+  }
+}
+
 // ---- OP_COPY, 4-byte path (unaligned pitches) ---------------------------------------------
 template <bool kNC>
 __device__ __forceinline__ void copy_rows_b32(const ExecParams &P, const DevItem &I) {
@@ -208,7 +225,9 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
     }
     __syncthreads();
     if (s_abort) return;  // the watchdog fired; the error word is set, leave the launch
-    if (I.op == OP_COPY) {
+    if (I.op == OP_COPY && (I.flags & kItemAtomic)) {
+      copy_rows_atomic(P, I);
+    } else if (I.op == OP_COPY) {
       const bool nc = readonly_kind(I.src_kind);
       if (V16) {
         if (nc) copy_rows_v16<true>(P, I);

@@ -93,6 +93,13 @@ __device__ __forceinline__ void bulk_s2g(void *gdst, const void *ssrc, uint32_t 
                "r"(smem_u32(ssrc)), "r"(bytes)
                : "memory");
 }
+// TMA bulk reduction: dst[i] += src[i] (fp32, element-wise atomic in L2) for `bytes` (16-B multiple)
+__device__ __forceinline__ void bulk_s2g_add_f32(void *gdst, const void *ssrc, uint32_t bytes) {
+  asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(
+                   gdst),
+               "r"(smem_u32(ssrc)), "r"(bytes)
+               : "memory");
+}
 __device__ __forceinline__ void bulk_commit() {
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
@@ -354,6 +361,38 @@ __device__ __forceinline__ void store_copy(const ExecParams &P, const DevItem &I
         }
       }
     }
+  }
+}
+
+// consumers: COPY item ADDED into its destination rows (ablation, option "atomic_backward"): every
+// consumer thread takes whole rows, one TMA bulk reduce-add (fp32 add in L2, atomic per element)
+// for the row's 16-B chunks and fp32 atomics for a partial last chunk (the destination is the
+// caller's emb_grad: nothing past the row is touched)
+__device__ __forceinline__ void store_copy_atomic(const ExecParams &P, const DevItem &I,
+                                                  const uint8_t *st, uint32_t tid, uint32_t T) {
+  const BufRef D = P.buf[I.dst_kind][I.dst_rank];
+  const int32_t *tab = I.dst < 0 ? reinterpret_cast<const int32_t *>(st + kTabDst) +
+                                       reinterpret_cast<const int32_t *>(st + kHdrInfo)[1]
+                                 : nullptr;
+  const uint32_t r16 = (uint32_t)P.row16;
+  const uint8_t *ops = st + kStageHdrBytes;
+  const uint32_t body = (uint32_t)P.row_bytes & ~15u;
+  const int tailw = (P.row_bytes - (int)body) / 4;
+  bool issued = false;
+  for (uint32_t r = tid; r < (uint32_t)I.rows; r += T) {
+    const int64_t drow = tab ? (int64_t)tab[r] : I.dst + r;
+    char *dp = D.ptr + drow * D.pitch;
+    if (body) {
+      bulk_s2g_add_f32(dp, ops + r * r16, body);
+      issued = true;
+    }
+    for (int w = 0; w < tailw; ++w)
+      atomicAdd(reinterpret_cast<float *>(dp + body) + w,
+                reinterpret_cast<const float *>(ops + r * r16 + body)[w]);
+  }
+  if (issued) {
+    bulk_commit();
+    bulk_wait_read();  // the stage may be reused once the reductions have read it
   }
 }
 
@@ -825,7 +864,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       // the launch's items, so e.g. a forward launch carries no fold code / registers)
       if ((kMask & kMaskCopy) && I.op == OP_COPY && !(I.flags & kItemDirect)) {
         const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
-        if (P.bulk_store && I.dst >= 0 && DB.pitch == (int64_t)P.row16) {
+        if (I.flags & kItemAtomic) {
+          store_copy_atomic(P, I, st, tid, T);
+        } else if (P.bulk_store && I.dst >= 0 && DB.pitch == (int64_t)P.row16) {
           // consecutive packed destination rows: kStoreSplit bulk (TMA) stores move the item,
           // issued by consumer warps (k * kStoreSplit + j) % n_cons_warps, so the stores of
           // several stages overlap while the other warps move on

@@ -32,7 +32,10 @@ void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim
     if (g.op == OP_COPY) {
       const int64_t srow = g.src_idx >= 0 ? low.idx[g.src_idx + i] : g.src_base + i;
       const float *s = row_ptr(B, g.src_kind, g.exec_rank, srow);
-      std::memcpy(d, s, sizeof(float) * dim);
+      if (g.atomic_add)
+        for (int c = 0; c < dim; ++c) d[c] += s[c];
+      else
+        std::memcpy(d, s, sizeof(float) * dim);
     } else {
       const int64_t t0 = low.term_ptr[g.term_ptr + i], t1 = low.term_ptr[g.term_ptr + i + 1];
       auto operand = [&](uint32_t term) -> const float * {
@@ -72,9 +75,14 @@ bool run_item(const Lowered &low, const DevItem &it, const std::vector<DevRun> &
       const DevRun &R = runs[it.tp + q];
       if (R.pos != covered || R.len < 1) return false;
       covered += R.len;
-      for (int32_t j = 0; j < R.len; ++j)
-        std::memcpy(row_ptr(B, it.dst_kind, it.dst_rank, R.dst + j),
-                    row_ptr(B, it.src_kind, it.exec_rank, R.src + j), sizeof(float) * dim);
+      for (int32_t j = 0; j < R.len; ++j) {
+        float *d = row_ptr(B, it.dst_kind, it.dst_rank, R.dst + j);
+        const float *s = row_ptr(B, it.src_kind, it.exec_rank, R.src + j);
+        if (it.flags & kItemAtomic)
+          for (int c = 0; c < dim; ++c) d[c] += s[c];
+        else
+          std::memcpy(d, s, sizeof(float) * dim);
+      }
     }
     return covered == it.rows;
   }

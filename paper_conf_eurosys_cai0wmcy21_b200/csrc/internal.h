@@ -74,7 +74,7 @@ struct DevGroup {
   int32_t wait_off;    // waits[wait_off .. wait_off + wait_n) on exec_rank's counters
   int32_t wait_n;
   int32_t term_mode;   // OP_FOLD terms: kTermLocal (SLOT/HGRAD of exec) or kTermRankHgrad
-  int32_t pad2;
+  int32_t atomic_add;  // OP_COPY: add the rows into the destination with atomics (ablation)
   int64_t n_rows;
   int64_t src_idx;     // offset into idx pool, or -1 => rows src_base + i
   int64_t src_base;
@@ -110,6 +110,9 @@ constexpr uint8_t kItemGather4 = 4; // COPY with short source runs (kind < kG4Ki
 // register executor ignores the flag): src = (segments << 40) | first segment in the run pool,
 // t0 = first staged term (shared-memory row of each term, per-program pool `sterms`)
 constexpr uint8_t kItemStaged = 8;
+// COPY whose rows are ADDED into the destination with atomic reductions (the paper's atomic
+// backward baseline, Table 9; ablation only: the order of the adds is not fixed)
+constexpr uint8_t kItemAtomic = 16;
 constexpr int kSegShift = 40;
 constexpr int kGather4MaxRowBytes = 1024;  // one tensor box (<= 256 fp32) per row
 

@@ -405,6 +405,36 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     }
   }
   L.direct_end = (int)L.groups.size();
+  // ---- loopback atomic backward (ablation, single-stage plans only) ----
+  // The paper's "Atomic" baseline (§6.2, Table 9): every requester adds
+  // its halo-gradient rows straight into the owner's rows with atomic reductions, one group per
+  // (requester c, owner p), rows in c's halo order (consecutive source rows).  Same sum, but the
+  // order of the adds is whatever the hardware makes it: not reproducible bit for bit.
+  if (K <= 1) {
+    std::vector<std::vector<std::pair<int64_t, int64_t>>> pairs((size_t)m * m);  // (pos_c, loc)
+    for (int64_t vi = 0; vi < NV; ++vi) {
+      const int64_t u = plan.order[vi];
+      for (int64_t q = rel.d_ptr[u]; q < rel.d_ptr[u + 1]; ++q)
+        pairs[(size_t)rel.d_gpu[q] * m + part[u]].push_back({rel.d_pos[q], loc[u]});
+    }
+    for (int c = 0; c < m; ++c)
+      for (int p = 0; p < m; ++p) {
+        auto &v = pairs[(size_t)c * m + p];
+        if (v.empty()) continue;
+        std::sort(v.begin(), v.end());
+        DevGroup g = base_group(OP_COPY, DIR_BWD, c, p, 1);
+        g.src_kind = K_HGRAD;
+        g.dst_kind = K_EGRAD;
+        g.atomic_add = 1;
+        std::vector<int64_t> src, dst;
+        for (auto &x : v) {
+          src.push_back(x.first);
+          dst.push_back(x.second);
+        }
+        flush_group(L.groups, g, src, dst);
+      }
+  }
+  L.atomic_end = (int)L.groups.size();
   L.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
 }
 
@@ -662,7 +692,8 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         // optional: items whose runs average fewer than `direct_copy_rows` rows are gathered by
         // the consumers with plain loads instead of one bulk copy per run (0 = never; measured
         // slower than per-row bulk copies on the BASELINE graphs)
-        if (g.op == OP_COPY && direct_copy_rows > 0 &&
+        if (g.atomic_add) it.flags |= kItemAtomic;
+        if (g.op == OP_COPY && direct_copy_rows > 0 && !g.atomic_add &&
             (int64_t)it.nterms * direct_copy_rows > (int64_t)it.rows)
           it.flags |= kItemDirect;
         // source rows in short runs (< 4 rows on average) of embeddings, halos (relay

@@ -64,6 +64,7 @@ struct Lowered {
   std::vector<DevGroup> groups;          // forward, backward, READY/WAIT, then direct-reduce
   int n_fwd_groups = 0;
   int direct_begin = 0, direct_end = 0;  // loopback direct-reduce backward groups (direct plans)
+  int atomic_end = 0;  // [direct_end, atomic_end): loopback atomic-add backward groups (ablation)
   std::vector<int32_t> idx;              // row index pool
   std::vector<int64_t> term_ptr;         // fold row pointers
   std::vector<uint32_t> terms;           // fold terms

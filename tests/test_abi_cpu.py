@@ -134,11 +134,14 @@ def _check_lowering(g, dims, topo, seed, options=None):
     return info
 
 
-@pytest.mark.parametrize("m,direct", [(2, 1), (3, 1), (8, 1), (3, 0), (8, 0)])
+@pytest.mark.parametrize("m,direct", [(2, 1), (3, 1), (8, 1), (3, 0), (8, 0), (3, 2), (8, 2)])
 def test_uniform_plan_and_lowering(m, direct):
-    """direct=1: loopback in-place reduce program; direct=0: push to slots + owner reduce."""
+    """direct=1: loopback in-place reduce program; direct=0: push to slots + owner reduce;
+    direct=2: the atomic-add ablation's groups (one per (requester, owner), run by the host in
+    requester order, i.e. the flat order)."""
     g = synth.make_graph(1500, 12000, m, graph_seed=m, part_seed=50 + m)
-    info = _check_lowering(g, [16, 5], None, seed=3, options={"direct_reduce": direct})
+    opts = {"atomic_backward": 1} if direct == 2 else {"direct_reduce": direct}
+    info = _check_lowering(g, [16, 5], None, seed=3, options=opts)
     assert info["n_stages"] == 1 and info["n_relay_rows"] == 0
 
 

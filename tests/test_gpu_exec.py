@@ -435,3 +435,35 @@ def test_wide_rows(dims):
     stage, so the register executor runs the launch."""
     g = synth.make_graph(600, 3000, 3, graph_seed=81, part_seed=82)
     _check_case(Case(g, dims))
+
+
+@pytest.mark.parametrize("small,dims", [(0, [64, 602]), (4 << 20, [16]), (0, [5])])
+def test_atomic_backward_ablation(small, dims):
+    """Option "atomic_backward" (ablation: the paper's Atomic baseline, Table 9):
+    requesters add their halo-gradient rows into the owners' rows with atomic reductions (TMA
+    bulk reduce-add; fp32 atomics for partial chunks and on the register path).  The order of
+    the adds is not fixed, so random inputs are held to the R6 tolerance against the flat
+    oracle; integer-valued inputs (every partial sum exact) must match bit for bit, and the
+    caller's emb_grad padding (pitch > dim) is never touched."""
+    g = synth.make_graph(6000, 60000, 4, graph_seed=21, part_seed=22)
+    c = Case(g, dims, seed=1, options={"atomic_backward": 1, "small_launch_bytes": small})
+    for layer, dim in enumerate(dims):
+        G, L = c.grads(layer)
+        p = c.pitch(layer)
+        if p > dim:
+            L[:, dim:] = 7.0
+        out = c.run_backward(layer, G, L)
+        if p > dim:
+            assert np.all(out[:, dim:] == 7.0)
+        Bf = halo.backward_flat(c.local(L, dim), c.halos(G, dim), c.R, c.g.part, c.loc)
+        absL = [np.abs(x) for x in c.local(L, dim)]
+        absG = [np.abs(x) for x in c.halos(G, dim)]
+        bound = halo.backward_flat(absL, absG, c.R, c.g.part, c.loc)
+        for d in range(c.m):
+            diff = np.abs(c.local(out, dim)[d].astype(np.float64) - Bf[d])
+            assert np.all(diff <= 1e-6 * bound[d]), "atomic tolerance rank %d" % d
+        Gi, Li = c.grads(layer, mode="int")
+        outi = c.run_backward(layer, Gi, Li)
+        Bi = halo.backward_flat(c.local(Li, dim), c.halos(Gi, dim), c.R, c.g.part, c.loc)
+        for d in range(c.m):
+            assert _eq(c.local(outi, dim)[d], Bi[d]), "atomic integer inputs rank %d" % d
