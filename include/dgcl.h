@@ -216,6 +216,11 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "stage_fold"     1 (default): backward folds bulk-copy all their operand rows into shared
  *                    memory (segments of consecutive rows) before adding them; 0: consumers
  *                    gather the operands with plain loads
+ *   "fanout"         0 (default) / 1: forward stage 1 as one fan-out item stream per owner — each
+ *                    embedding row read once and stored into every first-hop receiver's row
+ *                    (kernel-level communication fusion) — instead of one COPY group
+ *                    per (owner, receiver).  Same result; measured slower on one B200 (the
+ *                    per-pair groups write long contiguous destination runs with TMA stores)
  *   "atomic_backward" 0 (default) / 1: ABLATION ONLY (the paper's "Atomic" baseline, Table 9
  *                    P:2531-2537): a fused loopback with a single-stage plan runs the backward as
  *                    requesters adding their halo-gradient rows into the owners' rows with atomic

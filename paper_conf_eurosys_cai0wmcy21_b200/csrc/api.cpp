@@ -93,6 +93,7 @@ struct dgcl_ctx {
   std::vector<int32_t> host_gids[2];  // group order of the host interpreter per direction
   bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
   bool atomic_backward = false;       // ablation: loopback backward with atomic adds
+  bool fanout = false;                // forward stage 1 as per-owner fan-out items (option)
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
@@ -279,8 +280,14 @@ void build_programs(dgcl_ctx *c) {
   c->n_prog_ranks = fused ? 1 : m;
   c->progs.assign((size_t)c->n_layers * 2 * c->n_prog_ranks, Program());
   const int ng = (int)L.groups.size();
+  // forward stage 1 as one fan-out group per owner (each row read once, stored into all its
+  // first-hop receivers) instead of one COPY group per (owner, receiver); per layer below
+  const bool fan_avail = c->fanout && L.fanout_end > L.atomic_end;
+  auto is_stage1_copy = [&](const DevGroup &g) {
+    return g.dir == DIR_FWD && g.op == OP_COPY && g.stage == 1 && g.src_kind == K_EMB;
+  };
   for (int dir = 0; dir < 2; ++dir) {
-    std::vector<std::vector<int32_t>> gids(c->n_prog_ranks);
+    std::vector<std::vector<int32_t>> gids(c->n_prog_ranks), gids_fan(c->n_prog_ranks);
     for (int r = 0; r < c->n_prog_ranks; ++r) {
       const bool want_rank = c->loopback || r == c->rank;
       if (!fused && !want_rank) continue;
@@ -288,16 +295,24 @@ void build_programs(dgcl_ctx *c) {
         for (int gi = 0; gi < ng; ++gi)
           if (L.groups[gi].op == OP_READY && L.groups[gi].exec_rank == r) gids[r].push_back(gi);
       }
+      gids_fan[r] = gids[r];
+      if (dir == DIR_FWD && fan_avail)
+        for (int gi = L.atomic_end; gi < L.fanout_end; ++gi)
+          if (fused || L.groups[gi].exec_rank == r) gids_fan[r].push_back(gi);
       for (int gi = 0; gi < ng; ++gi) {
         const DevGroup &g = L.groups[gi];
         if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
-        if (gi >= L.direct_begin && gi < L.atomic_end) continue;
+        if (gi >= L.direct_begin && gi < L.fanout_end) continue;
         if (!fused && g.exec_rank != r) continue;
         gids[r].push_back(gi);
+        if (!(fan_avail && is_stage1_copy(g))) gids_fan[r].push_back(gi);
       }
       if (!fused && dir == DIR_FWD && m > 1) {
         for (int gi = 0; gi < ng; ++gi)
-          if (L.groups[gi].op == OP_WAIT && L.groups[gi].exec_rank == r) gids[r].push_back(gi);
+          if (L.groups[gi].op == OP_WAIT && L.groups[gi].exec_rank == r) {
+            gids[r].push_back(gi);
+            gids_fan[r].push_back(gi);
+          }
       }
     }
     // fused loopback, single-stage plan: the owner folds its requesters' halo gradients in place
@@ -318,21 +333,28 @@ void build_programs(dgcl_ctx *c) {
     if (direct || atomic) {
       c->host_gids[dir] = gids[0];
     } else {
+      if (dir == DIR_FWD && fan_avail)
+        for (int gi = L.atomic_end; gi < L.fanout_end; ++gi) c->host_gids[dir].push_back(gi);
       for (int gi = 0; gi < ng; ++gi) {
         const DevGroup &g = L.groups[gi];
         if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
-        if (gi >= L.direct_begin && gi < L.atomic_end) continue;
+        if (gi >= L.direct_begin && gi < L.fanout_end) continue;
+        if (fan_avail && is_stage1_copy(g)) continue;
         c->host_gids[dir].push_back(gi);
       }
     }
     for (int l = 0; l < c->n_layers; ++l) {
       for (int r = 0; r < c->n_prog_ranks; ++r) {
         Program &P = c->progs[c->prog_index(l, dir, r)];
-        const std::vector<uint8_t> need = needed_counters(L, gids[r]);
         const int64_t row_bytes = (int64_t)c->dims[l] * 4, row16 = (row_bytes + 15) / 16 * 16;
+        // fan-out items stage a row plus its destination words: rows up to half a DUAL stage
+        const bool fan = fan_avail && dir == DIR_FWD && 2 * (row16 + 128) <= kGeoDual.stage_bytes -
+                                                                               kStageHdrBytes;
+        const std::vector<int32_t> &G = fan ? gids_fan[r] : gids[r];
+        const std::vector<uint8_t> need = needed_counters(L, G);
         auto build = [&](int geo) {
           P.geo = geo;
-          build_items(L, gids[r], row_bytes,
+          build_items(L, G, row_bytes,
                       item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
                                   (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm),
                       !fused, need,
@@ -349,6 +371,7 @@ void build_programs(dgcl_ctx *c) {
               fold_terms += it.nterms;
             }
             if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
+            if (it.op == OP_FANOUT) P.op_mask |= kMaskFanout;
           }
           P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
           P.g4_kinds = 0;
@@ -358,6 +381,8 @@ void build_programs(dgcl_ctx *c) {
           for (const DevItem &it : P.items)
             if (it.op == OP_COPY || it.op == OP_FOLD)
               P.bytes += (int64_t)(it.rows + (it.op == OP_FOLD ? it.nterms : 0)) * row16;
+            else if (it.op == OP_FANOUT)
+              P.bytes += (int64_t)(it.rows + it.nterms) * row16;
         };
         if (c->geometry) {
           build(c->geometry - 1);
@@ -373,11 +398,15 @@ void build_programs(dgcl_ctx *c) {
         bool waits = false;
         for (const DevItem &it : P.items) {
           waits = waits || (it.wait_n > 0 && (it.op == OP_COPY || it.op == OP_FOLD));
+          if (it.op == OP_FANOUT) {  // one bulk copy per item
+            bytes += (int64_t)it.rows * row16;
+            ops += 1;
+          }
           if (it.op != OP_COPY) continue;
           bytes += (int64_t)it.rows * row16;
           ops += (it.flags & kItemGather4) ? (it.rows + 3) / 4 : it.nterms;
         }
-        const bool copy_only = (P.op_mask & ~kMaskCopy) == 0;
+        const bool copy_only = (P.op_mask & ~(kMaskCopy | kMaskFanout)) == 0;
         if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & kMaskFold) || waits)
           build(0);
       }
@@ -1144,6 +1173,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "stage_fold") {  // bulk-copy FOLD operand rows into the stage (bulk-copy executor)
     c->stage_fold = value != 0;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "fanout") {  // forward stage 1: per-owner fan-out items (1) or per-pair COPY items (0)
+    c->fanout = value != 0;
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }

@@ -182,6 +182,31 @@ __device__ __forceinline__ void fold_rows(const ExecParams &P, const DevItem &I)
   }
 }
 
+// ---- OP_FANOUT: flat (destination pair, chunk) space — each pair (dest word, source row) copies
+// the source row into one receiver's row (halo / relay staging, library-owned: whole chunks) ----
+template <bool V16>
+__device__ __forceinline__ void fanout_rows(const ExecParams &P, const DevItem &I,
+                                            uint32_t *s_cnt) {
+  const BufRef S = P.buf[I.src_kind][I.exec_rank];
+  const uint32_t *pw = P.terms + I.t0;
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)(I.nterms >> 1) * nch;
+  const bool sig = (I.flags & kItemSignal) != 0;
+  for (uint32_t e = threadIdx.x; e < total; e += blockDim.x) {
+    const uint32_t j = fdiv(e, P);
+    const uint32_t col = e - j * nch;
+    const uint32_t d = __ldg(pw + 2 * j), r = __ldg(pw + 2 * j + 1);
+    const BufRef D = P.buf[(d & kFanRelay) ? K_RELAY : K_HALO][d >> 28];
+    const char *sp = S.ptr + (int64_t)r * S.pitch;
+    char *dp = D.ptr + (int64_t)(d & kFanRowMask) * D.pitch;
+    if (V16)
+      st_v4(dp + col * 16, ld_nc_v4(sp + col * 16));
+    else
+      st_part(dp + col * 4, ld_part<true>(sp + col * 4, 4), 4);
+    if (sig && col == 0) atomicAdd(&s_cnt[d >> 28], 1u);
+  }
+}
+
 template <bool V16>
 __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant__ ExecParams P) {
   __shared__ int s_abort;
@@ -189,6 +214,8 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
   // per executing rank: the wait list last found satisfied (monotonic counters, fixed targets)
   __shared__ int32_t s_wait_ok[kMaxRanks];
   __shared__ uint32_t s_ready_ok;
+  __shared__ uint32_t s_cnt[kMaxRanks];  // fan-out rows per receiver of the current item
+  if (threadIdx.x < kMaxRanks) s_cnt[threadIdx.x] = 0;
   if (threadIdx.x < kMaxRanks) s_wait_ok[threadIdx.x] = -1;
   if (threadIdx.x == 0) s_ready_ok = 0;
   for (int it = blockIdx.x; it < P.n_items; it += gridDim.x) {
@@ -216,6 +243,12 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
                       1000 + I.group);
         if (ok) s_ready_ok |= 1u << I.ready_rank;
       }
+      if (P.use_ready && I.ready_rank == kReadyAll)  // fan-out: every receiver's buffers free
+        for (int s = 0; s < P.world && ok; ++s)
+          if (s != I.exec_rank && !((s_ready_ok >> s) & 1u)) {
+            ok = wait_geq(P.flags[I.exec_rank] + kReadyBase + s, P.seq, P, 1000 + I.group);
+            if (ok) s_ready_ok |= 1u << s;
+          }
       if (ok && I.wait_n > 0 && s_wait_ok[I.exec_rank] != I.wait_off) {
         ok = wait_item_sources(P, I, 100000 + I.group);
         if (ok) s_wait_ok[I.exec_rank] = I.wait_off;
@@ -238,12 +271,21 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
       }
     } else if (I.op == OP_FOLD) {
       fold_rows<V16>(P, I);
+    } else if (I.op == OP_FANOUT) {
+      fanout_rows<V16>(P, I, s_cnt);
     }
     if (P.trace) {
       __syncthreads();
       if (threadIdx.x == 0) P.trace[it].t_done = globaltimer();
     }
-    if (I.flags & kItemSignal) {
+    if ((I.flags & kItemSignal) && I.op == OP_FANOUT) {
+      __threadfence_system();
+      __syncthreads();
+      if (threadIdx.x < (unsigned)P.world && s_cnt[threadIdx.x]) {
+        release_rows(P.flags[threadIdx.x] + I.sig_ctr, (uint64_t)s_cnt[threadIdx.x], true);
+        s_cnt[threadIdx.x] = 0;
+      }
+    } else if (I.flags & kItemSignal) {
       __threadfence_system();  // this thread's row stores are visible system-wide ...
       __syncthreads();         // ... for every thread of the CTA ...
       release_rows(P.flags[I.dst_rank] + I.sig_ctr, (uint64_t)I.rows,

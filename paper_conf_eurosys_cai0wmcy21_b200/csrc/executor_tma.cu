@@ -27,10 +27,14 @@ using namespace dev;
 
 namespace {
 
+#ifndef DGCL_FAN_BULK_ROW
+#define DGCL_FAN_BULK_ROW 1024
+#endif
 #ifndef DGCL_STORE_SPLIT
 #define DGCL_STORE_SPLIT 15  // every consumer warp stores its share (measured best, Reddit)
 #endif
 constexpr int kStoreSplit = DGCL_STORE_SPLIT;  // bulk stores per COPY item (<= consumer warps)
+constexpr int kFanBulkRowBytes = DGCL_FAN_BULK_ROW;  // fan-out rows stored by bulk stores
 constexpr int kMetaSlots = 4;         // run windows prefetched kMetaAhead items ahead
 constexpr int kMetaAhead = 3;
 constexpr int kDescAhead = 6;         // descriptors prefetched further ahead (ring of kDescSlots)
@@ -228,6 +232,7 @@ __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const Dev
     return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;  // source-row window only
   }
   if (is_staged(I)) return staged_rows(I) * (uint32_t)P.row16 + window(I.t0, I.nterms, 4).bytes;
+  if (I.op == OP_FANOUT) return (uint32_t)I.rows * (uint32_t)P.row16 + window(I.t0, I.nterms, 4).bytes;
   return window(I.t0, I.nterms, 4).bytes;
 }
 
@@ -257,6 +262,21 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     if (wdst.bytes) bulk_g2s(st + kTabDst, P.idx + wdst.a, wdst.bytes, full);
   }
   uint8_t *ops = st + kStageHdrBytes;
+  if (I.op == OP_FANOUT) {
+    // consecutive source rows: one bulk copy (packed rows), then the destination words
+    const BufRef S = P.buf[I.src_kind][I.exec_rank];
+    if (S.pitch == (int64_t)r16) {
+      if (lane == 0) bulk_g2s(ops, S.ptr + I.src * S.pitch, (uint32_t)I.rows * r16, full);
+    } else {
+      for (int r = lane; r < I.rows; r += 32)
+        bulk_g2s(ops + (size_t)r * r16, S.ptr + (I.src + r) * S.pitch, r16, full);
+    }
+    if (lane == 0) {
+      const Win wt = window(I.t0, I.nterms, 4);
+      bulk_g2s(ops + (size_t)I.rows * r16, P.terms + wt.a, wt.bytes, full);
+    }
+    return;
+  }
   if (I.op == OP_COPY && (I.flags & kItemDirect)) {
     // short runs: stage only the source-row window; the consumers gather the rows
     if (lane == 0 && I.src < 0) {
@@ -359,6 +379,55 @@ __device__ __forceinline__ void store_copy(const ExecParams &P, const DevItem &I
           const uint32_t col = e - r * nch;
           st_v4(dbase + (int64_t)tab[r] * dpitch + col * 16, lds_v4(ops + r * r16 + col * 16));
         }
+      }
+    }
+  }
+}
+
+// consumers: FANOUT item — the staged rows stored into all their receivers' rows (halo or relay
+// staging, library-owned: whole 16-B chunks).  Flat (destination pair, chunk) index space over the
+// consumer threads, kUnroll independent chunks per thread in flight (as store_copy); with
+// signalling on, the thread holding a pair's chunk 0 counts it for its receiver (published at the
+// next FLUSH / END)
+__device__ __forceinline__ void store_fanout(const ExecParams &P, const DevItem &I,
+                                             const uint8_t *st, uint32_t tid, uint32_t T,
+                                             uint32_t *s_pend) {
+  const uint32_t r16 = (uint32_t)P.row16;
+  const uint8_t *ops = st + kStageHdrBytes;
+  const uint32_t *pw = reinterpret_cast<const uint32_t *>(ops + (size_t)I.rows * r16) +
+                       window(I.t0, I.nterms, 4).skew;
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)(I.nterms >> 1) * nch;
+  const bool sig = (I.flags & kItemSignal) != 0;
+  const uint32_t src0 = (uint32_t)I.src;
+  if (P.bulk_store && r16 >= (uint32_t)kFanBulkRowBytes) {
+    // rows of >= 1 KB: one bulk (TMA) store per (row, receiver) pair, issued by every consumer
+    // thread for its pairs; the stage is released once the stores have read it
+    const uint32_t np = (uint32_t)(I.nterms >> 1);
+    for (uint32_t j = tid; j < np; j += T) {
+      const uint32_t d = pw[2 * j], r = pw[2 * j + 1] - src0;
+      const BufRef D = P.buf[(d & kFanRelay) ? K_RELAY : K_HALO][d >> 28];
+      bulk_s2g(D.ptr + (int64_t)(d & kFanRowMask) * D.pitch, ops + r * r16, r16);
+      if (sig) atomicAdd(&s_pend[I.exec_rank * kMaxRanks + (d >> 28)], 1u);
+    }
+    if (tid < np) {
+      bulk_commit();
+      bulk_wait_read();
+    }
+    return;
+  }
+  for (uint32_t e0 = tid; e0 < total; e0 += T * kUnroll) {
+#pragma unroll
+    for (int q = 0; q < kUnroll; ++q) {
+      const uint32_t e = e0 + q * T;
+      if (e < total) {
+        const uint32_t j = fdiv(e, P);
+        const uint32_t col = e - j * nch;
+        const uint32_t d = pw[2 * j], r = pw[2 * j + 1] - src0;
+        const BufRef D = P.buf[(d & kFanRelay) ? K_RELAY : K_HALO][d >> 28];
+        st_v4(D.ptr + (int64_t)(d & kFanRowMask) * D.pitch + col * 16,
+              lds_v4(ops + r * r16 + col * 16));
+        if (sig && col == 0) atomicAdd(&s_pend[I.exec_rank * kMaxRanks + (d >> 28)], 1u);
       }
     }
   }
@@ -757,7 +826,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         if (lane == 0 && !known_sources(I)) w = wait_item_sources(P, I, 200000 + I.group) ? 1 : 0;
         ok = __shfl_sync(0xffffffffu, w, 0) != 0;
         if (!ok) break;
-      } else if (I.op == OP_COPY || I.op == OP_FOLD) {
+      } else if (I.op == OP_COPY || I.op == OP_FOLD || I.op == OP_FANOUT) {
         // Done counts are published in batches (FLUSH markers): before this producer could
         // block on a wait, and whenever the counter family (direction, stage) changes.
         const bool sig = (I.flags & kItemSignal) != 0;
@@ -768,6 +837,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
             ready = known_sources(I) || waits_ready(P, I) ? 1 : 0;
             if (ready && P.use_ready && I.ready_rank >= 0 && !((ready_ok >> I.ready_rank) & 1u))
               ready = ld_acquire_sys(P.flags[I.exec_rank] + kReadyBase + I.ready_rank) >= P.seq;
+            if (ready && P.use_ready && I.ready_rank == kReadyAll)
+              for (int s = 0; s < P.world && ready; ++s)
+                if (s != I.exec_rank && !((ready_ok >> s) & 1u))
+                  ready = ld_acquire_sys(P.flags[I.exec_rank] + kReadyBase + s) >= P.seq;
           }
           ready = __shfl_sync(0xffffffffu, ready, 0);
           if (!ready || (sig && key != pend_key)) {
@@ -787,6 +860,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
                          1000 + I.group) ? 1 : 0;
             if (w) ready_ok |= 1u << I.ready_rank;
           }
+          if (w && P.use_ready && I.ready_rank == kReadyAll)  // fan-out: every receiver
+            for (int s = 0; s < P.world && w; ++s)
+              if (s != I.exec_rank && !((ready_ok >> s) & 1u)) {
+                w = wait_geq(P.flags[I.exec_rank] + kReadyBase + s, P.seq, P, 1000 + I.group) ? 1 : 0;
+                if (w) ready_ok |= 1u << s;
+              }
         }
         ok = __shfl_sync(0xffffffffu, w, 0) != 0;
         if (!ok) break;
@@ -886,6 +965,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         } else {
           store_copy(P, I, st, tid, T);
         }
+      } else if ((kMask & kMaskFanout) && I.op == OP_FANOUT) {
+        store_fanout(P, I, st, tid, T, s_pend);
+        if ((I.flags & kItemSignal) && tid == 0) s_pend_base = I.sig_ctr - I.exec_rank;
       } else if ((kMask & kMaskDirect) && I.op == OP_COPY) {
         store_copy_direct(P, I, st, tid, T);
       } else if ((kMask & kMaskStaged) && is_staged(I)) {
@@ -899,7 +981,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       }
       if (P.trace && tid == 0)  // this warp's share of the item is stored
         P.trace[reinterpret_cast<const int32_t *>(st + kHdrInfo)[2]].t_done = globaltimer();
-      if ((I.flags & kItemSignal) && tid == 0) {
+      if ((I.flags & kItemSignal) && tid == 0 && I.op != OP_FANOUT) {
         // counted now, published by the next FLUSH / END marker (done flags)
         atomicAdd(&s_pend[I.exec_rank * kMaxRanks + I.dst_rank], (uint32_t)I.rows);
         s_pend_base = I.sig_ctr - I.exec_rank;
@@ -930,7 +1012,7 @@ int launch_mask(const ExecParams &p, int grid, int block, cudaStream_t s) {
   return (int)cudaGetLastError();
 }
 
-constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged;
+constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged | kMaskFanout;
 
 }  // namespace
 
@@ -938,6 +1020,9 @@ int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream) 
   cudaStream_t s = (cudaStream_t)stream;
   switch (p.op_mask) {
     case kMaskCopy: return launch_mask<kMaskCopy>(p, grid, block, s);
+    // forward with fan-out stage 1 (uniform plans), plus relay copies (relay plans)
+    case kMaskFanout: return launch_mask<kMaskFanout>(p, grid, block, s);
+    case kMaskFanout | kMaskCopy: return launch_mask<kMaskFanout | kMaskCopy>(p, grid, block, s);
     case kMaskFold:
       // fold-only launches of unstaged folds are latency-bound gathers by the consumer warps:
       // the host may run them with 1024 threads (31 consumer warps, <= 64 registers) for twice

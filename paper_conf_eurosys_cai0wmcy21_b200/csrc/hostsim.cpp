@@ -24,8 +24,27 @@ inline float *row_ptr(const HostBufs &B, int kind, int rank, int64_t row) {
   return B.base[kind][rank] + row * B.pitch;
 }
 
+// OP_FANOUT rows [r0, r0 + rows) of group g: each source row into all its receivers' rows
+bool run_fanout(const Lowered &low, const DevGroup &g, int64_t r0, int64_t rows,
+                const HostBufs &B, int dim) {
+  for (int64_t r = r0; r < r0 + rows; ++r) {
+    const float *s = row_ptr(B, g.src_kind, g.exec_rank, g.src_base + r);
+    for (int64_t t = low.term_ptr[g.term_ptr + r]; t < low.term_ptr[g.term_ptr + r + 1]; t += 2) {
+      const uint32_t d = low.terms[t];
+      if ((int64_t)low.terms[t + 1] != g.src_base + r) return false;  // (source row of the pair)
+      std::memcpy(row_ptr(B, (d & kFanRelay) ? K_RELAY : K_HALO, (int)(d >> 28), d & kFanRowMask),
+                  s, sizeof(float) * dim);
+    }
+  }
+  return true;
+}
+
 void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim) {
   if (g.op == OP_READY || g.op == OP_WAIT) return;
+  if (g.op == OP_FANOUT) {
+    run_fanout(low, g, 0, g.n_rows, B, dim);
+    return;
+  }
   for (int64_t i = 0; i < g.n_rows; ++i) {
     const int64_t drow = g.dst_idx >= 0 ? low.idx[g.dst_idx + i] : g.dst_base + i;
     float *d = row_ptr(B, g.dst_kind, g.dst_rank, drow);
@@ -66,8 +85,17 @@ void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim
 // returns false if the item is malformed (shape checks the device executor relies on)
 bool run_item(const Lowered &low, const DevItem &it, const std::vector<DevRun> &runs,
               const std::vector<uint32_t> &sterms, const HostBufs &B, int dim) {
-  if (it.op != OP_COPY && it.op != OP_FOLD) return it.rows == 0;
+  if (it.op != OP_COPY && it.op != OP_FOLD && it.op != OP_FANOUT) return it.rows == 0;
   if (it.rows <= 0 || it.rows > (it.op == OP_COPY ? kMaxItemRows : kMaxFoldRows)) return false;
+  if (it.op == OP_FANOUT) {
+    const DevGroup &g = low.groups[it.group];
+    const int64_t r0 = it.src - g.src_base;
+    if (it.tp != g.term_ptr + r0 || it.t0 != low.term_ptr[it.tp] ||
+        it.nterms != low.term_ptr[it.tp + it.rows] - it.t0 || it.nterms < 1 ||
+        it.nterms > kMaxItemTerms)
+      return false;
+    return run_fanout(low, g, r0, it.rows, B, dim);
+  }
   auto drow = [&](int64_t r) { return it.dst >= 0 ? it.dst + r : (int64_t)low.idx[~it.dst + r]; };
   if (it.op == OP_COPY) {
     int64_t covered = 0;

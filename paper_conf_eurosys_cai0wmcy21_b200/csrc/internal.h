@@ -37,8 +37,17 @@ enum Op : int32_t {
   OP_READY = 2,  // write ready[exec_rank] = seq into every peer's flag region
   OP_WAIT = 3,   // wait on the group's wait list (forward completion)
   OP_END = 4,    // (device only) end-of-stream marker from the producer warp to the consumers
-  OP_FLUSH = 5   // (device only) publish the done counts accumulated since the last flush
+  OP_FLUSH = 5,  // (device only) publish the done counts accumulated since the last flush
+  OP_FANOUT = 6  // forward stage 1, per owner: read each embedding row once and store it into
+                 // every requester's halo (or relay) row: dests(i) = terms[term_ptr[i]..)
 };
+
+// OP_FANOUT destinations (terms pool): word pairs (dest, source row); dest bits 31..28 = receiving
+// rank, bit 27 = relay staging (else halo), bits 26..0 = row in that buffer
+constexpr uint32_t kFanRelay = 1u << 27;
+constexpr uint32_t kFanRowMask = (1u << 27) - 1;
+// DevItem::ready_rank of an item that writes to several ranks (OP_FANOUT): wait for every peer
+constexpr int8_t kReadyAll = -2;
 
 enum Dir : int32_t { DIR_FWD = 0, DIR_BWD = 1 };
 
@@ -185,7 +194,7 @@ DGCL_HD inline uint32_t trace_tag(const DevItem &I, int stage) {
   return (uint32_t)I.op | (uint32_t)I.dir << 4 | (uint32_t)I.exec_rank << 8 |
          (uint32_t)I.dst_rank << 16 | (uint32_t)stage << 24;
 }
-constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8;
+constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8, kMaskFanout = 16;
 
 // A run of `len` rows whose source rows src.. and destination rows dst.. are both consecutive;
 // `pos` is the first row's index inside its item.  One bulk copy moves a run when the pitches

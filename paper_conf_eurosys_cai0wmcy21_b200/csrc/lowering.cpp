@@ -435,6 +435,60 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       }
   }
   L.atomic_end = (int)L.groups.size();
+  // ---- forward stage 1 as fan-out groups (one per owner) ----
+  // Every stage-1 tree edge leaves the owner (the root), so stage 1 is "each owner sends each of
+  // its rows to the requesters of that row" (P:1458-1462 packs one (d_i, d_j) tuple at a time).
+  // A fan-out group reads each embedding row ONCE and stores it into all its first-hop receivers
+  // (halo row, or relay staging for a forwarding GPU) — the kernel-level form of the paper's
+  // communication fusion: HBM reads drop from one per delivery to one per row.
+  // Rows are the owner's local rows in loc order (consecutive sources: one bulk copy per item);
+  // dests per row in ascending receiver id, as word pairs in the terms pool: (receiver << 28 |
+  // relay bit | destination row, source row) — the executor maps (pair, chunk) to threads.
+  {
+    int64_t N = (int64_t)loc.size();
+    std::vector<int64_t> vi_of(N, -1);
+    for (int64_t vi = 0; vi < NV; ++vi) vi_of[plan.order[vi]] = vi;
+    std::vector<std::vector<int64_t>> rows_of(m);  // owner -> vertices in loc order
+    for (int64_t u = 0; u < N; ++u) rows_of[part[u]].push_back(u);
+    bool fits = true;
+    std::vector<std::pair<int, uint32_t>> ds;
+    for (int p = 0; p < m && fits; ++p) {
+      DevGroup g = base_group(OP_FANOUT, DIR_FWD, p, p, 1);
+      g.src_kind = K_EMB;
+      g.dst_kind = K_HALO;
+      g.n_rows = (int64_t)rows_of[p].size();
+      g.src_base = 0;
+      g.dst_base = 0;
+      g.sig_ctr = (int32_t)ctr_index(DIR_FWD, 1, p);
+      g.ready_rank = kReadyAll;
+      g.term_ptr = (int64_t)L.term_ptr.size();
+      const size_t t_begin = L.terms.size();
+      L.term_ptr.push_back((int64_t)L.terms.size());
+      for (int64_t u : rows_of[p]) {
+        const int64_t vi = vi_of[u];
+        if (vi >= 0) {
+          ds.clear();
+          for (int64_t e = plan.e_ptr[vi]; e < plan.e_ptr[vi + 1]; ++e) {
+            if (plan.e_parent[e] != p) continue;
+            const int c = plan.e_child[e];
+            const int64_t row = child_pos[e] >= 0 ? child_pos[e] : relay_row[e];
+            if (row > (int64_t)kFanRowMask) fits = false;
+            ds.push_back({c, ((uint32_t)c << 28) | (child_pos[e] >= 0 ? 0u : kFanRelay) |
+                                 ((uint32_t)row & kFanRowMask)});
+          }
+          std::sort(ds.begin(), ds.end());
+          for (auto &d : ds) {
+            L.terms.push_back(d.second);
+            L.terms.push_back((uint32_t)loc[u]);
+          }
+        }
+        L.term_ptr.push_back((int64_t)L.terms.size());
+      }
+      if (L.terms.size() > t_begin) L.groups.push_back(g);
+    }
+    if (!fits) L.groups.resize(L.atomic_end);  // rows beyond the 27-bit dest field: per-pair groups
+  }
+  L.fanout_end = (int)L.groups.size();
   L.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
 }
 
@@ -529,6 +583,9 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
   size_t i = 0;
   std::vector<std::vector<int32_t>> bounds;  // per group of the stage: chunk start rows + end
   std::vector<uint8_t> staged;               // per group of the stage: FOLD items are staged
+  // per group of the stage: OP_FANOUT items as row ranges [first, second) (runs of rows without
+  // receivers between them are skipped, so items are not contiguous in the group's rows)
+  std::vector<std::vector<std::pair<int64_t, int64_t>>> franges;
   // staged FOLD item: operand rows (destination rows of the fold start + one per term) and the
   // staged-term window share one stage; segments (<= one per operand row) fill one meta slot
   const int64_t stage_rows_cap = std::min<int64_t>(lim.max_rows, lim.operand_bytes / row16);
@@ -547,6 +604,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     if (j == i) j = i + 1;
     bounds.assign(j - i, std::vector<int32_t>());
     staged.assign(j - i, 0);
+    franges.assign(j - i, {});
     size_t max_chunks = 0;
     // small stages: cut COPY items finer so that every co-resident CTA gets work (latency-bound
     // launches, e.g. the tiny config or the last relay stage), down to 4 rows per item
@@ -631,6 +689,36 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
           acc += cost;
         }
         b.push_back((int32_t)g.n_rows);
+      } else if (g.op == OP_FANOUT) {
+        // the source rows of an item are consecutive (one bulk copy) and its operands — rows and
+        // destination words — fit one stage; >= 8 rows without receivers end an item and are
+        // skipped (every row an item carries is read from HBM)
+        auto nd = [&](int64_t r) {
+          return low.term_ptr[g.term_ptr + r + 1] - low.term_ptr[g.term_ptr + r];
+        };
+        auto& fr = franges[q - i];
+        const int64_t max_rows = std::min<int64_t>(lim.max_rows, kMaxFoldRows);
+        int64_t r = 0;
+        while (r < g.n_rows) {
+          while (r < g.n_rows && nd(r) == 0) ++r;
+          if (r >= g.n_rows) break;
+          const int64_t r0 = r;
+          int64_t nt = 0, last = r;  // last row with receivers + 1
+          while (r < g.n_rows) {
+            const int64_t c = nd(r);
+            if (c == 0 && r - last + 1 >= 8) break;
+            const int64_t rows = r - r0 + 1;
+            if (rows > 1 && (rows > max_rows || nt + c > kMaxItemTerms ||
+                             rows * row16 + ((nt + c) * 4 + 15) / 16 * 16 + 16 > cap))
+              break;
+            nt += c;
+            ++r;
+            if (c) last = r;
+          }
+          fr.push_back({r0, last});
+          r = last;
+        }
+        b.assign(fr.size() + 1, 0);
       } else if (g.op != OP_FOLD && g.op != OP_COPY) {
         b.push_back(0);  // READY / WAIT: one empty item
       }
@@ -642,8 +730,9 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         const DevGroup &g = low.groups[gids[q]];
         const std::vector<int32_t> &b = bounds[q - i];
         if (c + 1 >= b.size()) continue;
-        const bool data = g.op == OP_COPY || g.op == OP_FOLD;
-        const int64_t rb = b[c];
+        const bool fan = g.op == OP_FANOUT;
+        const bool data = g.op == OP_COPY || g.op == OP_FOLD || fan;
+        const int64_t rb = fan ? franges[q - i][c].first : b[c];
         DevItem it;
         std::memset(&it, 0, sizeof(it));
         it.op = (uint8_t)g.op;
@@ -659,10 +748,15 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         it.wait_off = g.wait_off;
         it.sig_ctr = g.sig_ctr;
         it.group = gids[q];
-        it.rows = data ? b[c + 1] - b[c] : 0;
+        it.rows = !data ? 0 : fan ? (int32_t)(franges[q - i][c].second - rb) : b[c + 1] - b[c];
         it.src = g.src_idx >= 0 ? ~(g.src_idx + rb) : g.src_base + rb;
         it.dst = g.dst_idx >= 0 ? ~(g.dst_idx + rb) : g.dst_base + rb;
-        if (g.op == OP_FOLD) {
+        if (fan) {
+          it.dst = 0;
+          it.tp = g.term_ptr + rb;
+          it.t0 = low.term_ptr[it.tp];
+          it.nterms = (int32_t)(low.term_ptr[it.tp + it.rows] - it.t0);
+        } else if (g.op == OP_FOLD) {
           it.tp = g.term_ptr + rb;
           it.t0 = low.term_ptr[it.tp];
           it.nterms = (int32_t)(low.term_ptr[it.tp + it.rows] - it.t0);
@@ -686,8 +780,13 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
           it.nterms = (int32_t)((int64_t)runs->size() - it.tp);
         }
         bool sig = data && g.sig_ctr >= 0;
-        if (sig && !signal_all)
+        if (sig && !signal_all && fan) {
+          sig = false;  // needed by some receiver of the owner's rows
+          for (int d = 0; d < low.m; ++d)
+            if (d != g.exec_rank && needed_ctr[(size_t)d * kFlagWords + g.sig_ctr]) sig = true;
+        } else if (sig && !signal_all) {
           sig = needed_ctr[(size_t)g.dst_rank * kFlagWords + g.sig_ctr] != 0;
+        }
         it.flags |= sig ? kItemSignal : 0;
         // optional: items whose runs average fewer than `direct_copy_rows` rows are gathered by
         // the consumers with plain loads instead of one bulk copy per run (0 = never; measured

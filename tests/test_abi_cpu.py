@@ -150,7 +150,8 @@ def test_uniform_plan_and_lowering(m, direct):
                                     (8, {"direct_reduce": 0, "item_bytes": 2048}),
                                     (3, {"gather4": 0, "stage_fold": 0}),
                                     (8, {"geometry": 1}), (8, {"geometry": 2}),
-                                    (4, {"geometry": 2, "direct_reduce": 0})])
+                                    (4, {"geometry": 2, "direct_reduce": 0}),
+                                    (8, {"fanout": 1}), (3, {"fanout": 1, "geometry": 2})])
 def test_work_items_host(m, opts):
     """The fused program's WORK ITEMS (not the groups) moved the way the bulk-copy executor moves
     them — COPY row runs, staged FOLD segments read back through the staged-term table — on the
@@ -159,11 +160,12 @@ def test_work_items_host(m, opts):
     _check_lowering(g, [16, 5, 602], None, seed=3, options=dict(opts, hostsim_items=1))
 
 
-@pytest.mark.parametrize("name,sf", [("dgx1_like", 1), ("ring", 1), ("ring", 0)])
-def test_work_items_host_relay(name, sf):
+@pytest.mark.parametrize("name,sf,fan", [("dgx1_like", 1, 0), ("ring", 1, 0), ("ring", 0, 0),
+                                        ("dgx1_like", 1, 1), ("ring", 1, 1)])
+def test_work_items_host_relay(name, sf, fan):
     g = synth.make_graph(500, 2500, 8, graph_seed=9, part_seed=19)
     _check_lowering(g, [12, 3], synth.topology.by_name(name), seed=5,
-                    options={"hostsim_items": 1, "stage_fold": sf})
+                    options={"hostsim_items": 1, "stage_fold": sf, "fanout": fan})
 
 
 def test_work_items_host_shuffled():

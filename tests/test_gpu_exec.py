@@ -159,24 +159,27 @@ def test_tiny_config_bit_exact(small):
     (8, {"direct_reduce": 0, "item_bytes": 4096}),
     (8, {"geometry": 1}), (8, {"geometry": 2}), (4, {"geometry": 2, "direct_reduce": 0}),
     (3, {"geometry": 1, "stage_fold": 0}),
+    (8, {"fanout": 1}), (4, {"fanout": 1, "tma": 0}), (8, {"fanout": 1, "geometry": 2}),
+    (3, {"fanout": 1, "bulk_store": 0}), (4, {"fanout": 1, "geometry": 1}),
 ])
 def test_uniform_loopback_fused(m, opts):
     """Executor variants: tma (bulk-copy executor vs the register LDG executor), direct_reduce
     (loopback in-place reduce vs push to slots + owner reduce, the multi-GPU form), bulk_store
     (TMA stores vs 16-B st.global), gather4 (TMA row gather of 4 rows per instruction vs one bulk
     copy per run), direct_copy_rows (consumer-side gathers for short runs), stage_fold (backward
-    folds with every operand row bulk-copied into shared memory vs consumer gathers)."""
+    folds with every operand row bulk-copied into shared memory vs consumer gathers), fanout
+    (forward stage 1 as per-owner fan-out items vs one COPY group per (owner, receiver))."""
     g = synth.make_graph(6000, 60000, m, graph_seed=m, part_seed=7 * m)
     _check_case(Case(g, [64, 5, 602, 32], options=opts))
 
 
-@pytest.mark.parametrize("m", [2, 8])
-def test_per_rank_flag_protocol(m):
+@pytest.mark.parametrize("m,fanout", [(2, 1), (8, 1), (8, 0)])
+def test_per_rank_flag_protocol(m, fanout):
     """Every virtual rank is its own launch on its own stream: ready handshake, done counters,
     forward completion waits — the multi-GPU protocol on one device; several calls in a row."""
     D = _D()
     g = synth.make_graph(5000, 40000, m, graph_seed=11, part_seed=12)
-    c = Case(g, [32, 7], flags=D.LOOPBACK_PER_RANK)
+    c = Case(g, [32, 7], flags=D.LOOPBACK_PER_RANK, options={"fanout": fanout})
     for _ in range(2):
         _check_case(c)
 
@@ -185,13 +188,17 @@ def test_per_rank_flag_protocol(m):
                                                ("dgx1_like", 1, 1, 1), ("ring", 1, 1, 1),
                                                ("ring", 0, 0, 1), ("dgx1_like", 1, 0, 1),
                                                ("ring", 1, 1, 0), ("dgx1_like", 0, 1, 0),
-                                               ("ring", 0, 1, 2), ("dgx1_like", 1, 1, 3)])
+                                               ("ring", 0, 1, 2), ("dgx1_like", 1, 1, 3),
+                                               ("dgx1_like", 0, 1, 4), ("ring", 1, 1, 4)])
 def test_relay_plans(name, flags, tma, sf):
-    """sf: stage_fold 0/1; 2, 3 = stage_fold with the DUAL / WIDE geometry forced."""
+    """sf: stage_fold 0/1; 2, 3 = stage_fold with the DUAL / WIDE geometry forced; 4 = fan-out
+    stage 1 (first hops into halos and relay staging, done counts per receiver)."""
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
     opts = {"tma": tma, "stage_fold": min(sf, 1)}
-    if sf >= 2:
+    if sf in (2, 3):
         opts["geometry"] = 2 if sf == 2 else 1
+    if sf == 4:
+        opts["fanout"] = 1
     c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags, options=opts)
     assert c.ctx.plan_info()["n_stages"] >= 2
     _check_case(c)
