@@ -156,8 +156,10 @@ def host_inputs(w, pitches, rows_order=None):
 
 
 # ---------------------------------------------------------------------------------------------
-def oracle_sample(w, emb, hg, eg, budget_s=15.0, ranks=None):
+def oracle_sample(w, emb, hg, eg, budget_s=15.0, ranks=None, threads=1):
     """Time the CPU oracle (as it stands) on destination/owner ranks until the budget is spent.
+    threads > 1: the ranks' oracle calls run concurrently in a thread pool (numpy's gathers and
+    adds release the GIL), all of ranks at once, wall-clock timed.
     Returns (GB/s, seconds, ranks used, threads)."""
     from oracle import halo
     c = w.cfg
@@ -166,6 +168,16 @@ def oracle_sample(w, emb, hg, eg, budget_s=15.0, ranks=None):
     loc, n_local = halo.local_rows(g.part, m)
     ro = np.concatenate([[0], np.cumsum(n_local)])
     R = [g.R(d) for d in range(m)]
+    if threads > 1:
+        from concurrent.futures import ThreadPoolExecutor
+        rk = list(ranks if ranks is not None else range(m))
+        one = lambda d: oracle_sample(w, emb, hg, eg, budget_s=0.0, ranks=[d])
+        with ThreadPoolExecutor(max_workers=min(threads, len(rk))) as ex:
+            t = time.perf_counter()
+            res = list(ex.map(one, rk))
+            secs = time.perf_counter() - t
+        nbytes = sum(r[0] * r[1] * 1e9 for r in res)
+        return nbytes / secs / 1e9, secs, rk, min(threads, len(rk))
     done_bytes, t_total, used = 0, 0.0, []
     for d in (ranks if ranks is not None else range(m)):
         t = time.perf_counter()
@@ -399,6 +411,14 @@ def run_ours_single(args, w):
         cpu = {"value": gbs, "unit": UNIT, "cores": thr, "kind": "oracle",
                "sample": "oracle forward (all layers) + flat backward for destination/owner "
                          "ranks %s of %d (%.1f s of CPU work)" % (used, c.m, secs)}
+        ncores = len(os.sched_getaffinity(0))
+        if ncores > 1 and not args.no_cpu_threads:
+            gbs_t, secs_t, used_t, thr_t = oracle_sample(w, emb_h, hg_h, eg_h, ranks=range(c.m),
+                                                         threads=ncores)
+            cpu["threaded"] = {"value": gbs_t, "unit": UNIT, "cores": thr_t,
+                               "host_cores": ncores,
+                               "sample": "all %d ranks' oracle calls concurrently (%.1f s wall)" %
+                                         (c.m, secs_t)}
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": K,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
@@ -464,6 +484,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-torch-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
+    ap.add_argument("--no-cpu-threads", action="store_true")
     ap.add_argument("--item-bytes", type=int, default=0)
     ap.add_argument("--opt", action="append", default=[], metavar="KEY=VALUE",
                     help="executor option (dgcl_set_option) before planning, e.g. stage_fold=0")
