@@ -216,6 +216,10 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "stage_fold"     1 (default): backward folds bulk-copy all their operand rows into shared
  *                    memory (segments of consecutive rows) before adding them; 0: consumers
  *                    gather the operands with plain loads
+ *   "align_sources"  1 (default): the forward COPY groups that read one rank's embeddings (one per
+ *                    receiver) are cut into items at common source rows, so the copies of a row
+ *                    to its receivers run close together (L2 reuse; rows <= 1 KB); 0: independent
+ *                    cuts
  *   "fanout"         0 (default) / 1: forward stage 1 as one fan-out item stream per owner — each
  *                    embedding row read once and stored into every first-hop receiver's row
  *                    (kernel-level communication fusion) — instead of one COPY group

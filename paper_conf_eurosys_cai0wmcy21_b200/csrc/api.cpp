@@ -94,6 +94,7 @@ struct dgcl_ctx {
   bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
   bool atomic_backward = false;       // ablation: loopback backward with atomic adds
   bool fanout = false;                // forward stage 1 as per-owner fan-out items (option)
+  bool align_sources = true;          // forward COPY items of one source rank cut at common rows
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
@@ -354,10 +355,10 @@ void build_programs(dgcl_ctx *c) {
         const std::vector<uint8_t> need = needed_counters(L, G);
         auto build = [&](int geo) {
           P.geo = geo;
-          build_items(L, G, row_bytes,
-                      item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
-                                  (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm),
-                      !fused, need,
+          ItemLimits lim = item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
+                                       (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm);
+          lim.align_sources = c->align_sources;
+          build_items(L, G, row_bytes, lim, !fused, need,
                       &P.items, &P.runs, c->direct_copy_rows,
                       c->stage_fold ? &P.sterms : nullptr);
           P.op_mask = 0;
@@ -1173,6 +1174,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "stage_fold") {  // bulk-copy FOLD operand rows into the stage (bulk-copy executor)
     c->stage_fold = value != 0;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "align_sources") {  // forward COPY groups of one source rank: common item boundaries
+    c->align_sources = value != 0;
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }

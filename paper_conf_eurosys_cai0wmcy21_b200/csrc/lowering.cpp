@@ -586,12 +586,21 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
   // per group of the stage: OP_FANOUT items as row ranges [first, second) (runs of rows without
   // receivers between them are skipped, so items are not contiguous in the group's rows)
   std::vector<std::vector<std::pair<int64_t, int64_t>>> franges;
+  std::vector<uint8_t> aligned;  // per group of the stage: bounds set jointly (source-aligned)
   // staged FOLD item: operand rows (destination rows of the fold start + one per term) and the
   // staged-term window share one stage; segments (<= one per operand row) fill one meta slot
   const int64_t stage_rows_cap = std::min<int64_t>(lim.max_rows, lim.operand_bytes / row16);
   auto staged_fits = [&](int64_t srows, int64_t nt) {
     return srows <= stage_rows_cap &&
            srows * row16 + (nt * 4 + 15) / 16 * 16 + 16 <= lim.operand_bytes;
+  };
+  auto src_row = [&](const DevGroup &h, int64_t r) -> int64_t {
+    return h.src_idx >= 0 ? (int64_t)low.idx[h.src_idx + r] : h.src_base + r;
+  };
+  auto ascending_src = [&](const DevGroup &h) {
+    for (int64_t r = 1; r < h.n_rows; ++r)
+      if (src_row(h, r) <= src_row(h, r - 1)) return false;
+    return true;
   };
   while (i < gids.size()) {
     // one stage (READY / WAIT are their own runs)
@@ -614,9 +623,74 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     int64_t spread_rpi = lim.max_rows;
     if (lim.min_items > 0 && copy_rows < lim.min_items * lim.max_rows)
       spread_rpi = std::max<int64_t>(4, (copy_rows + lim.min_items - 1) / lim.min_items);
+    auto copy_rpi = [&](int64_t spread) {
+      int64_t rpi = std::min<int64_t>(std::min(lim.max_rows, spread),
+                                      std::max<int64_t>(1, cap / row16));
+      if (row16 <= kGather4MaxRowBytes && rpi >= 4) rpi = rpi / 4 * 4;
+      return rpi;
+    };
+    // Forward COPY groups that read the same rank's embeddings (one per receiver) get item
+    // boundaries at the SAME source rows: chunk c of every such group covers source rows
+    // [B_c, B_c+1), and chunks are interleaved, so the copies of one row to its receivers run
+    // close together and all but the first hit L2 (independent cuts drift apart over a long
+    // launch: the Com-Orkut forward re-read 0.7 GB on top of its 1.6 GB of rows, ncu r1i).  A
+    // cut falls where the first group of the set reaches `rpi` rows, so no item exceeds it.
+    // Applied to rows <= 1 KB (the per-row gather regime): measured Web-Google-4 forward 0.345
+    // -> 0.308 ms, Com-Orkut 1.62 -> 1.60, Web-Google-8 0.448 -> 0.445; the Reddit dim-602
+    // forward, whose rows already come once from DRAM, lost 2 % to the smaller items.
+    aligned.assign(j - i, 0);
+    if (lim.align_sources && row16 <= kGather4MaxRowBytes) {
+      auto alignable = [&](const DevGroup &h) {
+        return h.op == OP_COPY && h.dir == DIR_FWD && h.src_kind == K_EMB && !h.atomic_add &&
+               h.n_rows > 0 && ascending_src(h);
+      };
+      const int64_t rpi = copy_rpi(spread_rpi);
+      for (size_t q = i; q < j; ++q) {
+        const DevGroup &g = low.groups[gids[q]];
+        if (aligned[q - i] || !alignable(g)) continue;
+        std::vector<size_t> set;
+        for (size_t q2 = q; q2 < j; ++q2) {
+          const DevGroup &h = low.groups[gids[q2]];
+          if (!aligned[q2 - i] && h.exec_rank == g.exec_rank && alignable(h)) set.push_back(q2);
+        }
+        if (set.size() < 2) continue;
+        std::vector<int64_t> ptr(set.size(), 0);
+        for (size_t t = 0; t < set.size(); ++t) {
+          aligned[set[t] - i] = 1;
+          bounds[set[t] - i].assign(1, 0);
+        }
+        for (;;) {
+          int64_t B = INT64_MAX;
+          bool left = false;
+          for (size_t t = 0; t < set.size(); ++t) {
+            const DevGroup &h = low.groups[gids[set[t]]];
+            if (ptr[t] >= h.n_rows) continue;
+            left = true;
+            if (ptr[t] + rpi < h.n_rows) B = std::min(B, src_row(h, ptr[t] + rpi));
+          }
+          if (!left) break;
+          for (size_t t = 0; t < set.size(); ++t) {
+            const DevGroup &h = low.groups[gids[set[t]]];
+            int64_t lo = B == INT64_MAX ? h.n_rows : ptr[t], hi = h.n_rows;
+            if (B != INT64_MAX)
+              while (lo < hi) {  // first row whose source is >= B (sources ascending)
+                const int64_t mid = (lo + hi) / 2;
+                if (src_row(h, mid) < B) lo = mid + 1; else hi = mid;
+              }
+            ptr[t] = lo;
+            bounds[set[t] - i].push_back((int32_t)lo);
+          }
+          if (B == INT64_MAX) break;
+        }
+      }
+    }
     for (size_t q = i; q < j; ++q) {
       const DevGroup &g = low.groups[gids[q]];
       std::vector<int32_t> &b = bounds[q - i];
+      if (aligned[q - i]) {
+        max_chunks = std::max(max_chunks, b.size() - 1);
+        continue;
+      }
       b.push_back(0);
       if (g.op == OP_FOLD && sterms) {
         // staged: every row must fit a stage on its own
@@ -629,9 +703,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       }
       if (g.op == OP_COPY) {
         // rows per item; a multiple of 4 when gather4 may apply (its groups are padded to 4 rows)
-        int64_t rpi = std::min<int64_t>(std::min(lim.max_rows, spread_rpi),
-                                        std::max<int64_t>(1, cap / row16));
-        if (row16 <= kGather4MaxRowBytes && rpi >= 4) rpi = rpi / 4 * 4;
+        const int64_t rpi = copy_rpi(spread_rpi);
         for (int64_t r = rpi; r < g.n_rows; r += rpi) b.push_back((int32_t)r);
         b.push_back((int32_t)g.n_rows);
       } else if (g.op == OP_FOLD && staged[q - i]) {
@@ -732,6 +804,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         if (c + 1 >= b.size()) continue;
         const bool fan = g.op == OP_FANOUT;
         const bool data = g.op == OP_COPY || g.op == OP_FOLD || fan;
+        if (data && !fan && b[c + 1] == b[c]) continue;  // (empty chunk of a source-aligned set)
         const int64_t rb = fan ? franges[q - i][c].first : b[c];
         DevItem it;
         std::memset(&it, 0, sizeof(it));
