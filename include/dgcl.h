@@ -216,6 +216,10 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "stage_fold"     1 (default): backward folds bulk-copy all their operand rows into shared
  *                    memory (segments of consecutive rows) before adding them; 0: consumers
  *                    gather the operands with plain loads
+ *   "pipeline_blocks" relay plans: vertex blocks of the stage chaining (1..8, default 1): stage k
+ *                    of a block waits only for stage k-1 of the same block, so consecutive stages
+ *                    may overlap; 1 = one done counter per (stage, source) as in §6.1.  Measured
+ *                    slower with more blocks on one B200 (smaller groups and items)
  *   "align_sources"  1 (default): the forward COPY groups that read one rank's embeddings (one per
  *                    receiver) are cut into items at common source rows, so the copies of a row
  *                    to its receivers run close together (L2 reuse; rows <= 1 KB); 0: independent
@@ -259,7 +263,8 @@ dgcl_status dgcl_set_option(dgcl_ctx *ctx, const char *key, int64_t value);
  * recs == NULL: *n = number of records.  Synchronizes the device. */
 typedef struct dgcl_trace_rec {
   uint64_t t_start, t_ready, t_done;
-  uint32_t sm, tag;  /* op | dir << 4 | exec rank << 8 | dst rank << 16 | stage << 24 */
+  uint32_t sm, tag;  /* op | dir << 4 | exec rank << 8 | dst rank << 16 | stage << 24 (5 bits)
+                        | vertex block << 29 (option "pipeline_blocks") */
 } dgcl_trace_rec;
 dgcl_status dgcl_trace_read(dgcl_ctx *ctx, int32_t layer, int32_t dir, int32_t rank,
                             dgcl_trace_rec *recs, int64_t *n);

@@ -95,6 +95,7 @@ struct dgcl_ctx {
   bool atomic_backward = false;       // ablation: loopback backward with atomic adds
   bool fanout = false;                // forward stage 1 as per-owner fan-out items (option)
   bool align_sources = true;          // forward COPY items of one source rank cut at common rows
+  int pipeline_blocks = 1;            // relay plans: vertex blocks of the stage chaining
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
@@ -283,7 +284,7 @@ void build_programs(dgcl_ctx *c) {
   const int ng = (int)L.groups.size();
   // forward stage 1 as one fan-out group per owner (each row read once, stored into all its
   // first-hop receivers) instead of one COPY group per (owner, receiver); per layer below
-  const bool fan_avail = c->fanout && L.fanout_end > L.atomic_end;
+  const bool fan_avail = c->fanout && L.fanout_end > L.atomic_end && L.n_blocks == 1;
   auto is_stage1_copy = [&](const DevGroup &g) {
     return g.dir == DIR_FWD && g.op == OP_COPY && g.stage == 1 && g.src_kind == K_EMB;
   };
@@ -700,7 +701,7 @@ dgcl_status plan_common(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *req_
               : spst_plan(c->topo, c->part.data(), c->rel, seed, &c->plan);
     if (!e.empty()) return fail(c, DGCL_EPLAN, "%s", e.c_str());
     if (c->plan.n_stages >= kMaxStages) return fail(c, DGCL_EPLAN, "too many stages");
-    lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low);
+    lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low, c->pipeline_blocks);
     c->halo_off.assign(c->world + 1, 0);
     for (int d = 0; d < c->world; ++d) c->halo_off[d + 1] = c->halo_off[d] + c->rel.n_halo[d];
     compute_layout(c);
@@ -1175,6 +1176,16 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   if (k == "stage_fold") {  // bulk-copy FOLD operand rows into the stage (bulk-copy executor)
     c->stage_fold = value != 0;
     if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "pipeline_blocks") {  // relay plans: stage chaining per vertex block (1..8)
+    if (value < 1 || value > kMaxBlocks) return fail(c, DGCL_EINVAL, "pipeline_blocks in 1..%d", kMaxBlocks);
+    c->pipeline_blocks = (int)value;
+    if (c->planned) {
+      lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low, c->pipeline_blocks);
+      compute_layout(c);
+      build_programs(c);
+    }
     return DGCL_OK;
   }
   if (k == "align_sources") {  // forward COPY groups of one source rank: common item boundaries

@@ -231,7 +231,7 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
         P.trace[it].t_start = globaltimer();
         P.trace[it].sm = smid;
-        P.trace[it].tag = trace_tag(I, P.groups[I.group].stage);
+        P.trace[it].tag = trace_tag(I, P.groups[I.group].stage, P.groups[I.group].block);
       }
       if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer

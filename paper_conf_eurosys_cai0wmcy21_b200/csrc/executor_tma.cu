@@ -809,7 +809,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
         P.trace[gidx].t_start = globaltimer();
         P.trace[gidx].sm = smid;
-        P.trace[gidx].tag = trace_tag(I, P.groups[I.group].stage);
+        P.trace[gidx].tag = trace_tag(I, P.groups[I.group].stage, P.groups[I.group].block);
       }
       if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer

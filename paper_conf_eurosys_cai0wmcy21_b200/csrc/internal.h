@@ -51,13 +51,17 @@ constexpr int8_t kReadyAll = -2;
 
 enum Dir : int32_t { DIR_FWD = 0, DIR_BWD = 1 };
 
-// flag region layout (uint64 words) at the start of every rank's workspace
-constexpr int64_t ctr_index(int dir, int stage, int src) {
-  return ((int64_t)dir * kMaxStages + stage) * kMaxRanks + src;
+// flag region layout (uint64 words) at the start of every rank's workspace: done counters per
+// (direction, stage, vertex block, source rank) — relay plans split their vertices into blocks
+// so that stage k of block b waits only for stage k-1 of block b (stages overlap) — then the
+// ready words
+constexpr int kMaxBlocks = 8;
+constexpr int64_t ctr_index(int dir, int stage, int src, int block = 0) {
+  return (((int64_t)dir * kMaxStages + stage) * kMaxBlocks + block) * kMaxRanks + src;
 }
-constexpr int64_t kReadyBase = 2 * kMaxStages * kMaxRanks;  // ready[src] words
+constexpr int64_t kReadyBase = 2 * kMaxStages * kMaxBlocks * kMaxRanks;  // ready[src] words
 constexpr int64_t kFlagWords = kReadyBase + kMaxRanks;
-constexpr int64_t kFlagBytes = 8192;  // region reserved (>= kFlagWords * 8)
+constexpr int64_t kFlagBytes = 40960;  // region reserved (>= kFlagWords * 8)
 static_assert(kFlagWords * 8 <= kFlagBytes, "flag region");
 
 // term encodings for OP_FOLD
@@ -84,6 +88,8 @@ struct DevGroup {
   int32_t wait_n;
   int32_t term_mode;   // OP_FOLD terms: kTermLocal (SLOT/HGRAD of exec) or kTermRankHgrad
   int32_t atomic_add;  // OP_COPY: add the rows into the destination with atomics (ablation)
+  int32_t block;       // vertex block (relay plans: stage chaining per block), 0..n_blocks-1
+  int32_t pad3;
   int64_t n_rows;
   int64_t src_idx;     // offset into idx pool, or -1 => rows src_base + i
   int64_t src_base;
@@ -182,7 +188,7 @@ struct alignas(64) ExecParams {
 // its source waits were satisfied (stage chaining), its rows were stored; and what it was.
 struct TraceRec {
   uint64_t t_start, t_ready, t_done;
-  uint32_t sm, tag;  /* op | dir << 4 | exec rank << 8 | dst rank << 16 | stage << 24 */
+  uint32_t sm, tag;  /* op | dir << 4 | exec << 8 | dst << 16 | stage << 24 | block << 29 */
 };
 static_assert(sizeof(TraceRec) == 32, "trace record");
 #ifdef __CUDACC__
@@ -190,9 +196,9 @@ static_assert(sizeof(TraceRec) == 32, "trace record");
 #else
 #define DGCL_HD
 #endif
-DGCL_HD inline uint32_t trace_tag(const DevItem &I, int stage) {
+DGCL_HD inline uint32_t trace_tag(const DevItem &I, int stage, int block) {
   return (uint32_t)I.op | (uint32_t)I.dir << 4 | (uint32_t)I.exec_rank << 8 |
-         (uint32_t)I.dst_rank << 16 | (uint32_t)stage << 24;
+         (uint32_t)I.dst_rank << 16 | (uint32_t)(stage & 31) << 24 | (uint32_t)(block & 7) << 29;
 }
 constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8, kMaskFanout = 16;
 

@@ -37,6 +37,13 @@ inline uint64_t pack_key(int stage, int exec, int dst, int a, int b) {
   return ((uint64_t)stage << 24) | ((uint64_t)exec << 16) | ((uint64_t)dst << 8) |
          ((uint64_t)a << 4) | (uint64_t)b;
 }
+// group key ordered (stage, block, exec, dst, a, b): groups of a stage come block by block
+inline uint64_t pack_key_b(int stage, int block, int exec, int dst, int a, int b) {
+  return ((uint64_t)stage << 32) | ((uint64_t)block << 24) | ((uint64_t)exec << 16) |
+         ((uint64_t)dst << 8) | ((uint64_t)a << 4) | (uint64_t)b;
+}
+inline int key_stage(uint64_t k) { return (int)(k >> 32); }
+inline int key_block(uint64_t k) { return (int)(k >> 24 & 0xFF); }
 
 // position of u on GPU d (its halo row), or -1 if d did not request u
 inline int32_t halo_pos(const Relation &rel, int64_t u, int d) {
@@ -48,7 +55,7 @@ inline int32_t halo_pos(const Relation &rel, int64_t u, int d) {
 }  // namespace
 
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
-                const std::vector<int64_t> &loc, Lowered *out) {
+                const std::vector<int64_t> &loc, Lowered *out, int n_blocks) {
   auto t0 = std::chrono::steady_clock::now();
   const int m = plan.m;
   const int K = plan.n_stages;
@@ -59,10 +66,31 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   L.n_halo = rel.n_halo;
   L.n_relay.assign(m, 0);
   L.n_slot.assign(m, 0);
-  L.rows_sd.assign((size_t)2 * kMaxStages * m * m, 0);
+  L.rows_sd.assign((size_t)2 * kMaxStages * kMaxBlocks * m * m, 0);
   const int64_t NE = (int64_t)plan.e_parent.size();
   L.n_tree_edges = NE;
   const int64_t NV = (int64_t)plan.order.size();
+
+  // Vertex blocks (relay plans): stage k of block b only waits for stage k-1 of block b, so a
+  // stage's tail overlaps the next stage's first blocks instead of the launch idling at every
+  // stage boundary.  Blocks are ranges of vertex ids holding about equal numbers of tree edges
+  // (halo rows are ordered by id within an owner, so a block keeps runs of consecutive rows).
+  const int NB = K >= 2 ? std::max(1, std::min(n_blocks, kMaxBlocks)) : 1;
+  L.n_blocks = NB;
+  std::vector<uint8_t> blk_of;  // per planned vertex index
+  {
+    const int64_t N = (int64_t)loc.size();
+    std::vector<int64_t> w(N, 0);
+    for (int64_t vi = 0; vi < NV; ++vi) w[plan.order[vi]] = plan.e_ptr[vi + 1] - plan.e_ptr[vi];
+    std::vector<uint8_t> bu(N, 0);
+    int64_t acc = 0;
+    for (int64_t u = 0; u < N; ++u) {
+      bu[u] = (uint8_t)std::min<int64_t>(NB - 1, NE > 0 ? acc * NB / NE : 0);
+      acc += w[u];
+    }
+    blk_of.resize(NV);
+    for (int64_t vi = 0; vi < NV; ++vi) blk_of[vi] = bu[plan.order[vi]];
+  }
 
   // edge -> vertex index
   std::vector<int64_t> e_vidx(NE);
@@ -174,7 +202,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
         dk = K_RELAY;
         drow[e] = relay_row[e];
       }
-      ent[e] = {pack_key(k, p, c, sk, dk), drow[e], e, vi};
+      ent[e] = {pack_key_b(k, blk_of[vi], p, c, sk, dk), drow[e], e, vi};
     }
     std::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
       return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
@@ -190,12 +218,14 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
         ++j;
       }
       const uint64_t key = ent[i].key;
-      const int k = (int)(key >> 24), p = (int)(key >> 16 & 0xFF), c = (int)(key >> 8 & 0xFF);
+      const int k = key_stage(key), bl = key_block(key);
+      const int p = (int)(key >> 16 & 0xFF), c = (int)(key >> 8 & 0xFF);
       DevGroup g = base_group(OP_COPY, DIR_FWD, p, c, k);
+      g.block = bl;
       g.src_kind = (int)(key >> 4 & 0xF);
       g.dst_kind = (int)(key & 0xF);
       flush_group(L.groups, g, src, dst);
-      L.rows_sd[((size_t)(DIR_FWD * kMaxStages + k) * m + p) * m + c] += (int64_t)dst.size();
+      L.rows_at(DIR_FWD, k, p, c, bl) += (int64_t)dst.size();
       i = j;
     }
     L.n_fwd_groups = (int)L.groups.size();
@@ -219,7 +249,8 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     for (int64_t e = 0; e < NE; ++e) {
       const int b = K - plan.e_stage[e] + 1;
       const int64_t sort2 = sig[e] == 0 ? (int64_t)child_pos[e] : plan.order[e_vidx[e]];
-      ent[e] = {pack_key(b, plan.e_child[e], plan.e_parent[e], sig[e], 0), sort2, e, e_vidx[e]};
+      ent[e] = {pack_key_b(b, blk_of[e_vidx[e]], plan.e_child[e], plan.e_parent[e], sig[e], 0),
+                sort2, e, e_vidx[e]};
     }
     std::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
       return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
@@ -272,11 +303,13 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       size_t j = i;
       while (j < ent.size() && ent[j].key == ent[i].key) ++j;
       const uint64_t key = ent[i].key;
-      const int b = (int)(key >> 24), c = (int)(key >> 16 & 0xFF), p = (int)(key >> 8 & 0xFF);
+      const int b = key_stage(key), bl = key_block(key);
+      const int c = (int)(key >> 16 & 0xFF), p = (int)(key >> 8 & 0xFF);
       const int s = (int)(key >> 4 & 0xF);
       src.clear();
       dst.clear();
       DevGroup g = base_group(s == 2 ? OP_FOLD : OP_COPY, DIR_BWD, c, p, b);
+      g.block = bl;
       g.dst_kind = K_SLOT;
       if (s == 2) {
         g.term_ptr = (int64_t)L.term_ptr.size();
@@ -301,15 +334,19 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       }
       g.src_kind = s == 0 ? K_HGRAD : K_SLOT;
       flush_group(L.groups, g, src, dst);
-      L.rows_sd[((size_t)(DIR_BWD * kMaxStages + b) * m + c) * m + p] += (int64_t)(j - i);
+      L.rows_at(DIR_BWD, b, c, p, bl) += (int64_t)(j - i);
       i = j;
     }
 
     // ---- RED: owner folds its slots into emb_grad, ascending child id, stage K + 1 ----
+    for (int bl = 0; bl < NB; ++bl)
     for (int s = 0; s < m; ++s) {
-      const std::vector<std::pair<int64_t, int64_t>> &rows = red_rows[s];  // (loc, vidx)
+      std::vector<std::pair<int64_t, int64_t>> rows;  // (loc, vidx) of block bl
+      for (const auto &r : red_rows[s])
+        if (blk_of[r.second] == bl) rows.push_back(r);
       if (rows.empty()) continue;
       DevGroup g = base_group(OP_FOLD, DIR_BWD, s, s, K + 1);
+      g.block = bl;
       g.dst_kind = K_EGRAD;
       g.fold_init = 1;
       g.term_ptr = (int64_t)L.term_ptr.size();
@@ -327,16 +364,17 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   }
 
   // ---- signals and waits (the ready/done protocol of §6.1) ----
-  // wait lists per (dir, stage, exec): every in-peer's counter of the previous stage
-  std::map<std::tuple<int, int, int>, std::pair<int32_t, int32_t>> wait_lists;
-  auto get_waits = [&](int dir, int stage_prev, int r) {
-    auto key = std::make_tuple(dir, stage_prev, r);
+  // wait lists per (dir, stage, exec, block): every in-peer's counter of the previous stage of
+  // the same vertex block
+  std::map<std::tuple<int, int, int, int>, std::pair<int32_t, int32_t>> wait_lists;
+  auto get_waits = [&](int dir, int stage_prev, int r, int bl) {
+    auto key = std::make_tuple(dir, stage_prev, r, bl);
     auto it = wait_lists.find(key);
     if (it != wait_lists.end()) return it->second;
     const int32_t off = (int32_t)L.waits.size();
     for (int s = 0; s < m; ++s) {
-      const int64_t rows = L.rows(dir, stage_prev, s, r);
-      if (rows > 0) L.waits.push_back({(int32_t)ctr_index(dir, stage_prev, s), 0, rows});
+      const int64_t rows = L.rows(dir, stage_prev, s, r, bl);
+      if (rows > 0) L.waits.push_back({(int32_t)ctr_index(dir, stage_prev, s, bl), 0, rows});
     }
     auto v = std::make_pair(off, (int32_t)L.waits.size() - off);
     wait_lists[key] = v;
@@ -344,7 +382,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   };
   for (DevGroup &g : L.groups) {
     if (g.dst_rank != g.exec_rank) {
-      g.sig_ctr = (int32_t)ctr_index(g.dir, g.stage, g.exec_rank);
+      g.sig_ctr = (int32_t)ctr_index(g.dir, g.stage, g.exec_rank, g.block);
       g.ready_rank = g.dst_rank;
     }
     bool reads_inflight;
@@ -353,7 +391,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     else
       reads_inflight = g.op == OP_FOLD || g.src_kind == K_SLOT;
     if (reads_inflight && g.stage >= 2) {
-      auto w = get_waits(g.dir, g.stage - 1, g.exec_rank);
+      auto w = get_waits(g.dir, g.stage - 1, g.exec_rank, g.block);
       g.wait_off = w.first;
       g.wait_n = w.second;
     }
@@ -367,10 +405,11 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     DevGroup g = base_group(OP_WAIT, DIR_FWD, r, r, K + 1);
     g.wait_off = (int32_t)L.waits.size();
     for (int k = 1; k <= K; ++k)
-      for (int s = 0; s < m; ++s) {
-        const int64_t rows = L.rows(DIR_FWD, k, s, r);
-        if (rows > 0) L.waits.push_back({(int32_t)ctr_index(DIR_FWD, k, s), 0, rows});
-      }
+      for (int bl = 0; bl < NB; ++bl)
+        for (int s = 0; s < m; ++s) {
+          const int64_t rows = L.rows(DIR_FWD, k, s, r, bl);
+          if (rows > 0) L.waits.push_back({(int32_t)ctr_index(DIR_FWD, k, s, bl), 0, rows});
+        }
     g.wait_n = (int32_t)L.waits.size() - g.wait_off;
     L.groups.push_back(g);
   }
@@ -607,6 +646,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     const DevGroup &g0 = low.groups[gids[i]];
     size_t j = i;
     while (j < gids.size() && low.groups[gids[j]].stage == g0.stage &&
+           low.groups[gids[j]].block == g0.block &&
            low.groups[gids[j]].op != OP_READY && low.groups[gids[j]].op != OP_WAIT &&
            g0.op != OP_READY && g0.op != OP_WAIT)
       ++j;
@@ -648,10 +688,20 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       for (size_t q = i; q < j; ++q) {
         const DevGroup &g = low.groups[gids[q]];
         if (aligned[q - i] || !alignable(g)) continue;
+        // (groups of about the same size only: relay plans' first hops are very uneven, and a
+        // dense group would cut a sparse one into many small items)
         std::vector<size_t> set;
+        int64_t big = 0;
         for (size_t q2 = q; q2 < j; ++q2) {
           const DevGroup &h = low.groups[gids[q2]];
-          if (!aligned[q2 - i] && h.exec_rank == g.exec_rank && alignable(h)) set.push_back(q2);
+          if (!aligned[q2 - i] && h.exec_rank == g.exec_rank && alignable(h))
+            big = std::max(big, h.n_rows);
+        }
+        for (size_t q2 = q; q2 < j; ++q2) {
+          const DevGroup &h = low.groups[gids[q2]];
+          if (!aligned[q2 - i] && h.exec_rank == g.exec_rank && alignable(h) &&
+              4 * h.n_rows >= 3 * big)
+            set.push_back(q2);
         }
         if (set.size() < 2) continue;
         std::vector<int64_t> ptr(set.size(), 0);

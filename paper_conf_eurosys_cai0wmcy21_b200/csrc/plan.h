@@ -72,10 +72,19 @@ struct Lowered {
   std::vector<DevWait> waits;
   // per-rank buffer rows
   std::vector<int64_t> n_halo, n_relay, n_slot;  // [m]
-  // rows in: [dir][stage][src][dst] flattened: ((dir*kMaxStages + k)*m + s)*m + d
+  int n_blocks = 1;  // vertex blocks of the stage chaining (relay plans), see ctr_index
+  // rows in: [dir][stage][block][src][dst] flattened
   std::vector<int64_t> rows_sd;
-  int64_t rows(int dir, int k, int s, int d) const {
-    return rows_sd[((size_t)(dir * kMaxStages + k) * m + s) * m + d];
+  int64_t &rows_at(int dir, int k, int s, int d, int b) {
+    return rows_sd[(((size_t)(dir * kMaxStages + k) * kMaxBlocks + b) * m + s) * m + d];
+  }
+  int64_t rows(int dir, int k, int s, int d, int b) const {
+    return rows_sd[(((size_t)(dir * kMaxStages + k) * kMaxBlocks + b) * m + s) * m + d];
+  }
+  int64_t rows(int dir, int k, int s, int d) const {  // all blocks
+    int64_t t = 0;
+    for (int b = 0; b < n_blocks; ++b) t += rows(dir, k, s, d, b);
+    return t;
   }
   int64_t n_relay_edges = 0;
   int64_t n_tree_edges = 0;
@@ -86,8 +95,10 @@ struct Lowered {
   }
 };
 
+// n_blocks: vertex blocks for the stage chaining of relay plans (1 = one counter per stage;
+// single-stage plans always use 1)
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
-                const std::vector<int64_t> &loc, Lowered *out);
+                const std::vector<int64_t> &loc, Lowered *out, int n_blocks = 1);
 
 // Work items for one launch: the groups `gids` (already in stage order, READY / WAIT groups
 // included by the caller) cut into row ranges of about item_bytes gathered bytes and interleaved

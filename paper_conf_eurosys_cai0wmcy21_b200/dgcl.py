@@ -201,7 +201,7 @@ class Context:
         out = {k: rec[k] for k in rec.dtype.names}
         t = rec["tag"]
         out.update(op=t & 15, dir=(t >> 4) & 15, exec=(t >> 8) & 255, dst=(t >> 16) & 255,
-                   stage=t >> 24)
+                   stage=(t >> 24) & 31, block=t >> 29)
         return out
 
     def plan_info(self):

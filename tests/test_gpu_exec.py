@@ -189,30 +189,36 @@ def test_per_rank_flag_protocol(m, fanout):
                                                ("ring", 0, 0, 1), ("dgx1_like", 1, 0, 1),
                                                ("ring", 1, 1, 0), ("dgx1_like", 0, 1, 0),
                                                ("ring", 0, 1, 2), ("dgx1_like", 1, 1, 3),
-                                               ("dgx1_like", 0, 1, 4), ("ring", 1, 1, 4)])
+                                               ("dgx1_like", 0, 1, 4), ("ring", 1, 1, 4),
+                                               ("ring", 0, 1, 5), ("dgx1_like", 1, 1, 6),
+                                               ("ring", 1, 0, 6)])
 def test_relay_plans(name, flags, tma, sf):
     """sf: stage_fold 0/1; 2, 3 = stage_fold with the DUAL / WIDE geometry forced; 4 = fan-out
-    stage 1 (first hops into halos and relay staging, done counts per receiver)."""
+    stage 1 (first hops into halos and relay staging, done counts per receiver); 5, 6 = one /
+    eight vertex blocks in the stage chaining (default 4)."""
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
     opts = {"tma": tma, "stage_fold": min(sf, 1)}
     if sf in (2, 3):
         opts["geometry"] = 2 if sf == 2 else 1
     if sf == 4:
         opts["fanout"] = 1
+    if sf in (5, 6):
+        opts["pipeline_blocks"] = 1 if sf == 5 else 8
     c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags, options=opts)
     assert c.ctx.plan_info()["n_stages"] >= 2
     _check_case(c)
 
 
-@pytest.mark.parametrize("tma,flags", [(1, 0), (0, 0), (1, 1)])
-def test_trace_stage_causality(tma, flags):
+@pytest.mark.parametrize("tma,flags,blocks", [(1, 0, 4), (0, 0, 4), (1, 1, 4), (1, 0, 1)])
+def test_trace_stage_causality(tma, flags, blocks):
     """Option "trace": per-item timelines of a relay plan's forward.  Stage chaining on device
-    flags means no stage-k item of GPU r passes its waits before every stage-(k-1) item into r
-    has stored its rows; every item is traced once, in order start <= ready <= done."""
+    flags means no stage-k item of GPU r passes its waits before every stage-(k-1) item of the
+    same vertex block into r has stored its rows; every item is traced once, in
+    order start <= ready <= done; with blocks, later blocks' stage k-1 may still be running."""
     D = _D()
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
     c = Case(g, [40], topo=synth.topology.by_name("dgx1_like"), seed=9, flags=flags,
-             options={"tma": tma, "trace": 1})
+             options={"tma": tma, "trace": 1, "pipeline_blocks": blocks})
     K = c.ctx.plan_info()["n_stages"]
     assert K >= 2
     _check_case(c, bwd=False)
@@ -225,10 +231,11 @@ def test_trace_stage_causality(tma, flags):
     assert np.all(T["t_ready"][data] <= T["t_done"][data])
     for r in range(c.m):
         for k in range(2, K + 1):
-            after = data & (T["exec"] == r) & (T["stage"] == k)
-            before = data & (T["dst"] == r) & (T["stage"] == k - 1)
-            if after.any() and before.any():
-                assert T["t_ready"][after].min() >= T["t_done"][before].max(), (r, k)
+            for b in range(8):
+                after = data & (T["exec"] == r) & (T["stage"] == k) & (T["block"] == b)
+                before = data & (T["dst"] == r) & (T["stage"] == k - 1) & (T["block"] == b)
+                if after.any() and before.any():
+                    assert T["t_ready"][after].min() >= T["t_done"][before].max(), (r, k, b)
 
 
 def test_unaligned_pitch_scalar_path():
