@@ -47,6 +47,11 @@ for direction in (0, 1):
     print("%s %s geo %d: launch %.3f ms (median of 5), %d items, %d SMs" %
           (name, "fwd" if direction == 0 else "bwd", geo, float(np.median(ts)), len(tr["tag"]),
            len(np.unique(tr["sm"]))))
+    for st, op in sorted(set(zip(tr["stage"].tolist(), tr["op"].tolist()))):
+        m = (tr["stage"] == st) & (tr["op"] == op)
+        busy = (tr["t_done"][m] - tr["t_ready"][m]).astype(np.int64)
+        print("    stage %d op %d: %5d items, ready->done busy sum %.0f us, med %.1f us" %
+              (st, op, m.sum(), busy.sum() / 1e3, np.median(busy) / 1e3))
     for st in np.unique(tr["stage"]):
         m = tr["stage"] == st
         busy = (tr["t_done"][m] - tr["t_start"][m]).astype(np.int64)
