@@ -258,9 +258,11 @@ def run_ours_single(args, w):
     ctx = D.loopback(c.m, g.part, list(c.dims), device=0)
     if args.item_bytes:
         ctx.set_option("item_bytes", args.item_bytes)
+    opts = {}
     for kv in args.opt:  # executor options (dgcl_set_option), for A/B runs
         k, v = kv.split("=")
         ctx.set_option(k, int(v))
+        opts[k] = int(v)
     t = time.time()
     ctx.build_plan(g.req_ptr, g.req_ids, seed=0, topology=topo)
     plan_s = time.time() - t
@@ -369,16 +371,20 @@ def run_ours_single(args, w):
     peaks, src = measured_peaks()
     nv = info["n_vertices_planned"]
     # relay plans (several stages) must move more than the direct minimum: every tree edge writes
-    # a row and every forwarding GPU re-reads the row it forwards; the backward pushes one
-    # partial-sum row per tree edge into a slot that the parent reads back.  Reported next to
-    # the direct minimum as plan_algorithmic_bytes / plan_frac.
+    # a row and every forwarding GPU re-reads the row it forwards; the staged backward
+    # (direct_reduce = 0) pushes one partial-sum row per tree edge into a slot that the parent
+    # reads back.  Reported next to the direct minimum as plan_algorithmic_bytes / plan_frac.
+    # (The default loopback backward of a relay plan folds each owner row's tree in one pass:
+    # its bytes are the direct minimum.)
     plan_rows = None
     if info["n_stages"] > 1:
         E = ctx.plan_export()                       # (u, parent, child, stage)
         owner = g.part[E[:, 0]]
         fwd_pairs = np.unique(E[E[:, 1] != owner][:, [0, 1]], axis=0).shape[0]
         ne = int(info["n_tree_edges"])
-        plan_rows = {"fwd": nv + fwd_pairs + ne, "bwd": w.S + 2 * ne + 2 * nv}
+        staged_bwd = opts.get("direct_reduce", 1) == 0
+        plan_rows = {"fwd": nv + fwd_pairs + ne,
+                     "bwd": w.S + 2 * ne + 2 * nv if staged_bwd else w.S + 2 * nv}
     kernels = {}
     for i, n in enumerate(names):
         l = (w.fwd_layers + w.bwd_layers)[i]
@@ -430,6 +436,11 @@ def run_ours_single(args, w):
                    "dims": list(c.dims), "fwd_layers": w.fwd_layers, "bwd_layers": w.bwd_layers,
                    "halo_rows_total": w.S, "halo_rows_per_rank": np.diff(g.req_ptr).tolist(),
                    "topology": c.topology, "parallelism": "loopback%d" % c.m,
+                   "options": opts,
+                   "backward": ("staged reversed plan (slots, stage by stage)"
+                                if opts.get("direct_reduce", 1) == 0 or c.m < 2 else
+                                "tree-order fold per owner row, one pass (loopback)"
+                                if info["n_stages"] > 1 else "fixed-order fold per owner row"),
                    "l2": "inputs larger than L2 (no flush needed)"},
         "ms_per_layer": per_op,
         "gbs_per_gpu": value,

@@ -44,6 +44,7 @@ struct Program {
   int geo = 0;             // bulk-copy launch geometry: 0 = kGeoWide, 1 = kGeoDual
   int64_t bytes = 0;       // operand rows moved (rows x 16-B-rounded row, + fold terms)
   int g4_kinds = 0;        // source kinds of its gather4 items (tensor maps the launch needs)
+  bool tree = false;       // carries tree-order FOLD programs (kTermRankTree)
   TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
 };
 
@@ -304,7 +305,7 @@ void build_programs(dgcl_ctx *c) {
       for (int gi = 0; gi < ng; ++gi) {
         const DevGroup &g = L.groups[gi];
         if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
-        if (gi >= L.direct_begin && gi < L.fanout_end) continue;
+        if (gi >= L.direct_begin && gi < L.tree_end) continue;
         if (!fused && g.exec_rank != r) continue;
         gids[r].push_back(gi);
         if (!(fan_avail && is_stage1_copy(g))) gids_fan[r].push_back(gi);
@@ -324,15 +325,18 @@ void build_programs(dgcl_ctx *c) {
                         L.atomic_end > L.direct_end;
     const bool direct = !atomic && fused && dir == DIR_BWD && c->direct_reduce &&
                         L.n_stages <= 1 && L.direct_end > L.direct_begin;
-    if (direct || atomic) {
+    // relay plans: each owner row folds its whole tree in the reversed plan's order in one pass
+    const bool tree = fused && dir == DIR_BWD && c->direct_reduce && L.n_stages >= 2 &&
+                      L.tree_end > L.fanout_end;
+    if (direct || atomic || tree) {
       gids[0].clear();
-      for (int gi = atomic ? L.direct_end : L.direct_begin; gi < (atomic ? L.atomic_end : L.direct_end);
-           ++gi)
-        gids[0].push_back(gi);
+      const int b = atomic ? L.direct_end : tree ? L.fanout_end : L.direct_begin;
+      const int e = atomic ? L.atomic_end : tree ? L.tree_end : L.direct_end;
+      for (int gi = b; gi < e; ++gi) gids[0].push_back(gi);
     }
     // the host interpreter runs the fused-order program of this direction
     c->host_gids[dir].clear();
-    if (direct || atomic) {
+    if (direct || atomic || tree) {
       c->host_gids[dir] = gids[0];
     } else {
       if (dir == DIR_FWD && fan_avail)
@@ -340,7 +344,7 @@ void build_programs(dgcl_ctx *c) {
       for (int gi = 0; gi < ng; ++gi) {
         const DevGroup &g = L.groups[gi];
         if (g.op == OP_READY || g.op == OP_WAIT || g.dir != dir) continue;
-        if (gi >= L.direct_begin && gi < L.fanout_end) continue;
+        if (gi >= L.direct_begin && gi < L.tree_end) continue;
         if (fan_avail && is_stage1_copy(g)) continue;
         c->host_gids[dir].push_back(gi);
       }
@@ -377,6 +381,9 @@ void build_programs(dgcl_ctx *c) {
           }
           P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
           P.g4_kinds = 0;
+          P.tree = false;
+          for (const DevItem &it : P.items)
+            if (it.op == OP_FOLD && it.term_mode == kTermRankTree) P.tree = true;
           for (const DevItem &it : P.items)
             if (it.op == OP_COPY && (it.flags & kItemGather4)) P.g4_kinds |= 1 << it.src_kind;
           P.bytes = 0;
@@ -436,7 +443,7 @@ int tma_block(const dgcl_ctx *c, const Program &pg) {
   if (c->threads_set) return c->threads;
   const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
   if (pg.geo == 0 && (pg.op_mask & kMaskFold))
-    return pg.op_mask == kMaskFold && pg.fold_wide ? 1024 : 512;
+    return pg.op_mask == kMaskFold && pg.fold_wide && !pg.tree ? 1024 : 512;
   return G.threads;
 }
 

@@ -96,6 +96,30 @@ __device__ __forceinline__ void add4(float4 &a, const int4 &b) {
   a.w = __fadd_rn(a.w, __int_as_float(b.w));
 }
 
+// kTermRankTree: one output chunk of a postfix fold program — every word pushes load(word), then
+// replaces the top two by (below + top) (word >> 24) & 15 times; the stack bottom is the starting
+// value.  The stack lives in local memory (dynamic depth), L1-resident.
+template <typename Load>
+__device__ __forceinline__ float4 fold_tree(float4 init, const uint32_t *prog, int n, Load load) {
+  float4 stk[kTreeMaxDepth];
+  int sp = 0;
+  stk[0] = init;
+  for (int j = 0; j < n; ++j) {
+    const uint32_t w = prog[j];
+    float4 t = load(w);
+    for (uint32_t a = (w >> kTreeAddShift) & 15u; a > 0; --a) {
+      const float4 b = stk[sp--];
+      t.x = __fadd_rn(b.x, t.x);
+      t.y = __fadd_rn(b.y, t.y);
+      t.z = __fadd_rn(b.z, t.z);
+      t.w = __fadd_rn(b.w, t.w);
+    }
+    stk[++sp] = t;
+  }
+  return stk[0];
+}
+
+
 // Spin until *p >= target (acquire, system scope), bounded by the watchdog.
 static __device__ __noinline__ bool wait_geq(const uint64_t *p, uint64_t target, const ExecParams &P,
                                       int code) {

@@ -153,6 +153,22 @@ __device__ __forceinline__ void fold_rows(const ExecParams &P, const DevItem &I)
     const uint32_t col = e - r * nch;
     const int nb = V16 ? (col + 1 == nch ? tail : 16) : 4;
     char *dp = D.ptr + row_of(didx, db, r) * D.pitch + (int64_t)col * (V16 ? 16 : 4);
+    if (mode == kTermRankTree) {  // loopback tree-order backward: postfix program per row
+      const int64_t t0 = __ldg(tp + r), t1 = __ldg(tp + r + 1);
+      const float4 acc = fold_tree(
+          as_f4(V16 && nb == 16 ? ld_cg_v4(dp) : ld_part<false>(dp, V16 ? nb : 4)),
+          P.terms + t0, (int)(t1 - t0), [&](uint32_t w) {
+            const BufRef &B = P.buf[K_HGRAD][w >> 28];
+            const char *p = B.ptr + (int64_t)(w & kTreeRowMask) * B.pitch +
+                            (int64_t)col * (V16 ? 16 : 4);
+            return as_f4(V16 && nb == 16 ? ld_nc_v4(p) : ld_part<true>(p, V16 ? nb : 4));
+          });
+      if (V16 && nb == 16)
+        st_v4(dp, as_i4(acc));
+      else
+        st_part(dp, as_i4(acc), V16 ? nb : 4);
+      continue;
+    }
     int64_t t = __ldg(tp + r);
     const int64_t t1 = __ldg(tp + r + 1);
     float4 acc;

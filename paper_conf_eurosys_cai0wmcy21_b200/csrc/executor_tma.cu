@@ -614,6 +614,7 @@ __device__ __forceinline__ void store_fold_staged(const ExecParams &P, const Dev
   const uint32_t total = (uint32_t)I.rows * nch;
   const int tail = P.row_bytes - (int)(nch - 1) * 16;
   const int64_t tbase = tp[0];
+  const bool tree = I.term_mode == kTermRankTree;
   for (uint32_t e = tid; e < total; e += T) {
     const uint32_t r = fdiv(e, P);
     const uint32_t col = e - r * nch;
@@ -621,6 +622,17 @@ __device__ __forceinline__ void store_fold_staged(const ExecParams &P, const Dev
     int j = (int)(tp[r] - tbase);
     const int je = (int)(tp[r + 1] - tbase);
     float4 acc;
+    if (tree) {  // postfix program over the staged rows (loopback tree-order backward)
+      acc = fold_tree(as_f4(lds_v4(oc + r * r16)), stt + j, je - j,
+                      [&](uint32_t s) { return as_f4(lds_v4(oc + (s & kTreeRowMask) * r16)); });
+      const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
+      char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
+      if (col + 1 < nch || tail == 16)
+        st_v4(dp, as_i4(acc));
+      else
+        st_part(dp, as_i4(acc), tail);
+      continue;
+    }
     if (init) {
       acc = as_f4(lds_v4(oc + r * r16));
     } else {
@@ -642,6 +654,40 @@ __device__ __forceinline__ void store_fold_staged(const ExecParams &P, const Dev
       st_v4(dp, as_i4(acc));
     else
       st_part(dp, as_i4(acc), tail);
+  }
+}
+
+// consumers: unstaged tree-order FOLD (kTermRankTree): each output chunk evaluates its row's
+// postfix program, operands gathered from the requesters' halo-gradient rows
+__device__ __forceinline__ void store_fold_tree(const ExecParams &P, const DevItem &I,
+                                                const uint8_t *st, uint32_t tid, uint32_t T) {
+  const BufRef D = P.buf[I.dst_kind][I.dst_rank];
+  const int32_t *info = reinterpret_cast<const int32_t *>(st + kHdrInfo);
+  const int64_t *tp = reinterpret_cast<const int64_t *>(st + kTabTp) + info[0];
+  const int32_t *tab = reinterpret_cast<const int32_t *>(st + kTabDst) + info[1];
+  const uint32_t *tm = reinterpret_cast<const uint32_t *>(st + kStageHdrBytes) +
+                       window(I.t0, I.nterms, 4).skew;
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  const int tail = P.row_bytes - (int)(nch - 1) * 16;
+  for (uint32_t e = tid; e < total; e += T) {
+    const uint32_t r = fdiv(e, P);
+    const uint32_t col = e - r * nch;
+    const int nb = col + 1 == nch ? tail : 16;
+    const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
+    char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
+    const float4 init = as_f4(nb == 16 ? ld_cg_v4(dp) : ld_part<false>(dp, nb));
+    const float4 acc = fold_tree(init, tm + (tp[r] - I.t0), (int)(tp[r + 1] - tp[r]),
+                                 [&](uint32_t w) {
+                                   const BufRef &B = P.buf[K_HGRAD][w >> 28];
+                                   const char *p = B.ptr + (int64_t)(w & kTreeRowMask) * B.pitch +
+                                                   (int64_t)col * 16;
+                                   return as_f4(nb == 16 ? ld_nc_v4(p) : ld_part<true>(p, nb));
+                                 });
+    if (nb == 16)
+      st_v4(dp, as_i4(acc));
+    else
+      st_part(dp, as_i4(acc), nb);
   }
 }
 
@@ -972,6 +1018,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         store_copy_direct(P, I, st, tid, T);
       } else if ((kMask & kMaskStaged) && is_staged(I)) {
         store_fold_staged(P, I, st, tid, T);
+      } else if ((kMask & kMaskFold) && kMaxThreads <= 512 && I.op == OP_FOLD &&
+                 I.term_mode == kTermRankTree) {
+        // (tree programs never run in the 1024-thread instance: its 64 registers would spill)
+        store_fold_tree(P, I, st, tid, T);
       } else if ((kMask & kMaskFold) && I.op == OP_FOLD) {
         // many terms per row: batch a row's terms; few: batch across output chunks
         if (I.nterms >= 4 * I.rows)

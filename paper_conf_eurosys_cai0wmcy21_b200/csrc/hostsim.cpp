@@ -39,6 +39,23 @@ bool run_fanout(const Lowered &low, const DevGroup &g, int64_t r0, int64_t rows,
   return true;
 }
 
+// kTermRankTree postfix program: each word pushes its operand, then (word >> 24) & 15 adds of
+// the top two (below + top); the stack bottom is the starting value
+template <typename Val>
+float eval_tree(float init, const uint32_t *prog, int64_t n, Val val) {
+  std::vector<float> stk(1, init);
+  for (int64_t j = 0; j < n; ++j) {
+    stk.push_back(val(prog[j]));
+    for (uint32_t a = (prog[j] >> kTreeAddShift) & 15u; a > 0; --a) {
+      if (stk.size() < 2) return std::nanf("");  // (malformed program poisons the row)
+      volatile float t = stk.back();
+      stk.pop_back();
+      stk.back() = stk.back() + t;
+    }
+  }
+  return stk.size() == 1 ? stk[0] : std::nanf("");
+}
+
 void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim) {
   if (g.op == OP_READY || g.op == OP_WAIT) return;
   if (g.op == OP_FANOUT) {
@@ -62,6 +79,13 @@ void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim
           return row_ptr(B, K_HGRAD, (int)(term >> 28), term & kTermRowMask);
         return row_ptr(B, (term & kTermSlot) ? K_SLOT : K_HGRAD, g.exec_rank, term & ~kTermSlot);
       };
+      if (g.term_mode == kTermRankTree) {
+        for (int c = 0; c < dim; ++c)
+          d[c] = eval_tree(d[c], low.terms.data() + t0, t1 - t0, [&](uint32_t w) {
+            return row_ptr(B, K_HGRAD, (int)(w >> 28), w & kTreeRowMask)[c];
+          });
+        continue;
+      }
       for (int c = 0; c < dim; ++c) {
         int64_t t = t0;
         float acc;
@@ -117,7 +141,7 @@ bool run_item(const Lowered &low, const DevItem &it, const std::vector<DevRun> &
   const int64_t *tp = low.term_ptr.data() + it.tp;
   if (it.flags & kItemStaged) {
     const int64_t nseg = it.src >> kSegShift, seg0 = it.src & ((1ll << kSegShift) - 1);
-    const int64_t nst = (it.fold_init ? it.rows : 0) + it.nterms;
+    const int64_t nst = (it.fold_init ? it.rows : 0) + it.nterms;  // stage rows reserved
     if (nst > kMaxItemRows || nseg < 1 || nseg > nst) return false;
     std::vector<float> stage((size_t)nst * B.pitch, std::nanf(""));
     std::vector<uint8_t> hit(nst, 0);
@@ -134,6 +158,13 @@ bool run_item(const Lowered &low, const DevItem &it, const std::vector<DevRun> &
     }
     for (int64_t r = 0; r < it.rows; ++r) {
       float *d = row_ptr(B, it.dst_kind, it.dst_rank, drow(r));
+      if (low.groups[it.group].term_mode == kTermRankTree) {
+        const int64_t j = tp[r] - tp[0], je = tp[r + 1] - tp[0];
+        for (int c = 0; c < dim; ++c)
+          d[c] = eval_tree(stage[(size_t)r * B.pitch + c], sterms.data() + it.t0 + j, je - j,
+                           [&](uint32_t s) { return stage[(size_t)(s & kTreeRowMask) * B.pitch + c]; });
+        continue;
+      }
       for (int c = 0; c < dim; ++c) {
         int64_t j = tp[r] - tp[0];
         const int64_t je = tp[r + 1] - tp[0];

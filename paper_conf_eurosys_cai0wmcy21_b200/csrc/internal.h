@@ -72,6 +72,16 @@ constexpr uint32_t kTermSlot = 0x80000000u;
 constexpr int32_t kTermLocal = 0;
 constexpr int32_t kTermRankHgrad = 1;
 constexpr uint32_t kTermRowMask = 0x0FFFFFFFu;
+//   kTermRankTree:  a postfix program: every term pushes an operand, then performs `adds` stack
+//                   adds (pop two, push below + top); bits 31..28 = rank r, 27..24 = adds,
+//                   23..0 = row of HGRAD(r).  The starting value (fold_init) is the stack
+//                   bottom.  The loopback tree-order backward of relay plans: each owner row
+//                   folds its whole tree in the reversed plan's order in one pass.
+//                   Staged items keep the adds in the staged-term words (stage row | adds << 24)
+constexpr int32_t kTermRankTree = 2;
+constexpr uint32_t kTreeRowMask = 0x00FFFFFFu;
+constexpr int kTreeAddShift = 24;
+constexpr int kTreeMaxDepth = 17;  // stack slots: bottom + one per tree level (<= kMaxRanks)
 
 struct DevGroup {
   int32_t op;

@@ -15,6 +15,7 @@
 // writer, no atomics — and additionally fixes the summation order (R6).
 
 #include <algorithm>
+#include <functional>
 #include <chrono>
 #include <cstring>
 #include <map>
@@ -528,6 +529,88 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     if (!fits) L.groups.resize(L.atomic_end);  // rows beyond the 27-bit dest field: per-pair groups
   }
   L.fanout_end = (int)L.groups.size();
+  // ---- loopback tree-order backward (relay plans) ----
+  // With every virtual rank on one device the owner can evaluate the reversed plan's whole fold
+  // for its row in one pass: the staged backward computes val_c(u) = ((own_c + val(y1)) +
+  // val(y2)) ... bottom-up along T_u and the owner emb_grad = ((L + val(c1)) +
+  // val(c2)) ...; here the same expression, same operands, same association, is one postfix
+  // program per owner row over the requesters' halo-gradient rows (kTermRankTree), so the
+  // result is bit-identical to the staged pushes without their slot round trips and stage
+  // barriers.  (The multi-GPU form, and loopback with direct_reduce = 0, run the stages.)
+  if (K >= 2) {
+    auto kids = [&](int64_t vi, int x, int64_t *outv) -> int {
+      int n = 0;
+      for (int64_t f = plan.e_ptr[vi]; f < plan.e_ptr[vi + 1]; ++f)
+        if (plan.e_parent[f] == x) outv[n++] = f;
+      std::sort(outv, outv + n,
+                [&](int64_t a, int64_t b) { return plan.e_child[a] < plan.e_child[b]; });
+      return n;
+    };
+    bool fits = true;
+    int depth = 0, max_depth = 0;
+    // postfix of val(x) for vertex vi: own(x) (if x requested u), then each child ascending,
+    // an add after every value but the first; an add is counted on the operand word just
+    // emitted (every add follows an operand or another add)
+    auto add_after_last = [&]() {
+      const uint32_t w = L.terms.back();
+      const uint32_t a = ((w >> kTreeAddShift) & 15u) + 1;
+      if (a > 15) fits = false;
+      L.terms.back() = (w & ~(15u << kTreeAddShift)) | ((a & 15u) << kTreeAddShift);
+      --depth;
+    };
+    std::function<void(int64_t, int)> emit = [&](int64_t vi, int x) {
+      const int64_t u = plan.order[vi];
+      int64_t ch[kMaxRanks];
+      const int n = kids(vi, x, ch);
+      const int32_t pos = halo_pos(rel, u, x);
+      bool have = false;
+      if (pos >= 0) {
+        if ((uint32_t)pos > kTreeRowMask) fits = false;
+        L.terms.push_back(((uint32_t)x << 28) | ((uint32_t)pos & kTreeRowMask));
+        max_depth = std::max(max_depth, ++depth);
+        have = true;
+      }
+      for (int t = 0; t < n; ++t) {
+        emit(vi, plan.e_child[ch[t]]);
+        if (have) add_after_last();
+        have = true;
+      }
+    };
+    std::vector<std::vector<std::pair<int64_t, int64_t>>> rows_of(m);  // (loc, vi)
+    for (int64_t vi = 0; vi < NV; ++vi)
+      if (plan.e_ptr[vi + 1] > plan.e_ptr[vi]) rows_of[part[plan.order[vi]]].push_back({loc[plan.order[vi]], vi});
+    const size_t t_begin = L.terms.size(), p_begin = L.term_ptr.size();
+    for (int s = 0; s < m && fits; ++s) {
+      auto &rows = rows_of[s];
+      if (rows.empty()) continue;
+      std::sort(rows.begin(), rows.end());
+      DevGroup g = base_group(OP_FOLD, DIR_BWD, s, s, 1);
+      g.dst_kind = K_EGRAD;
+      g.fold_init = 1;
+      g.term_mode = kTermRankTree;
+      g.term_ptr = (int64_t)L.term_ptr.size();
+      L.term_ptr.push_back((int64_t)L.terms.size());
+      std::vector<int64_t> src, dst;
+      int64_t ch[kMaxRanks];
+      for (auto &r : rows) {
+        dst.push_back(r.first);
+        const int n = kids(r.second, s, ch);
+        for (int t = 0; t < n; ++t) {  // ((L + val(c1)) + val(c2)) ...: L is the stack bottom
+          depth = 1;
+          emit(r.second, plan.e_child[ch[t]]);
+          add_after_last();
+        }
+        L.term_ptr.push_back((int64_t)L.terms.size());
+      }
+      flush_group(L.groups, g, src, dst);
+    }
+    if (!fits || max_depth + 1 > kTreeMaxDepth) {  // (cannot happen with <= 16 ranks)
+      L.groups.resize(L.fanout_end);
+      L.terms.resize(t_begin);
+      L.term_ptr.resize(p_begin);
+    }
+  }
+  L.tree_end = (int)L.groups.size();
   L.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
 }
 
@@ -566,7 +649,10 @@ void stage_fold_item(const Lowered &low, const DevGroup &g, DevItem *it, std::ve
   for (int64_t t = it->t0; t < it->t0 + it->nterms; ++t) {
     const uint32_t x = low.terms[t];
     Ref f;
-    if (g.term_mode == kTermRankHgrad) {
+    if (g.term_mode == kTermRankTree) {
+      f.key = (K_HGRAD << 8) | (int32_t)(x >> 28);
+      f.row = (int32_t)(x & kTreeRowMask);
+    } else if (g.term_mode == kTermRankHgrad) {
       f.key = (K_HGRAD << 8) | (int32_t)(x >> 28);
       f.row = (int32_t)(x & kTermRowMask);
     } else if (x & kTermSlot) {
@@ -591,8 +677,10 @@ void stage_fold_item(const Lowered &low, const DevGroup &g, DevItem *it, std::ve
     runs->push_back({refs[a].row, refs[a].key, (int32_t)(e - a), (int32_t)(base + (int64_t)a)});
     a = e;
   }
-  for (size_t a = 0; a < refs.size(); ++a)
-    (*sterms)[st0 + (refs[a].t - it->t0)] = (uint32_t)(base + (int64_t)a);
+  for (size_t a = 0; a < refs.size(); ++a)  // (tree programs keep each term's adds)
+    (*sterms)[st0 + (refs[a].t - it->t0)] =
+        (uint32_t)(base + (int64_t)a) |
+        (g.term_mode == kTermRankTree ? low.terms[refs[a].t] & (15u << kTreeAddShift) : 0u);
   it->flags |= kItemStaged;
   it->src = ((int64_t)((int64_t)runs->size() - seg0) << kSegShift) | seg0;
   it->t0 = st0;

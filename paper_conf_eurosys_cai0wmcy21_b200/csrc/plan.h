@@ -66,6 +66,7 @@ struct Lowered {
   int direct_begin = 0, direct_end = 0;  // loopback direct-reduce backward groups (direct plans)
   int atomic_end = 0;  // [direct_end, atomic_end): loopback atomic-add backward groups (ablation)
   int fanout_end = 0;  // [atomic_end, fanout_end): forward stage-1 fan-out groups, one per owner
+  int tree_end = 0;    // [fanout_end, tree_end): loopback tree-order backward (relay plans)
   std::vector<int32_t> idx;              // row index pool
   std::vector<int64_t> term_ptr;         // fold row pointers
   std::vector<uint32_t> terms;           // fold terms

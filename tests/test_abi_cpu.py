@@ -163,13 +163,16 @@ def test_work_items_host(m, opts):
 @pytest.mark.parametrize("name,sf,fan,nb", [("dgx1_like", 1, 0, 4), ("ring", 1, 0, 4),
                                            ("ring", 0, 0, 4), ("dgx1_like", 1, 1, 1),
                                            ("ring", 1, 1, 1), ("ring", 1, 0, 8),
-                                           ("dgx1_like", 0, 0, 1)])
+                                           ("dgx1_like", 0, 0, 1), ("ring", 1, 0, -1),
+                                           ("dgx1_like", 0, 0, -4)])
 def test_work_items_host_relay(name, sf, fan, nb):
-    """nb: vertex blocks of the stage chaining (fan-out stage 1 needs nb = 1)."""
+    """nb: vertex blocks of the stage chaining (fan-out stage 1 needs nb = 1); nb < 0: the staged
+    reversed-plan backward (direct_reduce = 0) with |nb| blocks instead of the loopback
+    tree-order programs."""
     g = synth.make_graph(500, 2500, 8, graph_seed=9, part_seed=19)
     _check_lowering(g, [12, 3], synth.topology.by_name(name), seed=5,
                     options={"hostsim_items": 1, "stage_fold": sf, "fanout": fan,
-                             "pipeline_blocks": nb})
+                             "pipeline_blocks": abs(nb), "direct_reduce": int(nb > 0)})
 
 
 def test_work_items_host_shuffled():

@@ -191,11 +191,15 @@ def test_per_rank_flag_protocol(m, fanout):
                                                ("ring", 0, 1, 2), ("dgx1_like", 1, 1, 3),
                                                ("dgx1_like", 0, 1, 4), ("ring", 1, 1, 4),
                                                ("ring", 0, 1, 5), ("dgx1_like", 1, 1, 6),
-                                               ("ring", 1, 0, 6)])
+                                               ("ring", 1, 0, 6), ("ring", 0, 1, 7),
+                                               ("dgx1_like", 0, 1, 7), ("ring", 1, 1, 7),
+                                               ("dgx1_like", 0, 0, 7)])
 def test_relay_plans(name, flags, tma, sf):
     """sf: stage_fold 0/1; 2, 3 = stage_fold with the DUAL / WIDE geometry forced; 4 = fan-out
     stage 1 (first hops into halos and relay staging, done counts per receiver); 5, 6 = one /
-    eight vertex blocks in the stage chaining (default 4)."""
+    eight vertex blocks in the stage chaining (default 1); 7 = the staged reversed-plan backward
+    (direct_reduce = 0: pushes into slots stage by stage, the multi-GPU form) instead of the
+    loopback tree-order programs."""
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
     opts = {"tma": tma, "stage_fold": min(sf, 1)}
     if sf in (2, 3):
@@ -204,6 +208,8 @@ def test_relay_plans(name, flags, tma, sf):
         opts["fanout"] = 1
     if sf in (5, 6):
         opts["pipeline_blocks"] = 1 if sf == 5 else 8
+    if sf == 7:
+        opts["direct_reduce"] = 0
     c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags, options=opts)
     assert c.ctx.plan_info()["n_stages"] >= 2
     _check_case(c)
