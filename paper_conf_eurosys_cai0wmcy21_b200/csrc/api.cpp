@@ -371,6 +371,8 @@ void build_programs(dgcl_ctx *c) {
           for (const DevItem &it : P.items) {
             if (it.op == OP_FOLD && (it.flags & kItemStaged)) {
               P.op_mask |= kMaskStaged;
+            } else if (it.op == OP_FOLD && it.term_mode == kTermRankTree) {
+              P.op_mask |= kMaskTree;
             } else if (it.op == OP_FOLD) {
               P.op_mask |= kMaskFold;
               fold_rows += it.rows;
@@ -416,7 +418,8 @@ void build_programs(dgcl_ctx *c) {
           ops += (it.flags & kItemGather4) ? (it.rows + 3) / 4 : it.nterms;
         }
         const bool copy_only = (P.op_mask & ~(kMaskCopy | kMaskFanout)) == 0;
-        if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & kMaskFold) || waits)
+        if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & (kMaskFold | kMaskTree)) ||
+            waits)
           build(0);
       }
     }
@@ -442,7 +445,7 @@ dgcl_status upload(dgcl_ctx *c, T **dptr, const std::vector<T> &v) {
 int tma_block(const dgcl_ctx *c, const Program &pg) {
   if (c->threads_set) return c->threads;
   const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
-  if (pg.geo == 0 && (pg.op_mask & kMaskFold))
+  if (pg.geo == 0 && (pg.op_mask & (kMaskFold | kMaskTree)))
     return pg.op_mask == kMaskFold && pg.fold_wide && !pg.tree ? 1024 : 512;
   return G.threads;
 }

@@ -98,7 +98,8 @@ __device__ __forceinline__ void add4(float4 &a, const int4 &b) {
 
 // kTermRankTree: one output chunk of a postfix fold program — every word pushes load(word), then
 // replaces the top two by (below + top) (word >> 24) & 15 times; the stack bottom is the starting
-// value.  The stack lives in local memory (dynamic depth), L1-resident.
+// value.  The stack is a small local array (dynamic depth; measured faster than a shifting
+// register stack, whose moves cost more than the L1 round trips).
 template <typename Load>
 __device__ __forceinline__ float4 fold_tree(float4 init, const uint32_t *prog, int n, Load load) {
   float4 stk[kTreeMaxDepth];
@@ -107,7 +108,7 @@ __device__ __forceinline__ float4 fold_tree(float4 init, const uint32_t *prog, i
   for (int j = 0; j < n; ++j) {
     const uint32_t w = prog[j];
     float4 t = load(w);
-    for (uint32_t a = (w >> kTreeAddShift) & 15u; a > 0; --a) {
+    for (uint32_t a = (w >> kTreeAddShift) & 15u; a > 0; --a) {  // t = pop() + t
       const float4 b = stk[sp--];
       t.x = __fadd_rn(b.x, t.x);
       t.y = __fadd_rn(b.y, t.y);
@@ -118,7 +119,6 @@ __device__ __forceinline__ float4 fold_tree(float4 init, const uint32_t *prog, i
   }
   return stk[0];
 }
-
 
 // Spin until *p >= target (acquire, system scope), bounded by the watchdog.
 static __device__ __noinline__ bool wait_geq(const uint64_t *p, uint64_t target, const ExecParams &P,

@@ -614,7 +614,25 @@ __device__ __forceinline__ void store_fold_staged(const ExecParams &P, const Dev
   const uint32_t total = (uint32_t)I.rows * nch;
   const int tail = P.row_bytes - (int)(nch - 1) * 16;
   const int64_t tbase = tp[0];
-  const bool tree = I.term_mode == kTermRankTree;
+  if (I.term_mode == kTermRankTree) {
+    // postfix programs over the staged rows (loopback tree-order backward), one chunk per thread
+    for (uint32_t e = tid; e < total; e += T) {
+      const uint32_t r = fdiv(e, P);
+      const uint32_t col = e - r * nch;
+      const uint8_t *oc = ops + col * 16;
+      const int j = (int)(tp[r] - tbase), je = (int)(tp[r + 1] - tbase);
+      const float4 acc =
+          fold_tree(as_f4(lds_v4(oc + r * r16)), stt + j, je - j,
+                    [&](uint32_t s) { return as_f4(lds_v4(oc + (s & kTreeRowMask) * r16)); });
+      const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
+      char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
+      if (col + 1 < nch || tail == 16)
+        st_v4(dp, as_i4(acc));
+      else
+        st_part(dp, as_i4(acc), tail);
+    }
+    return;
+  }
   for (uint32_t e = tid; e < total; e += T) {
     const uint32_t r = fdiv(e, P);
     const uint32_t col = e - r * nch;
@@ -622,17 +640,6 @@ __device__ __forceinline__ void store_fold_staged(const ExecParams &P, const Dev
     int j = (int)(tp[r] - tbase);
     const int je = (int)(tp[r + 1] - tbase);
     float4 acc;
-    if (tree) {  // postfix program over the staged rows (loopback tree-order backward)
-      acc = fold_tree(as_f4(lds_v4(oc + r * r16)), stt + j, je - j,
-                      [&](uint32_t s) { return as_f4(lds_v4(oc + (s & kTreeRowMask) * r16)); });
-      const int64_t drow = I.dst >= 0 ? I.dst + r : (int64_t)tab[r];
-      char *dp = D.ptr + drow * D.pitch + (int64_t)col * 16;
-      if (col + 1 < nch || tail == 16)
-        st_v4(dp, as_i4(acc));
-      else
-        st_part(dp, as_i4(acc), tail);
-      continue;
-    }
     if (init) {
       acc = as_f4(lds_v4(oc + r * r16));
     } else {
@@ -1018,9 +1025,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         store_copy_direct(P, I, st, tid, T);
       } else if ((kMask & kMaskStaged) && is_staged(I)) {
         store_fold_staged(P, I, st, tid, T);
-      } else if ((kMask & kMaskFold) && kMaxThreads <= 512 && I.op == OP_FOLD &&
-                 I.term_mode == kTermRankTree) {
-        // (tree programs never run in the 1024-thread instance: its 64 registers would spill)
+      } else if ((kMask & kMaskTree) && I.op == OP_FOLD && I.term_mode == kTermRankTree) {
+        // (unstaged tree programs have their own kernel instance: the register stack would
+        // crowd the other fold paths)
         store_fold_tree(P, I, st, tid, T);
       } else if ((kMask & kMaskFold) && I.op == OP_FOLD) {
         // many terms per row: batch a row's terms; few: batch across output chunks
@@ -1062,7 +1069,7 @@ int launch_mask(const ExecParams &p, int grid, int block, cudaStream_t s) {
   return (int)cudaGetLastError();
 }
 
-constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged | kMaskFanout;
+constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged | kMaskFanout | kMaskTree;
 
 }  // namespace
 
@@ -1073,6 +1080,9 @@ int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream) 
     // forward with fan-out stage 1 (uniform plans), plus relay copies (relay plans)
     case kMaskFanout: return launch_mask<kMaskFanout>(p, grid, block, s);
     case kMaskFanout | kMaskCopy: return launch_mask<kMaskFanout | kMaskCopy>(p, grid, block, s);
+    // loopback tree-order backward (relay plans): staged programs, plus unstaged ones
+    case kMaskTree: return launch_mask<kMaskTree>(p, grid, block, s);
+    case kMaskTree | kMaskStaged: return launch_mask<kMaskTree | kMaskStaged>(p, grid, block, s);
     case kMaskFold:
       // fold-only launches of unstaged folds are latency-bound gathers by the consumer warps:
       // the host may run them with 1024 threads (31 consumer warps, <= 64 registers) for twice

@@ -81,7 +81,7 @@ constexpr uint32_t kTermRowMask = 0x0FFFFFFFu;
 constexpr int32_t kTermRankTree = 2;
 constexpr uint32_t kTreeRowMask = 0x00FFFFFFu;
 constexpr int kTreeAddShift = 24;
-constexpr int kTreeMaxDepth = 17;  // stack slots: bottom + one per tree level (<= kMaxRanks)
+constexpr int kTreeMaxDepth = 8;  // register stack slots (bottom included); deeper trees: staged
 
 struct DevGroup {
   int32_t op;
@@ -210,7 +210,8 @@ DGCL_HD inline uint32_t trace_tag(const DevItem &I, int stage, int block) {
   return (uint32_t)I.op | (uint32_t)I.dir << 4 | (uint32_t)I.exec_rank << 8 |
          (uint32_t)I.dst_rank << 16 | (uint32_t)(stage & 31) << 24 | (uint32_t)(block & 7) << 29;
 }
-constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8, kMaskFanout = 16;
+constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8, kMaskFanout = 16,
+                  kMaskTree = 32;  // unstaged tree-order FOLD items (their own instance)
 
 // A run of `len` rows whose source rows src.. and destination rows dst.. are both consecutive;
 // `pos` is the first row's index inside its item.  One bulk copy moves a run when the pitches

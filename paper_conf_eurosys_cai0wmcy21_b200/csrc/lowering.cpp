@@ -604,7 +604,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       }
       flush_group(L.groups, g, src, dst);
     }
-    if (!fits || max_depth + 1 > kTreeMaxDepth) {  // (cannot happen with <= 16 ranks)
+    if (!fits || max_depth > kTreeMaxDepth) {  // too deep for the register stack: staged form
       L.groups.resize(L.fanout_end);
       L.terms.resize(t_begin);
       L.term_ptr.resize(p_begin);
