@@ -98,26 +98,38 @@ __device__ __forceinline__ void add4(float4 &a, const int4 &b) {
 
 // kTermRankTree: one output chunk of a postfix fold program — every word pushes load(word), then
 // replaces the top two by (below + top) (word >> 24) & 15 times; the stack bottom is the starting
-// value.  The stack is a small local array (dynamic depth; measured faster than a shifting
-// register stack, whose moves cost more than the L1 round trips).
+// value.  The top of the stack lives in a register and only the entries below it in a small
+// local array, so a word with adds >= 1 consumes the register top without memory traffic: a
+// direct (relay-free) tree, ((L + o1) + o2) ..., runs entirely in registers, and only relay
+// subtrees (a word with no adds pushes) touch local memory.
 template <typename Load>
 __device__ __forceinline__ float4 fold_tree(float4 init, const uint32_t *prog, int n, Load load) {
-  float4 stk[kTreeMaxDepth];
-  int sp = 0;
-  stk[0] = init;
+  float4 below[kTreeMaxDepth];
+  int nb = 0;
+  float4 top = init;
   for (int j = 0; j < n; ++j) {
     const uint32_t w = prog[j];
     float4 t = load(w);
-    for (uint32_t a = (w >> kTreeAddShift) & 15u; a > 0; --a) {  // t = pop() + t
-      const float4 b = stk[sp--];
+    uint32_t a = (w >> kTreeAddShift) & 15u;
+    if (a == 0) {  // push: the old top goes below
+      below[nb++] = top;
+      top = t;
+      continue;
+    }
+    t.x = __fadd_rn(top.x, t.x);  // the first add consumes the register top
+    t.y = __fadd_rn(top.y, t.y);
+    t.z = __fadd_rn(top.z, t.z);
+    t.w = __fadd_rn(top.w, t.w);
+    for (; a > 1; --a) {
+      const float4 b = below[--nb];
       t.x = __fadd_rn(b.x, t.x);
       t.y = __fadd_rn(b.y, t.y);
       t.z = __fadd_rn(b.z, t.z);
       t.w = __fadd_rn(b.w, t.w);
     }
-    stk[++sp] = t;
+    top = t;
   }
-  return stk[0];
+  return top;
 }
 
 // Spin until *p >= target (acquire, system scope), bounded by the watchdog.
