@@ -213,6 +213,11 @@ dgcl_status init_common(int32_t rank, int32_t world, int32_t dev, int64_t n, con
 
 bool has_device(dgcl_ctx *c) { return c->device >= 0; }
 
+void relower(dgcl_ctx *c) {
+  lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low, c->pipeline_blocks,
+             c->atomic_backward, c->fanout);
+}
+
 void compute_layout(dgcl_ctx *c) {
   const int m = c->world;
   const Lowered &L = c->low;
@@ -711,7 +716,7 @@ dgcl_status plan_common(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *req_
               : spst_plan(c->topo, c->part.data(), c->rel, seed, &c->plan);
     if (!e.empty()) return fail(c, DGCL_EPLAN, "%s", e.c_str());
     if (c->plan.n_stages >= kMaxStages) return fail(c, DGCL_EPLAN, "too many stages");
-    lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low, c->pipeline_blocks);
+    relower(c);
     c->halo_off.assign(c->world + 1, 0);
     for (int d = 0; d < c->world; ++d) c->halo_off[d + 1] = c->halo_off[d] + c->rel.n_halo[d];
     compute_layout(c);
@@ -1192,7 +1197,7 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (value < 1 || value > kMaxBlocks) return fail(c, DGCL_EINVAL, "pipeline_blocks in 1..%d", kMaxBlocks);
     c->pipeline_blocks = (int)value;
     if (c->planned) {
-      lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low, c->pipeline_blocks);
+      relower(c);
       compute_layout(c);
       build_programs(c);
     }
@@ -1205,12 +1210,20 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "fanout") {  // forward stage 1: per-owner fan-out items (1) or per-pair COPY items (0)
     c->fanout = value != 0;
-    if (c->planned) build_programs(c);
+    if (c->planned) {  // its groups are lowered only when asked for
+      relower(c);
+      compute_layout(c);
+      build_programs(c);
+    }
     return DGCL_OK;
   }
   if (k == "atomic_backward") {  // ablation: loopback single-stage backward with atomic adds
     c->atomic_backward = value != 0;
-    if (c->planned) build_programs(c);
+    if (c->planned) {  // its groups are lowered only when asked for
+      relower(c);
+      compute_layout(c);
+      build_programs(c);
+    }
     return DGCL_OK;
   }
   if (k == "direct_reduce") {

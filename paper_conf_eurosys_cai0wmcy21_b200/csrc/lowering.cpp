@@ -56,7 +56,8 @@ inline int32_t halo_pos(const Relation &rel, int64_t u, int d) {
 }  // namespace
 
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
-                const std::vector<int64_t> &loc, Lowered *out, int n_blocks) {
+                const std::vector<int64_t> &loc, Lowered *out, int n_blocks, bool with_atomic,
+                bool with_fanout) {
   auto t0 = std::chrono::steady_clock::now();
   const int m = plan.m;
   const int K = plan.n_stages;
@@ -450,7 +451,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   // its halo-gradient rows straight into the owner's rows with atomic reductions, one group per
   // (requester c, owner p), rows in c's halo order (consecutive source rows).  Same sum, but the
   // order of the adds is whatever the hardware makes it: not reproducible bit for bit.
-  if (K <= 1) {
+  if (K <= 1 && with_atomic) {
     std::vector<std::vector<std::pair<int64_t, int64_t>>> pairs((size_t)m * m);  // (pos_c, loc)
     for (int64_t vi = 0; vi < NV; ++vi) {
       const int64_t u = plan.order[vi];
@@ -484,7 +485,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   // Rows are the owner's local rows in loc order (consecutive sources: one bulk copy per item);
   // dests per row in ascending receiver id, as word pairs in the terms pool: (receiver << 28 |
   // relay bit | destination row, source row) — the executor maps (pair, chunk) to threads.
-  {
+  if (with_fanout) {
     int64_t N = (int64_t)loc.size();
     std::vector<int64_t> vi_of(N, -1);
     for (int64_t vi = 0; vi < NV; ++vi) vi_of[plan.order[vi]] = vi;
@@ -768,26 +769,35 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     // forward, whose rows already come once from DRAM, lost 2 % to the smaller items.
     aligned.assign(j - i, 0);
     if (lim.align_sources && row16 <= kGather4MaxRowBytes) {
+      // (groups whose sources come in short runs, < 4 rows on average — the per-row gather
+      // regime; long runs already stream each row once)
+      auto short_runs = [&](const DevGroup &h) {
+        int64_t runs = 1;
+        for (int64_t r = 1; r < h.n_rows; ++r) runs += src_row(h, r) != src_row(h, r - 1) + 1;
+        return runs * 4 > h.n_rows;
+      };
       auto alignable = [&](const DevGroup &h) {
         return h.op == OP_COPY && h.dir == DIR_FWD && h.src_kind == K_EMB && !h.atomic_add &&
-               h.n_rows > 0 && ascending_src(h);
+               h.n_rows > 0 && ascending_src(h) && short_runs(h);
       };
       const int64_t rpi = copy_rpi(spread_rpi);
+      std::vector<uint8_t> can(j - i);  // alignable, evaluated once per group (O(rows))
+      for (size_t q = i; q < j; ++q) can[q - i] = alignable(low.groups[gids[q]]) ? 1 : 0;
       for (size_t q = i; q < j; ++q) {
         const DevGroup &g = low.groups[gids[q]];
-        if (aligned[q - i] || !alignable(g)) continue;
+        if (aligned[q - i] || !can[q - i]) continue;
         // (groups of about the same size only: relay plans' first hops are very uneven, and a
         // dense group would cut a sparse one into many small items)
         std::vector<size_t> set;
         int64_t big = 0;
         for (size_t q2 = q; q2 < j; ++q2) {
           const DevGroup &h = low.groups[gids[q2]];
-          if (!aligned[q2 - i] && h.exec_rank == g.exec_rank && alignable(h))
+          if (!aligned[q2 - i] && h.exec_rank == g.exec_rank && can[q2 - i])
             big = std::max(big, h.n_rows);
         }
         for (size_t q2 = q; q2 < j; ++q2) {
           const DevGroup &h = low.groups[gids[q2]];
-          if (!aligned[q2 - i] && h.exec_rank == g.exec_rank && alignable(h) &&
+          if (!aligned[q2 - i] && h.exec_rank == g.exec_rank && can[q2 - i] &&
               4 * h.n_rows >= 3 * big)
             set.push_back(q2);
         }

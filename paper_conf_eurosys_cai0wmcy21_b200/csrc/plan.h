@@ -97,9 +97,11 @@ struct Lowered {
 };
 
 // n_blocks: vertex blocks for the stage chaining of relay plans (1 = one counter per stage;
-// single-stage plans always use 1)
+// single-stage plans always use 1); with_atomic / with_fanout: also build the ablation groups
+// (atomic backward, fan-out forward) — only when their option is set (they cost lowering time)
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
-                const std::vector<int64_t> &loc, Lowered *out, int n_blocks = 1);
+                const std::vector<int64_t> &loc, Lowered *out, int n_blocks = 1,
+                bool with_atomic = false, bool with_fanout = false);
 
 // Work items for one launch: the groups `gids` (already in stage order, READY / WAIT groups
 // included by the caller) cut into row ranges of about item_bytes gathered bytes and interleaved
