@@ -28,6 +28,13 @@ using namespace dev;
 namespace {
 
 constexpr int kMaxFoldPrefetch = 4;
+#ifndef DGCL_REG_MINB
+#define DGCL_REG_MINB 2  // 2 x 512 threads per SM (64 registers): twice the loads in flight
+#endif
+#ifndef DGCL_COPY_UNROLL
+#define DGCL_COPY_UNROLL 2  // A/B on B200: 2 beat 4 and 8 (fewest spills at 64 registers per thread)
+#endif
+constexpr int kCopyUnroll = DGCL_COPY_UNROLL;  // 16-B loads in flight per thread (whole-chunk copies)
 
 __device__ __forceinline__ const int32_t *idx_of(const ExecParams &P, int64_t enc) {
   return enc < 0 ? P.idx + ~enc : nullptr;
@@ -46,6 +53,7 @@ __device__ __forceinline__ void copy_rows_v16(const ExecParams &P, const DevItem
   const uint32_t total = (uint32_t)I.rows * nch;
   const int tail = P.row_bytes - (int)(nch - 1) * 16;  // bytes in each row's last chunk (1..16)
   const uint32_t T = blockDim.x;
+#pragma unroll 1
   for (uint32_t e0 = threadIdx.x; e0 < total; e0 += T * kUnroll) {
     int4 v[kUnroll];
     char *dp[kUnroll];
@@ -70,6 +78,42 @@ __device__ __forceinline__ void copy_rows_v16(const ExecParams &P, const DevItem
       else if (nb[j] > 0)
         st_part(dp[j], v[j], nb[j]);
     }
+  }
+}
+
+// whole-chunk rows (row_bytes % 16 == 0): destinations kept as (row, chunk) 32-bit pairs instead
+// of pointers until the store loop, so the kUnroll vectors in flight fit 64 registers unspilled
+template <bool kNC>
+__device__ __forceinline__ void copy_rows_full(const ExecParams &P, const DevItem &I) {
+  const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
+  const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
+  char *dbase = P.buf[I.dst_kind][I.dst_rank].ptr;
+  const int64_t dpitch = P.buf[I.dst_kind][I.dst_rank].pitch;
+  const int32_t *sidx = idx_of(P, I.src), *didx = idx_of(P, I.dst);
+  const int64_t sb = I.src, db = I.dst;
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  const uint32_t T = blockDim.x;
+#pragma unroll 1
+  for (uint32_t e0 = threadIdx.x; e0 < total; e0 += T * kCopyUnroll) {
+    int4 v[kCopyUnroll];
+    int32_t drow[kCopyUnroll];
+    uint32_t dcol[kCopyUnroll];
+#pragma unroll
+    for (int j = 0; j < kCopyUnroll; ++j) {
+      const uint32_t e = e0 + j * T;
+      drow[j] = -1;
+      if (e < total) {
+        const uint32_t r = fdiv(e, P);
+        dcol[j] = e - r * nch;
+        drow[j] = (int32_t)row_of(didx, db, r);
+        const char *sp = sbase + row_of(sidx, sb, r) * spitch + (int64_t)dcol[j] * 16;
+        v[j] = kNC ? ld_nc_v4(sp) : ld_cg_v4(sp);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < kCopyUnroll; ++j)
+      if (drow[j] >= 0) st_v4(dbase + (int64_t)drow[j] * dpitch + (int64_t)dcol[j] * 16, v[j]);
   }
 }
 
@@ -102,6 +146,7 @@ __device__ __forceinline__ void copy_rows_b32(const ExecParams &P, const DevItem
   const uint32_t nch = (uint32_t)P.n_chunks;
   const uint32_t total = (uint32_t)I.rows * nch;
   const uint32_t T = blockDim.x;
+#pragma unroll 1
   for (uint32_t e0 = threadIdx.x; e0 < total; e0 += T * kUnroll) {
     int v[kUnroll];
     char *dp[kUnroll];
@@ -223,9 +268,21 @@ __device__ __forceinline__ void fanout_rows(const ExecParams &P, const DevItem &
   }
 }
 
-template <bool V16>
-__global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant__ ExecParams P) {
-  __shared__ int s_abort;
+// Done counts are published lazily: an item's (counter, rows) goes into a small per-CTA table, and
+// the table is flushed (every thread fences at system scope, then one red.release.sys per counter)
+// only before this CTA could block on a wait, when the table is full, and at the end.  A CTA never
+// waits while holding unpublished counts, so the co-resident grid stays deadlock-free; a fence per
+// item (a store drain every 64 KB) held the path at ~0.25 of HBM peak.
+constexpr int kPendMax = 16;
+
+// kCopyOnly: the instance for launches whose data items are all COPY (op_mask == kMaskCopy): no
+// fold / fan-out code, so the copy loop keeps its loaded vectors in registers under the 64-register
+// cap (the general instance spills there)
+template <bool V16, bool kCopyOnly>
+__global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __grid_constant__ ExecParams P) {
+  __shared__ int s_abort, s_flush, s_npend;
+  __shared__ uint64_t *s_pend_ctr[kPendMax];
+  __shared__ uint64_t s_pend_rows[kPendMax];
   __shared__ DevItem s_item;
   // per executing rank: the wait list last found satisfied (monotonic counters, fixed targets)
   __shared__ int32_t s_wait_ok[kMaxRanks];
@@ -233,13 +290,34 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
   __shared__ uint32_t s_cnt[kMaxRanks];  // fan-out rows per receiver of the current item
   if (threadIdx.x < kMaxRanks) s_cnt[threadIdx.x] = 0;
   if (threadIdx.x < kMaxRanks) s_wait_ok[threadIdx.x] = -1;
-  if (threadIdx.x == 0) s_ready_ok = 0;
+  if (threadIdx.x == 0) s_ready_ok = 0, s_npend = 0;
+  auto flush = [&]() {  // all threads: publish the pending done counts
+    __threadfence_system();  // this thread's row stores are visible system-wide ...
+    __syncthreads();         // ... for every thread of the CTA ...
+    if (threadIdx.x == 0) {  // ... before a receiver can observe the counts
+      for (int i = 0; i < s_npend; ++i) release_rows(s_pend_ctr[i], s_pend_rows[i], true);
+      s_npend = 0;
+    }
+    __syncthreads();
+  };
   for (int it = blockIdx.x; it < P.n_items; it += gridDim.x) {
     if (threadIdx.x < 4)
       reinterpret_cast<int4 *>(&s_item)[threadIdx.x] =
           __ldg(reinterpret_cast<const int4 *>(P.items + it) + threadIdx.x);
     __syncthreads();
     const DevItem I = s_item;
+    if (threadIdx.x == 0) {  // could this item block (an uncached wait)?  Or is the table full?
+      bool may_block = s_npend == kPendMax;
+      if (P.use_ready && I.ready_rank >= 0 && !((s_ready_ok >> I.ready_rank) & 1u))
+        may_block = true;
+      if (P.use_ready && I.ready_rank == kReadyAll)
+        for (int s = 0; s < P.world; ++s)
+          if (s != I.exec_rank && !((s_ready_ok >> s) & 1u)) may_block = true;
+      if (I.wait_n > 0 && s_wait_ok[I.exec_rank] != I.wait_off) may_block = true;
+      s_flush = may_block && s_npend > 0;
+    }
+    __syncthreads();
+    if (s_flush) flush();
     if (threadIdx.x == 0) {
       bool ok = true;
       if (P.trace) {
@@ -279,12 +357,14 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
     } else if (I.op == OP_COPY) {
       const bool nc = readonly_kind(I.src_kind);
       if (V16) {
-        if (nc) copy_rows_v16<true>(P, I);
-        else copy_rows_v16<false>(P, I);
+        const bool full = (P.row_bytes & 15) == 0;
+        if (nc) full ? copy_rows_full<true>(P, I) : copy_rows_v16<true>(P, I);
+        else full ? copy_rows_full<false>(P, I) : copy_rows_v16<false>(P, I);
       } else {
         if (nc) copy_rows_b32<true>(P, I);
         else copy_rows_b32<false>(P, I);
       }
+    } else if (kCopyOnly) {
     } else if (I.op == OP_FOLD) {
       fold_rows<V16>(P, I);
     } else if (I.op == OP_FANOUT) {
@@ -301,14 +381,16 @@ __global__ void __launch_bounds__(512, 1) executor_kernel(const __grid_constant_
         release_rows(P.flags[threadIdx.x] + I.sig_ctr, (uint64_t)s_cnt[threadIdx.x], true);
         s_cnt[threadIdx.x] = 0;
       }
-    } else if (I.flags & kItemSignal) {
-      __threadfence_system();  // this thread's row stores are visible system-wide ...
-      __syncthreads();         // ... for every thread of the CTA ...
-      release_rows(P.flags[I.dst_rank] + I.sig_ctr, (uint64_t)I.rows,
-                   threadIdx.x == 0);  // ... before the receiver can observe the count
+    } else if ((I.flags & kItemSignal) && threadIdx.x == 0) {  // deferred (see kPendMax)
+      uint64_t *ctr = P.flags[I.dst_rank] + I.sig_ctr;
+      int i = 0;
+      while (i < s_npend && s_pend_ctr[i] != ctr) ++i;
+      if (i == s_npend) s_pend_ctr[s_npend++] = ctr, s_pend_rows[i] = 0;
+      s_pend_rows[i] += (uint64_t)I.rows;
     }
     __syncthreads();
   }
+  if (s_npend > 0) flush();
 }
 
 }  // namespace
@@ -321,10 +403,15 @@ int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   if (grid <= 0) return 0;
   if (p.use_tma) return launch_tma_executor(p, grid, block, stream);
   cudaStream_t s = (cudaStream_t)stream;
-  if (p.vec16)
-    executor_kernel<true><<<grid, block, 0, s>>>(p);
+  const bool copy_only = p.op_mask == kMaskCopy;
+  if (p.vec16 && copy_only)
+    executor_kernel<true, true><<<grid, block, 0, s>>>(p);
+  else if (p.vec16)
+    executor_kernel<true, false><<<grid, block, 0, s>>>(p);
+  else if (copy_only)
+    executor_kernel<false, true><<<grid, block, 0, s>>>(p);
   else
-    executor_kernel<false><<<grid, block, 0, s>>>(p);
+    executor_kernel<false, false><<<grid, block, 0, s>>>(p);
   return (int)cudaGetLastError();
 }
 
@@ -334,9 +421,9 @@ int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm) {
 
 int executor_occupancy(int block, int *ctas_per_sm) {
   int a = 0, b = 0;
-  cudaError_t ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, executor_kernel<true>, block, 0);
+  cudaError_t ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, executor_kernel<true, false>, block, 0);
   if (ce != cudaSuccess) return (int)ce;
-  ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, executor_kernel<false>, block, 0);
+  ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, executor_kernel<false, false>, block, 0);
   if (ce != cudaSuccess) return (int)ce;
   *ctas_per_sm = a < b ? a : b;
   return 0;
