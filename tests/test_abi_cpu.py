@@ -288,3 +288,25 @@ def test_plan_is_dim_independent():
     a = _ctx(g, [3], synth.dgx1_like() if False else None, seed=2).plan_export()
     b = _ctx(g, [602, 256], None, seed=2).plan_export()
     assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("topo_name", ["dgx1_like", "ring"])
+def test_single_shared_hop_cost_closed_form(topo_name):
+    """tools/cost_fit.py's loopback model: when every link is the same single hop of w ticks per
+    row, the §5.1 rules (a stage costs the max over hops of load x w, stages add)
+    reduce to t(S) = (number of tree edges) x w for any plan — checked on relay plans re-costed
+    through dgcl_build_plan_from_trees, and against the oracle's plan_cost."""
+    from oracle import cost
+    from synth.topology import Topology
+    D = _D()
+    g = synth.make_graph(900, 7000, 8, graph_seed=51, part_seed=52)
+    a = _ctx(g, [8], synth.topology.by_name(topo_name), seed=2)
+    E = a.plan_export()
+    assert a.plan_info()["n_stages"] >= 2
+    one = Topology("one_hop", 8, [123.0], ["hbm"])
+    one.links = {(i, j): [0] for i in range(8) for j in range(8) if i != j}
+    w = one.hop_ticks[0]
+    b = D.loopback(g.m, g.part, [8], device=-1)
+    b.build_plan(g.req_ptr, g.req_ids, topology=one, trees=E)
+    assert b.plan_info()["model_cost_ticks"] == len(E) * w
+    assert cost.plan_cost(one, [(int(u), int(p), int(c), int(k)) for u, p, c, k in E])[0] == len(E) * w
