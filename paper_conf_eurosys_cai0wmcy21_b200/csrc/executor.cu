@@ -275,10 +275,11 @@ __device__ __forceinline__ void fanout_rows(const ExecParams &P, const DevItem &
 // item (a store drain every 64 KB) held the path at ~0.25 of HBM peak.
 constexpr int kPendMax = 16;
 
-// kCopyOnly: the instance for launches whose data items are all COPY (op_mask == kMaskCopy): no
-// fold / fan-out code, so the copy loop keeps its loaded vectors in registers under the 64-register
-// cap (the general instance spills there)
-template <bool V16, bool kCopyOnly>
+// kCopy: the instance per launch kind — 0 general; for launches whose data items are all COPY
+// (op_mask == kMaskCopy) 1 = whole 16-B chunks (or 4-B rows): no fold / fan-out / ragged-tail
+// code, spill-free under the 64-register cap; 2 = ragged 16-B rows (e.g. dim 602: 2408 B) without
+// the fold / fan-out code (the general instance spills far more there)
+template <bool V16, int kCopy>
 __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __grid_constant__ ExecParams P) {
   __shared__ int s_abort, s_flush, s_npend;
   __shared__ uint64_t *s_pend_ctr[kPendMax];
@@ -357,14 +358,16 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
     } else if (I.op == OP_COPY) {
       const bool nc = readonly_kind(I.src_kind);
       if (V16) {
-        const bool full = (P.row_bytes & 15) == 0;
+        // the copy-only instance runs whole-chunk rows only (the ragged loop, inlined, made the
+        // whole kernel spill at 64 registers)
+        const bool full = kCopy == 1 || (kCopy == 0 && (P.row_bytes & 15) == 0);
         if (nc) full ? copy_rows_full<true>(P, I) : copy_rows_v16<true>(P, I);
         else full ? copy_rows_full<false>(P, I) : copy_rows_v16<false>(P, I);
       } else {
         if (nc) copy_rows_b32<true>(P, I);
         else copy_rows_b32<false>(P, I);
       }
-    } else if (kCopyOnly) {
+    } else if (kCopy != 0) {
     } else if (I.op == OP_FOLD) {
       fold_rows<V16>(P, I);
     } else if (I.op == OP_FANOUT) {
@@ -404,14 +407,17 @@ int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   if (p.use_tma) return launch_tma_executor(p, grid, block, stream);
   cudaStream_t s = (cudaStream_t)stream;
   const bool copy_only = p.op_mask == kMaskCopy;
-  if (p.vec16 && copy_only)
-    executor_kernel<true, true><<<grid, block, 0, s>>>(p);
+  const bool whole = !p.vec16 || (p.row_bytes & 15) == 0;
+  if (p.vec16 && copy_only && whole)
+    executor_kernel<true, 1><<<grid, block, 0, s>>>(p);
+  else if (p.vec16 && copy_only)
+    executor_kernel<true, 2><<<grid, block, 0, s>>>(p);
   else if (p.vec16)
-    executor_kernel<true, false><<<grid, block, 0, s>>>(p);
+    executor_kernel<true, 0><<<grid, block, 0, s>>>(p);
   else if (copy_only)
-    executor_kernel<false, true><<<grid, block, 0, s>>>(p);
+    executor_kernel<false, 1><<<grid, block, 0, s>>>(p);
   else
-    executor_kernel<false, false><<<grid, block, 0, s>>>(p);
+    executor_kernel<false, 0><<<grid, block, 0, s>>>(p);
   return (int)cudaGetLastError();
 }
 
@@ -421,9 +427,9 @@ int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm) {
 
 int executor_occupancy(int block, int *ctas_per_sm) {
   int a = 0, b = 0;
-  cudaError_t ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, executor_kernel<true, false>, block, 0);
+  cudaError_t ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, executor_kernel<true, 0>, block, 0);
   if (ce != cudaSuccess) return (int)ce;
-  ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, executor_kernel<false, false>, block, 0);
+  ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, executor_kernel<false, 0>, block, 0);
   if (ce != cudaSuccess) return (int)ce;
   *ctas_per_sm = a < b ? a : b;
   return 0;
