@@ -278,7 +278,8 @@ constexpr int kPendMax = 16;
 // kCopy: the instance per launch kind — 0 general; for launches whose data items are all COPY
 // (op_mask == kMaskCopy) 1 = whole 16-B chunks (or 4-B rows): no fold / fan-out / ragged-tail
 // code, spill-free under the 64-register cap; 2 = ragged 16-B rows (e.g. dim 602: 2408 B) without
-// the fold / fan-out code (the general instance spills far more there)
+// the fold / fan-out code (the general instance spills far more there); 3 = fold-only launches
+// (owner reduces, tree-order folds: no copy / fan-out code)
 template <bool V16, int kCopy>
 __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __grid_constant__ ExecParams P) {
   __shared__ int s_abort, s_flush, s_npend;
@@ -353,7 +354,9 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
     }
     __syncthreads();
     if (s_abort) return;  // the watchdog fired; the error word is set, leave the launch
-    if (I.op == OP_COPY && (I.flags & kItemAtomic)) {
+    if (kCopy == 3) {  // fold-only instance
+      if (I.op == OP_FOLD) fold_rows<V16>(P, I);
+    } else if (I.op == OP_COPY && (I.flags & kItemAtomic)) {
       copy_rows_atomic(P, I);
     } else if (I.op == OP_COPY) {
       const bool nc = readonly_kind(I.src_kind);
@@ -408,10 +411,13 @@ int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   cudaStream_t s = (cudaStream_t)stream;
   const bool copy_only = p.op_mask == kMaskCopy;
   const bool whole = !p.vec16 || (p.row_bytes & 15) == 0;
+  const bool fold_only = !(p.op_mask & (kMaskCopy | kMaskFanout));
   if (p.vec16 && copy_only && whole)
     executor_kernel<true, 1><<<grid, block, 0, s>>>(p);
   else if (p.vec16 && copy_only)
     executor_kernel<true, 2><<<grid, block, 0, s>>>(p);
+  else if (p.vec16 && fold_only)
+    executor_kernel<true, 3><<<grid, block, 0, s>>>(p);
   else if (p.vec16)
     executor_kernel<true, 0><<<grid, block, 0, s>>>(p);
   else if (copy_only)
