@@ -355,53 +355,52 @@ void build_programs(dgcl_ctx *c) {
       }
     }
     for (int l = 0; l < c->n_layers; ++l) {
-      for (int r = 0; r < c->n_prog_ranks; ++r) {
-        Program &P = c->progs[c->prog_index(l, dir, r)];
-        const int64_t row_bytes = (int64_t)c->dims[l] * 4, row16 = (row_bytes + 15) / 16 * 16;
-        // fan-out items stage a row plus its destination words: rows up to half a DUAL stage
-        const bool fan = fan_avail && dir == DIR_FWD && 2 * (row16 + 128) <= kGeoDual.stage_bytes -
-                                                                               kStageHdrBytes;
+      const int64_t row_bytes = (int64_t)c->dims[l] * 4, row16 = (row_bytes + 15) / 16 * 16;
+      // fan-out items stage a row plus its destination words: rows up to half a DUAL stage
+      const bool fan = fan_avail && dir == DIR_FWD &&
+                       2 * (row16 + 128) <= kGeoDual.stage_bytes - kStageHdrBytes;
+      auto build = [&](Program &P, int r, int geo) {
         const std::vector<int32_t> &G = fan ? gids_fan[r] : gids[r];
         const std::vector<uint8_t> need = needed_counters(L, G);
-        auto build = [&](int geo) {
-          P.geo = geo;
-          ItemLimits lim = item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
-                                       (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm);
-          lim.align_sources = c->align_sources;
-          build_items(L, G, row_bytes, lim, !fused, need,
-                      &P.items, &P.runs, c->direct_copy_rows,
-                      c->stage_fold ? &P.sterms : nullptr);
-          P.op_mask = 0;
-          int64_t fold_rows = 0, fold_terms = 0;
-          for (const DevItem &it : P.items) {
-            if (it.op == OP_FOLD && (it.flags & kItemStaged)) {
-              P.op_mask |= kMaskStaged;
-            } else if (it.op == OP_FOLD && it.term_mode == kTermRankTree) {
-              P.op_mask |= kMaskTree;
-            } else if (it.op == OP_FOLD) {
-              P.op_mask |= kMaskFold;
-              fold_rows += it.rows;
-              fold_terms += it.nterms;
-            }
-            if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
-            if (it.op == OP_FANOUT) P.op_mask |= kMaskFanout;
+        P.geo = geo;
+        ItemLimits lim = item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
+                                     (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm);
+        lim.align_sources = c->align_sources;
+        build_items(L, G, row_bytes, lim, !fused, need, &P.items, &P.runs, c->direct_copy_rows,
+                    c->stage_fold ? &P.sterms : nullptr);
+        P.op_mask = 0;
+        int64_t fold_rows = 0, fold_terms = 0;
+        for (const DevItem &it : P.items) {
+          if (it.op == OP_FOLD && (it.flags & kItemStaged)) {
+            P.op_mask |= kMaskStaged;
+          } else if (it.op == OP_FOLD && it.term_mode == kTermRankTree) {
+            P.op_mask |= kMaskTree;
+          } else if (it.op == OP_FOLD) {
+            P.op_mask |= kMaskFold;
+            fold_rows += it.rows;
+            fold_terms += it.nterms;
           }
-          P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
-          P.g4_kinds = 0;
-          P.tree = false;
-          for (const DevItem &it : P.items)
-            if (it.op == OP_FOLD && it.term_mode == kTermRankTree) P.tree = true;
-          for (const DevItem &it : P.items)
-            if (it.op == OP_COPY && (it.flags & kItemGather4)) P.g4_kinds |= 1 << it.src_kind;
-          P.bytes = 0;
-          for (const DevItem &it : P.items)
-            if (it.op == OP_COPY || it.op == OP_FOLD)
-              P.bytes += (int64_t)(it.rows + (it.op == OP_FOLD ? it.nterms : 0)) * row16;
-            else if (it.op == OP_FANOUT)
-              P.bytes += (int64_t)(it.rows + it.nterms) * row16;
-        };
+          if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
+          if (it.op == OP_FANOUT) P.op_mask |= kMaskFanout;
+        }
+        P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
+        P.g4_kinds = 0;
+        P.tree = false;
+        for (const DevItem &it : P.items)
+          if (it.op == OP_FOLD && it.term_mode == kTermRankTree) P.tree = true;
+        for (const DevItem &it : P.items)
+          if (it.op == OP_COPY && (it.flags & kItemGather4)) P.g4_kinds |= 1 << it.src_kind;
+        P.bytes = 0;
+        for (const DevItem &it : P.items)
+          if (it.op == OP_COPY || it.op == OP_FOLD)
+            P.bytes += (int64_t)(it.rows + (it.op == OP_FOLD ? it.nterms : 0)) * row16;
+          else if (it.op == OP_FANOUT)
+            P.bytes += (int64_t)(it.rows + it.nterms) * row16;
+      };
+      for (int r = 0; r < c->n_prog_ranks; ++r) {
+        Program &P = c->progs[c->prog_index(l, dir, r)];
         if (c->geometry) {
-          build(c->geometry - 1);
+          build(P, r, c->geometry - 1);
           continue;
         }
         // auto: DUAL (two producer warps per SM) unless the launch is bulk-copy friendly —
@@ -409,7 +408,7 @@ void build_programs(dgcl_ctx *c) {
         // (consumer gathers, which want more consumer warps), or chains stages on flags (relay
         // plans: DUAL's forward time was bimodal, 0.83 / 2.1 ms, on the Web-Google dgx1_like
         // plan, WIDE a steady 0.9-1.1 ms); see TmaGeometry
-        build(1);
+        build(P, r, 1);
         int64_t ops = 0, bytes = 0;
         bool waits = false;
         for (const DevItem &it : P.items) {
@@ -425,7 +424,22 @@ void build_programs(dgcl_ctx *c) {
         const bool copy_only = (P.op_mask & ~(kMaskCopy | kMaskFanout)) == 0;
         if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & (kMaskFold | kMaskTree)) ||
             waits)
-          build(0);
+          build(P, r, 0);
+      }
+      // per-rank loopback: the ranks' launches run concurrently on one device and their CTAs wait
+      // on each other's flags, so together they must be co-resident.  A WIDE CTA (one per SM by
+      // shared memory) cannot share an SM with a DUAL one: every rank of a (layer, direction)
+      // takes the geometry of the largest program (launch() likewise picks one executor for all)
+      if (c->loopback && !fused && c->n_prog_ranks > 1) {
+        int big = 0;
+        for (int r = 1; r < c->n_prog_ranks; ++r)
+          if (c->progs[c->prog_index(l, dir, r)].bytes > c->progs[c->prog_index(l, dir, big)].bytes)
+            big = r;
+        const int geo = c->progs[c->prog_index(l, dir, big)].geo;
+        for (int r = 0; r < c->n_prog_ranks; ++r) {
+          Program &P = c->progs[c->prog_index(l, dir, r)];
+          if (P.geo != geo) build(P, r, geo);
+        }
       }
     }
   }
@@ -503,8 +517,22 @@ bool encode_rows_tmap(dgcl_ctx *c, unsigned char *out, const void *base, int64_t
   return true;
 }
 
+// the context's device is current for the launches (and the caller's restored afterwards)
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
 dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_pitch,
                    float *out, int64_t out_pitch, cudaStream_t stream) {
+  DeviceGuard guard(c->device);
   const int m = c->world;
   ExecParams P;
   std::memset(&P, 0, sizeof(P));
@@ -584,7 +612,8 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     }
   };
   // one program's launch: its items, kernel instance, CTA shape and bulk-copy geometry
-  auto launch_program = [&](const Program &pg, int grid_div, cudaStream_t st) -> int {
+  auto launch_program = [&](const Program &pg, int grid_div, cudaStream_t st,
+                            int64_t sel_bytes) -> int {
     ExecParams Pp = P;
     Pp.items = c->d_items + pg.dev_off;
     Pp.op_mask = pg.op_mask;
@@ -598,7 +627,8 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     int block = c->threads, grid_all = c->grid;
     // latency-bound launches (a few MB) skip the bulk-copy pipeline: the register executor's
     // single round trip per item is shorter (tiny config: 10 vs 14-19 us per launch)
-    const bool small = pg.bytes < c->small_launch_bytes;
+    // (sel_bytes: per-rank loopback decides for all ranks of a launch together, co-residency)
+    const bool small = sel_bytes < c->small_launch_bytes;
     if (Pp.use_tma && !small && Pp.row16 <= G.stage_bytes - kStageHdrBytes && tctas > 0) {
       block = tblock;
       grid_all = c->n_sm * tctas;
@@ -618,7 +648,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     const int r = fused ? 0 : c->rank;
     const Program &pg = c->progs[c->prog_index(layer, dir, fused ? 0 : (c->loopback ? r : r))];
     if (pg.items.empty()) return DGCL_OK;
-    int e = launch_program(pg, 1, stream);
+    int e = launch_program(pg, 1, stream, pg.bytes);
     if (e != 0) return fail(c, DGCL_ECUDA, "executor launch failed: %s",
                             cudaGetErrorString((cudaError_t)e));
     c->launches++;
@@ -626,11 +656,13 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   }
   // loopback, one launch per virtual rank on its own stream (full flag protocol)
   CUDA_TRY(c, cudaEventRecord(c->fork_event, stream));
+  int64_t sel_bytes = 0;  // one executor for every rank's launch: the largest program decides
+  for (int r = 0; r < m; ++r) sel_bytes = std::max(sel_bytes, c->progs[c->prog_index(layer, dir, r)].bytes);
   for (int r = 0; r < m; ++r) {
     const Program &pg = c->progs[c->prog_index(layer, dir, r)];
     CUDA_TRY(c, cudaStreamWaitEvent(c->rank_streams[r], c->fork_event, 0));
     if (!pg.items.empty() && r != c->debug_skip_rank) {
-      int e = launch_program(pg, m, c->rank_streams[r]);
+      int e = launch_program(pg, m, c->rank_streams[r], sel_bytes);
       if (e != 0) return fail(c, DGCL_ECUDA, "executor launch failed: %s",
                               cudaGetErrorString((cudaError_t)e));
       c->launches++;

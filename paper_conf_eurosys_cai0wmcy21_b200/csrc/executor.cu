@@ -409,9 +409,14 @@ int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   if (grid <= 0) return 0;
   if (p.use_tma) return launch_tma_executor(p, grid, block, stream);
   cudaStream_t s = (cudaStream_t)stream;
-  const bool copy_only = p.op_mask == kMaskCopy;
+  // copy-only: every data item is a COPY (bulk-path or consumer-gather kind: the register path
+  // runs both the same way); fold-only: no COPY of any kind and no FANOUT (the kCopy == 3
+  // instance runs OP_FOLD items only, so a direct COPY must never reach it)
+  const int copies = kMaskCopy | kMaskDirect;
+  const int folds = kMaskFold | kMaskStaged | kMaskTree;
+  const bool copy_only = p.op_mask != 0 && (p.op_mask & ~copies) == 0;
   const bool whole = !p.vec16 || (p.row_bytes & 15) == 0;
-  const bool fold_only = !(p.op_mask & (kMaskCopy | kMaskFanout));
+  const bool fold_only = p.op_mask != 0 && (p.op_mask & ~folds) == 0;
   if (p.vec16 && copy_only && whole)
     executor_kernel<true, 1><<<grid, block, 0, s>>>(p);
   else if (p.vec16 && copy_only)

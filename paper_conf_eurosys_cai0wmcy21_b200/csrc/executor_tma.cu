@@ -978,12 +978,13 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         }
         __threadfence_system();
         consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
-        if (tid < (uint32_t)(kMaxRanks * kMaxRanks)) {
-          const uint32_t amt = s_pend[tid];
+        // (strided: there are fewer consumer threads than (source, receiver) entries)
+        for (uint32_t i = tid; i < (uint32_t)(kMaxRanks * kMaxRanks); i += T) {
+          const uint32_t amt = s_pend[i];
           if (amt) {
-            const int ex = (int)(tid / kMaxRanks), dst = (int)(tid % kMaxRanks);
+            const int ex = (int)(i / kMaxRanks), dst = (int)(i % kMaxRanks);
             red_release_sys_add(P.flags[dst] + s_pend_base + ex, amt);
-            s_pend[tid] = 0;
+            s_pend[i] = 0;
           }
         }
         consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
@@ -1056,13 +1057,17 @@ namespace {
 
 template <int kMask, int kThreads = 512>
 int launch_mask(const ExecParams &p, int grid, int block, cudaStream_t s) {
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kMask, kThreads>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)kSmemMax);
+  // kernel attributes are per device (context): set once per device this process launches on
+  static unsigned long long attr_set = 0;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return (int)e;
+  const unsigned long long bit = 1ull << (dev & 63);
+  if (!(attr_set & bit)) {
+    e = cudaFuncSetAttribute(executor_tma_kernel<kMask, kThreads>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemMax);
     if (e != cudaSuccess) return (int)e;
-    attr = true;
+    attr_set |= bit;
   }
   const TmaGeometry g = {p.tma_stages, p.tma_buf, p.meta_bytes, block, 0, 0};
   executor_tma_kernel<kMask, kThreads><<<grid, block, tma_smem_bytes(g), s>>>(p);

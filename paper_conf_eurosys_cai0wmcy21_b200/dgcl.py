@@ -157,8 +157,32 @@ class Context:
         check(lib().dgcl_ipc_import(self.handle, data, _abi.IPC_BLOB_BYTES), self.handle)
 
     # ---- hot path ---------------------------------------------------------------------------
+    def _rows(self):
+        return int(len(self.part)) if self.loopback else int(self.n_local[self.rank])
+
+    def _check_arg(self, name, t, layer, rows):
+        """The C side sees a pointer and a pitch only: refuse what it cannot check (dtype, device,
+        column stride, row count, pitch >= dim) before any out-of-bounds access could happen."""
+        import torch
+        if not isinstance(t, torch.Tensor):
+            raise TypeError("%s must be a torch tensor" % name)
+        if t.dtype != torch.float32:
+            raise TypeError("%s must be float32 (got %s)" % (name, t.dtype))
+        if not t.is_cuda or t.device.index != self.device:
+            raise ValueError("%s must live on cuda:%d (got %s)" % (name, self.device, t.device))
+        if t.dim() != 2 or (t.shape[0] > 0 and t.stride(1) != 1):
+            raise ValueError("%s must be a 2-D row-major [rows x pitch] tensor" % name)
+        if t.shape[0] < rows:
+            raise ValueError("%s has %d rows < %d" % (name, t.shape[0], rows))
+        if t.shape[1] < self.dims[layer] or (rows > 1 and t.stride(0) < self.dims[layer]):
+            raise ValueError("%s: pitch < dim %d" % (name, self.dims[layer]))
+
+    def _halo_rows(self):
+        return int(self.halo_off[-1]) if self.loopback else int(self.n_halo[self.rank])
+
     def forward(self, layer, emb, halo=None, stream=None):
         """graphAllgather forward: emb (device float32 [rows x pitch]) -> the halo view."""
+        self._check_arg("emb", emb, layer, self._rows())
         h = halo if halo is not None else None
         check(lib().dgcl_dispatch_forward(
             self.handle, layer, ctypes.c_void_p(emb.data_ptr()), emb.stride(0),
@@ -168,6 +192,8 @@ class Context:
 
     def backward(self, layer, halo_grad, emb_grad, stream=None):
         """emb_grad (in/out) += fixed-order fold of halo_grad along the reversed plan."""
+        self._check_arg("halo_grad", halo_grad, layer, self._halo_rows())
+        self._check_arg("emb_grad", emb_grad, layer, self._rows())
         check(lib().dgcl_dispatch_backward(
             self.handle, layer, ctypes.c_void_p(halo_grad.data_ptr()), halo_grad.stride(0),
             ctypes.c_void_p(emb_grad.data_ptr()), emb_grad.stride(0), _stream_ptr(stream)),

@@ -126,6 +126,23 @@ def test_backward_closed_form_fanout_from_edges():
         assert out[part[u]][loc[u], 0] == fan[u] and out[part[u]][loc[u], 1] == fan[u]
 
 
+def test_fanout_is_edge_counted_requesters():
+    """halo.fanout (|D_u|, which drives the GPU closed-form test) against |D_u| counted from the
+    EDGE LIST by explicit loops (distinct foreign GPUs among u's out-neighbours, R3), and against
+    the H2 literal (its all-ones backward owner rows are exactly the fan-outs)."""
+    for m, seed in ((2, 61), (4, 62), (5, 63)):
+        n, m, part, edges, R = _tiny(m=m, seed=seed)
+        f = halo.fanout(R, n)
+        for u in range(n):
+            want = len({int(part[v]) for (a, v) in edges if a == u and part[v] != part[u]})
+            assert f[u] == want, (m, u)
+    g, part = _h2()
+    loc, _ = halo.local_rows(part, 3)
+    f = halo.fanout(g["R"], g["n"])
+    for v in range(g["n"]):
+        assert f[v] == g["all_ones_backward_owner_rows"][part[v]][loc[v]]
+
+
 def test_backward_integer_inputs_any_order():
     n, m, part, edges, R = _tiny(m=4, seed=33)
     loc, n_local = halo.local_rows(part, m)

@@ -194,3 +194,77 @@ def test_shuffle_is_a_permutation_and_seeded():
     assert sorted(a) == list(range(50))
     assert a == spst.shuffle_order(range(50), 9)
     assert a != spst.shuffle_order(range(50), 10)
+
+
+# ---- negative pins of oracle.invariants.check_plan: each invariant broken once ----------------
+# A checker that let a broken plan pass would let every planner test pass silently; each case
+# below breaks exactly one of (i)-(v) of SURVEY §8(c) step 7 on a known-good plan and must fail.
+
+def _chain3():
+    """3 GPUs on a chain 0 -> 1 -> 2 (links 0->1, 1->0, 1->2, 2->1 only: 0->2 does not exist)."""
+    t = synth.Topology("chain3", 3, [100.0] * 4, ["h01", "h10", "h12", "h21"])
+    t.links = {(0, 1): [0], (1, 0): [1], (1, 2): [2], (2, 1): [3]}
+    return t
+
+
+def _good_chain_plan():
+    """u=0 owned by GPU 0, requested by 1 and 2: T = 0->1 (stage 1), 1->2 (stage 2);
+    u=1 owned by GPU 2, requested by 0 through the relay 1 (1 did not ask): 2->1, 1->0."""
+    owner = {0: 0, 1: 2}
+    D = {0: [1, 2], 1: [0]}
+    edges = [(0, 0, 1, 1), (0, 1, 2, 2), (1, 2, 1, 1), (1, 1, 0, 2)]
+    total, _ = cost.plan_cost(_chain3(), edges)
+    return owner, D, edges, total
+
+
+def test_check_plan_accepts_the_good_plan():
+    owner, D, edges, total = _good_chain_plan()
+    # by hand: every hop is 100 GB/s = 1000 ticks per row; stage 1 carries 0->1 and 2->1 (one row
+    # on each of two hops), stage 2 carries 1->2 and 1->0 (likewise): t(S) = 1000 + 1000
+    assert total == 2000
+    assert invariants.check_plan(_chain3(), edges, owner, D, total) == 1   # one relay (u=1 on 1)
+
+
+@pytest.mark.parametrize("case", [
+    "stage_not_depth",       # (i)  stage label != tree depth
+    "stage_too_deep",        # (i)  a stage-3 edge in a 3-GPU plan (> m - 1, and != its depth)
+    "edge_into_root",        # (i)  the owner receives its own vertex
+    "cycle",                 # (i)  nodes that never reach the root
+    "duplicate_delivery",    # (ii) a GPU reached twice
+    "missing_delivery",      # (ii) a requester never reached
+    "useless_leaf",          # (iii) a leaf outside D_u (delivery to a GPU that did not ask)
+    "missing_link",          # (iv) an edge on a link the topology does not have
+    "wrong_cost",            # (v)  reported t(S) != recomputed
+    "unplanned_vertex",      # planned set != {u : D_u non-empty}
+    "planned_extra_vertex",  # a vertex nobody requested gets a tree
+])
+def test_check_plan_rejects(case):
+    t = _chain3()
+    owner, D, edges, total = _good_chain_plan()
+    reported = None          # structural cases: the cost check is not what must fire
+    if case == "stage_not_depth":
+        edges[1] = (0, 1, 2, 1)
+    elif case == "stage_too_deep":
+        edges[1] = (0, 1, 2, 3)
+    elif case == "edge_into_root":
+        edges.append((0, 1, 0, 2))
+    elif case == "cycle":
+        edges[0:2] = [(0, 2, 1, 1), (0, 1, 2, 2)]     # u=0: 1 and 2 point at each other
+    elif case == "duplicate_delivery":
+        edges.append((0, 2, 1, 3))                     # 1 reached again, from 2
+    elif case == "missing_delivery":
+        del edges[1]                                   # 2 asked for u=0, never gets it
+    elif case == "useless_leaf":
+        D[0] = [1]                                     # 2 no longer asks for u=0: 1->2 is useless
+    elif case == "missing_link":
+        edges[0:2] = [(0, 0, 1, 1), (0, 0, 2, 1)]     # 0->2 does not exist
+    elif case == "wrong_cost":
+        reported = total + 1
+    elif case == "unplanned_vertex":
+        D[5] = [1]
+        owner[5] = 0
+    elif case == "planned_extra_vertex":
+        edges.append((7, 0, 1, 1))
+        owner[7] = 0
+    with pytest.raises(AssertionError):
+        invariants.check_plan(t, edges, owner, D, reported)
