@@ -130,6 +130,21 @@ class Workload:
         self.fwd_layers = list(range(len(c.dims)))
         self.bwd_layers = list(c.backward_layers)
 
+    @classmethod
+    def from_parts(cls, cfg, world, part, req_ptr, req_ids):
+        """The same workload re-partitioned `world`-way (the N > 1 leg's partition)."""
+        import dataclasses
+        import synth
+        w = cls.__new__(cls)
+        w.cfg = dataclasses.replace(cfg, m=world)
+        w.g = synth.Graph(cfg.n, world, None, None, part, req_ptr, req_ids)
+        w.gen_s = 0.0
+        w.S = int(req_ptr[-1])
+        w.order = np.argsort(part, kind="stable")
+        w.fwd_layers = list(range(len(cfg.dims)))
+        w.bwd_layers = list(cfg.backward_layers)
+        return w
+
     def step_payload_bytes(self, ranks=None):
         """Halo payload one step delivers (forward) and returns (backward), algorithmic bytes."""
         ptr = self.g.req_ptr
@@ -158,8 +173,13 @@ def host_inputs(w, pitches, rows_order=None):
 # ---------------------------------------------------------------------------------------------
 def oracle_sample(w, emb, hg, eg, budget_s=15.0, ranks=None, threads=1):
     """Time the CPU oracle (as it stands) on destination/owner ranks until the budget is spent.
-    threads > 1: the ranks' oracle calls run concurrently in a thread pool (numpy's gathers and
-    adds release the GIL), all of ranks at once, wall-clock timed.
+
+    A unit of work is (rank d, chunk j of J): the forward of halo rows R_d[chunk j] (every
+    layer) and the flat backward of the owner-d vertices in vertex-id chunk j (the backward
+    layers) — oracle.halo calls on sub-lists, nothing re-implemented.  threads == 1: J = 1, ranks
+    in order until the budget is spent.  threads > 1: J chunks per rank so that there are >= 2
+    units per thread, every unit of the given ranks run in a thread pool over `threads` host
+    cores (numpy's gathers and adds release the GIL), wall-clock timed.
     Returns (GB/s, seconds, ranks used, threads)."""
     from oracle import halo
     c = w.cfg
@@ -168,41 +188,49 @@ def oracle_sample(w, emb, hg, eg, budget_s=15.0, ranks=None, threads=1):
     loc, n_local = halo.local_rows(g.part, m)
     ro = np.concatenate([[0], np.cumsum(n_local)])
     R = [g.R(d) for d in range(m)]
-    if threads > 1:
-        from concurrent.futures import ThreadPoolExecutor
-        rk = list(ranks if ranks is not None else range(m))
-        one = lambda d: oracle_sample(w, emb, hg, eg, budget_s=0.0, ranks=[d])
-        with ThreadPoolExecutor(max_workers=min(threads, len(rk))) as ex:
-            t = time.perf_counter()
-            res = list(ex.map(one, rk))
-            secs = time.perf_counter() - t
-        nbytes = sum(r[0] * r[1] * 1e9 for r in res)
-        return nbytes / secs / 1e9, secs, rk, min(threads, len(rk))
-    done_bytes, t_total, used = 0, 0.0, []
-    for d in (ranks if ranks is not None else range(m)):
-        t = time.perf_counter()
+    ptr = g.req_ptr
+    empty = np.zeros(0, np.int64)
+
+    def unit(d, j, J):
+        nb = 0
+        a, b = int(ptr[d]), int(ptr[d + 1])
+        lo, hi = a + (b - a) * j // J, a + (b - a) * (j + 1) // J
         for l in w.fwd_layers:
             dim = c.dims[l]
             local = [emb[l][ro[s]:ro[s + 1], :dim] for s in range(m)]
-            Rd = [R[q] if q == d else np.zeros(0, np.int64) for q in range(m)]
+            Rd = [g.req_ids[lo:hi] if q == d else empty for q in range(m)]
             halo.forward(local, Rd, g.part, loc)
+            nb += (hi - lo) * 4 * dim
+        vlo, vhi = g.n * j // J, g.n * (j + 1) // J
         for l in w.bwd_layers:
             dim = c.dims[l]
-            L = [eg[l][ro[s]:ro[s + 1], :dim] if s == d else np.zeros((n_local[s], dim), np.float32)
+            L = [eg[l][ro[s]:ro[s + 1], :dim] if s == d else np.zeros((0, dim), np.float32)
                  for s in range(m)]
-            ptr = g.req_ptr
             G = [hg[l][ptr[q]:ptr[q + 1], :dim] for q in range(m)]
-            # owner d's rows: every contributor's rows for vertices owned by d
-            Rd = [R[q][g.part[R[q]] == d] for q in range(m)]
-            Gd = [G[q][g.part[R[q]] == d] for q in range(m)]
+            # owner d's rows in the chunk: every contributor's rows for those vertices
+            sel = [(g.part[R[q]] == d) & (R[q] >= vlo) & (R[q] < vhi) for q in range(m)]
+            Rd = [R[q][sel[q]] for q in range(m)]
+            Gd = [G[q][sel[q]] for q in range(m)]
             halo.backward_flat(L, Gd, Rd, g.part, loc)
+            nb += sum(len(r) for r in Rd) * 4 * dim
+        return nb
+
+    rk = list(ranks if ranks is not None else range(m))
+    if threads > 1:
+        from concurrent.futures import ThreadPoolExecutor
+        J = max(1, -(-2 * threads // len(rk)))
+        units = [(d, j, J) for d in rk for j in range(J)]
+        with ThreadPoolExecutor(max_workers=threads) as ex:
+            t = time.perf_counter()
+            nbytes = sum(ex.map(lambda u: unit(*u), units))
+            secs = time.perf_counter() - t
+        return nbytes / secs / 1e9, secs, rk, threads
+    done_bytes, t_total, used = 0, 0.0, []
+    for d in rk:
+        t = time.perf_counter()
+        done_bytes += unit(d, 0, 1)
         t_total += time.perf_counter() - t
         used.append(d)
-        ptr = g.req_ptr
-        fwd_b = int(ptr[d + 1] - ptr[d]) * 4 * sum(c.dims[l] for l in w.fwd_layers)
-        owned_in = sum(int(np.count_nonzero(g.part[R[q]] == d)) for q in range(m))
-        bwd_b = owned_in * 4 * sum(c.dims[l] for l in w.bwd_layers)
-        done_bytes += fwd_b + bwd_b
         if t_total >= budget_s:
             break
     return done_bytes / t_total / 1e9, t_total, used, 1
@@ -423,8 +451,8 @@ def run_ours_single(args, w):
                                                          threads=ncores)
             cpu["threaded"] = {"value": gbs_t, "unit": UNIT, "cores": thr_t,
                                "host_cores": ncores,
-                               "sample": "all %d ranks' oracle calls concurrently (%.1f s wall)" %
-                                         (c.m, secs_t)}
+                               "sample": "all %d ranks' oracle work as (rank, row-chunk) units on "
+                                         "%d threads (%.1f s wall)" % (c.m, thr_t, secs_t)}
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": K,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
@@ -484,6 +512,27 @@ def run_reference(args, w):
                     "d2h_bytes_per_step": 0}}
 
 
+def spawn_ranks(args):
+    """`bench.py --gpus N` outside torchrun: start N ranks (one process per GPU) through
+    torch.distributed.run on 127.0.0.1 with the same arguments; rank 0's JSON line is the
+    output.  Refuses to run with fewer visible GPUs than N (unless --share-gpu, test mode)."""
+    import socket
+    import torch
+    n_dev = torch.cuda.device_count()
+    if n_dev < args.gpus and not args.share_gpu:
+        log("bench.py: --gpus %d but only %d CUDA device(s) visible" % (args.gpus, n_dev))
+        return 2
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           "--nproc-per-node", str(args.gpus), "--master-addr", "127.0.0.1",
+           "--master-port", str(port), os.path.join(ROOT, "bench.py")] + sys.argv[1:]
+    subprocess.check_call(["make", "-s", "-C", ROOT, "all"])
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -499,6 +548,11 @@ def main():
     ap.add_argument("--item-bytes", type=int, default=0)
     ap.add_argument("--opt", action="append", default=[], metavar="KEY=VALUE",
                     help="executor option (dgcl_set_option) before planning, e.g. stage_fold=0")
+    ap.add_argument("--calls", type=int, default=50,
+                    help="N > 1: timed calls per launch in the per-call protocol (device start "
+                         "barrier, max over ranks, median / p10 / p90 / mean of the first 10)")
+    ap.add_argument("--no-p2p-baseline", action="store_true",
+                    help="N > 1: skip the NCCL pack + send/recv + unpack baseline")
     ap.add_argument("--share-gpu", action="store_true", help=argparse.SUPPRESS)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
@@ -506,6 +560,10 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "ours":
+        sys.exit(spawn_ranks(args))
+    if args.impl == "ours" and world != args.gpus and "WORLD_SIZE" in os.environ:
+        raise SystemExit("bench.py: --gpus %d but WORLD_SIZE=%d" % (args.gpus, world))
     subprocess.check_call(["make", "-s", "-C", ROOT, "all"]) if rank == 0 and world == 1 else None
 
     if args.impl == "reference":
@@ -522,7 +580,9 @@ def main():
         return
 
     from bench_multi import run_multi
-    out = run_multi(args, METRIC, UNIT, rank, world, local_rank, ClockSampler)
+    out = run_multi(args, METRIC, UNIT, rank, world, local_rank, ClockSampler,
+                    make_workload=Workload.from_parts, oracle_sample=oracle_sample,
+                    host_inputs=host_inputs)
     if rank == 0:
         print(json.dumps(out), flush=True)
     import torch.distributed as dist

@@ -269,6 +269,16 @@ typedef struct dgcl_trace_rec {
 dgcl_status dgcl_trace_read(dgcl_ctx *ctx, int32_t layer, int32_t dir, int32_t rank,
                             dgcl_trace_rec *recs, int64_t *n);
 
+/* Device start barrier over the ranks (timing protocol of SURVEY.md §8(d) / a13; PAPER.md times
+ * communication "after warm-up", averaged over 10 runs): a one-warp kernel on
+ * `stream` in which this rank releases arrived[rank] = n into every peer's flag region (n = this
+ * context's barrier call count) and acquire-waits until every peer's arrived word reaches n.  Work
+ * queued after it on `stream` starts only once all ranks have reached the same barrier call.  A
+ * collective: every rank calls it the same number of times.  Loopback contexts run all virtual
+ * ranks in the one warp.  world == 1: no-op.  Errors: DGCL_ESTATE before registration / import;
+ * a peer that never arrives trips the watchdog (dgcl_check -> DGCL_ETIMEOUT). */
+dgcl_status dgcl_device_barrier(dgcl_ctx *ctx, void *stream);
+
 /* Number of executor kernel launches issued so far by this context. */
 dgcl_status dgcl_launch_count(dgcl_ctx *ctx, uint64_t *count);
 

@@ -22,7 +22,8 @@ SYMBOLS = [
     "dgcl_workspace_bytes", "dgcl_register_workspace", "dgcl_halo_view", "dgcl_rank_rows",
     "dgcl_ipc_export", "dgcl_ipc_import", "dgcl_dispatch_forward", "dgcl_dispatch_backward",
     "dgcl_forward_host", "dgcl_backward_host", "dgcl_plan_info", "dgcl_plan_counts",
-    "dgcl_plan_export", "dgcl_set_option", "dgcl_trace_read", "dgcl_launch_count", "dgcl_check",
+    "dgcl_plan_export", "dgcl_set_option", "dgcl_trace_read", "dgcl_device_barrier",
+    "dgcl_launch_count", "dgcl_check",
     "dgcl_last_error",
     "dgcl_strerror", "dgcl_destroy", "dgcl_debug_hostsim_forward", "dgcl_debug_hostsim_backward",
 ]
@@ -85,6 +86,7 @@ def lib():
             "dgcl_plan_export": [P, ctypes.POINTER(I64), P, P, P, P],
             "dgcl_set_option": [P, ctypes.c_char_p, I64],
             "dgcl_trace_read": [P, I32, I32, I32, P, ctypes.POINTER(I64)],
+            "dgcl_device_barrier": [P, P],
             "dgcl_launch_count": [P, ctypes.POINTER(U64)],
             "dgcl_check": [P],
             "dgcl_destroy": [P],

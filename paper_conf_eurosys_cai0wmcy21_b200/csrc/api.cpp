@@ -108,6 +108,7 @@ struct dgcl_ctx {
   int n_prog_ranks = 1;        // programs per (layer, dir)
 
   uint64_t seq = 0, epoch[2] = {0, 0};
+  uint64_t barrier_seq = 0;  // dgcl_device_barrier calls
   int *err_host = nullptr, *err_dev = nullptr;
   int threads = 512, ctas_per_sm = 0, grid = 0, n_sm = 0, use_tma = 1;
   int64_t item_bytes = kTmaBufBytes, timeout_ms = 20000;
@@ -1055,6 +1056,29 @@ static dgcl_status stage_out(dgcl_ctx *c, void *host, const void *dev, size_t by
   if ((s = stream_after(c, st, c->d2h_stream)) != DGCL_OK) return s;
   if (!c->host_async) CUDA_TRY(c, cudaStreamSynchronize(st));
   return check_dead(c);
+}
+
+dgcl_status dgcl_device_barrier(dgcl_ctx *c, void *stream) {
+  if (!c) return DGCL_EINVAL;
+  if (!has_device(c)) return fail(c, DGCL_ESTATE, "host-only context");
+  if (!c->registered) return fail(c, DGCL_ESTATE, "workspace not registered");
+  if (!c->loopback && c->world > 1 && !c->imported) return fail(c, DGCL_ESTATE, "peers not imported");
+  dgcl_status s = check_dead(c);
+  if (s != DGCL_OK) return s;
+  if (c->world == 1) return DGCL_OK;
+  DeviceGuard guard(c->device);
+  ExecParams P;
+  std::memset(&P, 0, sizeof(P));
+  for (int r = 0; r < c->world; ++r) P.flags[r] = (uint64_t *)(c->base[r] + c->off_flags[r]);
+  P.world = c->world;
+  P.seq = ++c->barrier_seq;
+  P.timeout_ns = (uint64_t)c->timeout_ms * 1000000ull;
+  P.err = c->err_dev;
+  // a fused loopback context is one launch stream: its virtual ranks arrive together
+  const int first = c->loopback ? 0 : c->rank, count = c->loopback ? c->world : 1;
+  const int e = launch_barrier(P, first, count, stream);
+  if (e != 0) return fail(c, DGCL_ECUDA, "barrier launch failed: %s", cudaGetErrorString((cudaError_t)e));
+  return DGCL_OK;
 }
 
 dgcl_status dgcl_forward_host(dgcl_ctx *c, int32_t layer, const float *host_emb, float *host_halo,

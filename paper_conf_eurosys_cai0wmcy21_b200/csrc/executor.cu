@@ -399,7 +399,26 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
   if (s_npend > 0) flush();
 }
 
+// Device start barrier (timing protocol: every timed call starts when all ranks
+// have arrived, so per-call times measure the exchange, not the ranks' launch skew).  Thread t
+// plays rank first + t; the ranks of a per-rank loopback context are threads of one warp, whose
+// spins make independent progress.
+__global__ void barrier_kernel(const __grid_constant__ ExecParams P, int first, int count) {
+  const int r = first + (int)threadIdx.x;
+  if ((int)threadIdx.x >= count) return;
+  for (int s = 0; s < P.world; ++s)
+    if (s != r) st_release_sys(P.flags[s] + kBarrierBase + r, P.seq);
+  for (int s = 0; s < P.world; ++s)
+    if (s != r && !wait_geq(P.flags[r] + kBarrierBase + s, P.seq, P, 3000000 + s)) return;
+}
+
 }  // namespace
+
+int launch_barrier(const ExecParams &p, int first, int count, void *stream) {
+  if (count <= 0) return 0;
+  barrier_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(p, first, count);
+  return (int)cudaGetLastError();
+}
 
 // executor_tma.cu
 int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream);

@@ -60,7 +60,8 @@ constexpr int64_t ctr_index(int dir, int stage, int src, int block = 0) {
   return (((int64_t)dir * kMaxStages + stage) * kMaxBlocks + block) * kMaxRanks + src;
 }
 constexpr int64_t kReadyBase = 2 * kMaxStages * kMaxBlocks * kMaxRanks;  // ready[src] words
-constexpr int64_t kFlagWords = kReadyBase + kMaxRanks;
+constexpr int64_t kBarrierBase = kReadyBase + kMaxRanks;  // device start barrier: arrived[src]
+constexpr int64_t kFlagWords = kBarrierBase + kMaxRanks;
 constexpr int64_t kFlagBytes = 40960;  // region reserved (>= kFlagWords * 8)
 static_assert(kFlagWords * 8 <= kFlagBytes, "flag region");
 
@@ -275,6 +276,9 @@ inline uint32_t fastdiv_host(uint32_t x, FastDiv f) {
 // launch wrapper implemented in executor.cu; returns a cudaError_t value
 int launch_executor(const ExecParams &p, int grid, int block, void *stream);
 int executor_occupancy(int block, int *ctas_per_sm);                          // register path
+// device start barrier: ranks first .. first+count-1 of this process (threads of one warp) each
+// release arrived[rank] = p.seq into every peer's flag region, then acquire-wait on every peer's
+int launch_barrier(const ExecParams &p, int first, int count, void *stream);
 int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm);  // bulk-copy path
 
 }  // namespace dgcl

@@ -162,20 +162,26 @@ class Context:
 
     def _check_arg(self, name, t, layer, rows):
         """The C side sees a pointer and a pitch only: refuse what it cannot check (dtype, device,
-        column stride, row count, pitch >= dim) before any out-of-bounds access could happen."""
+        column stride, row count, pitch >= dim) before any out-of-bounds access could happen.
+        Raises DGCLError(EINVAL) like the library's own argument checks."""
         import torch
+
+        def bad(msg):
+            raise DGCLError(_abi.EINVAL, "%s: %s" % (name, msg))
         if not isinstance(t, torch.Tensor):
-            raise TypeError("%s must be a torch tensor" % name)
+            bad("must be a torch tensor")
         if t.dtype != torch.float32:
-            raise TypeError("%s must be float32 (got %s)" % (name, t.dtype))
+            bad("must be float32 (got %s)" % t.dtype)
         if not t.is_cuda or t.device.index != self.device:
-            raise ValueError("%s must live on cuda:%d (got %s)" % (name, self.device, t.device))
+            bad("must live on cuda:%d (got %s)" % (self.device, t.device))
         if t.dim() != 2 or (t.shape[0] > 0 and t.stride(1) != 1):
-            raise ValueError("%s must be a 2-D row-major [rows x pitch] tensor" % name)
+            bad("must be a 2-D row-major [rows x pitch] tensor")
         if t.shape[0] < rows:
-            raise ValueError("%s has %d rows < %d" % (name, t.shape[0], rows))
-        if t.shape[1] < self.dims[layer] or (rows > 1 and t.stride(0) < self.dims[layer]):
-            raise ValueError("%s: pitch < dim %d" % (name, self.dims[layer]))
+            bad("has %d rows < %d" % (t.shape[0], rows))
+        if 0 <= layer < len(self.dims):   # (a bad layer is the library's EINVAL)
+            dim = self.dims[layer]
+            if t.shape[1] < dim or (t.shape[0] > 1 and t.stride(0) < dim):
+                bad("pitch < dim %d" % dim)
 
     def _halo_rows(self):
         return int(self.halo_off[-1]) if self.loopback else int(self.n_halo[self.rank])
@@ -255,6 +261,10 @@ class Context:
         check(lib().dgcl_plan_export(self.handle, ctypes.byref(n), u.ctypes.data, p.ctypes.data,
                                      c.ctypes.data, k.ctypes.data), self.handle)
         return np.stack([u, p.astype(np.int64), c.astype(np.int64), k.astype(np.int64)], axis=1)
+
+    def device_barrier(self, stream=None):
+        """Device-side start barrier over the ranks on `stream` (timing protocol)."""
+        check(lib().dgcl_device_barrier(self.handle, _stream_ptr(stream)), self.handle)
 
     def launch_count(self):
         v = ctypes.c_uint64(0)

@@ -360,6 +360,22 @@ def test_argument_errors():
     with pytest.raises(D.DGCLError) as e:
         c.ctx.forward(0, torch.zeros(g.n, 8, device="cuda"))            # pitch < dim
     assert e.value.status == 1
+    # what only the binding can see (the C side gets a pointer and a pitch): dtype, device,
+    # column stride, row count
+    for bad in (torch.zeros(g.n, 16, device="cuda", dtype=torch.bfloat16),
+                torch.zeros(g.n, 16),                                   # host tensor
+                torch.zeros(16, g.n, device="cuda").t(),                # column-strided
+                torch.zeros(g.n - 1, 16, device="cuda")):               # too few rows
+        with pytest.raises(D.DGCLError) as e:
+            c.ctx.forward(0, bad)
+        assert e.value.status == 1
+    hg = torch.zeros(c.S, 16, device="cuda")
+    with pytest.raises(D.DGCLError) as e:
+        c.ctx.backward(0, hg[:-1], torch.zeros(g.n, 16, device="cuda"))  # halo_grad too short
+    assert e.value.status == 1
+    with pytest.raises(D.DGCLError) as e:
+        c.ctx.backward(0, hg, torch.zeros(g.n, 16, device="cuda", dtype=torch.float16))
+    assert e.value.status == 1
 
 
 def test_autograd_graph_allgather():
