@@ -422,8 +422,14 @@ def run_ours_single(args, w):
         else:
             alg = (w.S + 2 * nv) * row
         ach = alg / (per_op[n] * 1e-3) / 1e9
+        # SURVEY §8(d)'s loopback formula, HBM r+w = 2 x deliveries x row (every delivery read
+        # AND written), reported beside it: it counts a row sent to k receivers as k DRAM reads,
+        # which L2 serves after the first (R20), so its "fraction" can exceed 1
+        survey = 2 * w.S * row
         kernels[n] = {"ms": per_op[n], "algorithmic_bytes": int(alg), "achieved_gbs": ach,
                       "frac": ach / peaks["hbm_gbs"],
+                      "survey_formula_bytes": int(survey),
+                      "survey_formula_frac": survey / (per_op[n] * 1e-3) / 1e9 / peaks["hbm_gbs"],
                       "traffic": profiled_traffic("%s/%s" % (c.name, n))}
         if plan_rows is not None:
             pb = plan_rows["fwd" if n.startswith("fwd") else "bwd"] * row
@@ -434,6 +440,11 @@ def run_ours_single(args, w):
                 "achieved": kernels[dom]["achieved_gbs"], "peak": peaks["hbm_gbs"],
                 "unit": "GB/s", "frac": kernels[dom]["frac"], "traffic": kernels[dom]["traffic"],
                 "algorithmic_bytes_per_launch": kernels[dom]["algorithmic_bytes"],
+                "algorithmic_bytes_definition": "compulsory DRAM bytes (DESIGN.md R20): unique "
+                                                "source rows read once + every destination row "
+                                                "written once (backward: halo-gradient rows read "
+                                                "+ owner rows with requesters read and written)",
+                "survey_formula_frac": kernels[dom]["survey_formula_frac"],
                 "peak_source": src + " (MEASURED_PEAKS.json hbm_gbs: copy read+write)",
                 "per_kernel": kernels}
 

@@ -239,6 +239,10 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "direct_copy_rows" COPY items whose runs average fewer rows are gathered by the consumer
  *                    warps with plain loads (default 0 = never)
  *   "trace"          1: record per-item timelines of every launch (dgcl_trace_read); default 0
+ *   "sm_budget"      SMs one executor launch may use (default 0 = all; any time): leaves SMs free
+ *                    for kernels that overlap the exchange (dgcl_stream_wait_arrival)
+ *   "signal_all"     fused loopback: every item publishes its done count, so arrival waits work
+ *                    (default 0: only counts some item of the launch waits on)
  *   "small_launch_bytes" launches moving fewer bytes (rows x row size) run the register
  *                    executor instead of the bulk-copy pipeline (latency; default 4 MiB, 0 = never)
  *   "host_async"     0 (default) / 1: dgcl_forward_host / dgcl_backward_host return before the
@@ -278,6 +282,19 @@ dgcl_status dgcl_trace_read(dgcl_ctx *ctx, int32_t layer, int32_t dir, int32_t r
  * ranks in the one warp.  world == 1: no-op.  Errors: DGCL_ESTATE before registration / import;
  * a peer that never arrives trips the watchdog (dgcl_check -> DGCL_ETIMEOUT). */
 dgcl_status dgcl_device_barrier(dgcl_ctx *ctx, void *stream);
+
+/* Arrival wait for overlapping work (the paper runs graph operations
+ * after graphAllgather returns, P:1554-1566 — this lets them start per source instead).
+ * Enqueues on `stream` a one-warp kernel that acquire-waits until rank `dst` (this rank; any
+ * virtual rank in loopback; -1 = this rank) has received, in the most recent dgcl_dispatch_forward
+ * call, every row that comes from rank `src` (single-stage plans: src's stage-1 done counter), or
+ * — for relay plans, or src = -1 — every incoming row of every stage.  Work queued after it on
+ * `stream` may read those halo rows while the exchange is still running on the dispatch stream.
+ * Use with option "sm_budget" < the SM count so that the overlapped kernels find free SMs.
+ * Fused loopback contexts need option "signal_all" (set before registration).  Errors: EINVAL
+ * for a bad (dst, src), ESTATE before registration / without signal_all; a row that never
+ * arrives trips the watchdog (dgcl_check -> DGCL_ETIMEOUT).  No forward call yet: no-op. */
+dgcl_status dgcl_stream_wait_arrival(dgcl_ctx *ctx, int32_t dst, int32_t src, void *stream);
 
 /* Number of executor kernel launches issued so far by this context. */
 dgcl_status dgcl_launch_count(dgcl_ctx *ctx, uint64_t *count);

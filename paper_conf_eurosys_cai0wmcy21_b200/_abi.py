@@ -23,6 +23,7 @@ SYMBOLS = [
     "dgcl_ipc_export", "dgcl_ipc_import", "dgcl_dispatch_forward", "dgcl_dispatch_backward",
     "dgcl_forward_host", "dgcl_backward_host", "dgcl_plan_info", "dgcl_plan_counts",
     "dgcl_plan_export", "dgcl_set_option", "dgcl_trace_read", "dgcl_device_barrier",
+    "dgcl_stream_wait_arrival",
     "dgcl_launch_count", "dgcl_check",
     "dgcl_last_error",
     "dgcl_strerror", "dgcl_destroy", "dgcl_debug_hostsim_forward", "dgcl_debug_hostsim_backward",
@@ -87,6 +88,7 @@ def lib():
             "dgcl_set_option": [P, ctypes.c_char_p, I64],
             "dgcl_trace_read": [P, I32, I32, I32, P, ctypes.POINTER(I64)],
             "dgcl_device_barrier": [P, P],
+            "dgcl_stream_wait_arrival": [P, I32, I32, P],
             "dgcl_launch_count": [P, ctypes.POINTER(U64)],
             "dgcl_check": [P],
             "dgcl_destroy": [P],

@@ -102,6 +102,9 @@ struct dgcl_ctx {
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
   bool hostsim_items = false;         // debug host interpreter: run the work items, not groups
   int geometry = 0;                   // bulk-copy geometry: 0 auto per program, 1 WIDE, 2 DUAL
+  int sm_budget = 0;                  // SMs an executor launch may use (0 = all): the rest stay
+                                      // free for kernels overlapping the exchange (NEXT-2)
+  bool signal_all = false;            // fused loopback: publish every done count (arrival waits)
   bool threads_set = false, ctas_set = false;  // user overrides of the CTA shape
   int sm_count = 148;  // SMs of the device (B200 until queried), for cutting small stages
   std::map<std::pair<int, int>, int> tma_ctas;  // (geo, block) -> co-resident CTAs per SM
@@ -367,7 +370,8 @@ void build_programs(dgcl_ctx *c) {
         ItemLimits lim = item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
                                      (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm);
         lim.align_sources = c->align_sources;
-        build_items(L, G, row_bytes, lim, !fused, need, &P.items, &P.runs, c->direct_copy_rows,
+        build_items(L, G, row_bytes, lim, !fused || c->signal_all, need, &P.items, &P.runs,
+                    c->direct_copy_rows,
                     c->stage_fold ? &P.sterms : nullptr);
         P.op_mask = 0;
         int64_t fold_rows = 0, fold_terms = 0;
@@ -625,14 +629,17 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     const int tblock = tma_block(c, pg);
     const auto occ = c->tma_ctas.find({pg.geo, tblock});
     const int tctas = occ == c->tma_ctas.end() ? 0 : occ->second;
-    int block = c->threads, grid_all = c->grid;
+    // (sm_budget: the grid covers only that many SMs, still co-resident; the other SMs run
+    // whatever the caller overlaps with the exchange)
+    const int sms = c->sm_budget > 0 ? std::min(c->sm_budget, c->n_sm) : c->n_sm;
+    int block = c->threads, grid_all = sms * c->ctas_per_sm;
     // latency-bound launches (a few MB) skip the bulk-copy pipeline: the register executor's
     // single round trip per item is shorter (tiny config: 10 vs 14-19 us per launch)
     // (sel_bytes: per-rank loopback decides for all ranks of a launch together, co-residency)
     const bool small = sel_bytes < c->small_launch_bytes;
     if (Pp.use_tma && !small && Pp.row16 <= G.stage_bytes - kStageHdrBytes && tctas > 0) {
       block = tblock;
-      grid_all = c->n_sm * tctas;
+      grid_all = sms * tctas;
       Pp.tma_stages = G.stages;
       Pp.tma_buf = G.stage_bytes;
       Pp.meta_bytes = G.meta_bytes;
@@ -1081,6 +1088,54 @@ dgcl_status dgcl_device_barrier(dgcl_ctx *c, void *stream) {
   return DGCL_OK;
 }
 
+dgcl_status dgcl_stream_wait_arrival(dgcl_ctx *c, int32_t dst, int32_t src, void *stream) {
+  if (!c) return DGCL_EINVAL;
+  if (!has_device(c)) return fail(c, DGCL_ESTATE, "host-only context");
+  if (!c->registered) return fail(c, DGCL_ESTATE, "workspace not registered");
+  if (!c->loopback && c->world > 1 && !c->imported) return fail(c, DGCL_ESTATE, "peers not imported");
+  if (dst < 0) dst = c->rank;
+  if (dst >= c->world || src < -1 || src >= c->world || src == dst)
+    return fail(c, DGCL_EINVAL, "bad (dst %d, src %d)", dst, src);
+  if (!c->loopback && dst != c->rank) return fail(c, DGCL_EINVAL, "dst must be this rank");
+  if (c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED && !c->signal_all)
+    return fail(c, DGCL_ESTATE, "fused loopback publishes arrivals only with option signal_all");
+  dgcl_status s = check_dead(c);
+  if (s != DGCL_OK) return s;
+  if (c->world == 1 || c->epoch[DIR_FWD] == 0) return DGCL_OK;
+  // the forward-completion wait list of dst: every incoming counter of every stage; a
+  // single-stage plan's entry for src is exactly "all rows from src have landed"
+  const Lowered &L = c->low;
+  int32_t off = -1, n = 0;
+  for (const DevGroup &g : L.groups)
+    if (g.op == OP_WAIT && g.exec_rank == dst) {
+      off = g.wait_off;
+      n = g.wait_n;
+    }
+  if (off < 0) return fail(c, DGCL_EPLAN, "no completion list for rank %d", dst);
+  if (src >= 0 && L.n_stages <= 1) {
+    const int32_t want = (int32_t)ctr_index(DIR_FWD, 1, src, 0);
+    int32_t hit = -1;
+    for (int32_t w = off; w < off + n; ++w)
+      if (L.waits[w].ctr == want) hit = w;
+    if (hit < 0) return DGCL_OK;  // nothing comes from src
+    off = hit;
+    n = 1;
+  }
+  if (n == 0) return DGCL_OK;
+  DeviceGuard guard(c->device);
+  ExecParams P;
+  std::memset(&P, 0, sizeof(P));
+  for (int r = 0; r < c->world; ++r) P.flags[r] = (uint64_t *)(c->base[r] + c->off_flags[r]);
+  P.world = c->world;
+  P.waits = c->d_waits;
+  P.epoch[DIR_FWD] = c->epoch[DIR_FWD];
+  P.timeout_ns = (uint64_t)c->timeout_ms * 1000000ull;
+  P.err = c->err_dev;
+  const int e = launch_wait(P, dst, off, n, stream);
+  if (e != 0) return fail(c, DGCL_ECUDA, "wait launch failed: %s", cudaGetErrorString((cudaError_t)e));
+  return DGCL_OK;
+}
+
 dgcl_status dgcl_forward_host(dgcl_ctx *c, int32_t layer, const float *host_emb, float *host_halo,
                               void *stream) {
   dgcl_status s = ready_to_dispatch(c, layer);
@@ -1193,6 +1248,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }
+  if (k == "sm_budget") {  // SMs per executor launch (0 = all); any time
+    if (value < 0) return fail(c, DGCL_EINVAL, "sm_budget must be >= 0");
+    c->sm_budget = (int)value;
+    return DGCL_OK;
+  }
   if (k == "trace") {  // per-item timelines of every launch (dgcl_trace_read)
     c->trace = value != 0;
     return DGCL_OK;
@@ -1257,6 +1317,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
       compute_layout(c);
       build_programs(c);
     }
+    return DGCL_OK;
+  }
+  if (k == "signal_all") {  // fused loopback: every item publishes its done count
+    c->signal_all = value != 0;
+    if (c->planned) build_programs(c);
     return DGCL_OK;
   }
   if (k == "align_sources") {  // forward COPY groups of one source rank: common item boundaries

@@ -412,7 +412,22 @@ __global__ void barrier_kernel(const __grid_constant__ ExecParams P, int first, 
     if (s != r && !wait_geq(P.flags[r] + kBarrierBase + s, P.seq, P, 3000000 + s)) return;
 }
 
+// Arrival wait: later work on the stream sees the rows counted by these counters (acquire).
+__global__ void wait_kernel(const __grid_constant__ ExecParams P, int exec, int off, int n) {
+  if (threadIdx.x != 0) return;
+  for (int w = off; w < off + n; ++w) {
+    const DevWait W = P.waits[w];
+    if (!wait_geq(P.flags[exec] + W.ctr, P.epoch[DIR_FWD] * (uint64_t)W.amount, P, 4000000 + w))
+      return;
+  }
+}
+
 }  // namespace
+
+int launch_wait(const ExecParams &p, int exec, int off, int n, void *stream) {
+  wait_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(p, exec, off, n);
+  return (int)cudaGetLastError();
+}
 
 int launch_barrier(const ExecParams &p, int first, int count, void *stream) {
   if (count <= 0) return 0;

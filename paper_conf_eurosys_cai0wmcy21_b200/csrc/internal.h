@@ -279,6 +279,9 @@ int executor_occupancy(int block, int *ctas_per_sm);                          //
 // device start barrier: ranks first .. first+count-1 of this process (threads of one warp) each
 // release arrived[rank] = p.seq into every peer's flag region, then acquire-wait on every peer's
 int launch_barrier(const ExecParams &p, int first, int count, void *stream);
+// arrival wait (overlap): one thread acquire-waits on rank `exec`'s counters
+// p.waits[off .. off + n) >= p.epoch[DIR_FWD] * amount, then the kernel ends
+int launch_wait(const ExecParams &p, int exec, int off, int n, void *stream);
 int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm);  // bulk-copy path
 
 }  // namespace dgcl

@@ -266,6 +266,12 @@ class Context:
         """Device-side start barrier over the ranks on `stream` (timing protocol)."""
         check(lib().dgcl_device_barrier(self.handle, _stream_ptr(stream)), self.handle)
 
+    def wait_arrival(self, src=-1, dst=-1, stream=None):
+        """Enqueue on `stream` a wait until the rows from `src` (-1: all sources) of the latest
+        forward call have landed on `dst` (-1: this rank; loopback: a virtual rank)."""
+        check(lib().dgcl_stream_wait_arrival(self.handle, dst, src, _stream_ptr(stream)),
+              self.handle)
+
     def launch_count(self):
         v = ctypes.c_uint64(0)
         check(lib().dgcl_launch_count(self.handle, ctypes.byref(v)), self.handle)
