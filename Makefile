@@ -7,7 +7,7 @@ NVCC     ?= $(CUDA)/bin/nvcc
 CXX      := $(shell test -x /usr/bin/g++ && echo /usr/bin/g++ || echo g++)
 GENCODE  := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS  := -O3 -std=c++17 $(GENCODE) -lineinfo -Xcompiler -fPIC -Xcompiler -Wall -Iinclude
-CXXFLAGS := -O3 -std=c++17 -fPIC -Wall -Wextra -Iinclude -I$(CUDA)/include
+CXXFLAGS := -O3 -std=c++17 -fPIC -fopenmp -Wall -Wextra -Iinclude -I$(CUDA)/include
 
 CSRC     := $(PKG)/csrc
 HOST_SRC := $(CSRC)/planner.cpp $(CSRC)/lowering.cpp $(CSRC)/api.cpp $(CSRC)/hostsim.cpp
@@ -33,7 +33,7 @@ build/%.o: $(CSRC)/%.cu $(HDRS)
 	$(NVCC) $(NVFLAGS) -Xptxas -v -c $< -o $@ 2> build/$*.ptxas.log || (cat build/$*.ptxas.log; false)
 
 $(PKG)/libdgcl.so: $(HOST_OBJ) $(CU_OBJ)
-	$(NVCC) $(GENCODE) -shared -Xcompiler -fPIC -cudart static $^ -o $@
+	$(NVCC) $(GENCODE) -shared -Xcompiler -fPIC -Xcompiler -fopenmp -cudart static $^ -o $@
 
 clean:
 	rm -rf build synth/_synth.so $(PKG)/libdgcl.so

@@ -15,6 +15,9 @@
 // writer, no atomics — and additionally fixes the summation order (R6).
 
 #include <algorithm>
+#include <parallel/algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <functional>
 #include <chrono>
 #include <cstring>
@@ -59,6 +62,16 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
                 const std::vector<int64_t> &loc, Lowered *out, int n_blocks, bool with_atomic,
                 bool with_fanout) {
   auto t0 = std::chrono::steady_clock::now();
+  // DGCL_TIMING=1: per-section wall times on stderr (planning at scale, NEXT-4)
+  static const bool timing = std::getenv("DGCL_TIMING") != nullptr;
+  auto tl = t0;
+  auto lap = [&](const char *what) {
+    if (!timing) return;
+    const auto now = std::chrono::steady_clock::now();
+    std::fprintf(stderr, "[dgcl lowering] %-24s %8.3f s\n", what,
+                 std::chrono::duration<double>(now - tl).count());
+    tl = now;
+  };
   const int m = plan.m;
   const int K = plan.n_stages;
   Lowered &L = *out;
@@ -100,6 +113,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     for (int64_t e = plan.e_ptr[i]; e < plan.e_ptr[i + 1]; ++e) e_vidx[e] = i;
   // is the child of edge e a requester (halo) or a pure relay?
   std::vector<int32_t> child_pos(NE);
+#pragma omp parallel for schedule(static)
   for (int64_t e = 0; e < NE; ++e)
     child_pos[e] = halo_pos(rel, plan.order[e_vidx[e]], plan.e_child[e]);
   // edge into node x of the same tree (for relay sources / children lists)
@@ -109,15 +123,75 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     return -1;
   };
 
+  // children index, built once (parallel over vertices): the tree edges out of the child node of
+  // every edge, and out of every tree's root, each list in ascending child id (the fixed
+  // contribution order, R6)
+  std::vector<int64_t> kid_eptr(NE + 1, 0), kid_rptr(NV + 1, 0), kid_elist, kid_rlist;
+  {
+#pragma omp parallel for schedule(static)
+    for (int64_t vi = 0; vi < NV; ++vi) {
+      const int root = part[plan.order[vi]];
+      int64_t nr = 0;
+      for (int64_t e = plan.e_ptr[vi]; e < plan.e_ptr[vi + 1]; ++e) {
+        int64_t nk = 0;
+        for (int64_t f = plan.e_ptr[vi]; f < plan.e_ptr[vi + 1]; ++f)
+          nk += plan.e_parent[f] == plan.e_child[e];
+        kid_eptr[e + 1] = nk;
+        nr += plan.e_parent[e] == root;
+      }
+      kid_rptr[vi + 1] = nr;
+    }
+    for (int64_t e = 0; e < NE; ++e) kid_eptr[e + 1] += kid_eptr[e];
+    for (int64_t vi = 0; vi < NV; ++vi) kid_rptr[vi + 1] += kid_rptr[vi];
+    kid_elist.resize(kid_eptr[NE]);
+    kid_rlist.resize(kid_rptr[NV]);
+    auto by_child = [&](int64_t a, int64_t b) { return plan.e_child[a] < plan.e_child[b]; };
+#pragma omp parallel for schedule(static)
+    for (int64_t vi = 0; vi < NV; ++vi) {
+      const int root = part[plan.order[vi]];
+      int64_t *rl = kid_rlist.data() + kid_rptr[vi];
+      int nr = 0;
+      for (int64_t e = plan.e_ptr[vi]; e < plan.e_ptr[vi + 1]; ++e) {
+        int64_t *el = kid_elist.data() + kid_eptr[e];
+        int nk = 0;
+        for (int64_t f = plan.e_ptr[vi]; f < plan.e_ptr[vi + 1]; ++f)
+          if (plan.e_parent[f] == plan.e_child[e]) el[nk++] = f;
+        std::sort(el, el + nk, by_child);
+        if (plan.e_parent[e] == root) rl[nr++] = e;
+      }
+      std::sort(rl, rl + nr, by_child);
+    }
+  }
+  // children (edge indices, ascending child id) of node x of tree vi: the root, or the child
+  // node of the tree's edge into x
+  auto children_of = [&](int64_t vi, int x, int64_t *outv) -> int {
+    const int64_t *b, *e;
+    if (x == part[plan.order[vi]]) {
+      b = kid_rlist.data() + kid_rptr[vi];
+      e = kid_rlist.data() + kid_rptr[vi + 1];
+    } else {
+      const int64_t in = edge_into(vi, x);
+      if (in < 0) return 0;
+      b = kid_elist.data() + kid_eptr[in];
+      e = kid_elist.data() + kid_eptr[in + 1];
+    }
+    int n = 0;
+    for (const int64_t *q = b; q < e; ++q) outv[n++] = *q;
+    return n;
+  };
+  lap("children index");
+
   // source buffer kind of every edge: the owner sends from its embeddings, a requester forwards
   // from its halo, a pure relay from its relay staging
   std::vector<int8_t> src_kind(NE);
+#pragma omp parallel for schedule(static)
   for (int64_t e = 0; e < NE; ++e) {
     const int64_t u = plan.order[e_vidx[e]];
     const int p = plan.e_parent[e];
     src_kind[e] = p == part[u] ? K_EMB : (halo_pos(rel, u, p) >= 0 ? K_HALO : K_RELAY);
   }
 
+  lap("blocks/child_pos/kinds");
   // ---- forward relay staging rows: contiguous per (receiver c, stage k, sender p, src kind) ----
   std::vector<int64_t> relay_row(NE, -1);
   {
@@ -127,7 +201,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
         rel_e.push_back({pack_key(plan.e_child[e], plan.e_stage[e], plan.e_parent[e],
                                   src_kind[e], 0),
                          e_vidx[e], e, e_vidx[e]});
-    std::sort(rel_e.begin(), rel_e.end(), [](const Entry &a, const Entry &b) {
+    __gnu_parallel::sort(rel_e.begin(), rel_e.end(), [](const Entry &a, const Entry &b) {
       return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
     });
     for (const Entry &x : rel_e) relay_row[x.edge] = L.n_relay[plan.e_child[x.edge]]++;
@@ -181,10 +255,12 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     return g;
   };
 
+  lap("relay rows");
   // ---- forward groups: key (k, p, c, src_kind, dst_kind), rows sorted by destination row ----
   {
     std::vector<Entry> ent(NE);
     std::vector<int64_t> srow(NE), drow(NE);
+#pragma omp parallel for schedule(static)
     for (int64_t e = 0; e < NE; ++e) {
       const int64_t vi = e_vidx[e];
       const int64_t u = plan.order[vi];
@@ -206,7 +282,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       }
       ent[e] = {pack_key_b(k, blk_of[vi], p, c, sk, dk), drow[e], e, vi};
     }
-    std::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
+    __gnu_parallel::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
       return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
     });
     std::vector<int64_t> src, dst;
@@ -233,11 +309,13 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     L.n_fwd_groups = (int)L.groups.size();
   }
 
+  lap("forward groups");
   // ---- backward pushes: key (b, c, p, sig) ----
   {
     // term signature of c's value for the vertex of edge e (c = child of e)
     std::vector<int8_t> sig(NE);
     std::vector<int8_t> nchild(NE, 0);
+#pragma omp parallel for schedule(static)
     for (int64_t e = 0; e < NE; ++e) {
       const int64_t vi = e_vidx[e];
       int nc = 0;
@@ -248,24 +326,19 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       sig[e] = (own && nc == 0) ? 0 : (!own && nc == 1) ? 1 : 2;
     }
     std::vector<Entry> ent(NE);
+#pragma omp parallel for schedule(static)
     for (int64_t e = 0; e < NE; ++e) {
       const int b = K - plan.e_stage[e] + 1;
       const int64_t sort2 = sig[e] == 0 ? (int64_t)child_pos[e] : plan.order[e_vidx[e]];
       ent[e] = {pack_key_b(b, blk_of[e_vidx[e]], plan.e_child[e], plan.e_parent[e], sig[e], 0),
                 sort2, e, e_vidx[e]};
     }
-    std::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
+    __gnu_parallel::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
       return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
     });
+    lap("  bwd sig + sort");
     // children of node x in tree vi, ascending id -> their edge indices
-    auto children_edges = [&](int64_t vi, int x, int64_t *outv) -> int {
-      int n = 0;
-      for (int64_t f = plan.e_ptr[vi]; f < plan.e_ptr[vi + 1]; ++f)
-        if (plan.e_parent[f] == x) outv[n++] = f;
-      std::sort(outv, outv + n,
-                [&](int64_t a, int64_t b) { return plan.e_child[a] < plan.e_child[b]; });
-      return n;
-    };
+    auto children_edges = children_of;
     // RED rows of every owner: (loc, vertex index) ascending
     std::vector<std::vector<std::pair<int64_t, int64_t>>> red_rows(m);
     for (int64_t vi = 0; vi < NV; ++vi) {
@@ -284,13 +357,15 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     // Web-Google ring 2.08 -> 1.92, Reddit dgx1_like 1.24 -> 1.18, Web-Google dgx1_like
     // 1.82 -> 1.91; against slots grouped per (consumer group, child) with pushes in consumer
     // order: 2.09 / 1.20 / 1.90.
+    lap("  bwd red_rows");
     std::vector<int64_t> slot_row(NE, -1);
     {
       int64_t chs[kMaxRanks];
-      for (const Entry &x : ent) {
-        const int c = plan.e_child[x.edge];
-        const int n = children_edges(x.vidx, c, chs);
-        for (int t = 0; t < n; ++t) slot_row[chs[t]] = L.n_slot[c]++;
+      for (const Entry &x : ent) {  // (the children of edge x's child node: its kid list)
+        const int64_t kb = kid_eptr[x.edge], ke = kid_eptr[x.edge + 1];
+        if (kb == ke) continue;
+        int64_t &ns = L.n_slot[plan.e_child[x.edge]];
+        for (int64_t q = kb; q < ke; ++q) slot_row[kid_elist[q]] = ns++;
       }
       for (int s = 0; s < m; ++s)
         for (auto &r : red_rows[s]) {
@@ -299,6 +374,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
         }
     }
 
+    lap("  bwd slot rows");
     std::vector<int64_t> src, dst;
     int64_t ch[kMaxRanks];
     for (size_t i = 0; i < ent.size();) {
@@ -319,18 +395,15 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       }
       for (size_t q = i; q < j; ++q) {
         const int64_t e = ent[q].edge;
-        const int64_t vi = ent[q].vidx;
         dst.push_back(slot_row[e]);
         if (s == 0) {
           src.push_back(child_pos[e]);
         } else if (s == 1) {
-          const int n = children_edges(vi, c, ch);
-          (void)n;
-          src.push_back(slot_row[ch[0]]);
+          src.push_back(slot_row[kid_elist[kid_eptr[e]]]);
         } else {
           if (child_pos[e] >= 0) L.terms.push_back((uint32_t)child_pos[e]);
-          const int n = children_edges(vi, c, ch);
-          for (int t = 0; t < n; ++t) L.terms.push_back(kTermSlot | (uint32_t)slot_row[ch[t]]);
+          for (int64_t q = kid_eptr[e]; q < kid_eptr[e + 1]; ++q)
+            L.terms.push_back(kTermSlot | (uint32_t)slot_row[kid_elist[q]]);
           L.term_ptr.push_back((int64_t)L.terms.size());
         }
       }
@@ -340,6 +413,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       i = j;
     }
 
+    lap("  bwd push groups");
     // ---- RED: owner folds its slots into emb_grad, ascending child id, stage K + 1 ----
     for (int bl = 0; bl < NB; ++bl)
     for (int s = 0; s < m; ++s) {
@@ -365,6 +439,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     }
   }
 
+  lap("backward pushes + RED");
   // ---- signals and waits (the ready/done protocol of §6.1) ----
   // wait lists per (dir, stage, exec, block): every in-peer's counter of the previous stage of
   // the same vertex block
@@ -415,6 +490,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     g.wait_n = (int32_t)L.waits.size() - g.wait_off;
     L.groups.push_back(g);
   }
+  lap("signals/waits");
   // ---- loopback direct reduce (single-stage plans only) ----
   // When every virtual rank lives on one device the owner can read its requesters' halo-gradient
   // rows in place: emb_grad[loc u] = ((emb_grad[loc u] + G_c1[pos]) + G_c2[pos]) + ..., c
@@ -446,6 +522,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     }
   }
   L.direct_end = (int)L.groups.size();
+  lap("direct reduce");
   // ---- loopback atomic backward (ablation, single-stage plans only) ----
   // The paper's "Atomic" baseline (§6.2, Table 9): every requester adds
   // its halo-gradient rows straight into the owner's rows with atomic reductions, one group per
@@ -530,6 +607,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     if (!fits) L.groups.resize(L.atomic_end);  // rows beyond the 27-bit dest field: per-pair groups
   }
   L.fanout_end = (int)L.groups.size();
+  lap("atomic/fanout groups");
   // ---- loopback tree-order backward (relay plans) ----
   // With every virtual rank on one device the owner can evaluate the reversed plan's whole fold
   // for its row in one pass: the staged backward computes val_c(u) = ((own_c + val(y1)) +
@@ -539,14 +617,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   // result is bit-identical to the staged pushes without their slot round trips and stage
   // barriers.  (The multi-GPU form, and loopback with direct_reduce = 0, run the stages.)
   if (K >= 2) {
-    auto kids = [&](int64_t vi, int x, int64_t *outv) -> int {
-      int n = 0;
-      for (int64_t f = plan.e_ptr[vi]; f < plan.e_ptr[vi + 1]; ++f)
-        if (plan.e_parent[f] == x) outv[n++] = f;
-      std::sort(outv, outv + n,
-                [&](int64_t a, int64_t b) { return plan.e_child[a] < plan.e_child[b]; });
-      return n;
-    };
+    auto kids = children_of;
     bool fits = true;
     int depth = 0, max_depth = 0;
     // postfix of val(x) for vertex vi: own(x) (if x requested u), then each child ascending,
@@ -612,6 +683,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     }
   }
   L.tree_end = (int)L.groups.size();
+  lap("tree programs");
   L.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
 }
 

@@ -15,3 +15,11 @@ for C in ${CFGS:-tiny reddit google2 google4 google8 orkut google8_dgx1 google8_
     > gpurun_out/${TAG}_${C}_prof.log 2>&1
   echo "$C bench+ncu rc=$?"
 done
+# summaries on the box (gpurun_out/ must stay < 64 MiB): raw CSV pages + markdown, then the
+# reports themselves are dropped (KEEP_REP=cfg keeps one)
+mkdir -p gpurun_out/${TAG}_profiles
+python tools/profile_summary.py ${TAG} "${CFGS// /,}" gpurun_out/${TAG}_profiles > /dev/null
+for f in gpurun_out/${TAG}_*_prof.ncu-rep; do
+  case "$f" in *"_${KEEP_REP:-none}_prof.ncu-rep") ;; *) rm -f "$f" ;; esac
+done
+du -sh gpurun_out

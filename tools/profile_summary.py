@@ -18,8 +18,13 @@ UNIT = {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1.0, "ms": 1e-3, "us":
 
 
 def raw(rep):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
-                         text=True).stdout
+    """Rows of the raw page: from the report (ncu -i), or from its saved CSV (<rep>.raw.csv)."""
+    if os.path.exists(rep):
+        out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
+                             text=True).stdout
+        open(rep[:-len(".ncu-rep")] + ".raw.csv", "w").write(out)
+    else:
+        out = open(rep[:-len(".ncu-rep")] + ".raw.csv").read()
     rows = list(csv.reader(io.StringIO(out)))
     hdr, units = rows[0], rows[1]
     return [{h: (r[i], units[i]) for i, h in enumerate(hdr)} for r in rows[2:]]
@@ -38,7 +43,8 @@ def num(d, k):
 def summarize(tag, cfg):
     rep = os.path.join(ROOT, "gpurun_out", "%s_%s_prof.ncu-rep" % (tag, cfg))
     bj = os.path.join(ROOT, "gpurun_out", "%s_%s_bench.json" % (tag, cfg))
-    if not os.path.exists(rep) or not os.path.exists(bj):
+    csvp = rep[:-len(".ncu-rep")] + ".raw.csv"
+    if not (os.path.exists(rep) or os.path.exists(csvp)) or not os.path.exists(bj):
         return None, {}
     bench = json.loads(open(bj).read().strip().splitlines()[-1])
     names = list(bench["ms_per_layer"])
@@ -77,7 +83,8 @@ def summarize(tag, cfg):
     return "\n".join(head + rows) + "\n", traffic
 
 
-def main(tag, cfgs):
+def main(tag, cfgs, outdir=None):
+    outdir = outdir or os.path.join(ROOT, "profiles")
     out = ["# ncu --set full, every executor launch of one step (%s)" % tag, "",
            "`tools/ncu_all.sh`: `ncu --set full --clock-control none --import-source on -k "
            "regex:executor -c <launches per step> python bench.py --config C --steps 1 --warmup 3` "
@@ -86,19 +93,23 @@ def main(tag, cfgs):
            "(DESIGN.md §4: unique source rows read once + every destination row written once; "
            "backward: halo-gradient rows read + owner rows with requesters read and written); "
            "plan = the relay plan's own minimum (every tree edge written, forwarded rows read).", ""]
-    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    tp = os.path.join(outdir, "traffic.json")
+    if not os.path.exists(tp) and os.path.exists(os.path.join(ROOT, "profiles", "traffic.json")):
+        tp0 = os.path.join(ROOT, "profiles", "traffic.json")
+        json.dump(json.load(open(tp0)), open(tp, "w"))
     traffic = json.load(open(tp)) if os.path.exists(tp) else {}
     for c in cfgs:
         s, t = summarize(tag, c)
         if s:
             out.append(s)
             traffic.update(t)
-    path = os.path.join(ROOT, "profiles", "%s_ncu_all_configs.md" % tag)
+    path = os.path.join(outdir, "%s_ncu_all_configs.md" % tag)
     open(path, "w").write("\n".join(out))
     json.dump(traffic, open(tp, "w"), indent=1, sort_keys=True)
     print("\n".join(out))
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2].split(",") if len(sys.argv) > 2 else
-         "tiny,reddit,google2,google4,google8,orkut,google8_dgx1,google8_ring,reddit_dgx1".split(","))
+    main(sys.argv[1], sys.argv[2].split(",") if len(sys.argv) > 2 and sys.argv[2] else
+         "tiny,reddit,google2,google4,google8,orkut,google8_dgx1,google8_ring,reddit_dgx1".split(","),
+         sys.argv[3] if len(sys.argv) > 3 else None)
