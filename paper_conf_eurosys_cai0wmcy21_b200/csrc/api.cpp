@@ -105,6 +105,8 @@ struct dgcl_ctx {
   int sm_budget = 0;                  // SMs an executor launch may use (0 = all): the rest stay
                                       // free for kernels overlapping the exchange (NEXT-2)
   bool signal_all = false;            // fused loopback: publish every done count (arrival waits)
+  int l2_policy = 0;                  // L2 eviction hints (executor_tma.cu), A/B option
+  bool force_sys_scope = false;       // loopback with the multi-GPU (.sys) flag scope (A/B)
   bool threads_set = false, ctas_set = false;  // user overrides of the CTA shape
   int sm_count = 148;  // SMs of the device (B200 until queried), for cutting small stages
   std::map<std::pair<int, int>, int> tma_ctas;  // (geo, block) -> co-resident CTAs per SM
@@ -583,6 +585,9 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
   P.runs = c->d_runs;
   P.sterms = c->d_sterms;
   P.bulk_store = (c->loopback ? c->bulk_store_local : c->bulk_store_peer) ? 1 : 0;
+  P.l2_policy = c->l2_policy;
+  // every rank on this device (loopback): the flag protocol needs only device scope
+  P.sys_scope = (c->loopback && !c->force_sys_scope) ? 0 : 1;
   // bulk-copy path: 16-B rows and every gathered item fits one shared-memory stage (checked
   // again per program against its geometry in launch_program)
   P.use_tma = (v16 && c->use_tma && P.row16 <= kTmaOperandBytes) ? 1 : 0;
@@ -1079,6 +1084,7 @@ dgcl_status dgcl_device_barrier(dgcl_ctx *c, void *stream) {
   for (int r = 0; r < c->world; ++r) P.flags[r] = (uint64_t *)(c->base[r] + c->off_flags[r]);
   P.world = c->world;
   P.seq = ++c->barrier_seq;
+  P.sys_scope = c->loopback ? 0 : 1;
   P.timeout_ns = (uint64_t)c->timeout_ms * 1000000ull;
   P.err = c->err_dev;
   // a fused loopback context is one launch stream: its virtual ranks arrive together
@@ -1131,6 +1137,7 @@ dgcl_status dgcl_stream_wait_arrival(dgcl_ctx *c, int32_t dst, int32_t src, void
   P.epoch[DIR_FWD] = c->epoch[DIR_FWD];
   P.timeout_ns = (uint64_t)c->timeout_ms * 1000000ull;
   P.err = c->err_dev;
+  P.sys_scope = c->loopback ? 0 : 1;
   const int e = launch_wait(P, dst, off, n, stream);
   if (e != 0) return fail(c, DGCL_ECUDA, "wait launch failed: %s", cudaGetErrorString((cudaError_t)e));
   return DGCL_OK;
@@ -1246,6 +1253,15 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->registered) return fail(c, DGCL_ESTATE, "geometry must be set before registration");
     c->geometry = (int)value;
     if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "sys_scope") {  // loopback: 1 = the multi-GPU system-scope flag protocol (A/B)
+    c->force_sys_scope = value != 0;
+    return DGCL_OK;
+  }
+  if (k == "l2_policy") {  // L2 eviction hints, bit mask (executor_tma.cu); any time
+    if (value < 0 || value > 15) return fail(c, DGCL_EINVAL, "l2_policy in 0..15");
+    c->l2_policy = (int)value;
     return DGCL_OK;
   }
   if (k == "sm_budget") {  // SMs per executor launch (0 = all); any time

@@ -23,6 +23,42 @@ __device__ __forceinline__ void st_release_sys(uint64_t *p, uint64_t v) {
 __device__ __forceinline__ void red_release_sys_add(uint64_t *p, uint64_t v) {
   asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+// The flag protocol's scope: system (.sys) when peers are other GPUs (NVLink peer memory, CUDA
+// IPC), device (.gpu) when every rank lives on this GPU (loopback) — ExecParams::sys_scope.  The
+// narrower scope is exact there and makes fences / releases far cheaper (MEMBAR.GPU vs .SYS).
+__device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint64_t *p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_release_gpu_add(uint64_t *p, uint64_t v) {
+  asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t *p, int sys) {
+  return sys ? ld_acquire_sys(p) : ld_acquire_gpu(p);
+}
+__device__ __forceinline__ void st_release(uint64_t *p, uint64_t v, int sys) {
+  if (sys)
+    st_release_sys(p, v);
+  else
+    st_release_gpu(p, v);
+}
+__device__ __forceinline__ void red_release_add(uint64_t *p, uint64_t v, int sys) {
+  if (sys)
+    red_release_sys_add(p, v);
+  else
+    red_release_gpu_add(p, v);
+}
+// this thread's earlier stores are visible at the protocol's scope before its later ones
+__device__ __forceinline__ void fence_scope(int sys) {
+  if (sys)
+    __threadfence_system();
+  else
+    __threadfence();
+}
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -135,11 +171,11 @@ __device__ __forceinline__ float4 fold_tree(float4 init, const uint32_t *prog, i
 // Spin until *p >= target (acquire, system scope), bounded by the watchdog.
 static __device__ __noinline__ bool wait_geq(const uint64_t *p, uint64_t target, const ExecParams &P,
                                       int code) {
-  if (ld_acquire_sys(p) >= target) return true;
+  if (ld_acquire(p, P.sys_scope) >= target) return true;
   const uint64_t t0 = globaltimer();
   for (uint32_t it = 1;; ++it) {
     __nanosleep(64);
-    if (ld_acquire_sys(p) >= target) return true;
+    if (ld_acquire(p, P.sys_scope) >= target) return true;
     if ((it & 255) == 0) {
       if (*(volatile int *)P.err != 0) return false;  // another CTA / peer already failed
       if (globaltimer() - t0 > P.timeout_ns) {
@@ -172,8 +208,8 @@ __device__ __forceinline__ int64_t row_of(const int32_t *idx, int64_t base, int6
 }
 
 // receiver-visible completion of an item: every thread's stores, then one counter add
-__device__ __forceinline__ void release_rows(uint64_t *ctr, uint64_t rows, bool leader) {
-  if (leader) red_release_sys_add(ctr, rows);
+__device__ __forceinline__ void release_rows(uint64_t *ctr, uint64_t rows, bool leader, int sys) {
+  if (leader) red_release_add(ctr, rows, sys);
 }
 
 }  // namespace dev

@@ -294,10 +294,11 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
   if (threadIdx.x < kMaxRanks) s_wait_ok[threadIdx.x] = -1;
   if (threadIdx.x == 0) s_ready_ok = 0, s_npend = 0;
   auto flush = [&]() {  // all threads: publish the pending done counts
-    __threadfence_system();  // this thread's row stores are visible system-wide ...
+    fence_scope(P.sys_scope);  // this thread's row stores are visible (peers: system-wide) ...
     __syncthreads();         // ... for every thread of the CTA ...
     if (threadIdx.x == 0) {  // ... before a receiver can observe the counts
-      for (int i = 0; i < s_npend; ++i) release_rows(s_pend_ctr[i], s_pend_rows[i], true);
+      for (int i = 0; i < s_npend; ++i)
+        release_rows(s_pend_ctr[i], s_pend_rows[i], true, P.sys_scope);
       s_npend = 0;
     }
     __syncthreads();
@@ -332,7 +333,7 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
       if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer
         for (int s = 0; s < P.world; ++s)
-          if (s != I.exec_rank) st_release_sys(P.flags[s] + kReadyBase + I.exec_rank, P.seq);
+          if (s != I.exec_rank) st_release(P.flags[s] + kReadyBase + I.exec_rank, P.seq, P.sys_scope);
       }
       if (P.use_ready && I.ready_rank >= 0 && !((s_ready_ok >> I.ready_rank) & 1u)) {
         ok = wait_geq(P.flags[I.exec_rank] + kReadyBase + I.ready_rank, P.seq, P,
@@ -381,10 +382,11 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
       if (threadIdx.x == 0) P.trace[it].t_done = globaltimer();
     }
     if ((I.flags & kItemSignal) && I.op == OP_FANOUT) {
-      __threadfence_system();
+      fence_scope(P.sys_scope);
       __syncthreads();
       if (threadIdx.x < (unsigned)P.world && s_cnt[threadIdx.x]) {
-        release_rows(P.flags[threadIdx.x] + I.sig_ctr, (uint64_t)s_cnt[threadIdx.x], true);
+        release_rows(P.flags[threadIdx.x] + I.sig_ctr, (uint64_t)s_cnt[threadIdx.x], true,
+                     P.sys_scope);
         s_cnt[threadIdx.x] = 0;
       }
     } else if ((I.flags & kItemSignal) && threadIdx.x == 0) {  // deferred (see kPendMax)
@@ -407,7 +409,7 @@ __global__ void barrier_kernel(const __grid_constant__ ExecParams P, int first, 
   const int r = first + (int)threadIdx.x;
   if ((int)threadIdx.x >= count) return;
   for (int s = 0; s < P.world; ++s)
-    if (s != r) st_release_sys(P.flags[s] + kBarrierBase + r, P.seq);
+    if (s != r) st_release(P.flags[s] + kBarrierBase + r, P.seq, P.sys_scope);
   for (int s = 0; s < P.world; ++s)
     if (s != r && !wait_geq(P.flags[r] + kBarrierBase + s, P.seq, P, 3000000 + s)) return;
 }

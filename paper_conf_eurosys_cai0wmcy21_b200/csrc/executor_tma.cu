@@ -92,6 +92,36 @@ __device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t 
       "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+// L2 eviction priority hints (option "l2_policy", ExecParams::l2_policy): a 64-bit cache policy
+// made once per thread by createpolicy, attached to the data bulk copies / stores
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void bulk_g2s_h(void *sdst, const void *gsrc, uint32_t bytes,
+                                           uint64_t *bar, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1], %2, [%3], %4;" ::"r"(smem_u32(sdst)),
+      "l"(gsrc), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_s2g_h(void *gdst, const void *ssrc, uint32_t bytes,
+                                           uint64_t pol) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(
+                   gdst),
+               "r"(smem_u32(ssrc)), "r"(bytes), "l"(pol)
+               : "memory");
+}
+// data movement with an optional policy (pol == 0: no hint)
+__device__ __forceinline__ void g2s(void *sdst, const void *gsrc, uint32_t bytes, uint64_t *bar,
+                                    uint64_t pol);
 __device__ __forceinline__ void bulk_s2g(void *gdst, const void *ssrc, uint32_t bytes) {
   asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst),
                "r"(smem_u32(ssrc)), "r"(bytes)
@@ -103,6 +133,19 @@ __device__ __forceinline__ void bulk_s2g_add_f32(void *gdst, const void *ssrc, u
                    gdst),
                "r"(smem_u32(ssrc)), "r"(bytes)
                : "memory");
+}
+__device__ __forceinline__ void g2s(void *sdst, const void *gsrc, uint32_t bytes, uint64_t *bar,
+                                    uint64_t pol) {
+  if (pol)
+    bulk_g2s_h(sdst, gsrc, bytes, bar, pol);
+  else
+    bulk_g2s(sdst, gsrc, bytes, bar);
+}
+__device__ __forceinline__ void s2g(void *gdst, const void *ssrc, uint32_t bytes, uint64_t pol) {
+  if (pol)
+    bulk_s2g_h(gdst, ssrc, bytes, pol);
+  else
+    bulk_s2g(gdst, ssrc, bytes);
 }
 __device__ __forceinline__ void bulk_commit() {
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
@@ -149,7 +192,7 @@ __device__ __forceinline__ void consumer_barrier(unsigned *count, volatile unsig
 __device__ __forceinline__ bool waits_ready(const ExecParams &P, const DevItem &I) {
   for (int w = 0; w < I.wait_n; ++w) {
     const DevWait W = P.waits[I.wait_off + w];
-    if (ld_acquire_sys(P.flags[I.exec_rank] + W.ctr) < P.epoch[I.dir] * (uint64_t)W.amount)
+    if (ld_acquire(P.flags[I.exec_rank] + W.ctr, P.sys_scope) < P.epoch[I.dir] * (uint64_t)W.amount)
       return false;
   }
   return true;
@@ -178,7 +221,16 @@ __device__ __forceinline__ bool uses_gather4(const ExecParams &P, const DevItem 
 }
 
 __device__ __forceinline__ void tma_gather4(void *sdst, const void *tmap, int32_t col, int32_t r0,
-                                            int32_t r1, int32_t r2, int32_t r3, uint64_t *bar) {
+                                            int32_t r1, int32_t r2, int32_t r3, uint64_t *bar,
+                                            uint64_t pol = 0) {
+  if (pol) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
+        ".L2::cache_hint [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(sdst)),
+        "l"(tmap), "r"(col), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(bar)), "l"(pol)
+        : "memory");
+    return;
+  }
   asm volatile(
       "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
       " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(sdst)),
@@ -241,7 +293,8 @@ __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const Dev
 // stage to be free and fenced the consumers' generic reads of it against the async proxy.
 __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I,
                                            const DevItem *Ism, uint8_t *st, const uint8_t *meta,
-                                           uint64_t *full, int lane, uint32_t item_index) {
+                                           uint64_t *full, int lane, uint32_t item_index,
+                                           uint64_t pol_copy, uint64_t pol_fold) {
   const uint32_t r16 = (uint32_t)P.row16;
   // consumer tables: term_ptr window (FOLD) and destination rows (when not consecutive)
   Win wtp = {0, 0, 0}, wdst = {0, 0, 0};
@@ -266,10 +319,10 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     // consecutive source rows: one bulk copy (packed rows), then the destination words
     const BufRef S = P.buf[I.src_kind][I.exec_rank];
     if (S.pitch == (int64_t)r16) {
-      if (lane == 0) bulk_g2s(ops, S.ptr + I.src * S.pitch, (uint32_t)I.rows * r16, full);
+      if (lane == 0) g2s(ops, S.ptr + I.src * S.pitch, (uint32_t)I.rows * r16, full, pol_copy);
     } else {
       for (int r = lane; r < I.rows; r += 32)
-        bulk_g2s(ops + (size_t)r * r16, S.ptr + (I.src + r) * S.pitch, r16, full);
+        g2s(ops + (size_t)r * r16, S.ptr + (I.src + r) * S.pitch, r16, full, pol_copy);
     }
     if (lane == 0) {
       const Win wt = window(I.t0, I.nterms, 4);
@@ -295,7 +348,7 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
       const int r = 4 * g, last = I.rows - 1;
       tma_gather4(ops + (size_t)r * r16, tmap, 0, base + sidx[r],
                   base + sidx[min(r + 1, last)], base + sidx[min(r + 2, last)],
-                  base + sidx[min(r + 3, last)], full);
+                  base + sidx[min(r + 3, last)], full, pol_copy);
     }
   } else if (I.op == OP_COPY) {
     // one bulk copy per run of consecutive source rows when rows are packed (pitch == row16)
@@ -305,15 +358,15 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     if (spitch == (int64_t)r16) {
       for (int q = lane; q < I.nterms; q += 32) {
         const DevRun R = runs[q];
-        bulk_g2s(ops + (size_t)R.pos * r16, sbase + (int64_t)R.src * spitch,
-                 (uint32_t)R.len * r16, full);
+        g2s(ops + (size_t)R.pos * r16, sbase + (int64_t)R.src * spitch, (uint32_t)R.len * r16,
+            full, pol_copy);
       }
     } else {
       for (int q = lane; q < I.nterms; q += 32) {
         const DevRun R = runs[q];
         for (int j = 0; j < R.len; ++j)
-          bulk_g2s(ops + (size_t)(R.pos + j) * r16, sbase + (int64_t)(R.src + j) * spitch, r16,
-                   full);
+          g2s(ops + (size_t)(R.pos + j) * r16, sbase + (int64_t)(R.src + j) * spitch, r16, full,
+              pol_copy);
       }
     }
   } else if (is_staged(I)) {
@@ -324,12 +377,12 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
       const DevRun R = segs[q];
       const BufRef B = P.buf[R.dst >> 8][R.dst & 255];
       if (B.pitch == (int64_t)r16) {
-        bulk_g2s(ops + (size_t)R.pos * r16, B.ptr + (int64_t)R.src * B.pitch,
-                 (uint32_t)R.len * r16, full);
+        g2s(ops + (size_t)R.pos * r16, B.ptr + (int64_t)R.src * B.pitch, (uint32_t)R.len * r16,
+            full, pol_fold);
       } else {
         for (int j = 0; j < R.len; ++j)
-          bulk_g2s(ops + (size_t)(R.pos + j) * r16, B.ptr + (int64_t)(R.src + j) * B.pitch, r16,
-                   full);
+          g2s(ops + (size_t)(R.pos + j) * r16, B.ptr + (int64_t)(R.src + j) * B.pitch, r16, full,
+              pol_fold);
       }
     }
     if (lane == 0) {
@@ -391,7 +444,7 @@ __device__ __forceinline__ void store_copy(const ExecParams &P, const DevItem &I
 // next FLUSH / END)
 __device__ __forceinline__ void store_fanout(const ExecParams &P, const DevItem &I,
                                              const uint8_t *st, uint32_t tid, uint32_t T,
-                                             uint32_t *s_pend) {
+                                             uint32_t *s_pend, uint64_t pol_st) {
   const uint32_t r16 = (uint32_t)P.row16;
   const uint8_t *ops = st + kStageHdrBytes;
   const uint32_t *pw = reinterpret_cast<const uint32_t *>(ops + (size_t)I.rows * r16) +
@@ -407,7 +460,7 @@ __device__ __forceinline__ void store_fanout(const ExecParams &P, const DevItem 
     for (uint32_t j = tid; j < np; j += T) {
       const uint32_t d = pw[2 * j], r = pw[2 * j + 1] - src0;
       const BufRef D = P.buf[(d & kFanRelay) ? K_RELAY : K_HALO][d >> 28];
-      bulk_s2g(D.ptr + (int64_t)(d & kFanRowMask) * D.pitch, ops + r * r16, r16);
+      s2g(D.ptr + (int64_t)(d & kFanRowMask) * D.pitch, ops + r * r16, r16, pol_st);
       if (sig) atomicAdd(&s_pend[I.exec_rank * kMaxRanks + (d >> 28)], 1u);
     }
     if (tid < np) {
@@ -788,6 +841,13 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   int32_t *s_wait_ok = reinterpret_cast<int32_t *>(dsmem + kPendOff + 1040);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
+  // L2 hints (option "l2_policy"): bit 0 data stores evict_first (write-once halo / relay /
+  // slot rows), bit 1 COPY / FANOUT source reads evict_last (a row sent to several receivers is
+  // read again soon), bit 2 COPY source reads evict_first, bit 3 FOLD operand reads evict_first
+  const int lp = P.l2_policy;
+  const uint64_t pol_st = (lp & 1) ? policy_evict_first() : 0;
+  const uint64_t pol_copy = (lp & 2) ? policy_evict_last() : (lp & 4) ? policy_evict_first() : 0;
+  const uint64_t pol_fold = (lp & 8) ? policy_evict_first() : 0;
   for (int i = threadIdx.x; i < kMaxRanks * kMaxRanks; i += blockDim.x) s_pend[i] = 0;
   if (threadIdx.x == 0) {
     s_pend_base = 0;
@@ -868,7 +928,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         // my buffers of every layer are free for this call: tell every peer
         if (lane == 0)
           for (int s = 0; s < P.world; ++s)
-            if (s != I.exec_rank) st_release_sys(P.flags[s] + kReadyBase + I.exec_rank, P.seq);
+            if (s != I.exec_rank)
+              st_release(P.flags[s] + kReadyBase + I.exec_rank, P.seq, P.sys_scope);
       } else if (I.op == OP_WAIT) {
         // forward completion: the launch ends only once every incoming row landed
         if (pend) {
@@ -889,11 +950,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           if (lane == 0) {
             ready = known_sources(I) || waits_ready(P, I) ? 1 : 0;
             if (ready && P.use_ready && I.ready_rank >= 0 && !((ready_ok >> I.ready_rank) & 1u))
-              ready = ld_acquire_sys(P.flags[I.exec_rank] + kReadyBase + I.ready_rank) >= P.seq;
+              ready = ld_acquire(P.flags[I.exec_rank] + kReadyBase + I.ready_rank, P.sys_scope) >=
+                      P.seq;
             if (ready && P.use_ready && I.ready_rank == kReadyAll)
               for (int s = 0; s < P.world && ready; ++s)
                 if (s != I.exec_rank && !((ready_ok >> s) & 1u))
-                  ready = ld_acquire_sys(P.flags[I.exec_rank] + kReadyBase + s) >= P.seq;
+                  ready = ld_acquire(P.flags[I.exec_rank] + kReadyBase + s, P.sys_scope) >= P.seq;
           }
           ready = __shfl_sync(0xffffffffu, ready, 0);
           if (!ready || (sig && key != pend_key)) {
@@ -931,7 +993,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         fence_proxy_async_smem();
         fenced = true;
         issue_item(P, I, Ism, stages + (size_t)stage * stage_bytes, meta_of(m), &full[stage],
-                   lane, gidx);
+                   lane, gidx, pol_copy, pol_fold);
         ++k;
         if (sig) {
           pend = true;
@@ -976,14 +1038,14 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           bulk_wait_all();
           fence_proxy_async_global();
         }
-        __threadfence_system();
+        fence_scope(P.sys_scope);
         consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
         // (strided: there are fewer consumer threads than (source, receiver) entries)
         for (uint32_t i = tid; i < (uint32_t)(kMaxRanks * kMaxRanks); i += T) {
           const uint32_t amt = s_pend[i];
           if (amt) {
             const int ex = (int)(i / kMaxRanks), dst = (int)(i % kMaxRanks);
-            red_release_sys_add(P.flags[dst] + s_pend_base + ex, amt);
+            red_release_add(P.flags[dst] + s_pend_base + ex, amt, P.sys_scope);
             s_pend[i] = 0;
           }
         }
@@ -1010,8 +1072,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
             const int64_t lo = (int64_t)I.rows * j / split;
             const int64_t hi = (int64_t)I.rows * (j + 1) / split;
             if (hi > lo) {
-              bulk_s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
-                       (uint32_t)((hi - lo) * P.row16));
+              s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
+                  (uint32_t)((hi - lo) * P.row16), pol_st);
               bulk_commit();
               bulk_wait_read();  // the stage may be reused once the bulk store has read it
             }
@@ -1020,7 +1082,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           store_copy(P, I, st, tid, T);
         }
       } else if ((kMask & kMaskFanout) && I.op == OP_FANOUT) {
-        store_fanout(P, I, st, tid, T, s_pend);
+        store_fanout(P, I, st, tid, T, s_pend, pol_st);
         if ((I.flags & kItemSignal) && tid == 0) s_pend_base = I.sig_ctr - I.exec_rank;
       } else if ((kMask & kMaskDirect) && I.op == OP_COPY) {
         store_copy_direct(P, I, st, tid, T);

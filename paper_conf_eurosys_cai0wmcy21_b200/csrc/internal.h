@@ -193,6 +193,8 @@ struct alignas(64) ExecParams {
   int32_t fold_wide;   // FOLD rows average >= 4 terms (selects the 1024-thread fold instance)
   const uint32_t *sterms;  // staged FOLD items: operand row (in the stage) of every term
   struct TraceRec *trace;  // option "trace": one record per item of this launch, or nullptr
+  int32_t l2_policy;       // option "l2_policy": L2 eviction hints of the bulk-copy executor
+  int32_t sys_scope;       // 1: flags / fences at system scope (peers are other GPUs); 0: .gpu
 };
 
 // Per-item timeline (%globaltimer ns), written when tracing is on: the executor reached the item,
