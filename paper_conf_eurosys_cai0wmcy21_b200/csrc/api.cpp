@@ -46,6 +46,7 @@ struct Program {
   int g4_kinds = 0;        // source kinds of its gather4 items (tensor maps the launch needs)
   bool tree = false;       // carries tree-order FOLD programs (kTermRankTree)
   TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
+  mutable uint64_t claims = 0;  // dynamic item claiming: claims consumed by earlier launches
 };
 
 }  // namespace
@@ -87,6 +88,8 @@ struct dgcl_ctx {
   DevItem *d_items = nullptr;
   DevRun *d_runs = nullptr;
   uint32_t *d_sterms = nullptr;
+  uint64_t *d_claims = nullptr;  // one item-claim counter per program (dynamic claiming)
+  bool dynamic_items = true;     // bulk-copy executor: dynamic item claiming (option)
   int64_t run_bytes = 0;
   bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
   bool bulk_store_peer = false;   // TMA stores into peer memory over NVLink (not yet validated)
@@ -653,6 +656,11 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     }
     encode_g4(Pp, pg.g4_kinds);
     const int grid = (int)std::min<int64_t>(std::max(1, grid_all / grid_div), Pp.n_items);
+    if (Pp.use_tma && c->dynamic_items && c->d_claims) {
+      Pp.claim = c->d_claims + (&pg - c->progs.data());
+      Pp.claim_base = pg.claims;
+      pg.claims += (uint64_t)Pp.n_items + (uint64_t)grid;
+    }
     return launch_executor(Pp, grid, block, st);
   };
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
@@ -849,6 +857,7 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   if ((s = upload(c, &c->d_items, all)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_runs, all_runs)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_sterms, all_sterms)) != DGCL_OK) return s;
+  if ((s = upload(c, &c->d_claims, std::vector<uint64_t>(c->progs.size(), 0))) != DGCL_OK) return s;
   c->run_bytes = (int64_t)(all_runs.size() * sizeof(DevRun) + all_sterms.size() * 4);
   if (c->trace)
     for (Program &p : c->progs)
@@ -1255,6 +1264,10 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }
+  if (k == "dynamic_items") {  // bulk-copy executor: 1 dynamic item claiming, 0 round-robin
+    c->dynamic_items = value != 0;
+    return DGCL_OK;
+  }
   if (k == "sys_scope") {  // loopback: 1 = the multi-GPU system-scope flag protocol (A/B)
     c->force_sys_scope = value != 0;
     return DGCL_OK;
@@ -1454,6 +1467,7 @@ dgcl_status dgcl_destroy(dgcl_ctx *c) {
     cudaFree(c->d_items);
     cudaFree(c->d_runs);
     cudaFree(c->d_sterms);
+    cudaFree(c->d_claims);
     for (Program &p : c->progs)
       if (p.d_trace) cudaFree(p.d_trace);
     for (auto &kv : c->stages) {

@@ -839,6 +839,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   // monotonic and their targets fixed for the launch, so it stays satisfied: later items of the
   // same (direction, stage, rank) skip the flag reads)
   int32_t *s_wait_ok = reinterpret_cast<int32_t *>(dsmem + kPendOff + 1040);
+  // producer-private: the launch index of the item in each descriptor ring slot
+  uint32_t *s_claim = reinterpret_cast<uint32_t *>(dsmem + kPendOff + 1104);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
   // L2 hints (option "l2_policy"): bit 0 data stores evict_first (write-once halo / relay /
@@ -869,13 +871,43 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     // item q of this CTA is P.items[blockIdx.x + q * gridDim.x]; its descriptor is bulk-copied
     // into ring slot q % kDescSlots kDescAhead items ahead, its row runs into meta slot
     // q % kMetaSlots kMetaAhead items ahead, so their latency never stalls the issue loop
+    // Items are claimed in list order: statically (item q of this CTA = blockIdx.x + q * G) or,
+    // with P.claim, dynamically from a launch-wide counter (claims hand out list positions in
+    // increasing order, so every CTA's queue stays in list (stage) order and the earliest
+    // unfinished item can always run: deadlock-free like the static order, and no CTA idles
+    // while another still holds a backlog — items cost very different times when their row
+    // runs differ).  nend = the first queue position without an item (known once a claim fails).
     const uint32_t G = gridDim.x;
-    const uint32_t nmine =
-        blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
-    auto request_desc = [&](uint32_t q) {  // lane 0, after a proxy fence
+    uint32_t nend = 0xffffffffu, nreq = 0;
+    if (!P.claim)
+      nend = blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
+    auto request_desc = [&](uint32_t q) -> bool {  // lane 0, after a proxy fence
+      uint64_t idx;
+      if (P.claim) {
+        idx = atomicAdd(reinterpret_cast<unsigned long long *>(P.claim), 1ull) - P.claim_base;
+        if (idx >= (uint64_t)P.n_items) return false;
+      } else {
+        idx = blockIdx.x + (uint64_t)q * G;
+      }
       const uint32_t s = q % kDescSlots;
+      s_claim[s] = (uint32_t)idx;
       mbar_expect_tx(&descb[s], (uint32_t)sizeof(DevItem));
-      bulk_g2s(descs + s, P.items + blockIdx.x + q * G, (uint32_t)sizeof(DevItem), &descb[s]);
+      bulk_g2s(descs + s, P.items + idx, (uint32_t)sizeof(DevItem), &descb[s]);
+      return true;
+    };
+    // request descriptors nreq .. upto-1 (fewer once the items run out); warp-uniform
+    auto request_upto = [&](uint32_t upto) {
+      int e = -1;
+      if (lane == 0)
+        for (uint32_t q = nreq; q < upto && q < nend; ++q)
+          if (!request_desc(q)) {
+            e = (int)q;
+            break;
+          }
+      e = __shfl_sync(0xffffffffu, e, 0);
+      if (e >= 0) nend = (uint32_t)e;
+      nreq = upto < nend ? upto : nend;
+      __syncwarp();
     };
     auto desc_ready = [&](uint32_t q) -> const DevItem & {
       mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
@@ -906,17 +938,16 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     // consumers, ordered by the empty barrier) the stage come before every bulk copy into them.
     // Prefetches are issued after the item, so the item's fence covers them too.
     fence_proxy_async_smem();
-    if (lane == 0)
-      for (uint32_t q = 0; q < (uint32_t)kDescAhead && q < nmine; ++q) request_desc(q);
-    for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nmine; ++q) {
+    request_upto((uint32_t)kDescAhead);
+    for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nend; ++q) {
       const DevItem Iq = desc_ready(q);
       if (lane == 0) issue_meta(P, Iq, meta_of(q), &metab[q % kMetaSlots]);
     }
-    for (; m < nmine; ++m) {
+    for (; m < nend; ++m) {
       const DevItem I = desc_ready(m);  // registers: no shared-memory reload per field
       const DevItem *Ism = &descs[m % kDescSlots];
       bool fenced = false;
-      const uint32_t gidx = blockIdx.x + m * G;  // the item's index in the launch
+      const uint32_t gidx = s_claim[m % kDescSlots];  // the item's index in the launch
       if (P.trace && lane == 0) {
         uint32_t smid;
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
@@ -1002,9 +1033,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       }
       __syncwarp();
       // prefetch: descriptor kDescAhead items ahead, row runs / segments kMetaAhead items ahead
-      if (!fenced && (m + kMetaAhead < nmine)) fence_proxy_async_smem();
-      if (lane == 0 && m + kDescAhead < nmine) request_desc(m + kDescAhead);
-      if (m + kMetaAhead < nmine) {
+      if (!fenced && (m + kMetaAhead < nend || m + kDescAhead < nend)) fence_proxy_async_smem();
+      if (m + kDescAhead < nend) request_upto(m + kDescAhead + 1);
+      if (m + kMetaAhead < nend) {
         const uint32_t q = m + kMetaAhead;
         const DevItem In = desc_ready(q);
         if (lane == 0) issue_meta(P, In, meta_of(q), &metab[q % kMetaSlots]);
@@ -1014,9 +1045,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       // watchdog abort: descriptor / metadata copies still in flight land before the CTA leaves
       // (item m aborted before its own prefetches: requested so far are descriptors < m +
       // kDescAhead and metadata < m + kMetaAhead)
-      for (uint32_t q = m; q < m + kDescAhead && q < nmine; ++q)
+      for (uint32_t q = m; q < nreq; ++q)
         mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
-      for (uint32_t q = m; q < m + kMetaAhead && q < nmine; ++q)
+      for (uint32_t q = m; q < m + kMetaAhead && q < nend; ++q)
         mbar_wait(&metab[q % kMetaSlots], (q / kMetaSlots) & 1u);
     }
     // END marker: consumers drain every issued stage, publish pending counts, then stop

@@ -195,6 +195,11 @@ struct alignas(64) ExecParams {
   struct TraceRec *trace;  // option "trace": one record per item of this launch, or nullptr
   int32_t l2_policy;       // option "l2_policy": L2 eviction hints of the bulk-copy executor
   int32_t sys_scope;       // 1: flags / fences at system scope (peers are other GPUs); 0: .gpu
+  // bulk-copy executor, dynamic item claiming: a launch-wide counter (nullptr = static
+  // round-robin).  Every CTA claims until one claim fails, so a launch consumes exactly
+  // n_items + grid claims; claim_base = the counter's value at launch (kept by the host)
+  uint64_t *claim;
+  uint64_t claim_base;
 };
 
 // Per-item timeline (%globaltimer ns), written when tracing is on: the executor reached the item,
