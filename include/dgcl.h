@@ -77,6 +77,7 @@ typedef struct {
   double lowering_seconds;
   int32_t n_fwd_groups;        /* (stage, src, dst, buffer-kind) tuples */
   int32_t n_bwd_groups;
+  int64_t n_multicast_rows;    /* rows sent through the NVSwitch multicast (option "multicast") */
 } dgcl_plan_stats;
 
 /* ---- lifecycle ---------------------------------------------------------------------------- */
@@ -239,6 +240,15 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "direct_copy_rows" COPY items whose runs average fewer rows are gathered by the consumer
  *                    warps with plain loads (default 0 = never)
  *   "trace"          1: record per-item timelines of every launch (dgcl_trace_read); default 0
+ *   "l2_policy"      L2 eviction hints of the bulk-copy executor, bit mask (any time): 1 data stores
+ *                    evict_first (default), 2 COPY source reads evict_last, 4 COPY source reads
+ *                    evict_first, 8 FOLD operand reads evict_first
+ *   "item_order"     bulk-copy executor item assignment (any time): 0 round-robin, 1 dynamic
+ *                    claiming from a launch-wide counter, 2 rotated rounds (default)
+ *   "sys_scope"      loopback contexts: 1 = use the multi-GPU system-scope flag protocol (A/B;
+ *                    default 0: device scope, exact when every rank is on this GPU)
+ *   "multicast"      NVSwitch multicast of high-fan-out rows (see dgcl_multicast_open): 0 off
+ *                    (default), 1 rows every peer requested, k >= 2 rows >= k GPUs requested
  *   "sm_budget"      SMs one executor launch may use (default 0 = all; any time): leaves SMs free
  *                    for kernels that overlap the exchange (dgcl_stream_wait_arrival)
  *   "signal_all"     fused loopback: every item publishes its done count, so arrival waits work
@@ -295,6 +305,36 @@ dgcl_status dgcl_device_barrier(dgcl_ctx *ctx, void *stream);
  * for a bad (dst, src), ESTATE before registration / without signal_all; a row that never
  * arrives trips the watchdog (dgcl_check -> DGCL_ETIMEOUT).  No forward call yet: no-op. */
 dgcl_status dgcl_stream_wait_arrival(dgcl_ctx *ctx, int32_t dst, int32_t src, void *stream);
+
+/* ---- NVSwitch multicast (the switch-level form of the paper's
+ * communication fusion, and of "forward to multiple destinations") ----
+ * With option "multicast" (1: rows every peer requested; k >= 2: rows >= k GPUs requested; set
+ * before dgcl_build_plan or re-lowered on set; single-stage plans only) the owner of such a row
+ * stores it ONCE through a multicast address (multimem.st): the NVSwitch replicates the write into
+ * every GPU's copy of a multicast region bound at the same offset (row mc_off[owner] + j), one
+ * multimem reduction bumps the owner's multicast done counter on every GPU, and each requester
+ * copies the row from its own region into its halo row (unpack, local HBM).  Owner egress drops
+ * from |D_u| row copies to one; the ingress bound is unchanged.  The backward keeps the fixed-order
+ * reduce (multimem.ld_reduce has no fixed order).  Setup, after dgcl_ipc_import, collective:
+ *   dgcl_multicast_open  rank 0 creates the object (cuMulticastCreate, POSIX fd handle) and returns
+ *                        *fd; every other rank passes that fd (received over a Unix socket:
+ *                        the Python setup does it) and imports it;
+ *   dgcl_multicast_add   every rank adds its device;    -- barrier --
+ *   dgcl_multicast_bind  every rank binds its memory and maps the unicast + multicast views.
+ * Loopback contexts emulate the multicast (one store per virtual rank's region copy, in the
+ * workspace).  Errors: ECUDA when the device has no multicast support (probe with
+ * dgcl_multicast_supported) or a driver call fails; ESTATE on a wrong order; dispatch refuses a
+ * multi-GPU context whose plan multicasts before dgcl_multicast_bind. */
+dgcl_status dgcl_multicast_supported(int32_t cuda_device, int32_t *supported);
+dgcl_status dgcl_multicast_bytes(dgcl_ctx *ctx, size_t *bytes, int64_t *rows);
+dgcl_status dgcl_multicast_open(dgcl_ctx *ctx, int32_t *fd);
+dgcl_status dgcl_multicast_add(dgcl_ctx *ctx);
+dgcl_status dgcl_multicast_bind(dgcl_ctx *ctx);
+/* Verification aid: a one-device multicast object on `cuda_device` (bytes of region), stores and
+ * a reduction through the multicast address, checked through the unicast view.  Writes a one-line
+ * result into msg.  DGCL_ECUDA if unsupported. */
+dgcl_status dgcl_debug_multicast_selftest(int32_t cuda_device, int64_t bytes, char *msg,
+                                          size_t msg_len);
 
 /* Number of executor kernel launches issued so far by this context. */
 dgcl_status dgcl_launch_count(dgcl_ctx *ctx, uint64_t *count);

@@ -23,7 +23,9 @@ SYMBOLS = [
     "dgcl_ipc_export", "dgcl_ipc_import", "dgcl_dispatch_forward", "dgcl_dispatch_backward",
     "dgcl_forward_host", "dgcl_backward_host", "dgcl_plan_info", "dgcl_plan_counts",
     "dgcl_plan_export", "dgcl_set_option", "dgcl_trace_read", "dgcl_device_barrier",
-    "dgcl_stream_wait_arrival",
+    "dgcl_stream_wait_arrival", "dgcl_multicast_supported", "dgcl_multicast_bytes",
+    "dgcl_multicast_open", "dgcl_multicast_add", "dgcl_multicast_bind",
+    "dgcl_debug_multicast_selftest",
     "dgcl_launch_count", "dgcl_check",
     "dgcl_last_error",
     "dgcl_strerror", "dgcl_destroy", "dgcl_debug_hostsim_forward", "dgcl_debug_hostsim_backward",
@@ -47,7 +49,8 @@ class PlanStats(ctypes.Structure):
                 ("n_tree_edges", ctypes.c_int64), ("n_relay_rows", ctypes.c_int64),
                 ("model_cost_ticks", ctypes.c_int64), ("table_bytes", ctypes.c_int64),
                 ("planner_seconds", ctypes.c_double), ("lowering_seconds", ctypes.c_double),
-                ("n_fwd_groups", ctypes.c_int32), ("n_bwd_groups", ctypes.c_int32)]
+                ("n_fwd_groups", ctypes.c_int32), ("n_bwd_groups", ctypes.c_int32),
+                ("n_multicast_rows", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -89,6 +92,12 @@ def lib():
             "dgcl_trace_read": [P, I32, I32, I32, P, ctypes.POINTER(I64)],
             "dgcl_device_barrier": [P, P],
             "dgcl_stream_wait_arrival": [P, I32, I32, P],
+            "dgcl_multicast_supported": [I32, ctypes.POINTER(I32)],
+            "dgcl_multicast_bytes": [P, ctypes.POINTER(SZ), ctypes.POINTER(I64)],
+            "dgcl_multicast_open": [P, ctypes.POINTER(I32)],
+            "dgcl_multicast_add": [P],
+            "dgcl_multicast_bind": [P],
+            "dgcl_debug_multicast_selftest": [I32, I64, ctypes.c_char_p, SZ],
             "dgcl_launch_count": [P, ctypes.POINTER(U64)],
             "dgcl_check": [P],
             "dgcl_destroy": [P],

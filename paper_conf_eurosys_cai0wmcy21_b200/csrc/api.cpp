@@ -89,7 +89,7 @@ struct dgcl_ctx {
   DevRun *d_runs = nullptr;
   uint32_t *d_sterms = nullptr;
   uint64_t *d_claims = nullptr;  // one item-claim counter per program (dynamic claiming)
-  bool dynamic_items = true;     // bulk-copy executor: dynamic item claiming (option)
+  int item_order = 2;  // bulk-copy executor: 0 round-robin, 1 dynamic claiming, 2 rotated rounds
   int64_t run_bytes = 0;
   bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
   bool bulk_store_peer = false;   // TMA stores into peer memory over NVLink (not yet validated)
@@ -98,6 +98,17 @@ struct dgcl_ctx {
   bool direct_reduce = true;          // fused loopback + single-stage plan: in-place reduce
   bool atomic_backward = false;       // ablation: loopback backward with atomic adds
   bool fanout = false;                // forward stage 1 as per-owner fan-out items (option)
+  // NVSwitch multicast (option "multicast": 0 off, 1 rows requested by every peer, k >= 2 rows
+  // requested by >= k GPUs).  Multi-GPU: a multicast object over every rank's device with this
+  // region bound at the same offset; loopback: emulated (one copy per virtual rank, workspace)
+  int multicast = 0;
+  std::vector<size_t> off_mc;   // loopback: each virtual rank's region copy in the workspace
+  std::vector<size_t> mc_layer_off;  // byte offset of each layer's rows in the region
+  size_t mc_bytes = 0;          // region bytes (flag page + every layer's rows)
+  CUmemGenericAllocationHandle mc_handle = 0, mc_mem = 0;  // multicast object, bound memory
+  bool mc_have_handle = false, mc_have_mem = false, mc_added = false;
+  char *mc_va = nullptr, *mc_uc = nullptr;  // multicast / unicast mappings of the region
+  size_t mc_map_bytes = 0;      // granularity-rounded size of the mappings
   bool align_sources = true;          // forward COPY items of one source rank cut at common rows
   int pipeline_blocks = 1;            // relay plans: vertex blocks of the stage chaining
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
@@ -108,7 +119,8 @@ struct dgcl_ctx {
   int sm_budget = 0;                  // SMs an executor launch may use (0 = all): the rest stay
                                       // free for kernels overlapping the exchange (NEXT-2)
   bool signal_all = false;            // fused loopback: publish every done count (arrival waits)
-  int l2_policy = 0;                  // L2 eviction hints (executor_tma.cu), A/B option
+  int l2_policy = 1;                  // L2 eviction hints (executor_tma.cu): stores evict_first
+                                      // (Com-Orkut forward 1.69 -> 1.63 ms, others neutral)
   bool force_sys_scope = false;       // loopback with the multi-GPU (.sys) flag scope (A/B)
   bool threads_set = false, ctas_set = false;  // user overrides of the CTA shape
   int sm_count = 148;  // SMs of the device (B200 until queried), for cutting small stages
@@ -222,9 +234,14 @@ dgcl_status init_common(int32_t rank, int32_t world, int32_t dev, int64_t n, con
 
 bool has_device(dgcl_ctx *c) { return c->device >= 0; }
 
+int mc_min_fanout(const dgcl_ctx *c) {
+  if (c->multicast <= 0 || c->world < 2) return 0;
+  return c->multicast == 1 ? c->world - 1 : c->multicast;
+}
+
 void relower(dgcl_ctx *c) {
   lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low, c->pipeline_blocks,
-             c->atomic_backward, c->fanout);
+             c->atomic_backward, c->fanout && !mc_min_fanout(c), mc_min_fanout(c));
 }
 
 void compute_layout(dgcl_ctx *c) {
@@ -277,15 +294,35 @@ void compute_layout(dgcl_ctx *c) {
       c->ws_need[r] = off;
     }
   }
+  // multicast region: [flag page][layer 0 rows][layer 1 rows] ... (same layout on every rank)
+  c->mc_layer_off.assign(c->n_layers, 0);
+  c->mc_bytes = 0;
+  c->off_mc.assign(m, 0);
+  if (L.mc_total > 0) {
+    size_t o = kMcFlagBytes;
+    for (int l = 0; l < c->n_layers; ++l) {
+      c->mc_layer_off[l] = o;
+      o = align_up(o + (size_t)L.mc_total * c->pitch[l] * 4);
+    }
+    c->mc_bytes = o;
+    if (c->loopback) {  // emulation: every virtual rank's copy after the workspace
+      size_t off = c->ws_need[0];
+      for (int r = 0; r < m; ++r) {
+        c->off_mc[r] = off;
+        off = align_up(off + c->mc_bytes);
+      }
+      for (int r = 0; r < m; ++r) c->ws_need[r] = off;
+    }
+  }
 }
 
 // counters some group of the given program waits on (fused loopback: only those need a signal)
 std::vector<uint8_t> needed_counters(const Lowered &L, const std::vector<int32_t> &gids) {
-  std::vector<uint8_t> need((size_t)kMaxRanks * kFlagWords, 0);
+  std::vector<uint8_t> need((size_t)kMaxRanks * kCtrSpace, 0);
   for (int32_t gi : gids) {
     const DevGroup &g = L.groups[gi];
     for (int w = 0; w < g.wait_n; ++w)
-      need[(size_t)g.exec_rank * kFlagWords + L.waits[g.wait_off + w].ctr] = 1;
+      need[(size_t)g.exec_rank * kCtrSpace + L.waits[g.wait_off + w].ctr] = 1;
   }
   return need;
 }
@@ -491,6 +528,127 @@ dgcl_status check_dead(dgcl_ctx *c) {
 
 inline bool al16(const void *p) { return ((uintptr_t)p & 15) == 0; }
 
+// CUDA driver entry points, resolved through the runtime (libdgcl does not link libcuda)
+template <typename F>
+F drv(const char *name) {
+  void *p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess ||
+      q != cudaDriverEntryPointSuccess)
+    return nullptr;
+  return (F)p;
+}
+
+// ---- NVSwitch multicast objects (cuMulticast*): the driver calls behind dgcl_multicast_* ----
+struct McDriver {
+  CUresult (*getAttr)(int *, CUdevice_attribute, CUdevice) = nullptr;
+  CUresult (*gran)(size_t *, const CUmulticastObjectProp *, CUmulticastGranularity_flags) = nullptr;
+  CUresult (*create)(CUmemGenericAllocationHandle *, const CUmulticastObjectProp *) = nullptr;
+  CUresult (*addDevice)(CUmemGenericAllocationHandle, CUdevice) = nullptr;
+  CUresult (*bindMem)(CUmemGenericAllocationHandle, size_t, CUmemGenericAllocationHandle, size_t,
+                      size_t, unsigned long long) = nullptr;
+  CUresult (*unbind)(CUmemGenericAllocationHandle, CUdevice, size_t, size_t) = nullptr;
+  CUresult (*memCreate)(CUmemGenericAllocationHandle *, size_t, const CUmemAllocationProp *,
+                        unsigned long long) = nullptr;
+  CUresult (*memRelease)(CUmemGenericAllocationHandle) = nullptr;
+  CUresult (*reserve)(CUdeviceptr *, size_t, size_t, CUdeviceptr, unsigned long long) = nullptr;
+  CUresult (*addrFree)(CUdeviceptr, size_t) = nullptr;
+  CUresult (*map)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle,
+                  unsigned long long) = nullptr;
+  CUresult (*unmap)(CUdeviceptr, size_t) = nullptr;
+  CUresult (*setAccess)(CUdeviceptr, size_t, const CUmemAccessDesc *, size_t) = nullptr;
+  CUresult (*exportH)(void *, CUmemGenericAllocationHandle, CUmemAllocationHandleType,
+                      unsigned long long) = nullptr;
+  CUresult (*importH)(CUmemGenericAllocationHandle *, void *, CUmemAllocationHandleType) = nullptr;
+  bool ok = false;
+  McDriver() {
+    getAttr = drv<decltype(getAttr)>("cuDeviceGetAttribute");
+    gran = drv<decltype(gran)>("cuMulticastGetGranularity");
+    create = drv<decltype(create)>("cuMulticastCreate");
+    addDevice = drv<decltype(addDevice)>("cuMulticastAddDevice");
+    bindMem = drv<decltype(bindMem)>("cuMulticastBindMem");
+    unbind = drv<decltype(unbind)>("cuMulticastUnbind");
+    memCreate = drv<decltype(memCreate)>("cuMemCreate");
+    memRelease = drv<decltype(memRelease)>("cuMemRelease");
+    reserve = drv<decltype(reserve)>("cuMemAddressReserve");
+    addrFree = drv<decltype(addrFree)>("cuMemAddressFree");
+    map = drv<decltype(map)>("cuMemMap");
+    unmap = drv<decltype(unmap)>("cuMemUnmap");
+    setAccess = drv<decltype(setAccess)>("cuMemSetAccess");
+    exportH = drv<decltype(exportH)>("cuMemExportToShareableHandle");
+    importH = drv<decltype(importH)>("cuMemImportFromShareableHandle");
+    ok = getAttr && gran && create && addDevice && bindMem && unbind && memCreate && memRelease &&
+         reserve && addrFree && map && unmap && setAccess && exportH && importH;
+  }
+};
+const McDriver &mcd() {
+  static McDriver d;
+  return d;
+}
+
+bool mc_supported(int dev) {
+  const McDriver &D = mcd();
+  int v = 0;
+  return D.ok && D.getAttr(&v, CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED, (CUdevice)dev) == CUDA_SUCCESS &&
+         v != 0;
+}
+
+CUmulticastObjectProp mc_prop(int n_devices, size_t bytes) {
+  CUmulticastObjectProp p;
+  std::memset(&p, 0, sizeof(p));
+  p.numDevices = (unsigned)n_devices;
+  p.size = bytes;
+  p.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+  return p;
+}
+
+// bind `bytes` of new device memory of `dev` to multicast object h at offset 0 and map it twice:
+// unicast (*uc) and through the multicast address (*mc)
+CUresult mc_bind_map(int dev, CUmemGenericAllocationHandle h, size_t bytes,
+                     CUmemGenericAllocationHandle *mem, char **uc, char **mc) {
+  const McDriver &D = mcd();
+  CUmemAllocationProp ap;
+  std::memset(&ap, 0, sizeof(ap));
+  ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  ap.location.id = dev;
+  CUresult r = D.memCreate(mem, bytes, &ap, 0);
+  if (r != CUDA_SUCCESS) return r;
+  if ((r = D.bindMem(h, 0, *mem, 0, bytes, 0)) != CUDA_SUCCESS) return r;
+  CUmemAccessDesc acc;
+  std::memset(&acc, 0, sizeof(acc));
+  acc.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  acc.location.id = dev;
+  acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  CUdeviceptr a = 0, b = 0;
+  if ((r = D.reserve(&a, bytes, 0, 0, 0)) != CUDA_SUCCESS) return r;
+  if ((r = D.map(a, bytes, 0, *mem, 0)) != CUDA_SUCCESS) return r;
+  if ((r = D.setAccess(a, bytes, &acc, 1)) != CUDA_SUCCESS) return r;
+  *uc = (char *)a;
+  if ((r = D.reserve(&b, bytes, 0, 0, 0)) != CUDA_SUCCESS) return r;
+  if ((r = D.map(b, bytes, 0, h, 0)) != CUDA_SUCCESS) return r;
+  if ((r = D.setAccess(b, bytes, &acc, 1)) != CUDA_SUCCESS) return r;
+  *mc = (char *)b;
+  return CUDA_SUCCESS;
+}
+
+void mc_teardown(int dev, CUmemGenericAllocationHandle h, bool have_h, CUmemGenericAllocationHandle mem,
+                 bool have_mem, char *uc, char *mc, size_t bytes) {
+  const McDriver &D = mcd();
+  if (!D.ok) return;
+  if (mc) {
+    D.unmap((CUdeviceptr)mc, bytes);
+    D.addrFree((CUdeviceptr)mc, bytes);
+  }
+  if (uc) {
+    D.unmap((CUdeviceptr)uc, bytes);
+    D.addrFree((CUdeviceptr)uc, bytes);
+  }
+  if (have_h && have_mem) D.unbind(h, (CUdevice)dev, 0, bytes);
+  if (have_mem) D.memRelease(mem);
+  if (have_h) D.memRelease(h);
+}
+
 // 2-D tensor map over `rows` packed rows of row_bytes (<= 1 KB) starting at `base`: box = one row,
 // for cp.async.bulk.tensor ... tile::gather4.  The driver entry point is resolved through the
 // runtime (no libcuda link).  Returns false if the map cannot be built (the launch then uses
@@ -554,6 +712,22 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     P.buf[K_HALO][r] = {b + c->off_halo[layer][r], hp};
     P.buf[K_RELAY][r] = {b + c->off_relay[layer][r], hp};
     P.buf[K_SLOT][r] = {b + c->off_slot[r], hp};
+  }
+  if (dir == DIR_FWD && c->low.mc_total > 0) {
+    const size_t lo = c->mc_layer_off[layer];
+    for (int r = 0; r < m; ++r) {
+      if (c->loopback) {
+        char *b = c->base[r] + c->off_mc[r];
+        P.buf[K_MCUC][r] = {b + lo, hp};
+        P.mcuc_flags[r] = (uint64_t *)b;
+      } else if (r == c->rank) {
+        P.buf[K_MCUC][r] = {c->mc_uc + lo, hp};
+        P.buf[K_MCAST][r] = {c->mc_va + lo, hp};
+        P.mcuc_flags[r] = (uint64_t *)c->mc_uc;
+        P.mc_flags = (uint64_t *)c->mc_va;
+      }
+    }
+    P.mc_emulate = c->loopback ? 1 : 0;
   }
   const int in_kind = dir == DIR_FWD ? K_EMB : K_HGRAD;
   for (int r = 0; r < m; ++r) {
@@ -656,7 +830,8 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     }
     encode_g4(Pp, pg.g4_kinds);
     const int grid = (int)std::min<int64_t>(std::max(1, grid_all / grid_div), Pp.n_items);
-    if (Pp.use_tma && c->dynamic_items && c->d_claims) {
+    Pp.item_order = c->item_order == 2 ? 1 : 0;
+    if (Pp.use_tma && c->item_order == 1 && c->d_claims) {
       Pp.claim = c->d_claims + (&pg - c->progs.data());
       Pp.claim_base = pg.claims;
       pg.claims += (uint64_t)Pp.n_items + (uint64_t)grid;
@@ -701,6 +876,8 @@ dgcl_status ready_to_dispatch(dgcl_ctx *c, int32_t layer) {
   if (!c->loopback && c->world > 1 && !c->imported)
     return fail(c, DGCL_ESTATE, "peers not imported");
   if (layer < 0 || layer >= c->n_layers) return fail(c, DGCL_EINVAL, "bad layer %d", layer);
+  if (!c->loopback && c->low.mc_total > 0 && !c->mc_uc)
+    return fail(c, DGCL_ESTATE, "multicast planned but the region is not bound (dgcl_multicast_bind)");
   return check_dead(c);
 }
 
@@ -825,6 +1002,8 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   // zero every flag region this context owns (monotonic counters start at 0)
   if (c->loopback) {
     CUDA_TRY(c, cudaMemset(c->ws, 0, (size_t)c->world * kFlagBytes));
+    for (int r = 0; r < c->world && c->mc_bytes; ++r)
+      CUDA_TRY(c, cudaMemset(c->ws + c->off_mc[r], 0, kMcFlagBytes));
   } else {
     CUDA_TRY(c, cudaMemset(c->ws, 0, kFlagBytes));
   }
@@ -1103,6 +1282,135 @@ dgcl_status dgcl_device_barrier(dgcl_ctx *c, void *stream) {
   return DGCL_OK;
 }
 
+dgcl_status dgcl_multicast_supported(int32_t cuda_device, int32_t *supported) {
+  if (!supported) return DGCL_EINVAL;
+  *supported = mc_supported(cuda_device) ? 1 : 0;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_multicast_bytes(dgcl_ctx *c, size_t *bytes, int64_t *rows) {
+  if (!c || !bytes) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  *bytes = c->mc_bytes;
+  if (rows) *rows = c->low.mc_total;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_multicast_open(dgcl_ctx *c, int32_t *fd) {
+  if (!c || !fd) return DGCL_EINVAL;
+  if (!c->registered) return fail(c, DGCL_ESTATE, "workspace not registered");
+  if (c->loopback) return fail(c, DGCL_ESTATE, "loopback contexts emulate the multicast");
+  if (c->mc_bytes == 0) return fail(c, DGCL_ESTATE, "no multicast rows planned (option multicast)");
+  if (c->mc_have_handle) return fail(c, DGCL_ESTATE, "multicast object already open");
+  if (!mc_supported(c->device))
+    return fail(c, DGCL_ECUDA, "device %d does not support multicast objects", c->device);
+  DeviceGuard guard(c->device);
+  const McDriver &D = mcd();
+  CUmulticastObjectProp prop = mc_prop(c->world, c->mc_bytes);
+  size_t g = 0;
+  CUresult r = D.gran(&g, &prop, CU_MULTICAST_GRANULARITY_MINIMUM);
+  if (r != CUDA_SUCCESS || g == 0) return fail(c, DGCL_ECUDA, "cuMulticastGetGranularity (%d)", (int)r);
+  c->mc_map_bytes = (c->mc_bytes + g - 1) / g * g;
+  prop.size = c->mc_map_bytes;
+  if (c->rank == 0) {
+    if ((r = D.create(&c->mc_handle, &prop)) != CUDA_SUCCESS)
+      return fail(c, DGCL_ECUDA, "cuMulticastCreate (%d)", (int)r);
+    c->mc_have_handle = true;
+    int out = -1;
+    if ((r = D.exportH(&out, c->mc_handle, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, 0)) != CUDA_SUCCESS)
+      return fail(c, DGCL_ECUDA, "cuMemExportToShareableHandle (%d)", (int)r);
+    *fd = out;
+  } else {
+    if ((r = D.importH(&c->mc_handle, (void *)(intptr_t)*fd, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR)) !=
+        CUDA_SUCCESS)
+      return fail(c, DGCL_ECUDA, "cuMemImportFromShareableHandle (%d)", (int)r);
+    c->mc_have_handle = true;
+  }
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_multicast_add(dgcl_ctx *c) {
+  if (!c) return DGCL_EINVAL;
+  if (!c->mc_have_handle) return fail(c, DGCL_ESTATE, "dgcl_multicast_open first");
+  if (c->mc_added) return fail(c, DGCL_ESTATE, "device already added");
+  DeviceGuard guard(c->device);
+  const CUresult r = mcd().addDevice(c->mc_handle, (CUdevice)c->device);
+  if (r != CUDA_SUCCESS) return fail(c, DGCL_ECUDA, "cuMulticastAddDevice (%d)", (int)r);
+  c->mc_added = true;
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_multicast_bind(dgcl_ctx *c) {
+  if (!c) return DGCL_EINVAL;
+  if (!c->mc_added) return fail(c, DGCL_ESTATE, "dgcl_multicast_add first (on every rank)");
+  if (c->mc_uc) return fail(c, DGCL_ESTATE, "already bound");
+  DeviceGuard guard(c->device);
+  const CUresult r = mc_bind_map(c->device, c->mc_handle, c->mc_map_bytes, &c->mc_mem, &c->mc_uc,
+                                 &c->mc_va);
+  c->mc_have_mem = c->mc_mem != 0;
+  if (r != CUDA_SUCCESS) return fail(c, DGCL_ECUDA, "multicast bind / map (%d)", (int)r);
+  CUDA_TRY(c, cudaMemset(c->mc_uc, 0, kMcFlagBytes));
+  CUDA_TRY(c, cudaDeviceSynchronize());
+  return DGCL_OK;
+}
+
+dgcl_status dgcl_debug_multicast_selftest(int32_t cuda_device, int64_t bytes, char *msg,
+                                          size_t msg_len) {
+  auto say = [&](const char *fmt, int v) {
+    if (msg && msg_len) std::snprintf(msg, msg_len, fmt, v);
+  };
+  if (bytes < 4096) bytes = 4096;
+  if (!mc_supported(cuda_device)) {
+    say("multicast not supported on device %d", cuda_device);
+    return DGCL_ECUDA;
+  }
+  if (cudaSetDevice(cuda_device) != cudaSuccess) return DGCL_ECUDA;
+  const McDriver &D = mcd();
+  CUmulticastObjectProp prop = mc_prop(1, (size_t)bytes);
+  size_t g = 0;
+  CUresult r = D.gran(&g, &prop, CU_MULTICAST_GRANULARITY_MINIMUM);
+  if (r != CUDA_SUCCESS) { say("cuMulticastGetGranularity %d", (int)r); return DGCL_ECUDA; }
+  const size_t sz = ((size_t)bytes + g - 1) / g * g;
+  prop.size = sz;
+  CUmemGenericAllocationHandle h = 0, mem = 0;
+  char *uc = nullptr, *mc = nullptr;
+  dgcl_status st = DGCL_OK;
+  if ((r = D.create(&h, &prop)) != CUDA_SUCCESS) { say("cuMulticastCreate %d", (int)r); return DGCL_ECUDA; }
+  if ((r = D.addDevice(h, (CUdevice)cuda_device)) != CUDA_SUCCESS) {
+    say("cuMulticastAddDevice %d", (int)r);
+    st = DGCL_ECUDA;
+  } else if ((r = mc_bind_map(cuda_device, h, sz, &mem, &uc, &mc)) != CUDA_SUCCESS) {
+    say("bind / map %d", (int)r);
+    st = DGCL_ECUDA;
+  } else {
+    // region = [flag 4 KB | data]: chunk i of the data through the multicast address
+    const int n16 = (int)((sz - 4096) / 16 < 65536 ? (sz - 4096) / 16 : 65536);
+    std::vector<int32_t> hostv((size_t)n16 * 4);
+    uint64_t flag = 0;
+    if (cudaMemset(uc, 0, sz) != cudaSuccess ||
+        launch_mc_selftest(mc + 4096, (uint64_t *)mc, n16, nullptr) != 0 ||
+        cudaDeviceSynchronize() != cudaSuccess ||
+        cudaMemcpy(hostv.data(), uc + 4096, hostv.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess ||
+        cudaMemcpy(&flag, uc, 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+      say("kernel / copy failed (%d)", (int)cudaGetLastError());
+      st = DGCL_ECUDA;
+    } else {
+      int bad = 0;
+      for (int i = 0; i < n16; ++i)
+        bad += hostv[4 * i] != i || hostv[4 * i + 1] != (i ^ 0x5a5a5a5a) || hostv[4 * i + 2] != ~i ||
+               hostv[4 * i + 3] != 7;
+      if (bad || flag != 5) {
+        say("wrong data through the unicast view (%d bad chunks)", bad);
+        st = DGCL_EPLAN;
+      } else {
+        say("ok: %d chunks stored through the multicast address, reduction seen", n16);
+      }
+    }
+  }
+  mc_teardown(cuda_device, h, true, mem, mem != 0, uc, mc, sz);
+  return st;
+}
+
 dgcl_status dgcl_stream_wait_arrival(dgcl_ctx *c, int32_t dst, int32_t src, void *stream) {
   if (!c) return DGCL_EINVAL;
   if (!has_device(c)) return fail(c, DGCL_ESTATE, "host-only context");
@@ -1214,6 +1522,7 @@ dgcl_status dgcl_plan_info(dgcl_ctx *c, dgcl_plan_stats *info) {
   }
   info->n_fwd_groups = nf;
   info->n_bwd_groups = nb;
+  info->n_multicast_rows = c->low.mc_total;
   return DGCL_OK;
 }
 
@@ -1264,8 +1573,9 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }
-  if (k == "dynamic_items") {  // bulk-copy executor: 1 dynamic item claiming, 0 round-robin
-    c->dynamic_items = value != 0;
+  if (k == "item_order") {  // bulk-copy executor: 0 round-robin, 1 dynamic claiming, 2 rotated
+    if (value < 0 || value > 2) return fail(c, DGCL_EINVAL, "item_order in 0..2");
+    c->item_order = (int)value;
     return DGCL_OK;
   }
   if (k == "sys_scope") {  // loopback: 1 = the multi-GPU system-scope flag protocol (A/B)
@@ -1356,6 +1666,16 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   if (k == "align_sources") {  // forward COPY groups of one source rank: common item boundaries
     c->align_sources = value != 0;
     if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "multicast") {  // NVSwitch multicast of high-fan-out rows (0 off, 1 all peers, k >= 2)
+    if (value < 0 || value > kMaxRanks) return fail(c, DGCL_EINVAL, "multicast in 0..%d", kMaxRanks);
+    c->multicast = (int)value;
+    if (c->planned) {
+      relower(c);
+      compute_layout(c);
+      build_programs(c);
+    }
     return DGCL_OK;
   }
   if (k == "fanout") {  // forward stage 1: per-owner fan-out items (1) or per-pair COPY items (0)
@@ -1482,6 +1802,8 @@ dgcl_status dgcl_destroy(dgcl_ctx *c) {
     for (cudaEvent_t e : c->rank_events)
       if (e) cudaEventDestroy(e);
     if (c->fork_event) cudaEventDestroy(c->fork_event);
+    mc_teardown(c->device, c->mc_handle, c->mc_have_handle, c->mc_mem, c->mc_have_mem, c->mc_uc,
+                c->mc_va, c->mc_map_bytes);
   }
   delete c;
   return DGCL_OK;

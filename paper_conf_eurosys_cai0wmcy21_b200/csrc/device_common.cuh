@@ -187,13 +187,47 @@ static __device__ __noinline__ bool wait_geq(const uint64_t *p, uint64_t target,
   }
 }
 
+// counter index -> word: the flag region, or (multicast done counters) the multicast flag page
+__device__ __forceinline__ uint64_t *ctr_ptr(const ExecParams &P, int rank, int64_t ctr) {
+  return ctr < kMcCtrBase ? P.flags[rank] + ctr : P.mcuc_flags[rank] + (ctr - kMcCtrBase);
+}
+
+// NVSwitch multicast: one store through the multicast address lands in every bound GPU's copy
+__device__ __forceinline__ void mm_st_v4(void *p, const int4 &v) {
+  asm volatile("multimem.st.relaxed.sys.global.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p),
+               "f"(__int_as_float(v.x)), "f"(__int_as_float(v.y)), "f"(__int_as_float(v.z)),
+               "f"(__int_as_float(v.w))
+               : "memory");
+}
+__device__ __forceinline__ void mm_red_release_add(uint64_t *p, uint64_t v) {
+  asm volatile("multimem.red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// a 16-B chunk of multicast region row `row` (layer pitch): every GPU's copy
+__device__ __forceinline__ void mc_store16(const ExecParams &P, int exec, int64_t row,
+                                           uint32_t col, const int4 &v) {
+  if (P.mc_emulate) {
+    for (int r = 0; r < P.world; ++r)
+      st_v4(P.buf[K_MCUC][r].ptr + row * P.buf[K_MCUC][r].pitch + (int64_t)col * 16, v);
+  } else {
+    mm_st_v4(P.buf[K_MCAST][exec].ptr + row * P.buf[K_MCAST][exec].pitch + (int64_t)col * 16, v);
+  }
+}
+// owner's multicast done counter += rows on every GPU (the caller fenced its stores)
+__device__ __forceinline__ void mc_publish(const ExecParams &P, int owner, uint64_t rows) {
+  if (P.mc_emulate) {
+    for (int r = 0; r < P.world; ++r) red_release_add(P.mcuc_flags[r] + owner, rows, P.sys_scope);
+  } else {
+    mm_red_release_add(P.mc_flags + owner, rows);
+  }
+}
+
 // counter waits of an item (all of them, blocking): its source rows are final
 __device__ __forceinline__ bool wait_item_sources(const ExecParams &P, const DevItem &I,
                                                   int code) {
   bool ok = true;
   for (int w = 0; ok && w < I.wait_n; ++w) {
     const DevWait W = P.waits[I.wait_off + w];
-    ok = wait_geq(P.flags[I.exec_rank] + W.ctr, P.epoch[I.dir] * (uint64_t)W.amount, P, code);
+    ok = wait_geq(ctr_ptr(P, I.exec_rank, W.ctr), P.epoch[I.dir] * (uint64_t)W.amount, P, code);
   }
   return ok;
 }

@@ -117,6 +117,21 @@ __device__ __forceinline__ void copy_rows_full(const ExecParams &P, const DevIte
   }
 }
 
+// ---- OP_COPY into the multicast region: every chunk once through the multicast address ----
+__device__ __forceinline__ void copy_rows_mc(const ExecParams &P, const DevItem &I) {
+  const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
+  const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
+  const int32_t *sidx = idx_of(P, I.src);
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  for (uint32_t e = threadIdx.x; e < total; e += blockDim.x) {
+    const uint32_t r = fdiv(e, P);
+    const uint32_t col = e - r * nch;
+    mc_store16(P, I.exec_rank, I.dst + r, col,
+               ld_nc_v4(sbase + row_of(sidx, I.src, r) * spitch + (int64_t)col * 16));
+  }
+}
+
 // ---- OP_COPY with atomic adds (ablation, option "atomic_backward"): one fp32 atomic per word --
 __device__ __forceinline__ void copy_rows_atomic(const ExecParams &P, const DevItem &I) {
   const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
@@ -357,6 +372,8 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
     if (s_abort) return;  // the watchdog fired; the error word is set, leave the launch
     if (kCopy == 3) {  // fold-only instance
       if (I.op == OP_FOLD) fold_rows<V16>(P, I);
+    } else if (I.op == OP_COPY && I.dst_kind == K_MCAST) {
+      copy_rows_mc(P, I);
     } else if (I.op == OP_COPY && (I.flags & kItemAtomic)) {
       copy_rows_atomic(P, I);
     } else if (I.op == OP_COPY) {
@@ -381,7 +398,11 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
       __syncthreads();
       if (threadIdx.x == 0) P.trace[it].t_done = globaltimer();
     }
-    if ((I.flags & kItemSignal) && I.op == OP_FANOUT) {
+    if ((I.flags & kItemSignal) && I.dst_kind == K_MCAST) {  // multicast counter: right away
+      fence_scope(1);
+      __syncthreads();
+      if (threadIdx.x == 0) mc_publish(P, I.exec_rank, (uint64_t)I.rows);
+    } else if ((I.flags & kItemSignal) && I.op == OP_FANOUT) {
       fence_scope(P.sys_scope);
       __syncthreads();
       if (threadIdx.x < (unsigned)P.world && s_cnt[threadIdx.x]) {
@@ -419,12 +440,29 @@ __global__ void wait_kernel(const __grid_constant__ ExecParams P, int exec, int 
   if (threadIdx.x != 0) return;
   for (int w = off; w < off + n; ++w) {
     const DevWait W = P.waits[w];
-    if (!wait_geq(P.flags[exec] + W.ctr, P.epoch[DIR_FWD] * (uint64_t)W.amount, P, 4000000 + w))
+    if (!wait_geq(ctr_ptr(P, exec, W.ctr), P.epoch[DIR_FWD] * (uint64_t)W.amount, P, 4000000 + w))
       return;
   }
 }
 
+// multicast self-test: chunk i of the region = (i, i ^ 0x5a5a5a5a, ~i, 7) through the multicast
+// address, then the flag word += 5 by one multimem reduction (release)
+__global__ void mc_selftest_kernel(char *mc, uint64_t *mcflag, int n16) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n16) mm_st_v4(mc + (int64_t)i * 16, make_int4(i, i ^ 0x5a5a5a5a, ~i, 7));
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence_system();
+    mm_red_release_add(mcflag, 5);
+  }
+}
+
 }  // namespace
+
+int launch_mc_selftest(void *mc, uint64_t *mcflag, int n16, void *stream) {
+  mc_selftest_kernel<<<(n16 + 255) / 256, 256, 0, (cudaStream_t)stream>>>((char *)mc, mcflag, n16);
+  return (int)cudaGetLastError();
+}
 
 int launch_wait(const ExecParams &p, int exec, int off, int n, void *stream) {
   wait_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(p, exec, off, n);

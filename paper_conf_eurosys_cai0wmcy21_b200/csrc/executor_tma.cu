@@ -192,7 +192,8 @@ __device__ __forceinline__ void consumer_barrier(unsigned *count, volatile unsig
 __device__ __forceinline__ bool waits_ready(const ExecParams &P, const DevItem &I) {
   for (int w = 0; w < I.wait_n; ++w) {
     const DevWait W = P.waits[I.wait_off + w];
-    if (ld_acquire(P.flags[I.exec_rank] + W.ctr, P.sys_scope) < P.epoch[I.dir] * (uint64_t)W.amount)
+    if (ld_acquire(ctr_ptr(P, I.exec_rank, W.ctr), P.sys_scope) <
+        P.epoch[I.dir] * (uint64_t)W.amount)
       return false;
   }
   return true;
@@ -434,6 +435,22 @@ __device__ __forceinline__ void store_copy(const ExecParams &P, const DevItem &I
         }
       }
     }
+  }
+}
+
+// consumers: COPY item into the multicast region (NVSwitch multicast):
+// every 16-B chunk goes out once through the multicast address (multimem.st) and lands in every
+// GPU's copy of the region; the destination rows are consecutive
+__device__ __forceinline__ void store_copy_mc(const ExecParams &P, const DevItem &I,
+                                              const uint8_t *st, uint32_t tid, uint32_t T) {
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t r16 = (uint32_t)P.row16;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  const uint8_t *ops = st + kStageHdrBytes;
+  for (uint32_t e = tid; e < total; e += T) {
+    const uint32_t r = fdiv(e, P);
+    const uint32_t col = e - r * nch;
+    mc_store16(P, I.exec_rank, I.dst + r, col, lds_v4(ops + r * r16 + col * 16));
   }
 }
 
@@ -879,13 +896,22 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     // runs differ).  nend = the first queue position without an item (known once a claim fails).
     const uint32_t G = gridDim.x;
     uint32_t nend = 0xffffffffu, nreq = 0;
+    // static orders: plain round-robin (round q: CTA b takes list position q * G + b), or
+    // rotated (position q * G + (b + q) % G): each round still covers the same G consecutive
+    // positions, but a CTA's items no longer all come from the same group when the number of
+    // interleaved groups divides G (e.g. the 2-way Web-Google forward: 2 groups, 296 CTAs)
+    const uint32_t R = (uint32_t)P.n_items / G, rem = (uint32_t)P.n_items % G;
     if (!P.claim)
-      nend = blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
+      nend = P.item_order == 1 ? R + ((blockIdx.x + R) % G < rem ? 1u : 0u)
+             : blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G
+                                                : 0;
     auto request_desc = [&](uint32_t q) -> bool {  // lane 0, after a proxy fence
       uint64_t idx;
       if (P.claim) {
         idx = atomicAdd(reinterpret_cast<unsigned long long *>(P.claim), 1ull) - P.claim_base;
         if (idx >= (uint64_t)P.n_items) return false;
+      } else if (P.item_order == 1) {
+        idx = (uint64_t)q * G + (blockIdx.x + q) % G;
       } else {
         idx = blockIdx.x + (uint64_t)q * G;
       }
@@ -1076,7 +1102,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           const uint32_t amt = s_pend[i];
           if (amt) {
             const int ex = (int)(i / kMaxRanks), dst = (int)(i % kMaxRanks);
-            red_release_add(P.flags[dst] + s_pend_base + ex, amt, P.sys_scope);
+            if (s_pend_base >= kMcCtrBase)  // multicast sends: every GPU's copy of ex's counter
+              mc_publish(P, ex, amt);
+            else
+              red_release_add(P.flags[dst] + s_pend_base + ex, amt, P.sys_scope);
             s_pend[i] = 0;
           }
         }
@@ -1090,7 +1119,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       // the launch's items, so e.g. a forward launch carries no fold code / registers)
       if ((kMask & kMaskCopy) && I.op == OP_COPY && !(I.flags & kItemDirect)) {
         const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
-        if (I.flags & kItemAtomic) {
+        if (I.dst_kind == K_MCAST) {
+          store_copy_mc(P, I, st, tid, T);
+        } else if (I.flags & kItemAtomic) {
           store_copy_atomic(P, I, st, tid, T);
         } else if (P.bulk_store && I.dst >= 0 && DB.pitch == (int64_t)P.row16) {
           // consecutive packed destination rows: kStoreSplit bulk (TMA) stores move the item,

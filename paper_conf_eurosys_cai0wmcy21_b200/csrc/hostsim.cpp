@@ -24,6 +24,17 @@ inline float *row_ptr(const HostBufs &B, int kind, int rank, int64_t row) {
   return B.base[kind][rank] + row * B.pitch;
 }
 
+// a row stored into destination (kind, rank, row): the multicast region kind reaches every
+// rank's copy (what one store through the multicast address does)
+inline void put_row(const HostBufs &B, int m, int kind, int rank, int64_t row, const float *s,
+                    int dim) {
+  if (kind == K_MCAST) {
+    for (int r = 0; r < m; ++r) std::memcpy(row_ptr(B, K_MCUC, r, row), s, sizeof(float) * dim);
+    return;
+  }
+  std::memcpy(row_ptr(B, kind, rank, row), s, sizeof(float) * dim);
+}
+
 // OP_FANOUT rows [r0, r0 + rows) of group g: each source row into all its receivers' rows
 bool run_fanout(const Lowered &low, const DevGroup &g, int64_t r0, int64_t rows,
                 const HostBufs &B, int dim) {
@@ -64,14 +75,14 @@ void run_group(const Lowered &low, const DevGroup &g, const HostBufs &B, int dim
   }
   for (int64_t i = 0; i < g.n_rows; ++i) {
     const int64_t drow = g.dst_idx >= 0 ? low.idx[g.dst_idx + i] : g.dst_base + i;
-    float *d = row_ptr(B, g.dst_kind, g.dst_rank, drow);
+    float *d = g.dst_kind == K_MCAST ? nullptr : row_ptr(B, g.dst_kind, g.dst_rank, drow);
     if (g.op == OP_COPY) {
       const int64_t srow = g.src_idx >= 0 ? low.idx[g.src_idx + i] : g.src_base + i;
       const float *s = row_ptr(B, g.src_kind, g.exec_rank, srow);
       if (g.atomic_add)
         for (int c = 0; c < dim; ++c) d[c] += s[c];
       else
-        std::memcpy(d, s, sizeof(float) * dim);
+        put_row(B, low.m, g.dst_kind, g.dst_rank, drow, s, dim);
     } else {
       const int64_t t0 = low.term_ptr[g.term_ptr + i], t1 = low.term_ptr[g.term_ptr + i + 1];
       auto operand = [&](uint32_t term) -> const float * {
@@ -128,12 +139,13 @@ bool run_item(const Lowered &low, const DevItem &it, const std::vector<DevRun> &
       if (R.pos != covered || R.len < 1) return false;
       covered += R.len;
       for (int32_t j = 0; j < R.len; ++j) {
-        float *d = row_ptr(B, it.dst_kind, it.dst_rank, R.dst + j);
         const float *s = row_ptr(B, it.src_kind, it.exec_rank, R.src + j);
-        if (it.flags & kItemAtomic)
+        if (it.flags & kItemAtomic) {
+          float *d = row_ptr(B, it.dst_kind, it.dst_rank, R.dst + j);
           for (int c = 0; c < dim; ++c) d[c] += s[c];
-        else
-          std::memcpy(d, s, sizeof(float) * dim);
+        } else {
+          put_row(B, low.m, it.dst_kind, it.dst_rank, R.dst + j, s, dim);
+        }
       }
     }
     return covered == it.rows;
@@ -197,6 +209,8 @@ void setup_bufs(const Lowered &low, const std::vector<int64_t> &row_off,
   const int m = low.m;
   relay.assign(m, {});
   slot.assign(m, {});
+  // (the multicast region copies live after the relay / slot buffers of `relay`)
+  relay.resize(2 * m);
   std::memset(B, 0, sizeof(*B));
   B->pitch = pitch;
   for (int r = 0; r < m; ++r) {
@@ -208,6 +222,8 @@ void setup_bufs(const Lowered &low, const std::vector<int64_t> &row_off,
     B->base[K_HGRAD][r] = const_cast<float *>(halo_grad) + (halo_grad ? halo_off[r] * pitch : 0);
     B->base[K_RELAY][r] = relay[r].data();
     B->base[K_SLOT][r] = slot[r].data();
+    relay[m + r].assign((size_t)low.mc_total * pitch, 0.f);
+    B->base[K_MCUC][r] = relay[m + r].data();
   }
 }
 

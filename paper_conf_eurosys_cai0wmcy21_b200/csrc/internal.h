@@ -24,7 +24,9 @@ enum Kind : int32_t {
   K_HGRAD = 3,  // user halo gradients, read-only
   K_SLOT = 4,   // backward gradient slots (workspace), written by tree children
   K_EGRAD = 5,  // user embedding gradients (in/out)
-  K_NKINDS = 6
+  K_MCAST = 6,  // multicast region through the NVSwitch multicast address (multimem stores)
+  K_MCUC = 7,   // this GPU's own copy of the multicast region (unicast reads)
+  K_NKINDS = 8
 };
 
 // source kinds a COPY item may gather with tile::gather4 (tensor map per kind, ExecParams::tmap)
@@ -62,6 +64,11 @@ constexpr int64_t ctr_index(int dir, int stage, int src, int block = 0) {
 constexpr int64_t kReadyBase = 2 * kMaxStages * kMaxBlocks * kMaxRanks;  // ready[src] words
 constexpr int64_t kBarrierBase = kReadyBase + kMaxRanks;  // device start barrier: arrived[src]
 constexpr int64_t kFlagWords = kBarrierBase + kMaxRanks;
+// multicast done counters mc_done[owner] live in the multicast region's flag page, not in the
+// flag region: counter indices kMcCtrBase + owner (DevGroup::sig_ctr, DevWait::ctr)
+constexpr int64_t kMcCtrBase = kFlagWords;
+constexpr int64_t kMcFlagBytes = 4096;  // flag page at the start of the multicast region
+constexpr int64_t kCtrSpace = kFlagWords + kMaxRanks;  // counter indices of one rank
 constexpr int64_t kFlagBytes = 40960;  // region reserved (>= kFlagWords * 8)
 static_assert(kFlagWords * 8 <= kFlagBytes, "flag region");
 
@@ -200,6 +207,13 @@ struct alignas(64) ExecParams {
   // n_items + grid claims; claim_base = the counter's value at launch (kept by the host)
   uint64_t *claim;
   uint64_t claim_base;
+  int32_t item_order;      // static orders (claim == nullptr): 0 round-robin, 1 rotated rounds
+  // multicast (option "multicast"): the multicast flag page (multimem reductions), every rank's
+  // unicast flag page (acquire waits; loopback: each virtual rank's copy), and whether the
+  // multicast is emulated by one store / reduction per rank (loopback: no multicast object)
+  uint64_t *mc_flags;
+  uint64_t *mcuc_flags[kMaxRanks];
+  int32_t mc_emulate;
 };
 
 // Per-item timeline (%globaltimer ns), written when tracing is on: the executor reached the item,
@@ -289,6 +303,8 @@ int launch_barrier(const ExecParams &p, int first, int count, void *stream);
 // arrival wait (overlap): one thread acquire-waits on rank `exec`'s counters
 // p.waits[off .. off + n) >= p.epoch[DIR_FWD] * amount, then the kernel ends
 int launch_wait(const ExecParams &p, int exec, int off, int n, void *stream);
+// multicast self-test kernel (dgcl_debug_multicast_selftest): multimem stores + one reduction
+int launch_mc_selftest(void *mc, uint64_t *mcflag, int n16, void *stream);
 int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm);  // bulk-copy path
 
 }  // namespace dgcl

@@ -60,7 +60,7 @@ inline int32_t halo_pos(const Relation &rel, int64_t u, int d) {
 
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
                 const std::vector<int64_t> &loc, Lowered *out, int n_blocks, bool with_atomic,
-                bool with_fanout) {
+                bool with_fanout, int mc_min_fanout) {
   auto t0 = std::chrono::steady_clock::now();
   // DGCL_TIMING=1: per-section wall times on stderr (planning at scale, NEXT-4)
   static const bool timing = std::getenv("DGCL_TIMING") != nullptr;
@@ -191,6 +191,25 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     src_kind[e] = p == part[u] ? K_EMB : (halo_pos(rel, u, p) >= 0 ? K_HALO : K_RELAY);
   }
 
+  // NVSwitch multicast (the switch-level form of communication fusion,
+  // P:1057-1065): single-stage plans only, every vertex requested by >= mc_min_fanout GPUs is
+  // sent once, by its owner, with multimem stores into the multicast region every GPU binds at
+  // the same offset (row mc_off[s] + j: the j-th such vertex of owner s in ascending id), then
+  // each requester copies it from its own region into its halo row (unpack, local HBM)
+  std::vector<uint8_t> mc_v(NV, 0);
+  L.mc_rows.assign(m, 0);
+  L.mc_off.assign(m + 1, 0);
+  if (mc_min_fanout > 0 && K == 1) {
+    for (int64_t vi = 0; vi < NV; ++vi) {
+      const int64_t u = plan.order[vi];
+      if (rel.d_ptr[u + 1] - rel.d_ptr[u] >= mc_min_fanout) {
+        mc_v[vi] = 1;
+        ++L.mc_rows[part[u]];
+      }
+    }
+    for (int d = 0; d < m; ++d) L.mc_off[d + 1] = L.mc_off[d] + L.mc_rows[d];
+  }
+  L.mc_total = L.mc_off[m];
   lap("blocks/child_pos/kinds");
   // ---- forward relay staging rows: contiguous per (receiver c, stage k, sender p, src kind) ----
   std::vector<int64_t> relay_row(NE, -1);
@@ -260,8 +279,13 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   {
     std::vector<Entry> ent(NE);
     std::vector<int64_t> srow(NE), drow(NE);
+    std::vector<uint8_t> keep(NE, 1);
 #pragma omp parallel for schedule(static)
     for (int64_t e = 0; e < NE; ++e) {
+      if (mc_v[e_vidx[e]]) {  // multicast vertex: its rows leave by the multicast groups
+        keep[e] = 0;
+        continue;
+      }
       const int64_t vi = e_vidx[e];
       const int64_t u = plan.order[vi];
       const int p = plan.e_parent[e], c = plan.e_child[e], k = plan.e_stage[e];
@@ -281,6 +305,12 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
         drow[e] = relay_row[e];
       }
       ent[e] = {pack_key_b(k, blk_of[vi], p, c, sk, dk), drow[e], e, vi};
+    }
+    if (L.mc_total > 0) {
+      size_t w = 0;
+      for (int64_t e = 0; e < NE; ++e)
+        if (keep[e]) ent[w++] = ent[e];
+      ent.resize(w);
     }
     __gnu_parallel::sort(ent.begin(), ent.end(), [](const Entry &a, const Entry &b) {
       return a.key != b.key ? a.key < b.key : a.sort2 < b.sort2;
@@ -305,6 +335,48 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       flush_group(L.groups, g, src, dst);
       L.rows_at(DIR_FWD, k, p, c, bl) += (int64_t)dst.size();
       i = j;
+    }
+    // multicast: per owner s one send group (its multicast vertices' embedding rows, ascending
+    // id, into region rows mc_off[s] ..), then per (receiver d, owner s) one unpack group (region
+    // rows of the s-vertices d requested -> d's halo rows), stage 2: after every send
+    if (L.mc_total > 0) {
+      std::vector<std::vector<int64_t>> mcv(m);  // multicast vertices of each owner, ascending
+      for (int64_t vi = 0; vi < NV; ++vi)
+        if (mc_v[vi]) mcv[part[plan.order[vi]]].push_back(plan.order[vi]);
+      for (auto &v : mcv) std::sort(v.begin(), v.end());
+      L.mc_begin = (int)L.groups.size();
+      for (int s = 0; s < m; ++s) {
+        if (mcv[s].empty()) continue;
+        src.clear();
+        dst.clear();
+        for (size_t j = 0; j < mcv[s].size(); ++j) {
+          src.push_back(loc[mcv[s][j]]);
+          dst.push_back(L.mc_off[s] + (int64_t)j);
+        }
+        DevGroup g = base_group(OP_COPY, DIR_FWD, s, s, 1);
+        g.src_kind = K_EMB;
+        g.dst_kind = K_MCAST;
+        flush_group(L.groups, g, src, dst);
+      }
+      for (int d = 0; d < m; ++d)
+        for (int s = 0; s < m; ++s) {
+          if (s == d || mcv[s].empty()) continue;
+          src.clear();
+          dst.clear();
+          for (size_t j = 0; j < mcv[s].size(); ++j) {
+            const int32_t pos = halo_pos(rel, mcv[s][j], d);
+            if (pos < 0) continue;  // (fan-out below m - 1: d did not ask for this one)
+            src.push_back(L.mc_off[s] + (int64_t)j);
+            dst.push_back(pos);
+          }
+          if (dst.empty()) continue;
+          DevGroup g = base_group(OP_COPY, DIR_FWD, d, d, 2);
+          g.src_kind = K_MCUC;
+          g.dst_kind = K_HALO;
+          g.block = s;  // (the owner whose multicast rows it unpacks; see the waits below)
+          flush_group(L.groups, g, src, dst);
+        }
+      L.mc_end = (int)L.groups.size();
     }
     L.n_fwd_groups = (int)L.groups.size();
   }
@@ -471,6 +543,24 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       auto w = get_waits(g.dir, g.stage - 1, g.exec_rank, g.block);
       g.wait_off = w.first;
       g.wait_n = w.second;
+    }
+  }
+  // multicast groups: a send signals the multicast done counter of its owner (one multimem
+  // reduction reaches every GPU's copy) and writes into every peer's region (all ready words);
+  // an unpack waits on the owner's multicast counter in this GPU's own region
+  for (int gi = L.mc_begin; gi < L.mc_end; ++gi) {
+    DevGroup &g = L.groups[gi];
+    g.wait_off = 0;
+    g.wait_n = 0;
+    if (g.dst_kind == K_MCAST) {
+      g.sig_ctr = (int32_t)(kMcCtrBase + g.exec_rank);
+      g.ready_rank = kReadyAll;
+    } else {
+      const int s_owner = g.block;
+      g.block = 0;
+      g.wait_off = (int32_t)L.waits.size();
+      g.wait_n = 1;
+      L.waits.push_back({(int32_t)(kMcCtrBase + s_owner), 0, L.mc_rows[s_owner]});
     }
   }
   // per-rank READY and forward-completion WAIT groups (used by per-rank programs only)
@@ -850,7 +940,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       };
       auto alignable = [&](const DevGroup &h) {
         return h.op == OP_COPY && h.dir == DIR_FWD && h.src_kind == K_EMB && !h.atomic_add &&
-               h.n_rows > 0 && ascending_src(h) && short_runs(h);
+               h.dst_kind != K_MCAST && h.n_rows > 0 && ascending_src(h) && short_runs(h);
       };
       const int64_t rpi = copy_rpi(spread_rpi);
       std::vector<uint8_t> can(j - i);  // alignable, evaluated once per group (O(rows))
@@ -1073,19 +1163,19 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
           it.nterms = (int32_t)((int64_t)runs->size() - it.tp);
         }
         bool sig = data && g.sig_ctr >= 0;
-        if (sig && !signal_all && fan) {
+        if (sig && !signal_all && (fan || g.dst_kind == K_MCAST)) {
           sig = false;  // needed by some receiver of the owner's rows
           for (int d = 0; d < low.m; ++d)
-            if (d != g.exec_rank && needed_ctr[(size_t)d * kFlagWords + g.sig_ctr]) sig = true;
+            if (d != g.exec_rank && needed_ctr[(size_t)d * kCtrSpace + g.sig_ctr]) sig = true;
         } else if (sig && !signal_all) {
-          sig = needed_ctr[(size_t)g.dst_rank * kFlagWords + g.sig_ctr] != 0;
+          sig = needed_ctr[(size_t)g.dst_rank * kCtrSpace + g.sig_ctr] != 0;
         }
         it.flags |= sig ? kItemSignal : 0;
         // optional: items whose runs average fewer than `direct_copy_rows` rows are gathered by
         // the consumers with plain loads instead of one bulk copy per run (0 = never; measured
         // slower than per-row bulk copies on the BASELINE graphs)
         if (g.atomic_add) it.flags |= kItemAtomic;
-        if (g.op == OP_COPY && direct_copy_rows > 0 && !g.atomic_add &&
+        if (g.op == OP_COPY && direct_copy_rows > 0 && !g.atomic_add && g.dst_kind != K_MCAST &&
             (int64_t)it.nterms * direct_copy_rows > (int64_t)it.rows)
           it.flags |= kItemDirect;
         // source rows in short runs (< 4 rows on average) of embeddings, halos (relay

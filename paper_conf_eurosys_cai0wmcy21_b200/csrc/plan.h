@@ -67,6 +67,12 @@ struct Lowered {
   int atomic_end = 0;  // [direct_end, atomic_end): loopback atomic-add backward groups (ablation)
   int fanout_end = 0;  // [atomic_end, fanout_end): forward stage-1 fan-out groups, one per owner
   int tree_end = 0;    // [fanout_end, tree_end): loopback tree-order backward (relay plans)
+  // multicast (option "multicast"): [mc_begin, mc_end) = per-owner send groups (dst K_MCAST) and
+  // per-(receiver, owner) unpack groups (src K_MCUC), inside the forward groups; the region holds
+  // mc_total rows, owner s's at mc_off[s] ..
+  int mc_begin = 0, mc_end = 0;
+  std::vector<int64_t> mc_rows, mc_off;
+  int64_t mc_total = 0;
   std::vector<int32_t> idx;              // row index pool
   std::vector<int64_t> term_ptr;         // fold row pointers
   std::vector<uint32_t> terms;           // fold terms
@@ -99,9 +105,11 @@ struct Lowered {
 // n_blocks: vertex blocks for the stage chaining of relay plans (1 = one counter per stage;
 // single-stage plans always use 1); with_atomic / with_fanout: also build the ablation groups
 // (atomic backward, fan-out forward) — only when their option is set (they cost lowering time)
+// mc_min_fanout > 0: multicast the rows of vertices requested by >= that many GPUs
+// (single-stage plans)
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
                 const std::vector<int64_t> &loc, Lowered *out, int n_blocks = 1,
-                bool with_atomic = false, bool with_fanout = false);
+                bool with_atomic = false, bool with_fanout = false, int mc_min_fanout = 0);
 
 // Work items for one launch: the groups `gids` (already in stage order, READY / WAIT groups
 // included by the caller) cut into row ranges of about item_bytes gathered bytes and interleaved
