@@ -150,6 +150,9 @@ def run_multi(args, metric, unit, rank, world, local_rank, ClockSampler, make_wo
     dist.all_gather_object(blobs, ctx.ipc_export())
     ctx.ipc_import(blobs)
     dist.barrier()
+    if ctx.multicast_bytes()[1] > 0:  # option multicast: NVSwitch multicast object
+        from paper_conf_eurosys_cai0wmcy21_b200.dgcl import _setup_multicast
+        _setup_multicast(ctx)
     info = ctx.plan_info()
     mine = np.nonzero(part == rank)[0]
     n_halo = int(ptr[rank + 1] - ptr[rank])

@@ -203,11 +203,12 @@ struct alignas(64) ExecParams {
   int32_t l2_policy;       // option "l2_policy": L2 eviction hints of the bulk-copy executor
   int32_t sys_scope;       // 1: flags / fences at system scope (peers are other GPUs); 0: .gpu
   // bulk-copy executor, dynamic item claiming: a launch-wide counter (nullptr = static
-  // round-robin).  Every CTA claims until one claim fails, so a launch consumes exactly
-  // n_items + grid claims; claim_base = the counter's value at launch (kept by the host)
+  // order).  Every CTA claims until one claim fails, so a launch consumes exactly
+  // n_items - claim_from + grid claims; claim_base = the counter's value at launch (host)
   uint64_t *claim;
   uint64_t claim_base;
-  int32_t item_order;      // static orders (claim == nullptr): 0 round-robin, 1 rotated rounds
+  int32_t item_order;      // static part: 0 round-robin, 1 rotated rounds
+  int64_t claim_from;      // with claim: list positions >= claim_from are claimed dynamically
   // multicast (option "multicast"): the multicast flag page (multimem reductions), every rank's
   // unicast flag page (acquire waits; loopback: each virtual rank's copy), and whether the
   // multicast is emulated by one store / reduction per rank (loopback: no multicast object)

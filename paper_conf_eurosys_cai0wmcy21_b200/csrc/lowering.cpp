@@ -41,12 +41,16 @@ inline uint64_t pack_key(int stage, int exec, int dst, int a, int b) {
   return ((uint64_t)stage << 24) | ((uint64_t)exec << 16) | ((uint64_t)dst << 8) |
          ((uint64_t)a << 4) | (uint64_t)b;
 }
-// group key ordered (stage, block, exec, dst, a, b): groups of a stage come block by block
+// group key ordered (stage + block, stage, block, exec, dst, a, b): with vertex blocks the
+// (stage, block) runs come in wavefront order — stage k of block b right after stage k - 1 of
+// block b + 1 — so the executor reaches stage k of the first blocks while the later blocks'
+// stage k - 1 still runs (every dependency, stage k - 1 of the same block, comes earlier);
+// without blocks this is plain stage order
 inline uint64_t pack_key_b(int stage, int block, int exec, int dst, int a, int b) {
-  return ((uint64_t)stage << 32) | ((uint64_t)block << 24) | ((uint64_t)exec << 16) |
-         ((uint64_t)dst << 8) | ((uint64_t)a << 4) | (uint64_t)b;
+  return ((uint64_t)(stage + block) << 40) | ((uint64_t)stage << 32) | ((uint64_t)block << 24) |
+         ((uint64_t)exec << 16) | ((uint64_t)dst << 8) | ((uint64_t)a << 4) | (uint64_t)b;
 }
-inline int key_stage(uint64_t k) { return (int)(k >> 32); }
+inline int key_stage(uint64_t k) { return (int)(k >> 32 & 0xFF); }
 inline int key_block(uint64_t k) { return (int)(k >> 24 & 0xFF); }
 
 // position of u on GPU d (its halo row), or -1 if d did not request u
@@ -912,7 +916,7 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     for (size_t q = i; q < j; ++q)
       if (low.groups[gids[q]].op == OP_COPY) copy_rows += low.groups[gids[q]].n_rows;
     int64_t spread_rpi = lim.max_rows;
-    if (lim.min_items > 0 && copy_rows < lim.min_items * lim.max_rows)
+    if (lim.min_items > 0 && low.n_blocks == 1 && copy_rows < lim.min_items * lim.max_rows)
       spread_rpi = std::max<int64_t>(4, (copy_rows + lim.min_items - 1) / lim.min_items);
     auto copy_rpi = [&](int64_t spread) {
       int64_t rpi = std::min<int64_t>(std::min(lim.max_rows, spread),

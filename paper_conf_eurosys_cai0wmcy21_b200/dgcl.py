@@ -272,6 +272,27 @@ class Context:
         check(lib().dgcl_stream_wait_arrival(self.handle, dst, src, _stream_ptr(stream)),
               self.handle)
 
+    # ---- NVSwitch multicast (option "multicast"; see dgcl.h) ---------------------------------
+    def multicast_bytes(self):
+        """(region bytes, multicast rows) of the plan (0, 0 when nothing is multicast)."""
+        b = ctypes.c_size_t(0)
+        r = ctypes.c_int64(0)
+        check(lib().dgcl_multicast_bytes(self.handle, ctypes.byref(b), ctypes.byref(r)),
+              self.handle)
+        return b.value, r.value
+
+    def multicast_open(self, fd=None):
+        """Rank 0: create the multicast object, return its POSIX fd.  Others: import `fd`."""
+        v = ctypes.c_int32(-1 if fd is None else int(fd))
+        check(lib().dgcl_multicast_open(self.handle, ctypes.byref(v)), self.handle)
+        return v.value
+
+    def multicast_add(self):
+        check(lib().dgcl_multicast_add(self.handle), self.handle)
+
+    def multicast_bind(self):
+        check(lib().dgcl_multicast_bind(self.handle), self.handle)
+
     def launch_count(self):
         v = ctypes.c_uint64(0)
         check(lib().dgcl_launch_count(self.handle, ctypes.byref(v)), self.handle)
@@ -292,6 +313,63 @@ class Context:
         assert emb_grad.dtype == np.float32 and emb_grad.flags.c_contiguous
         check(lib().dgcl_debug_hostsim_backward(self.handle, layer, halo_grad.ctypes.data,
                                                 emb_grad.ctypes.data), self.handle)
+
+
+def multicast_supported(device=0):
+    """CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED of `device`."""
+    v = ctypes.c_int32(0)
+    check(lib().dgcl_multicast_supported(int(device), ctypes.byref(v)))
+    return bool(v.value)
+
+
+def multicast_selftest(device=0, nbytes=1 << 21):
+    """(status, message) of the library's one-device multicast self-test (dgcl.h)."""
+    buf = ctypes.create_string_buffer(256)
+    st = lib().dgcl_debug_multicast_selftest(int(device), int(nbytes), buf, 256)
+    return st, buf.value.decode()
+
+
+def _setup_multicast(ctx, group=None):
+    """Collective: rank 0 creates the multicast object and hands its POSIX fd to every other rank
+    over a Unix socket (SCM_RIGHTS), every rank adds its device, then binds and maps its memory
+    (dgcl_multicast_open / _add / _bind)."""
+    import os
+    import socket
+    import uuid
+
+    import torch.distributed as dist
+    rank = dist.get_rank(group)
+    world = dist.get_world_size(group)
+    srv = None
+    name = [None]
+    if rank == 0:
+        name = ["\0dgcl-mc-%d-%s" % (os.getpid(), uuid.uuid4().hex)]
+        srv = socket.socket(socket.AF_UNIX, socket.SOCK_STREAM)
+        srv.bind(name[0])
+        srv.listen(world)
+    dist.broadcast_object_list(name, src=0, group=group)
+    try:
+        if rank == 0:
+            fd = ctx.multicast_open()
+            for _ in range(world - 1):
+                conn, _ = srv.accept()
+                socket.send_fds(conn, [b"m"], [fd])
+                conn.close()
+            os.close(fd)
+        else:
+            s = socket.socket(socket.AF_UNIX, socket.SOCK_STREAM)
+            s.connect(name[0])
+            _msg, fds, _flags, _addr = socket.recv_fds(s, 1, 1)
+            s.close()
+            ctx.multicast_open(fds[0])
+            os.close(fds[0])
+    finally:
+        if srv is not None:
+            srv.close()
+    ctx.multicast_add()
+    dist.barrier(group=group)
+    ctx.multicast_bind()
+    dist.barrier(group=group)
 
 
 def _host_ptr(a):
@@ -360,6 +438,8 @@ def setup_distributed(part, dims, my_required, topology=None, seed=0, group=None
     if world > 1:
         ctx.ipc_import(blobs)
     dist.barrier(group=group)
+    if world > 1 and ctx.multicast_bytes()[1] > 0:
+        _setup_multicast(ctx, group)
     return ctx
 
 

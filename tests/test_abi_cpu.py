@@ -310,3 +310,40 @@ def test_single_shared_hop_cost_closed_form(topo_name):
     b.build_plan(g.req_ptr, g.req_ids, topology=one, trees=E)
     assert b.plan_info()["model_cost_ticks"] == len(E) * w
     assert cost.plan_cost(one, [(int(u), int(p), int(c), int(k)) for u, p, c, k in E])[0] == len(E) * w
+
+
+@pytest.mark.parametrize("m,mc", [(2, 1), (4, 1), (8, 1), (8, 5), (3, 2)])
+def test_multicast_lowering_host(m, mc):
+    """Option multicast (NEXT-1): rows of vertices requested by >= k GPUs (1: every peer) leave
+    by one multicast group per owner + per-requester unpack groups.  The host interpreter runs the
+    groups and the work items (a multicast store reaching every rank's region copy) and the halos
+    equal oracle.halo.forward bit for bit; the number of multicast rows is the number of vertices
+    whose fan-out, counted by the oracle, reaches the threshold; the backward is untouched."""
+    import paper_conf_eurosys_cai0wmcy21_b200 as D
+    g = synth.make_graph(3000, 60000, m, graph_seed=3 + m, part_seed=4)
+    ctx = D.loopback(m, g.part, [24], device=-1)
+    ctx.set_option("multicast", mc)
+    ctx.build_plan(g.req_ptr, g.req_ids)
+    k = m - 1 if mc == 1 else mc
+    R = [g.R(d) for d in range(m)]
+    assert ctx.plan_info()["n_multicast_rows"] == int((halo.fanout(R, g.n) >= k).sum()) > 0
+    order = np.argsort(g.part, kind="stable")
+    loc, nl = halo.local_rows(g.part, m)
+    ro = np.concatenate([[0], np.cumsum(nl)])
+    emb = synth.fill_values(g.n, 24, keys=order)
+    Ho = halo.forward([emb[ro[d]:ro[d + 1]] for d in range(m)], R, g.part, loc)
+    for items in (0, 1):
+        ctx.set_option("hostsim_items", items)
+        H = np.zeros((int(g.req_ptr[-1]), 24), np.float32)
+        ctx.debug_hostsim_forward(0, emb, H)
+        for d in range(m):
+            a, b = int(g.req_ptr[d]), int(g.req_ptr[d + 1])
+            assert np.array_equal(H[a:b].view(np.uint32), Ho[d].view(np.uint32))
+    Gr = synth.fill_values(int(g.req_ptr[-1]), 24, seed=4)
+    L = synth.fill_values(g.n, 24, keys=order, seed=5)
+    out = L.copy()
+    ctx.debug_hostsim_backward(0, Gr, out)
+    Bf = halo.backward_flat([L[ro[d]:ro[d + 1]] for d in range(m)],
+                            [Gr[g.req_ptr[d]:g.req_ptr[d + 1]] for d in range(m)], R, g.part, loc)
+    for d in range(m):
+        assert np.array_equal(out[ro[d]:ro[d + 1]].view(np.uint32), Bf[d].view(np.uint32))

@@ -166,6 +166,10 @@ def test_tiny_config_bit_exact(small):
     (3, {"geometry": 1, "stage_fold": 0}),
     (8, {"fanout": 1}), (4, {"fanout": 1, "tma": 0}), (8, {"fanout": 1, "geometry": 2}),
     (3, {"fanout": 1, "bulk_store": 0}), (4, {"fanout": 1, "geometry": 1}),
+    # NVSwitch multicast of high-fan-out rows, emulated on one GPU (one store per virtual rank's
+    # region copy): send + unpack groups, multicast done counters
+    (8, {"multicast": 1}), (4, {"multicast": 2}), (4, {"multicast": 1, "tma": 0}),
+    (3, {"multicast": 1, "geometry": 2}), (8, {"multicast": 3, "small_launch_bytes": 4 << 20}),
 ])
 def test_uniform_loopback_fused(m, opts):
     """Executor variants: tma (bulk-copy executor vs the register LDG executor), direct_reduce
@@ -178,13 +182,17 @@ def test_uniform_loopback_fused(m, opts):
     _check_case(Case(g, [64, 5, 602, 32], options=opts))
 
 
-@pytest.mark.parametrize("m,fanout", [(2, 1), (8, 1), (8, 0)])
-def test_per_rank_flag_protocol(m, fanout):
+@pytest.mark.parametrize("m,fanout,mc", [(2, 1, 0), (8, 1, 0), (8, 0, 0), (8, 0, 1), (4, 0, 2)])
+def test_per_rank_flag_protocol(m, fanout, mc):
     """Every virtual rank is its own launch on its own stream: ready handshake, done counters,
-    forward completion waits — the multi-GPU protocol on one device; several calls in a row."""
+    forward completion waits — the multi-GPU protocol on one device; several calls in a row.
+    mc: the (emulated) multicast path, whose sends wait on every peer's ready word and whose
+    unpacks wait on the owners' multicast counters."""
     D = _D()
     g = synth.make_graph(5000, 40000, m, graph_seed=11, part_seed=12)
-    c = Case(g, [32, 7], flags=D.LOOPBACK_PER_RANK, options={"fanout": fanout})
+    c = Case(g, [32, 7], flags=D.LOOPBACK_PER_RANK, options={"fanout": fanout, "multicast": mc})
+    if mc:
+        assert c.ctx.plan_info()["n_multicast_rows"] > 0
     for _ in range(2):
         _check_case(c)
 
