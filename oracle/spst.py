@@ -106,8 +106,8 @@ def _dijkstra(topo, state, nsrc_depth):
 def spst(topo, owner, D, seed, order=None):
     """Algorithm 1.  owner: dict u -> s_u; D: dict u -> set of requesting GPUs (D_u).
 
-    Returns (edges, cost): edges = list of (u, parent, child, stage) in planning order, and the
-    final costFunc(S).  Raises ValueError if some d in D_u is unreachable."""
+    Returns (edges, cost): edges = list of (u, parent, child, stage), vertices in planning order,
+    each tree's edges in (stage, child) order (R26), and the final costFunc(S).  Raises ValueError if some d in D_u is unreachable."""
     if order is None:
         order = shuffle_order(sorted(u for u in D if D[u]), seed)
     state = CostState(topo)
@@ -116,6 +116,7 @@ def spst(topo, owner, D, seed, order=None):
         su = owner[u]
         depth = {su: 0}                       # N_src with tree depths
         remaining = set(D[u]) - {su}
+        tree = []
         while remaining:
             # line 6 (Algorithm 2) is evaluated inside _dijkstra on demand; S is fixed meanwhile
             label, pred = _dijkstra(topo, state, depth)
@@ -132,9 +133,11 @@ def spst(topo, owner, D, seed, order=None):
             for (p, c) in path:                # lines 9-10
                 k = depth[p] + 1
                 depth[c] = k
-                edges.append((u, p, c, k))
+                tree.append((u, p, c, k))
                 state.add(k, (p, c))
                 remaining.discard(c)
+        # T_u is a set of edges: listed in the canonical (stage, child) order (R26)
+        edges.extend(sorted(tree, key=lambda e: (e[3], e[2])))
     return edges, state.cost_func()
 
 

@@ -95,6 +95,7 @@ struct dgcl_ctx {
   // 4 auto: 3 for launches of few groups (<= 12: the 2- and 4-way forwards, whose per-group item
   // costs differ: Web-Google-2 0.228 -> 0.199 ms), 0 otherwise (Reddit forward 3 % slower with 3)
   int item_order = 4;
+  bool spst_fast = true;  // uniform switch: SPST's closed form (parallel) instead of the loop
   int64_t run_bytes = 0;
   bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
   bool bulk_store_peer = false;   // TMA stores into peer memory over NVLink (not yet validated)
@@ -955,7 +956,7 @@ dgcl_status plan_common(dgcl_ctx *c, const int64_t *req_ptr, const int64_t *req_
     for (int d = 0; d < c->world; ++d)
       if (req_ptr[d + 1] - req_ptr[d] > INT32_MAX) return fail(c, DGCL_EINVAL, "halo too large");
     e = trees ? import_plan(c->topo, c->part.data(), c->rel, n_edges, tu, tp, tc, ts, &c->plan)
-              : spst_plan(c->topo, c->part.data(), c->rel, seed, &c->plan);
+              : spst_plan(c->topo, c->part.data(), c->rel, seed, &c->plan, c->spst_fast);
     if (!e.empty()) return fail(c, DGCL_EPLAN, "%s", e.c_str());
     if (c->plan.n_stages >= kMaxStages) return fail(c, DGCL_EPLAN, "too many stages");
     relower(c);
@@ -1583,6 +1584,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->registered) return fail(c, DGCL_ESTATE, "geometry must be set before registration");
     c->geometry = (int)value;
     if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "spst_fast") {  // before dgcl_build_plan: 0 = always run Algorithm 1's loop
+    if (c->planned) return fail(c, DGCL_ESTATE, "spst_fast must be set before dgcl_build_plan");
+    c->spst_fast = value != 0;
     return DGCL_OK;
   }
   if (k == "item_order") {  // bulk-copy executor: 0 round-robin, 1 dynamic claiming, 2 rotated

@@ -40,15 +40,18 @@ struct Plan {
   std::vector<int32_t> e_parent, e_child, e_stage;
   int64_t cost = 0;                // t(S) in ticks
   double seconds = 0;
+  bool closed_form = false;        // planned by the uniform-switch closed form (parallel)
 };
 
 // Build the relation from the required lists; returns "" or an error message (EINVAL).
 std::string build_relation(int64_t n, int m, const int32_t *part, const int64_t *req_ptr,
                            const int64_t *req_ids, Relation *out);
 
-// SPST, Algorithm 1 + 2 (§5.2).  Returns "" or an error message (EPLAN).
+// SPST, Algorithm 1 + 2 (§5.2).  Returns "" or an error message (EPLAN).  allow_fast: on the
+// uniform switch model use SPST's closed form (every tree a direct star; parallel), which gives
+// the same plan as the general loop (tested)
 std::string spst_plan(const Topology &topo, const int32_t *part, const Relation &rel,
-                      uint64_t seed, Plan *out);
+                      uint64_t seed, Plan *out, bool allow_fast = true);
 
 // A saved plan (trees, as dgcl_plan_export gives them) instead of SPST; the plan invariants are
 // checked and t(S) recomputed.  Returns "" or an error message (EPLAN).

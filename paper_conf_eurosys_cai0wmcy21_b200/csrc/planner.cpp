@@ -92,10 +92,37 @@ inline uint64_t mix64(uint64_t z) {
 
 constexpr int64_t kInf = INT64_MAX;
 
+// Is the topology the uniform switch model (link i->j = {egress_i, ingress_j}, every hop the same
+// cost, egress and ingress hops all distinct)?  Then SPST provably plans every delivery directly
+// in stage 1, in any vertex order: stage 2 carries no load (induction), so any 2-hop path costs at
+// least C(2, .) = w, while a direct link costs C(1, s->d) = max((c+1) w) - t^1 <= w (t^1 >= c w for
+// every stage-1 hop) and wins ties on depth (R8); the trees are stars, t(S) = w x the largest
+// egress / ingress row count.  (the closed form behind the parallel planner.)
+bool uniform_switch(const Topology &t) {
+  const int m = t.m;
+  if (m < 2 || t.w.empty()) return false;
+  std::vector<int32_t> eg(m, -1), ig(m, -1);
+  for (int i = 0; i < m; ++i)
+    for (int j = 0; j < m; ++j) {
+      if (i == j) continue;
+      const int64_t a = t.link_ptr[(size_t)i * m + j], b = t.link_ptr[(size_t)i * m + j + 1];
+      if (b - a != 2) return false;
+      const int32_t h0 = t.link_hops[a], h1 = t.link_hops[a + 1];
+      if (t.w[h0] != t.w[0] || t.w[h1] != t.w[0] || h0 == h1) return false;
+      if ((eg[i] >= 0 && eg[i] != h0) || (ig[j] >= 0 && ig[j] != h1)) return false;
+      eg[i] = h0;
+      ig[j] = h1;
+    }
+  std::vector<int32_t> all(eg);
+  all.insert(all.end(), ig.begin(), ig.end());
+  std::sort(all.begin(), all.end());
+  return std::adjacent_find(all.begin(), all.end()) == all.end();
+}
+
 }  // namespace
 
 std::string spst_plan(const Topology &topo, const int32_t *part, const Relation &rel,
-                      uint64_t seed, Plan *out) {
+                      uint64_t seed, Plan *out, bool allow_fast) {
   auto t0 = std::chrono::steady_clock::now();
   const int m = topo.m;
   Plan &P = *out;
@@ -114,6 +141,40 @@ std::string spst_plan(const Topology &topo, const int32_t *part, const Relation 
     }
   }
   const int H = (int)topo.w.size();
+  if (allow_fast && uniform_switch(topo)) {
+    // the closed form of SPST on the uniform switch (above): every vertex's tree is the star
+    // owner -> each requester (ascending id: the canonical edge order), built in parallel
+    const int64_t NV = (int64_t)order.size();
+    P.e_ptr.assign(NV + 1, 0);
+    for (int64_t i = 0; i < NV; ++i)
+      P.e_ptr[i + 1] = P.e_ptr[i] + (rel.d_ptr[order[i] + 1] - rel.d_ptr[order[i]]);
+    const int64_t NE = P.e_ptr[NV];
+    P.e_parent.assign(NE, 0);
+    P.e_child.assign(NE, 0);
+    P.e_stage.assign(NE, 1);
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < NV; ++i) {
+      const int64_t u = order[i];
+      int64_t e = P.e_ptr[i];
+      for (int64_t q = rel.d_ptr[u]; q < rel.d_ptr[u + 1]; ++q, ++e) {
+        P.e_parent[e] = part[u];
+        P.e_child[e] = rel.d_gpu[q];
+      }
+    }
+    std::vector<int64_t> out_rows(m, 0), in_rows(m, 0);
+    for (int64_t u = 0; u < rel.n; ++u)
+      for (int64_t q = rel.d_ptr[u]; q < rel.d_ptr[u + 1]; ++q) {
+        ++out_rows[part[u]];
+        ++in_rows[rel.d_gpu[q]];
+      }
+    int64_t mx = 0;
+    for (int d = 0; d < m; ++d) mx = std::max(mx, std::max(out_rows[d], in_rows[d]));
+    P.n_stages = NE > 0 ? 1 : 0;
+    P.cost = mx * topo.w[0];
+    P.closed_form = true;
+    P.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    return "";
+  }
   // c_h^k and t^k, k in 1..m-1 (row 0 unused)
   std::vector<int64_t> load((size_t)m * H, 0);
   std::vector<int64_t> tk(m, 0);
@@ -216,6 +277,29 @@ std::string spst_plan(const Topology &topo, const int32_t *part, const Relation 
           const int64_t v = ld[h] * topo.w[h];
           if (v > tk[k]) tk[k] = v;
         }
+      }
+    }
+    // canonical edge order within T_u: (stage, child) — a tree is a set of edges; this order
+    // keeps parents before children (R26)
+    {
+      const int64_t b = P.e_ptr.back(), e = (int64_t)P.e_parent.size();
+      int64_t idx[kMaxRanks];
+      int32_t pp[kMaxRanks], cc[kMaxRanks], kk[kMaxRanks];
+      const int n = (int)(e - b);
+      for (int i = 0; i < n; ++i) idx[i] = b + i;
+      std::sort(idx, idx + n, [&](int64_t x, int64_t y) {
+        return P.e_stage[x] != P.e_stage[y] ? P.e_stage[x] < P.e_stage[y]
+                                            : P.e_child[x] < P.e_child[y];
+      });
+      for (int i = 0; i < n; ++i) {
+        pp[i] = P.e_parent[idx[i]];
+        cc[i] = P.e_child[idx[i]];
+        kk[i] = P.e_stage[idx[i]];
+      }
+      for (int i = 0; i < n; ++i) {
+        P.e_parent[b + i] = pp[i];
+        P.e_child[b + i] = cc[i];
+        P.e_stage[b + i] = kk[i];
       }
     }
     P.e_ptr.push_back((int64_t)P.e_parent.size());

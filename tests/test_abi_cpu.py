@@ -347,3 +347,24 @@ def test_multicast_lowering_host(m, mc):
                             [Gr[g.req_ptr[d]:g.req_ptr[d + 1]] for d in range(m)], R, g.part, loc)
     for d in range(m):
         assert np.array_equal(out[ro[d]:ro[d + 1]].view(np.uint32), Bf[d].view(np.uint32))
+
+
+@pytest.mark.parametrize("m,explicit", [(2, False), (4, False), (8, False), (8, True), (16, False)])
+def test_uniform_closed_form_equals_spst_loop(m, explicit):
+    """Planning at scale (NEXT-4): on the uniform switch model SPST's result is the direct star of
+    every vertex (DESIGN.md §11 proof), computed in parallel.  It must equal Algorithm 1's loop
+    (option spst_fast = 0) edge for edge, with the same t(S); the topology may also be given
+    explicitly (dgcl_set_topology with synth.uniform_nvswitch)."""
+    import paper_conf_eurosys_cai0wmcy21_b200 as D
+    g = synth.make_graph(4000, 50000, m, graph_seed=70 + m, part_seed=71)
+    plans, costs = [], []
+    for fast in (1, 0):
+        ctx = D.loopback(m, g.part, [8], device=-1)
+        ctx.set_option("spst_fast", fast)
+        ctx.build_plan(g.req_ptr, g.req_ids, seed=13,
+                       topology=synth.uniform_nvswitch(m) if explicit else None)
+        plans.append(ctx.plan_export())
+        costs.append(ctx.plan_info()["model_cost_ticks"])
+        ctx.destroy()
+    assert np.array_equal(plans[0], plans[1]) and costs[0] == costs[1]
+    assert np.all(plans[0][:, 3] == 1)
