@@ -243,10 +243,6 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "l2_policy"      L2 eviction hints of the bulk-copy executor, bit mask (any time): 1 data stores
  *                    evict_first (default), 2 COPY source reads evict_last, 4 COPY source reads
  *                    evict_first, 8 FOLD operand reads evict_first
- *   "item_order"     bulk-copy executor item assignment (any time): 0 round-robin, 1 dynamic
- *                    claiming from a launch-wide counter, 2 rotated rounds, 3 round-robin for the
- *                    first 3/4 of the items and dynamic claiming for the tail, 4 (default) 3 for
- *                    launches of <= 12 groups, else 0
  *   "sys_scope"      loopback contexts: 1 = use the multi-GPU system-scope flag protocol (A/B;
  *                    default 0: device scope, exact when every rank is on this GPU)
  *   "multicast"      NVSwitch multicast of high-fan-out rows (see dgcl_multicast_open): 0 off

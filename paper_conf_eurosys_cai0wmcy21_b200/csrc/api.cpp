@@ -46,8 +46,6 @@ struct Program {
   int g4_kinds = 0;        // source kinds of its gather4 items (tensor maps the launch needs)
   bool tree = false;       // carries tree-order FOLD programs (kTermRankTree)
   TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
-  mutable uint64_t claims = 0;  // dynamic item claiming: claims consumed by earlier launches
-  int n_groups = 0;             // data groups (COPY / FOLD / FANOUT) of the program
 };
 
 }  // namespace
@@ -89,12 +87,6 @@ struct dgcl_ctx {
   DevItem *d_items = nullptr;
   DevRun *d_runs = nullptr;
   uint32_t *d_sterms = nullptr;
-  uint64_t *d_claims = nullptr;  // one item-claim counter per program (dynamic claiming)
-  // bulk-copy executor item assignment: 0 round-robin; 1 dynamic claiming; 2 rotated rounds;
-  // 3 round-robin for the first 3/4 of the items (whole rounds), dynamic claiming for the rest;
-  // 4 auto: 3 for launches of few groups (<= 12: the 2- and 4-way forwards, whose per-group item
-  // costs differ: Web-Google-2 0.228 -> 0.199 ms), 0 otherwise (Reddit forward 3 % slower with 3)
-  int item_order = 4;
   bool spst_fast = true;  // uniform switch: SPST's closed form (parallel) instead of the loop
   int64_t run_bytes = 0;
   bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
@@ -437,11 +429,6 @@ void build_programs(dgcl_ctx *c) {
           if (it.op == OP_FANOUT) P.op_mask |= kMaskFanout;
         }
         P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
-        P.n_groups = 0;
-        for (int32_t gi : G) {
-          const int op = L.groups[gi].op;
-          P.n_groups += op == OP_COPY || op == OP_FOLD || op == OP_FANOUT;
-        }
         P.g4_kinds = 0;
         P.tree = false;
         for (const DevItem &it : P.items)
@@ -841,14 +828,6 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     }
     encode_g4(Pp, pg.g4_kinds);
     const int grid = (int)std::min<int64_t>(std::max(1, grid_all / grid_div), Pp.n_items);
-    Pp.item_order = c->item_order == 2 ? 1 : 0;
-    const int order = c->item_order == 4 ? (pg.n_groups <= 12 ? 3 : 0) : c->item_order;
-    if (Pp.use_tma && (order == 1 || order == 3) && c->d_claims) {
-      Pp.claim = c->d_claims + (&pg - c->progs.data());
-      Pp.claim_base = pg.claims;
-      Pp.claim_from = order == 1 ? 0 : (int64_t)Pp.n_items * 3 / 4 / grid * grid;
-      pg.claims += (uint64_t)(Pp.n_items - Pp.claim_from) + (uint64_t)grid;
-    }
     return launch_executor(Pp, grid, block, st);
   };
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
@@ -1049,7 +1028,6 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   if ((s = upload(c, &c->d_items, all)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_runs, all_runs)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_sterms, all_sterms)) != DGCL_OK) return s;
-  if ((s = upload(c, &c->d_claims, std::vector<uint64_t>(c->progs.size(), 0))) != DGCL_OK) return s;
   c->run_bytes = (int64_t)(all_runs.size() * sizeof(DevRun) + all_sterms.size() * 4);
   if (c->trace)
     for (Program &p : c->progs)
@@ -1591,11 +1569,6 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     c->spst_fast = value != 0;
     return DGCL_OK;
   }
-  if (k == "item_order") {  // bulk-copy executor: 0 round-robin, 1 dynamic claiming, 2 rotated
-    if (value < 0 || value > 4) return fail(c, DGCL_EINVAL, "item_order in 0..4");
-    c->item_order = (int)value;
-    return DGCL_OK;
-  }
   if (k == "sys_scope") {  // loopback: 1 = the multi-GPU system-scope flag protocol (A/B)
     c->force_sys_scope = value != 0;
     return DGCL_OK;
@@ -1805,7 +1778,6 @@ dgcl_status dgcl_destroy(dgcl_ctx *c) {
     cudaFree(c->d_items);
     cudaFree(c->d_runs);
     cudaFree(c->d_sterms);
-    cudaFree(c->d_claims);
     for (Program &p : c->progs)
       if (p.d_trace) cudaFree(p.d_trace);
     for (auto &kv : c->stages) {

@@ -42,7 +42,6 @@ constexpr int kHdrInfo = 64;         // stage: int32 info words after the 64-B i
 constexpr int kTabTp = 128;          // stage: term_ptr window (FOLD)
 constexpr int kTabDst = 2176;        // stage: destination-row window
 constexpr int kDescSlots = 8;        // producer descriptor ring
-constexpr int kPendSlots = 32;       // distinct done counters pending between two FLUSH markers
 static_assert(kDescAhead > kMetaAhead && kDescAhead < kDescSlots && kMetaAhead < kMetaSlots,
               "prefetch distances");
 // shared-memory carve-up (internal.h, tma_smem_bytes): offsets depend on the launch geometry
@@ -187,20 +186,6 @@ __device__ __forceinline__ void consumer_barrier(unsigned *count, volatile unsig
     __threadfence_block();
   }
   __syncwarp();
-}
-
-// pending-count table (one consumer thread at a time): add rows to key's entry, or append it
-// (the producer guarantees at most kPendSlots distinct keys between two FLUSH markers)
-__device__ __forceinline__ void pend_add(uint32_t *keys, uint32_t *cnt, int &n, uint32_t key,
-                                         uint32_t rows) {
-  int i = 0;
-  while (i < n && keys[i] != key) ++i;
-  if (i == n) {
-    keys[n] = key;
-    cnt[n] = 0;
-    ++n;
-  }
-  cnt[i] += rows;
 }
 
 // non-blocking: are all counter waits of I already satisfied?
@@ -472,8 +457,8 @@ __device__ __forceinline__ void store_copy_mc(const ExecParams &P, const DevItem
 // consumers: FANOUT item — the staged rows stored into all their receivers' rows (halo or relay
 // staging, library-owned: whole 16-B chunks).  Flat (destination pair, chunk) index space over the
 // consumer threads, kUnroll independent chunks per thread in flight (as store_copy); with
-// signalling on, the thread holding a pair's chunk 0 counts it for its receiver in s_pend[16]
-// (the caller moves them into the pending-count table after the item)
+// signalling on, the thread holding a pair's chunk 0 counts it for its receiver (published at the
+// next FLUSH / END)
 __device__ __forceinline__ void store_fanout(const ExecParams &P, const DevItem &I,
                                              const uint8_t *st, uint32_t tid, uint32_t T,
                                              uint32_t *s_pend, uint64_t pol_st) {
@@ -493,7 +478,7 @@ __device__ __forceinline__ void store_fanout(const ExecParams &P, const DevItem 
       const uint32_t d = pw[2 * j], r = pw[2 * j + 1] - src0;
       const BufRef D = P.buf[(d & kFanRelay) ? K_RELAY : K_HALO][d >> 28];
       s2g(D.ptr + (int64_t)(d & kFanRowMask) * D.pitch, ops + r * r16, r16, pol_st);
-      if (sig) atomicAdd(&s_pend[d >> 28], 1u);
+      if (sig) atomicAdd(&s_pend[I.exec_rank * kMaxRanks + (d >> 28)], 1u);
     }
     if (tid < np) {
       bulk_commit();
@@ -512,7 +497,7 @@ __device__ __forceinline__ void store_fanout(const ExecParams &P, const DevItem 
         const BufRef D = P.buf[(d & kFanRelay) ? K_RELAY : K_HALO][d >> 28];
         st_v4(D.ptr + (int64_t)(d & kFanRowMask) * D.pitch + col * 16,
               lds_v4(ops + r * r16 + col * 16));
-        if (sig && col == 0) atomicAdd(&s_pend[d >> 28], 1u);
+        if (sig && col == 0) atomicAdd(&s_pend[I.exec_rank * kMaxRanks + (d >> 28)], 1u);
       }
     }
   }
@@ -863,24 +848,14 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   uint8_t *stages = dsmem + kStageOff;
   // rows stored since the last flush per (source, receiver), their counter family, and the
   // consumer barrier words: carved from the dynamic region (no static shared memory)
-  // pending done counts (published at FLUSH / END): up to kPendSlots (counter key, rows) entries,
-  // key = receiver << 16 | counter index (ctr_index, or kMcCtrBase + owner for the multicast
-  // counters); the producer bounds the distinct keys between two FLUSH markers
-  uint32_t *s_pkey = reinterpret_cast<uint32_t *>(dsmem + kPendOff);
-  uint32_t *s_pcnt = reinterpret_cast<uint32_t *>(dsmem + kPendOff + 4 * kPendSlots);
-  uint32_t *s_pend = reinterpret_cast<uint32_t *>(dsmem + kPendOff + 8 * kPendSlots);  // fan-out
-  int &s_npend = *reinterpret_cast<int *>(dsmem + kPendOff + 8 * kPendSlots + 64);
-  uint32_t *s_prodkey = reinterpret_cast<uint32_t *>(dsmem + kPendOff + 8 * kPendSlots + 128);
+  uint32_t *s_pend = reinterpret_cast<uint32_t *>(dsmem + kPendOff);
+  int &s_pend_base = *reinterpret_cast<int *>(dsmem + kPendOff + 1024);
   unsigned &s_bar_count = *reinterpret_cast<unsigned *>(dsmem + kPendOff + 1028);
   volatile unsigned &s_bar_gen = *reinterpret_cast<volatile unsigned *>(dsmem + kPendOff + 1032);
   // producer-private: per executing rank, the wait list last found satisfied (counters are
   // monotonic and their targets fixed for the launch, so it stays satisfied: later items of the
   // same (direction, stage, rank) skip the flag reads)
-  // (4 most recent wait lists per executing rank: relay plans with vertex blocks alternate
-  // between the lists of neighbouring (stage, block) runs)
-  int32_t *s_wait_ok = reinterpret_cast<int32_t *>(dsmem + kPendOff + 512);
-  // producer-private: the launch index of the item in each descriptor ring slot
-  uint32_t *s_claim = reinterpret_cast<uint32_t *>(dsmem + kPendOff + 1104);
+  int32_t *s_wait_ok = reinterpret_cast<int32_t *>(dsmem + kPendOff + 1040);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
   // L2 hints (option "l2_policy"): bit 0 data stores evict_first (write-once halo / relay /
@@ -890,12 +865,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   const uint64_t pol_st = (lp & 1) ? policy_evict_first() : 0;
   const uint64_t pol_copy = (lp & 2) ? policy_evict_last() : (lp & 4) ? policy_evict_first() : 0;
   const uint64_t pol_fold = (lp & 8) ? policy_evict_first() : 0;
-  for (int i = threadIdx.x; i < kMaxRanks; i += blockDim.x) s_pend[i] = 0;
+  for (int i = threadIdx.x; i < kMaxRanks * kMaxRanks; i += blockDim.x) s_pend[i] = 0;
   if (threadIdx.x == 0) {
-    s_npend = 0;
+    s_pend_base = 0;
     s_bar_count = 0;
     s_bar_gen = 0;
-    for (int r = 0; r < 4 * kMaxRanks; ++r) s_wait_ok[r] = -1;
+    for (int r = 0; r < kMaxRanks; ++r) s_wait_ok[r] = -1;
     for (int s = 0; s < (int)NS; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], n_cons_warps);
@@ -911,49 +886,13 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     // item q of this CTA is P.items[blockIdx.x + q * gridDim.x]; its descriptor is bulk-copied
     // into ring slot q % kDescSlots kDescAhead items ahead, its row runs into meta slot
     // q % kMetaSlots kMetaAhead items ahead, so their latency never stalls the issue loop
-    // Items are taken in list order: statically (round q: CTA b takes list position q * G + b,
-    // or q * G + (b + q) % G with rotated rounds) up to position claim_from, then — with
-    // P.claim — claimed dynamically from a launch-wide counter.  Claims hand out positions in
-    // increasing order, so every CTA's queue stays in list (stage) order and the earliest
-    // unfinished item can always run: deadlock-free like the static order; a dynamic tail lets
-    // CTAs that drew cheaper items take more (per-item costs differ with the row runs).
-    // nend = the first queue position without an item (known once a claim fails).
     const uint32_t G = gridDim.x;
-    const uint32_t S0 = P.claim ? (uint32_t)P.claim_from : (uint32_t)P.n_items;
-    const uint32_t R = S0 / G, rem = S0 % G;
-    const uint32_t nstat = P.item_order == 1 ? R + ((blockIdx.x + R) % G < rem ? 1u : 0u)
-                           : blockIdx.x < S0 ? (S0 - blockIdx.x + G - 1) / G
-                                             : 0;
-    uint32_t nend = P.claim ? 0xffffffffu : nstat, nreq = 0;
-    auto request_desc = [&](uint32_t q) -> bool {  // lane 0, after a proxy fence
-      uint64_t idx;
-      if (q >= nstat) {  // (only with P.claim)
-        idx = S0 + atomicAdd(reinterpret_cast<unsigned long long *>(P.claim), 1ull) - P.claim_base;
-        if (idx >= (uint64_t)P.n_items) return false;
-      } else if (P.item_order == 1) {
-        idx = (uint64_t)q * G + (blockIdx.x + q) % G;
-      } else {
-        idx = blockIdx.x + (uint64_t)q * G;
-      }
+    const uint32_t nmine =
+        blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
+    auto request_desc = [&](uint32_t q) {  // lane 0, after a proxy fence
       const uint32_t s = q % kDescSlots;
-      s_claim[s] = (uint32_t)idx;
       mbar_expect_tx(&descb[s], (uint32_t)sizeof(DevItem));
-      bulk_g2s(descs + s, P.items + idx, (uint32_t)sizeof(DevItem), &descb[s]);
-      return true;
-    };
-    // request descriptors nreq .. upto-1 (fewer once the items run out); warp-uniform
-    auto request_upto = [&](uint32_t upto) {
-      int e = -1;
-      if (lane == 0)
-        for (uint32_t q = nreq; q < upto && q < nend; ++q)
-          if (!request_desc(q)) {
-            e = (int)q;
-            break;
-          }
-      e = __shfl_sync(0xffffffffu, e, 0);
-      if (e >= 0) nend = (uint32_t)e;
-      nreq = upto < nend ? upto : nend;
-      __syncwarp();
+      bulk_g2s(descs + s, P.items + blockIdx.x + q * G, (uint32_t)sizeof(DevItem), &descb[s]);
     };
     auto desc_ready = [&](uint32_t q) -> const DevItem & {
       mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
@@ -964,28 +903,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     bool ok = true;
     uint32_t ready_ok = 0;  // lane 0: destinations whose ready word reached seq (bit per rank)
     auto known_sources = [&](const DevItem &I) {
-      if (I.wait_n == 0) return true;
-      const int32_t *c = s_wait_ok + 4 * I.exec_rank;
-      return c[0] == I.wait_off || c[1] == I.wait_off || c[2] == I.wait_off || c[3] == I.wait_off;
+      return I.wait_n == 0 || s_wait_ok[I.exec_rank] == I.wait_off;
     };
-    // counter keys of the signalling items issued since the last FLUSH (s_prodkey, lane 0)
-    int npk = 0;
-    bool pend = false;
-    // keys item I adds (a fan-out item: one per possible receiver); returns how many are new
-    auto new_keys = [&](const DevItem &I, bool add) -> int {
-      int nnew = 0;
-      for (int d = 0; d < (I.op == OP_FANOUT ? P.world : 1); ++d) {
-        const int dst = I.op == OP_FANOUT ? d : I.dst_rank;
-        if (I.op == OP_FANOUT && d == I.exec_rank) continue;
-        const uint32_t key = (uint32_t)dst << 16 | (uint32_t)I.sig_ctr;
-        bool found = false;
-        for (int i = 0; i < npk && !found; ++i) found = s_prodkey[i] == key;
-        if (found) continue;
-        ++nnew;
-        if (add) s_prodkey[npk++] = key;
-      }
-      return nnew;
-    };
+    bool pend = false;  // signalling items issued since the last FLUSH
+    int pend_key = -1;  // their counter family: ctr_index(dir, stage, 0)
     auto emit_marker = [&](uint8_t op) {  // header-only stage: FLUSH or END
       uint32_t stage, use;
       ring_pos(k, NS, stage, use);
@@ -1002,16 +923,17 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     // consumers, ordered by the empty barrier) the stage come before every bulk copy into them.
     // Prefetches are issued after the item, so the item's fence covers them too.
     fence_proxy_async_smem();
-    request_upto((uint32_t)kDescAhead);
-    for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nend; ++q) {
+    if (lane == 0)
+      for (uint32_t q = 0; q < (uint32_t)kDescAhead && q < nmine; ++q) request_desc(q);
+    for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nmine; ++q) {
       const DevItem Iq = desc_ready(q);
       if (lane == 0) issue_meta(P, Iq, meta_of(q), &metab[q % kMetaSlots]);
     }
-    for (; m < nend; ++m) {
+    for (; m < nmine; ++m) {
       const DevItem I = desc_ready(m);  // registers: no shared-memory reload per field
       const DevItem *Ism = &descs[m % kDescSlots];
       bool fenced = false;
-      const uint32_t gidx = s_claim[m % kDescSlots];  // the item's index in the launch
+      const uint32_t gidx = blockIdx.x + m * G;  // the item's index in the launch
       if (P.trace && lane == 0) {
         uint32_t smid;
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
@@ -1030,7 +952,6 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         if (pend) {
           emit_marker(OP_FLUSH);
           pend = false;
-          npk = 0;
         }
         int w = 1;
         if (lane == 0 && !known_sources(I)) w = wait_item_sources(P, I, 200000 + I.group) ? 1 : 0;
@@ -1038,8 +959,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         if (!ok) break;
       } else if (I.op == OP_COPY || I.op == OP_FOLD || I.op == OP_FANOUT) {
         // Done counts are published in batches (FLUSH markers): before this producer could
-        // block on a wait, and when this item's counters would not fit the pending table.
+        // block on a wait, and whenever the counter family (direction, stage) changes.
         const bool sig = (I.flags & kItemSignal) != 0;
+        const int key = sig ? I.sig_ctr - I.exec_rank : -1;
         if (pend) {
           int ready = 1;
           if (lane == 0) {
@@ -1052,14 +974,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
                 if (s != I.exec_rank && !((ready_ok >> s) & 1u))
                   ready = ld_acquire(P.flags[I.exec_rank] + kReadyBase + s, P.sys_scope) >= P.seq;
           }
-          int full_tab = 0;
-          if (lane == 0 && sig) full_tab = npk + new_keys(I, false) > kPendSlots ? 1 : 0;
           ready = __shfl_sync(0xffffffffu, ready, 0);
-          full_tab = __shfl_sync(0xffffffffu, full_tab, 0);
-          if (!ready || full_tab) {
+          if (!ready || (sig && key != pend_key)) {
             emit_marker(OP_FLUSH);
             pend = false;
-            npk = 0;
           }
         }
         int w = 1;
@@ -1067,13 +985,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           // sources final (stage chaining) and the destination's buffers free (ready word)
           if (!known_sources(I)) {
             w = wait_item_sources(P, I, 100000 + I.group) ? 1 : 0;
-            if (w) {
-              int32_t *c = s_wait_ok + 4 * I.exec_rank;
-              c[3] = c[2];
-              c[2] = c[1];
-              c[1] = c[0];
-              c[0] = I.wait_off;
-            }
+            if (w) s_wait_ok[I.exec_rank] = I.wait_off;
           }
           if (w && P.use_ready && I.ready_rank >= 0 && !((ready_ok >> I.ready_rank) & 1u)) {
             w = wait_geq(P.flags[I.exec_rank] + kReadyBase + I.ready_rank, P.seq, P,
@@ -1102,15 +1014,14 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         ++k;
         if (sig) {
           pend = true;
-          if (lane == 0) new_keys(I, true);
-          npk = __shfl_sync(0xffffffffu, npk, 0);
+          pend_key = key;
         }
       }
       __syncwarp();
       // prefetch: descriptor kDescAhead items ahead, row runs / segments kMetaAhead items ahead
-      if (!fenced && (m + kMetaAhead < nend || m + kDescAhead < nend)) fence_proxy_async_smem();
-      if (m + kDescAhead < nend) request_upto(m + kDescAhead + 1);
-      if (m + kMetaAhead < nend) {
+      if (!fenced && (m + kMetaAhead < nmine)) fence_proxy_async_smem();
+      if (lane == 0 && m + kDescAhead < nmine) request_desc(m + kDescAhead);
+      if (m + kMetaAhead < nmine) {
         const uint32_t q = m + kMetaAhead;
         const DevItem In = desc_ready(q);
         if (lane == 0) issue_meta(P, In, meta_of(q), &metab[q % kMetaSlots]);
@@ -1120,9 +1031,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       // watchdog abort: descriptor / metadata copies still in flight land before the CTA leaves
       // (item m aborted before its own prefetches: requested so far are descriptors < m +
       // kDescAhead and metadata < m + kMetaAhead)
-      for (uint32_t q = m; q < nreq; ++q)
+      for (uint32_t q = m; q < m + kDescAhead && q < nmine; ++q)
         mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
-      for (uint32_t q = m; q < m + kMetaAhead && q < nend; ++q)
+      for (uint32_t q = m; q < m + kMetaAhead && q < nmine; ++q)
         mbar_wait(&metab[q % kMetaSlots], (q / kMetaSlots) & 1u);
     }
     // END marker: consumers drain every issued stage, publish pending counts, then stop
@@ -1146,16 +1057,19 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         }
         fence_scope(P.sys_scope);
         consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
-        for (uint32_t i = tid; i < (uint32_t)s_npend; i += T) {
-          const uint32_t key = s_pkey[i], amt = s_pcnt[i];
-          const uint32_t ctr = key & 0xffffu;
-          if (ctr >= (uint32_t)kMcCtrBase)  // multicast sends: every GPU's copy of the counter
-            mc_publish(P, (int)(ctr - kMcCtrBase), amt);
-          else
-            red_release_add(P.flags[key >> 16] + ctr, amt, P.sys_scope);
+        // (strided: there are fewer consumer threads than (source, receiver) entries)
+        for (uint32_t i = tid; i < (uint32_t)(kMaxRanks * kMaxRanks); i += T) {
+          const uint32_t amt = s_pend[i];
+          if (amt) {
+            const int ex = (int)(i / kMaxRanks), dst = (int)(i % kMaxRanks);
+            if (s_pend_base >= kMcCtrBase)  // multicast sends: every GPU's copy of ex's counter
+              mc_publish(P, ex, amt);
+            else
+              red_release_add(P.flags[dst] + s_pend_base + ex, amt, P.sys_scope);
+            s_pend[i] = 0;
+          }
         }
         consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
-        if (tid == 0) s_npend = 0;
         if (I.op == OP_END) break;
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[stage]);
@@ -1191,17 +1105,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         }
       } else if ((kMask & kMaskFanout) && I.op == OP_FANOUT) {
         store_fanout(P, I, st, tid, T, s_pend, pol_st);
-        if (I.flags & kItemSignal) {  // the item's per-receiver counts -> the pending table
-          consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
-          if (tid == 0)
-            for (int d = 0; d < P.world; ++d)
-              if (s_pend[d]) {
-                pend_add(s_pkey, s_pcnt, s_npend, (uint32_t)d << 16 | (uint32_t)I.sig_ctr,
-                         s_pend[d]);
-                s_pend[d] = 0;
-              }
-          consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
-        }
+        if ((I.flags & kItemSignal) && tid == 0) s_pend_base = I.sig_ctr - I.exec_rank;
       } else if ((kMask & kMaskDirect) && I.op == OP_COPY) {
         store_copy_direct(P, I, st, tid, T);
       } else if ((kMask & kMaskStaged) && is_staged(I)) {
@@ -1219,10 +1123,11 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       }
       if (P.trace && tid == 0)  // this warp's share of the item is stored
         P.trace[reinterpret_cast<const int32_t *>(st + kHdrInfo)[2]].t_done = globaltimer();
-      if ((I.flags & kItemSignal) && tid == 0 && I.op != OP_FANOUT)
+      if ((I.flags & kItemSignal) && tid == 0 && I.op != OP_FANOUT) {
         // counted now, published by the next FLUSH / END marker (done flags)
-        pend_add(s_pkey, s_pcnt, s_npend, (uint32_t)I.dst_rank << 16 | (uint32_t)I.sig_ctr,
-                 (uint32_t)I.rows);
+        atomicAdd(&s_pend[I.exec_rank * kMaxRanks + I.dst_rank], (uint32_t)I.rows);
+        s_pend_base = I.sig_ctr - I.exec_rank;
+      }
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // this warp is done reading the stage
     }

@@ -202,13 +202,6 @@ struct alignas(64) ExecParams {
   struct TraceRec *trace;  // option "trace": one record per item of this launch, or nullptr
   int32_t l2_policy;       // option "l2_policy": L2 eviction hints of the bulk-copy executor
   int32_t sys_scope;       // 1: flags / fences at system scope (peers are other GPUs); 0: .gpu
-  // bulk-copy executor, dynamic item claiming: a launch-wide counter (nullptr = static
-  // order).  Every CTA claims until one claim fails, so a launch consumes exactly
-  // n_items - claim_from + grid claims; claim_base = the counter's value at launch (host)
-  uint64_t *claim;
-  uint64_t claim_base;
-  int32_t item_order;      // static part: 0 round-robin, 1 rotated rounds
-  int64_t claim_from;      // with claim: list positions >= claim_from are claimed dynamically
   // multicast (option "multicast"): the multicast flag page (multimem reductions), every rank's
   // unicast flag page (acquire waits; loopback: each virtual rank's copy), and whether the
   // multicast is emulated by one store / reduction per rank (loopback: no multicast object)
