@@ -122,7 +122,8 @@ struct dgcl_ctx {
   bool force_sys_scope = false;       // loopback with the multi-GPU (.sys) flag scope (A/B)
   bool threads_set = false, ctas_set = false;  // user overrides of the CTA shape
   int sm_count = 148;  // SMs of the device (B200 until queried), for cutting small stages
-  std::map<std::pair<int, int>, int> tma_ctas;  // (geo, block) -> co-resident CTAs per SM
+  // (geo, block, instance mask or -1) -> co-resident CTAs per SM
+  std::map<std::tuple<int, int, int>, int> tma_ctas;
   int n_prog_ranks = 1;        // programs per (layer, dir)
 
   uint64_t seq = 0, epoch[2] = {0, 0};
@@ -450,9 +451,7 @@ void build_programs(dgcl_ctx *c) {
         }
         // auto: DUAL (two producer warps per SM) unless the launch is bulk-copy friendly —
         // copies only, >= 8 KB per bulk operation (long runs of rows) — or carries unstaged folds
-        // (consumer gathers, which want more consumer warps), or chains stages on flags (relay
-        // plans: DUAL's forward time was bimodal, 0.83 / 2.1 ms, on the Web-Google dgx1_like
-        // plan, WIDE a steady 0.9-1.1 ms); see TmaGeometry
+        // (consumer gathers, which want more consumer warps); see TmaGeometry
         build(P, r, 1);
         int64_t ops = 0, bytes = 0;
         bool waits = false;
@@ -467,8 +466,10 @@ void build_programs(dgcl_ctx *c) {
           ops += (it.flags & kItemGather4) ? (it.rows + 3) / 4 : it.nterms;
         }
         const bool copy_only = (P.op_mask & ~(kMaskCopy | kMaskFanout)) == 0;
-        if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & (kMaskFold | kMaskTree)) ||
-            waits)
+        // (relay forwards chained on flags now run DUAL too: 1.08 -> 1.01 ms on the Web-Google
+        // ring plan, 0.83 -> 0.81 dgx1_like, no bimodality with device-scope flags, A/B r2j/r2k)
+        (void)waits;
+        if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & (kMaskFold | kMaskTree)))
           build(P, r, 0);
       }
       // per-rank loopback: the ranks' launches run concurrently on one device and their CTAs wait
@@ -512,6 +513,12 @@ int tma_block(const dgcl_ctx *c, const Program &pg) {
   if (pg.geo == 0 && (pg.op_mask & (kMaskFold | kMaskTree)))
     return pg.op_mask == kMaskFold && pg.fold_wide && !pg.tree ? 1024 : 512;
   return G.threads;
+}
+
+// occupancy key of a program's launch: its own instance when it runs alone on the device; the
+// worst case over instances when per-rank loopback launches share the device concurrently
+int occ_mask(const dgcl_ctx *c, const Program &pg) {
+  return (c->loopback && c->lb_flags == DGCL_LOOPBACK_PER_RANK) ? -1 : pg.op_mask;
 }
 
 dgcl_status check_dead(dgcl_ctx *c) {
@@ -807,7 +814,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     Pp.trace = pg.d_trace;
     const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
     const int tblock = tma_block(c, pg);
-    const auto occ = c->tma_ctas.find({pg.geo, tblock});
+    const auto occ = c->tma_ctas.find({pg.geo, tblock, occ_mask(c, pg)});
     const int tctas = occ == c->tma_ctas.end() ? 0 : occ->second;
     // (sm_budget: the grid covers only that many SMs, still co-resident; the other SMs run
     // whatever the caller overlaps with the exchange)
@@ -1047,14 +1054,15 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   // bulk-copy executor: co-resident CTAs per SM for every (geometry, CTA size) a program uses
   for (const Program &pg : c->progs) {
     const int block = tma_block(c, pg);
-    if (c->tma_ctas.count({pg.geo, block})) continue;
+    const int mk = occ_mask(c, pg);
+    if (c->tma_ctas.count({pg.geo, block, mk})) continue;
     const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
     int n = 0;
-    e = executor_tma_occupancy(block, tma_smem_bytes(G), &n);
+    e = executor_tma_occupancy(mk, block, tma_smem_bytes(G), &n);
     if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");
     n = std::min(n, G.ctas_per_sm);
     if (c->ctas_set) n = std::min(n, c->ctas_per_sm);
-    c->tma_ctas[{pg.geo, block}] = n;
+    c->tma_ctas[{pg.geo, block, mk}] = n;
   }
   if (c->ctas_per_sm <= 0) c->ctas_per_sm = std::min(occ, 4);
   c->ctas_per_sm = std::max(1, std::min(c->ctas_per_sm, occ));

@@ -477,7 +477,7 @@ int launch_barrier(const ExecParams &p, int first, int count, void *stream) {
 
 // executor_tma.cu
 int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream);
-int tma_executor_occupancy(int block, size_t smem_bytes, int *ctas_per_sm);
+int tma_executor_occupancy(int op_mask, int block, size_t smem_bytes, int *ctas_per_sm);
 
 int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   if (grid <= 0) return 0;
@@ -506,8 +506,8 @@ int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   return (int)cudaGetLastError();
 }
 
-int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm) {
-  return tma_executor_occupancy(block, smem_bytes, ctas_per_sm);
+int executor_tma_occupancy(int op_mask, int block, size_t smem_bytes, int *ctas_per_sm) {
+  return tma_executor_occupancy(op_mask, block, smem_bytes, ctas_per_sm);
 }
 
 int executor_occupancy(int block, int *ctas_per_sm) {

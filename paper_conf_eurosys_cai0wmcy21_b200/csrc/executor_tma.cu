@@ -1186,24 +1186,44 @@ int launch_tma_executor(const ExecParams &p, int grid, int block, void *stream) 
   }
 }
 
-// co-resident CTAs per SM of the worst-case instance at this geometry (the persistent grid must
-// be fully resident: CTAs wait on flags other CTAs set)
-int tma_executor_occupancy(int block, size_t smem_bytes, int *ctas_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kAll>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)kSmemMax);
-  if (e != cudaSuccess) return (int)e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, executor_tma_kernel<kAll>,
-                                                    block, smem_bytes);
-  if (e != cudaSuccess || block != 1024) return (int)e;
-  int c2 = 0;
-  e = cudaFuncSetAttribute(executor_tma_kernel<kMaskFold, 1024>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemMax);
+namespace {
+template <int kMask, int kThreads = 512>
+int occupancy_of(int block, size_t smem_bytes, int *ctas_per_sm) {
+  cudaError_t e = cudaFuncSetAttribute(executor_tma_kernel<kMask, kThreads>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemMax);
   if (e == cudaSuccess)
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c2, executor_tma_kernel<kMaskFold, 1024>,
-                                                      1024, smem_bytes);
-  *ctas_per_sm = c2;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm,
+                                                      executor_tma_kernel<kMask, kThreads>, block,
+                                                      smem_bytes);
   return (int)e;
+}
+}  // namespace
+
+// co-resident CTAs per SM (the persistent grid must be fully resident: CTAs wait on flags other
+// CTAs set) of the instance launch_tma_executor picks for op_mask, or (op_mask < 0) of the
+// worst-case instance — for launches that share the device with other programs' launches
+int tma_executor_occupancy(int op_mask, int block, size_t smem_bytes, int *ctas_per_sm) {
+  switch (op_mask) {
+    case kMaskCopy: return occupancy_of<kMaskCopy>(block, smem_bytes, ctas_per_sm);
+    case kMaskFanout: return occupancy_of<kMaskFanout>(block, smem_bytes, ctas_per_sm);
+    case kMaskFanout | kMaskCopy:
+      return occupancy_of<kMaskFanout | kMaskCopy>(block, smem_bytes, ctas_per_sm);
+    case kMaskTree: return occupancy_of<kMaskTree>(block, smem_bytes, ctas_per_sm);
+    case kMaskTree | kMaskStaged:
+      return occupancy_of<kMaskTree | kMaskStaged>(block, smem_bytes, ctas_per_sm);
+    case kMaskFold:
+      if (block == 1024) return occupancy_of<kMaskFold, 1024>(1024, smem_bytes, ctas_per_sm);
+      return occupancy_of<kMaskFold>(block, smem_bytes, ctas_per_sm);
+    case kMaskCopy | kMaskFold:
+      return occupancy_of<kMaskCopy | kMaskFold>(block, smem_bytes, ctas_per_sm);
+    case kMaskStaged: return occupancy_of<kMaskStaged>(block, smem_bytes, ctas_per_sm);
+    case kMaskCopy | kMaskStaged:
+      return occupancy_of<kMaskCopy | kMaskStaged>(block, smem_bytes, ctas_per_sm);
+    default: break;
+  }
+  int e = occupancy_of<kAll>(block == 1024 ? 512 : block, smem_bytes, ctas_per_sm);
+  if (e != 0 || block != 1024) return e;
+  return occupancy_of<kMaskFold, 1024>(1024, smem_bytes, ctas_per_sm);
 }
 
 }  // namespace dgcl

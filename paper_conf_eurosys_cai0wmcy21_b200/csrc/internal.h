@@ -253,7 +253,16 @@ struct TmaGeometry {
   int32_t stages, stage_bytes, meta_bytes, threads, ctas_per_sm, max_item_rows;
 };
 constexpr TmaGeometry kGeoWide = {3, 64 * 1024, 8 * 1024, 256, 1, 464};
-constexpr TmaGeometry kGeoDual = {2, 47 * 1024, 4 * 1024, 256, 2, 240};
+#ifndef DGCL_DUAL_STAGES  // (build-time A/B of the DUAL geometry, tools/build_variant.sh)
+#define DGCL_DUAL_STAGES 2
+#define DGCL_DUAL_STAGE_KB 47
+#define DGCL_DUAL_CTAS 2
+#define DGCL_DUAL_META_KB 4
+#endif
+constexpr TmaGeometry kGeoDual = {DGCL_DUAL_STAGES, DGCL_DUAL_STAGE_KB * 1024,
+                                  DGCL_DUAL_META_KB * 1024, 256, DGCL_DUAL_CTAS,
+                                  DGCL_DUAL_META_KB * 1024 / 16 < 240 ? DGCL_DUAL_META_KB * 1024 / 16
+                                                                       : 240};
 constexpr int kMaxTmaStages = 3;
 constexpr int kStageHdrBytes = 4096;
 constexpr int kTmaBufBytes = kGeoWide.stage_bytes;          // largest stage
@@ -262,7 +271,7 @@ constexpr size_t tma_smem_bytes(const TmaGeometry &g) {
   return 256 + 4 * (size_t)g.meta_bytes + 8 * 64 + (size_t)g.stages * g.stage_bytes + 1152;
 }
 static_assert(tma_smem_bytes(kGeoWide) <= 227 * 1024, "WIDE: one CTA per SM");
-static_assert(tma_smem_bytes(kGeoDual) <= 113 * 1024, "DUAL: two CTAs per SM");
+static_assert(tma_smem_bytes(kGeoDual) * DGCL_DUAL_CTAS <= 227 * 1024, "DUAL: CTAs per SM");
 static_assert(kGeoWide.max_item_rows * 16 <= kGeoWide.meta_bytes &&
                   kGeoDual.max_item_rows * 16 <= kGeoDual.meta_bytes,
               "a meta slot holds an item's 16-B runs");
@@ -299,6 +308,7 @@ int launch_barrier(const ExecParams &p, int first, int count, void *stream);
 int launch_wait(const ExecParams &p, int exec, int off, int n, void *stream);
 // multicast self-test kernel (dgcl_debug_multicast_selftest): multimem stores + one reduction
 int launch_mc_selftest(void *mc, uint64_t *mcflag, int n16, void *stream);
-int executor_tma_occupancy(int block, size_t smem_bytes, int *ctas_per_sm);  // bulk-copy path
+// bulk-copy path: the instance for op_mask (< 0: the worst case over instances)
+int executor_tma_occupancy(int op_mask, int block, size_t smem_bytes, int *ctas_per_sm);
 
 }  // namespace dgcl
