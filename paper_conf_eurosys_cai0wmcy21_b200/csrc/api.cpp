@@ -46,6 +46,8 @@ struct Program {
   int g4_kinds = 0;        // source kinds of its gather4 items (tensor maps the launch needs)
   bool tree = false;       // carries tree-order FOLD programs (kTermRankTree)
   TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
+  mutable uint64_t claims = 0;  // dynamic item claiming: the counter's value before the next launch
+  bool relay_fwd = false;       // a forward program with stage chaining (waits on counters)
 };
 
 }  // namespace
@@ -87,6 +89,10 @@ struct dgcl_ctx {
   DevItem *d_items = nullptr;
   DevRun *d_runs = nullptr;
   uint32_t *d_sterms = nullptr;
+  uint64_t *d_claims = nullptr;  // one item-claim counter per program (dynamic claiming)
+  // dynamic item claiming (bulk-copy executor): -1 auto (batches of 4 for relay forwards, whose
+  // stage boundaries wait for the slowest CTA), 0 round-robin everywhere, k >= 1 batches of k
+  int claim_batch = -1;
   bool spst_fast = true;  // uniform switch: SPST's closed form (parallel) instead of the loop
   int64_t run_bytes = 0;
   bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
@@ -430,6 +436,9 @@ void build_programs(dgcl_ctx *c) {
           if (it.op == OP_FANOUT) P.op_mask |= kMaskFanout;
         }
         P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
+        P.relay_fwd = false;
+        for (const DevItem &it : P.items)
+          if (it.dir == DIR_FWD && it.op == OP_COPY && it.wait_n > 0) P.relay_fwd = true;
         P.g4_kinds = 0;
         P.tree = false;
         for (const DevItem &it : P.items)
@@ -835,6 +844,13 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     }
     encode_g4(Pp, pg.g4_kinds);
     const int grid = (int)std::min<int64_t>(std::max(1, grid_all / grid_div), Pp.n_items);
+    const int cb = c->claim_batch < 0 ? (pg.relay_fwd ? 4 : 0) : c->claim_batch;
+    if (Pp.use_tma && cb > 0 && c->d_claims) {
+      Pp.claim = c->d_claims + (&pg - c->progs.data());
+      Pp.claim_base = pg.claims;
+      Pp.claim_batch = cb;
+      pg.claims += (uint64_t)cb * ((uint64_t)(Pp.n_items + cb - 1) / cb + (uint64_t)grid);
+    }
     return launch_executor(Pp, grid, block, st);
   };
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
@@ -1035,6 +1051,7 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
   if ((s = upload(c, &c->d_items, all)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_runs, all_runs)) != DGCL_OK) return s;
   if ((s = upload(c, &c->d_sterms, all_sterms)) != DGCL_OK) return s;
+  if ((s = upload(c, &c->d_claims, std::vector<uint64_t>(c->progs.size(), 0))) != DGCL_OK) return s;
   c->run_bytes = (int64_t)(all_runs.size() * sizeof(DevRun) + all_sterms.size() * 4);
   if (c->trace)
     for (Program &p : c->progs)
@@ -1434,16 +1451,30 @@ dgcl_status dgcl_stream_wait_arrival(dgcl_ctx *c, int32_t dst, int32_t src, void
       n = g.wait_n;
     }
   if (off < 0) return fail(c, DGCL_EPLAN, "no completion list for rank %d", dst);
+  // multicast: the rows of src that came through the multicast region land with dst's unpack
+  int32_t mc_w = -1;
+  if (!L.mc_unpack_wait.empty()) {
+    if (src >= 0) {
+      mc_w = L.mc_unpack_wait[(size_t)dst * c->world + src];
+    } else {
+      for (int s2 = 0; s2 < c->world; ++s2) {  // every source: one wait launch per unpack
+        const int32_t w = L.mc_unpack_wait[(size_t)dst * c->world + s2];
+        if (w >= 0) {
+          dgcl_status st = dgcl_stream_wait_arrival(c, dst, s2, stream);
+          if (st != DGCL_OK) return st;
+        }
+      }
+    }
+  }
   if (src >= 0 && L.n_stages <= 1) {
     const int32_t want = (int32_t)ctr_index(DIR_FWD, 1, src, 0);
     int32_t hit = -1;
     for (int32_t w = off; w < off + n; ++w)
       if (L.waits[w].ctr == want) hit = w;
-    if (hit < 0) return DGCL_OK;  // nothing comes from src
     off = hit;
-    n = 1;
+    n = hit < 0 ? 0 : 1;  // (hit < 0: nothing comes from src directly)
   }
-  if (n == 0) return DGCL_OK;
+  if (n == 0 && mc_w < 0) return DGCL_OK;
   DeviceGuard guard(c->device);
   ExecParams P;
   std::memset(&P, 0, sizeof(P));
@@ -1454,7 +1485,8 @@ dgcl_status dgcl_stream_wait_arrival(dgcl_ctx *c, int32_t dst, int32_t src, void
   P.timeout_ns = (uint64_t)c->timeout_ms * 1000000ull;
   P.err = c->err_dev;
   P.sys_scope = c->loopback ? 0 : 1;
-  const int e = launch_wait(P, dst, off, n, stream);
+  int e = n > 0 ? launch_wait(P, dst, off, n, stream) : 0;
+  if (e == 0 && mc_w >= 0) e = launch_wait(P, dst, mc_w, 1, stream);
   if (e != 0) return fail(c, DGCL_ECUDA, "wait launch failed: %s", cudaGetErrorString((cudaError_t)e));
   return DGCL_OK;
 }
@@ -1575,6 +1607,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   if (k == "spst_fast") {  // before dgcl_build_plan: 0 = always run Algorithm 1's loop
     if (c->planned) return fail(c, DGCL_ESTATE, "spst_fast must be set before dgcl_build_plan");
     c->spst_fast = value != 0;
+    return DGCL_OK;
+  }
+  if (k == "claim_batch") {  // dynamic item claiming: -1 auto, 0 off, k >= 1 batch size; any time
+    if (value < -1 || value > 64) return fail(c, DGCL_EINVAL, "claim_batch in -1..64");
+    c->claim_batch = (int)value;
     return DGCL_OK;
   }
   if (k == "sys_scope") {  // loopback: 1 = the multi-GPU system-scope flag protocol (A/B)
@@ -1786,6 +1823,7 @@ dgcl_status dgcl_destroy(dgcl_ctx *c) {
     cudaFree(c->d_items);
     cudaFree(c->d_runs);
     cudaFree(c->d_sterms);
+    cudaFree(c->d_claims);
     for (Program &p : c->progs)
       if (p.d_trace) cudaFree(p.d_trace);
     for (auto &kv : c->stages) {

@@ -856,6 +856,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   // monotonic and their targets fixed for the launch, so it stays satisfied: later items of the
   // same (direction, stage, rank) skip the flag reads)
   int32_t *s_wait_ok = reinterpret_cast<int32_t *>(dsmem + kPendOff + 1040);
+  // producer-private (dynamic claiming): the launch index of the item in each descriptor slot
+  uint32_t *s_claim = reinterpret_cast<uint32_t *>(dsmem + kPendOff + 1104);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
   // L2 hints (option "l2_policy"): bit 0 data stores evict_first (write-once halo / relay /
@@ -887,12 +889,47 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     // into ring slot q % kDescSlots kDescAhead items ahead, its row runs into meta slot
     // q % kMetaSlots kMetaAhead items ahead, so their latency never stalls the issue loop
     const uint32_t G = gridDim.x;
-    const uint32_t nmine =
-        blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
-    auto request_desc = [&](uint32_t q) {  // lane 0, after a proxy fence
+    // Items are taken in list order: round-robin (item q of this CTA at list position
+    // blockIdx.x + q * G), or — with P.claim — in batches of P.claim_batch consecutive positions
+    // claimed from a launch-wide counter (claims hand out positions in increasing order, so every
+    // CTA's queue stays in list = stage order and the earliest unfinished item can always run:
+    // deadlock-free like round-robin; CTAs that drew cheaper items take more, which removes the
+    // per-SM speed spread at stage boundaries).  nmine: this CTA's item count (dynamic: known
+    // once a claim fails).
+    uint32_t nmine = P.claim ? 0xffffffffu
+                             : blockIdx.x < (uint32_t)P.n_items
+                                   ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G
+                                   : 0;
+    uint64_t bnext = 0;
+    uint32_t bleft = 0;                        // (lane 0) unissued positions of the batch
+    auto request_desc = [&](uint32_t q) -> bool {  // lane 0, after a proxy fence
       const uint32_t s = q % kDescSlots;
+      uint64_t idx;
+      if (P.claim) {
+        if (bleft == 0) {
+          const uint64_t b0 = atomicAdd(reinterpret_cast<unsigned long long *>(P.claim),
+                                        (unsigned long long)P.claim_batch) - P.claim_base;
+          if (b0 >= (uint64_t)P.n_items) return false;
+          bnext = b0;
+          bleft = (uint32_t)min((uint64_t)P.claim_batch, (uint64_t)P.n_items - b0);
+        }
+        idx = bnext++;
+        --bleft;
+        s_claim[s] = (uint32_t)idx;
+      } else {
+        idx = blockIdx.x + (uint64_t)q * G;
+      }
       mbar_expect_tx(&descb[s], (uint32_t)sizeof(DevItem));
-      bulk_g2s(descs + s, P.items + blockIdx.x + q * G, (uint32_t)sizeof(DevItem), &descb[s]);
+      bulk_g2s(descs + s, P.items + idx, (uint32_t)sizeof(DevItem), &descb[s]);
+      return true;
+    };
+    auto req = [&](uint32_t q) {  // warp-collective: request q, learn the end when claiming
+      int ok_q = 1;
+      if (lane == 0) ok_q = request_desc(q) ? 1 : 0;
+      if (P.claim) {
+        ok_q = __shfl_sync(0xffffffffu, ok_q, 0);
+        if (!ok_q && q < nmine) nmine = q;
+      }
     };
     auto desc_ready = [&](uint32_t q) -> const DevItem & {
       mbar_wait(&descb[q % kDescSlots], (q / kDescSlots) & 1u);
@@ -923,8 +960,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     // consumers, ordered by the empty barrier) the stage come before every bulk copy into them.
     // Prefetches are issued after the item, so the item's fence covers them too.
     fence_proxy_async_smem();
-    if (lane == 0)
-      for (uint32_t q = 0; q < (uint32_t)kDescAhead && q < nmine; ++q) request_desc(q);
+    for (uint32_t q = 0; q < (uint32_t)kDescAhead && q < nmine; ++q) req(q);
     for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nmine; ++q) {
       const DevItem Iq = desc_ready(q);
       if (lane == 0) issue_meta(P, Iq, meta_of(q), &metab[q % kMetaSlots]);
@@ -933,7 +969,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       const DevItem I = desc_ready(m);  // registers: no shared-memory reload per field
       const DevItem *Ism = &descs[m % kDescSlots];
       bool fenced = false;
-      const uint32_t gidx = blockIdx.x + m * G;  // the item's index in the launch
+      const uint32_t gidx = P.claim ? s_claim[m % kDescSlots] : blockIdx.x + m * G;  // (launch)
       if (P.trace && lane == 0) {
         uint32_t smid;
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
@@ -1020,7 +1056,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       __syncwarp();
       // prefetch: descriptor kDescAhead items ahead, row runs / segments kMetaAhead items ahead
       if (!fenced && (m + kMetaAhead < nmine)) fence_proxy_async_smem();
-      if (lane == 0 && m + kDescAhead < nmine) request_desc(m + kDescAhead);
+      if (m + kDescAhead < nmine) req(m + kDescAhead);
       if (m + kMetaAhead < nmine) {
         const uint32_t q = m + kMetaAhead;
         const DevItem In = desc_ready(q);

@@ -202,6 +202,13 @@ struct alignas(64) ExecParams {
   struct TraceRec *trace;  // option "trace": one record per item of this launch, or nullptr
   int32_t l2_policy;       // option "l2_policy": L2 eviction hints of the bulk-copy executor
   int32_t sys_scope;       // 1: flags / fences at system scope (peers are other GPUs); 0: .gpu
+  // bulk-copy executor, dynamic item claiming (option "claim_batch"): a launch-wide counter
+  // (nullptr = round-robin).  Every CTA claims batches of claim_batch list positions until a
+  // claim fails, so a launch adds exactly claim_batch * (ceil(n_items / claim_batch) + grid) to
+  // the counter; claim_base = its value at launch (kept by the host, never reset)
+  uint64_t *claim;
+  uint64_t claim_base;
+  int32_t claim_batch;
   // multicast (option "multicast"): the multicast flag page (multimem reductions), every rank's
   // unicast flag page (acquire waits; loopback: each virtual rank's copy), and whether the
   // multicast is emulated by one store / reduction per rank (loopback: no multicast object)

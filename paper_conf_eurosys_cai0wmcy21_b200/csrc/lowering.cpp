@@ -552,6 +552,10 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
   // multicast groups: a send signals the multicast done counter of its owner (one multimem
   // reduction reaches every GPU's copy) and writes into every peer's region (all ready words);
   // an unpack waits on the owner's multicast counter in this GPU's own region
+  // an unpack signals its own GPU's stage-2 counter of the owner s (arrival waits, R25: the rows
+  // of s that came by multicast are in the halo once it reaches its target); its wait entry is
+  // kept for dgcl_stream_wait_arrival
+  L.mc_unpack_wait.assign((size_t)m * m, -1);
   for (int gi = L.mc_begin; gi < L.mc_end; ++gi) {
     DevGroup &g = L.groups[gi];
     g.wait_off = 0;
@@ -565,6 +569,9 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
       g.wait_off = (int32_t)L.waits.size();
       g.wait_n = 1;
       L.waits.push_back({(int32_t)(kMcCtrBase + s_owner), 0, L.mc_rows[s_owner]});
+      g.sig_ctr = (int32_t)ctr_index(DIR_FWD, 2, s_owner, 0);
+      L.mc_unpack_wait[(size_t)g.exec_rank * m + s_owner] = (int32_t)L.waits.size();
+      L.waits.push_back({g.sig_ctr, 0, g.n_rows});
     }
   }
   // per-rank READY and forward-completion WAIT groups (used by per-rank programs only)

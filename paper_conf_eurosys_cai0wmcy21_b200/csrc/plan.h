@@ -76,6 +76,7 @@ struct Lowered {
   int mc_begin = 0, mc_end = 0;
   std::vector<int64_t> mc_rows, mc_off;
   int64_t mc_total = 0;
+  std::vector<int32_t> mc_unpack_wait;  // [d * m + s]: waits index of d's unpack of s, or -1
   std::vector<int32_t> idx;              // row index pool
   std::vector<int64_t> term_ptr;         // fold row pointers
   std::vector<uint32_t> terms;           // fold terms

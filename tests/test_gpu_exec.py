@@ -556,3 +556,39 @@ def test_atomic_backward_ablation(small, dims):
         Bi = halo.backward_flat(c.local(Li, dim), c.halos(Gi, dim), c.R, c.g.part, c.loc)
         for d in range(c.m):
             assert _eq(c.local(outi, dim)[d], Bi[d]), "atomic integer inputs rank %d" % d
+
+
+@pytest.mark.parametrize("flags,opts", [(1, {}), (0, {"signal_all": 1}),
+                                        (1, {"tma": 0}), (0, {"signal_all": 1, "multicast": 1})])
+def test_wait_arrival_per_source(flags, opts):
+    """dgcl_stream_wait_arrival (overlap, NEXT-2): on a second stream, after the wait for
+    (receiver d, source s), the halo rows d received from s equal the oracle's — the halo was
+    zeroed before the call, so a read ahead of the rows would show; a device start barrier
+    precedes each call (dgcl_device_barrier)."""
+    torch = _torch()
+    g = synth.make_graph(6000, 60000, 4, graph_seed=91, part_seed=92)
+    c = Case(g, [64], flags=flags, options=dict({"sm_budget": 100}, **opts))
+    emb = c.emb(0)
+    Ho = halo.forward(c.local(emb, 64), c.R, g.part, c.loc)
+    e = c.dev(emb)
+    side = torch.cuda.Stream()
+    for rep in range(2):
+        c.ctx.halo(0).zero_()
+        torch.cuda.synchronize()
+        main = torch.cuda.current_stream()
+        c.ctx.device_barrier(main)
+        c.ctx.forward(0, e, stream=main)
+        got = {}
+        with torch.cuda.stream(side):
+            for d in range(c.m):
+                for s in range(c.m):
+                    if s == d:
+                        continue
+                    c.ctx.wait_arrival(src=s, dst=d, stream=side)
+                    a, b = int(g.req_ptr[d]), int(g.req_ptr[d + 1])
+                    got[(d, s)] = c.ctx.halo(0)[a:b, :64].clone()
+        torch.cuda.synchronize()
+        c.ctx.check()
+        for (d, s), h in got.items():
+            sel = g.part[c.R[d]] == s
+            assert _eq(h.cpu().numpy()[sel], Ho[d][sel]), (rep, d, s)
