@@ -244,8 +244,8 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    evict_first (default), 2 COPY source reads evict_last, 4 COPY source reads
  *                    evict_first, 8 FOLD operand reads evict_first
  *   "claim_batch"    bulk-copy executor item assignment (any time): -1 (default) auto = dynamic
- *                    claiming in batches of 4 for relay forwards, round-robin otherwise; 0
- *                    round-robin everywhere; k >= 1 dynamic batches of k list positions
+ *                    claiming in batches of 4 for relay forwards, of 2 for jobs of <= 4 ranks,
+ *                    round-robin otherwise; 0 round-robin everywhere; k >= 1 batches of k
  *   "sys_scope"      loopback contexts: 1 = use the multi-GPU system-scope flag protocol (A/B;
  *                    default 0: device scope, exact when every rank is on this GPU)
  *   "multicast"      NVSwitch multicast of high-fan-out rows (see dgcl_multicast_open): 0 off

@@ -90,8 +90,8 @@ struct dgcl_ctx {
   DevRun *d_runs = nullptr;
   uint32_t *d_sterms = nullptr;
   uint64_t *d_claims = nullptr;  // one item-claim counter per program (dynamic claiming)
-  // dynamic item claiming (bulk-copy executor): -1 auto (batches of 4 for relay forwards, whose
-  // stage boundaries wait for the slowest CTA), 0 round-robin everywhere, k >= 1 batches of k
+  // dynamic item claiming (bulk-copy executor): -1 auto (batches of 4 for relay forwards, of 2
+  // for jobs of <= 4 ranks, else round-robin), 0 round-robin everywhere, k >= 1 batches of k
   int claim_batch = -1;
   bool spst_fast = true;  // uniform switch: SPST's closed form (parallel) instead of the loop
   int64_t run_bytes = 0;
@@ -844,7 +844,15 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     }
     encode_g4(Pp, pg.g4_kinds);
     const int grid = (int)std::min<int64_t>(std::max(1, grid_all / grid_div), Pp.n_items);
-    const int cb = c->claim_batch < 0 ? (pg.relay_fwd ? 4 : 0) : c->claim_batch;
+    // auto: batches of 4 for relay forwards (stage boundaries wait for the slowest CTA: Web-Google
+    // dgx1_like 0.815 -> 0.730 ms, ring 1.017 -> 0.969, Reddit dgx1_like 0.516 -> 0.482), of 2
+    // for jobs of <= 4 ranks (per-SM speed spread: Web-Google-2 fwd 0.211 -> 0.185, bwd 0.275 ->
+    // 0.255), none for the 8-way single-stage launches (Reddit fwd602 0.741 -> 0.765 with 4: the
+    // claims cost more than the spread), A/B r2n
+    const int cb = c->claim_batch >= 0 ? c->claim_batch
+                   : pg.relay_fwd     ? 4
+                   : m <= 4           ? 2
+                                      : 0;
     if (Pp.use_tma && cb > 0 && c->d_claims) {
       Pp.claim = c->d_claims + (&pg - c->progs.data());
       Pp.claim_base = pg.claims;
