@@ -93,6 +93,7 @@ struct dgcl_ctx {
   // dynamic item claiming (bulk-copy executor): -1 auto (batches of 4 for relay forwards, of 2
   // for jobs of <= 4 ranks, else round-robin), 0 round-robin everywhere, k >= 1 batches of k
   int claim_batch = -1;
+  bool lsu_gather = false;  // short-run COPY items gathered by consumer cp.async (A/B option)
   bool spst_fast = true;  // uniform switch: SPST's closed form (parallel) instead of the loop
   int64_t run_bytes = 0;
   bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
@@ -417,6 +418,7 @@ void build_programs(dgcl_ctx *c) {
         ItemLimits lim = item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
                                      (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm);
         lim.align_sources = c->align_sources;
+        lim.lsu_gather = c->lsu_gather && c->use_tma;
         build_items(L, G, row_bytes, lim, !fused || c->signal_all, need, &P.items, &P.runs,
                     c->direct_copy_rows,
                     c->stage_fold ? &P.sterms : nullptr);
@@ -1704,6 +1706,11 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "signal_all") {  // fused loopback: every item publishes its done count
     c->signal_all = value != 0;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "lsu_gather") {  // short-run COPY items: consumer cp.async gathers (bulk-copy executor)
+    c->lsu_gather = value != 0;
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }

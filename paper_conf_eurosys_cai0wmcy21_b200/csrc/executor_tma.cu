@@ -270,7 +270,7 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
     bulk_g2s(meta, P.runs + (I.src & ((1ll << kSegShift) - 1)), tx, bar);
     return;
   }
-  const uint32_t tx = (I.op == OP_COPY && !(I.flags & kItemDirect))
+  const uint32_t tx = (I.op == OP_COPY && !(I.flags & (kItemDirect | kItemLsu)))
                           ? (uint32_t)I.nterms * (uint32_t)sizeof(DevRun)
                           : 0u;
   mbar_expect_tx(bar, tx);
@@ -281,6 +281,7 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
 __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const DevItem &I) {
   if (I.op == OP_COPY) {
     if (uses_gather4(P, I)) return (uint32_t)((I.rows + 3) / 4 * 4) * (uint32_t)P.row16;
+    if (I.flags & kItemLsu) return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;
     if (!(I.flags & kItemDirect)) return (uint32_t)I.rows * (uint32_t)P.row16;
     return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;  // source-row window only
   }
@@ -336,6 +337,12 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     if (lane == 0 && I.src < 0) {
       const Win ws = window(~I.src, I.rows, 4);
       bulk_g2s(ops, P.idx + ws.a, ws.bytes, full);
+    }
+  } else if (I.op == OP_COPY && (I.flags & kItemLsu)) {
+    // consumer cp.async gathers: the source-row window goes after the item's rows
+    if (lane == 0 && I.src < 0) {
+      const Win ws = window(~I.src, I.rows, 4);
+      bulk_g2s(ops + (size_t)I.rows * r16, P.idx + ws.a, ws.bytes, full);
     }
   } else if (uses_gather4(P, I)) {
     // four rows per instruction (the last group repeats the item's last row; the stage holds
@@ -533,6 +540,32 @@ __device__ __forceinline__ void store_copy_atomic(const ExecParams &P, const Dev
     bulk_commit();
     bulk_wait_read();  // the stage may be reused once the reductions have read it
   }
+}
+
+// consumers: LSU item — gather the item's rows into the stage with 16-B cp.async (every consumer
+// thread many chunks in flight), then make them visible to the async proxy for the bulk stores
+__device__ __forceinline__ void gather_lsu(const ExecParams &P, const DevItem &I, uint8_t *st,
+                                           uint32_t tid, uint32_t T) {
+  const uint32_t r16 = (uint32_t)P.row16;
+  uint8_t *ops = st + kStageHdrBytes;
+  const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
+  const int64_t spitch = P.buf[I.src_kind][I.exec_rank].pitch;
+  const int32_t *sidx = I.src < 0 ? reinterpret_cast<const int32_t *>(ops + (size_t)I.rows * r16) +
+                                        window(~I.src, I.rows, 4).skew
+                                  : nullptr;
+  const uint32_t nch = (uint32_t)P.n_chunks;
+  const uint32_t total = (uint32_t)I.rows * nch;
+  for (uint32_t e = tid; e < total; e += T) {
+    const uint32_t r = fdiv(e, P);
+    const uint32_t col = e - r * nch;
+    const int64_t srow = sidx ? (int64_t)sidx[r] : I.src + r;
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(ops + r * r16 + col * 16)),
+                 "l"(sbase + srow * spitch + (int64_t)col * 16)
+                 : "memory");
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
+  fence_proxy_async_smem();  // (this thread's shared-memory writes -> the TMA stores' reads)
 }
 
 // consumers: COPY item with short runs — gather each row chunk straight from memory (8 loads in
@@ -1115,6 +1148,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       // the launch's items, so e.g. a forward launch carries no fold code / registers)
       if ((kMask & kMaskCopy) && I.op == OP_COPY && !(I.flags & kItemDirect)) {
         const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
+        if (I.flags & kItemLsu) {  // rows gathered by every consumer thread, then stored as usual
+          gather_lsu(P, I, const_cast<uint8_t *>(st), tid, T);
+          consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
+        }
         if (I.dst_kind == K_MCAST) {
           store_copy_mc(P, I, st, tid, T);
         } else if (I.flags & kItemAtomic) {

@@ -146,6 +146,11 @@ constexpr uint8_t kItemStaged = 8;
 // COPY whose rows are ADDED into the destination with atomic reductions (the paper's atomic
 // backward baseline, Table 9; ablation only: the order of the adds is not fixed)
 constexpr uint8_t kItemAtomic = 16;
+// COPY with short source runs (option "lsu_gather", bulk-copy executor): the consumer threads
+// gather the rows into the stage with 16-B cp.async (LDGSTS, many in flight, no per-instruction
+// issue loop on the producer), then the stage is stored as usual (TMA bulk stores); the
+// producer stages only the source-row window, after the rows
+constexpr uint8_t kItemLsu = 32;
 constexpr int kSegShift = 40;
 constexpr int kGather4MaxRowBytes = 1024;  // one tensor box (<= 256 fp32) per row
 

@@ -926,8 +926,10 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     if (lim.min_items > 0 && low.n_blocks == 1 && copy_rows < lim.min_items * lim.max_rows)
       spread_rpi = std::max<int64_t>(4, (copy_rows + lim.min_items - 1) / lim.min_items);
     auto copy_rpi = [&](int64_t spread) {
+      // (lsu_gather: the source-row window shares the stage with the rows)
+      const int64_t per_row = lim.lsu_gather ? row16 + 4 : row16;
       int64_t rpi = std::min<int64_t>(std::min(lim.max_rows, spread),
-                                      std::max<int64_t>(1, cap / row16));
+                                      std::max<int64_t>(1, (cap - (lim.lsu_gather ? 32 : 0)) / per_row));
       if (row16 <= kGather4MaxRowBytes && rpi >= 4) rpi = rpi / 4 * 4;
       return rpi;
     };
@@ -1194,6 +1196,9 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
         // rows per TMA instruction instead of one bulk copy per run (used only when the launch
         // provides the kind's tensor map, see ExecParams::gather4_mask)
         // (a 4-row group must start 128-B aligned in shared memory: row16 % 32 == 0)
+        else if (g.op == OP_COPY && lim.lsu_gather && g.dst_kind != K_MCAST && g.src_idx >= 0 &&
+                 row16 <= kGather4MaxRowBytes && (int64_t)it.nterms * 4 > (int64_t)it.rows)
+          it.flags |= kItemLsu;
         else if (g.op == OP_COPY && g.src_kind < kG4Kinds && g.src_idx >= 0 &&
                  row16 <= kGather4MaxRowBytes && row16 % 32 == 0 &&
                  (int64_t)it.nterms * 4 > (int64_t)it.rows)

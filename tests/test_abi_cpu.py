@@ -151,7 +151,9 @@ def test_uniform_plan_and_lowering(m, direct):
                                     (3, {"gather4": 0, "stage_fold": 0}),
                                     (8, {"geometry": 1}), (8, {"geometry": 2}),
                                     (4, {"geometry": 2, "direct_reduce": 0}),
-                                    (8, {"fanout": 1}), (3, {"fanout": 1, "geometry": 2})])
+                                    (8, {"fanout": 1}), (3, {"fanout": 1, "geometry": 2}),
+                                    (8, {"lsu_gather": 1}), (4, {"lsu_gather": 1, "geometry": 1}),
+                                    (8, {"multicast": 1, "lsu_gather": 1})])
 def test_work_items_host(m, opts):
     """The fused program's WORK ITEMS (not the groups) moved the way the bulk-copy executor moves
     them — COPY row runs, staged FOLD segments read back through the staged-term table — on the

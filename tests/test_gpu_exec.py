@@ -170,6 +170,9 @@ def test_tiny_config_bit_exact(small):
     # region copy): send + unpack groups, multicast done counters
     (8, {"multicast": 1}), (4, {"multicast": 2}), (4, {"multicast": 1, "tma": 0}),
     (3, {"multicast": 1, "geometry": 2}), (8, {"multicast": 3, "small_launch_bytes": 4 << 20}),
+    # consumer cp.async gathers for short-run items (option lsu_gather), both geometries
+    (8, {"lsu_gather": 1}), (4, {"lsu_gather": 1, "geometry": 1}),
+    (3, {"lsu_gather": 1, "bulk_store": 0}), (4, {"lsu_gather": 1, "direct_reduce": 0}),
 ])
 def test_uniform_loopback_fused(m, opts):
     """Executor variants: tma (bulk-copy executor vs the register LDG executor), direct_reduce
