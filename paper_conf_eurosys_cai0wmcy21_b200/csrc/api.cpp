@@ -1575,6 +1575,12 @@ dgcl_status dgcl_plan_counts(dgcl_ctx *c, int64_t *rows) {
     for (int s = 0; s < m; ++s)
       for (int d = 0; d < m; ++d)
         rows[((size_t)(k - 1) * m + s) * m + d] = c->low.rows(DIR_FWD, k, s, d);
+  // multicast deliveries are stage-1 rows s -> d too (their counters are the multicast ones)
+  for (size_t i = 0; i < c->low.mc_unpack_wait.size(); ++i)
+    if (c->low.mc_unpack_wait[i] >= 0) {
+      const int d = (int)(i / m), s = (int)(i % m);
+      rows[(size_t)s * m + d] += c->low.waits[c->low.mc_unpack_wait[i]].amount;
+    }
   return DGCL_OK;
 }
 
