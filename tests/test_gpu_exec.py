@@ -283,14 +283,27 @@ def test_empty_halo_rank_and_no_requests():
     _check_case(Case(g, [4]))
 
 
-def test_closed_form_ones_and_integer_inputs():
-    g = synth.make_graph(5000, 50000, 4, graph_seed=21, part_seed=22)
-    c = Case(g, [16], topo=synth.dgx1_like() if False else None)
+@pytest.mark.parametrize("topo,flags,opts", [(None, 0, {}), ("ring", 0, {}), ("dgx1_like", 1, {}),
+                                             ("ring", 0, {"direct_reduce": 0}),
+                                             (None, 1, {"tma": 0})])
+def test_closed_form_ones_and_integer_inputs(topo, flags, opts):
+    """Backward closed forms on direct and relay plans: G = 1, L = 0 gives |D_u| (counted by the
+    oracle from the required lists) in every column; integer-valued inputs (|x| <= 8, every
+    partial sum exact in fp32) make every summation order exact, so the result must equal the
+    flat oracle bit for bit whatever the tree."""
+    g = synth.make_graph(5000, 50000, 8 if topo else 4, graph_seed=21, part_seed=22)
+    t = synth.topology.by_name(topo) if topo else None
+    c = Case(g, [16], topo=t, seed=2, flags=flags, options=opts)
     G, L = c.grads(0, mode="ones")
     out = c.run_backward(0, G, np.zeros_like(L))
     fan = halo.fanout(c.R, g.n)
     want = fan[c.order].astype(np.float32)
     assert np.array_equal(out[:, 0], want) and np.array_equal(out[:, 15], want)
+    Gi, Li = c.grads(0, mode="int")
+    outi = c.run_backward(0, Gi, Li)
+    Bf = halo.backward_flat(c.local(Li, 16), c.halos(Gi, 16), c.R, g.part, c.loc)
+    for d in range(c.m):
+        assert _eq(c.local(outi, 16)[d], Bf[d]), "integer inputs rank %d" % d
 
 
 def test_host_buffer_entry_points():
