@@ -855,13 +855,16 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
                    : pg.relay_fwd     ? 4
                    : m <= 4           ? 2
                                       : 0;
+    uint64_t claimed = 0;
     if (Pp.use_tma && cb > 0 && c->d_claims) {
       Pp.claim = c->d_claims + (&pg - c->progs.data());
       Pp.claim_base = pg.claims;
       Pp.claim_batch = cb;
-      pg.claims += (uint64_t)cb * ((uint64_t)(Pp.n_items + cb - 1) / cb + (uint64_t)grid);
+      claimed = (uint64_t)cb * ((uint64_t)(Pp.n_items + cb - 1) / cb + (uint64_t)grid);
     }
-    return launch_executor(Pp, grid, block, st);
+    const int rc = launch_executor(Pp, grid, block, st);
+    if (rc == 0) pg.claims += claimed;  // (a launch that never ran added nothing on the device)
+    return rc;
   };
   const bool fused = c->loopback && c->lb_flags == DGCL_LOOPBACK_FUSED;
   P.use_ready = (!fused && m > 1) ? 1 : 0;
