@@ -27,6 +27,9 @@ using namespace dev;
 
 namespace {
 
+#ifndef DGCL_G4_LANE0
+#define DGCL_G4_LANE0 0  // 0: one gather4 per lane (default); k > 0: lane 0 issues k per step
+#endif
 #ifndef DGCL_FAN_BULK_ROW
 #define DGCL_FAN_BULK_ROW 1024
 #endif
@@ -352,12 +355,31 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     const int32_t base = P.tmap_row_off[I.src_kind][I.exec_rank];
     const void *tmap = P.tmap[I.src_kind];
     const int ng = (I.rows + 3) / 4;
+#if DGCL_G4_LANE0
+    // variant: lane 0 issues every gather, DGCL_G4_LANE0 per loop iteration (independent
+    // operand registers, so consecutive TMA instructions need not wait for each other's
+    // uniform-register operands)
+    if (lane == 0) {
+      const int last = I.rows - 1;
+      for (int g = 0; g < ng; g += DGCL_G4_LANE0) {
+#pragma unroll
+        for (int j = 0; j < DGCL_G4_LANE0; ++j) {
+          const int r = 4 * (g + j);
+          if (g + j < ng)
+            tma_gather4(ops + (size_t)r * r16, tmap, 0, base + sidx[r],
+                        base + sidx[min(r + 1, last)], base + sidx[min(r + 2, last)],
+                        base + sidx[min(r + 3, last)], full, pol_copy);
+        }
+      }
+    }
+#else
     for (int g = lane; g < ng; g += 32) {
       const int r = 4 * g, last = I.rows - 1;
       tma_gather4(ops + (size_t)r * r16, tmap, 0, base + sidx[r],
                   base + sidx[min(r + 1, last)], base + sidx[min(r + 2, last)],
                   base + sidx[min(r + 3, last)], full, pol_copy);
     }
+#endif
   } else if (I.op == OP_COPY) {
     // one bulk copy per run of consecutive source rows when rows are packed (pitch == row16)
     const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
