@@ -256,6 +256,7 @@ __device__ __forceinline__ uint32_t n_segments(const DevItem &I) {
 
 // producer lane 0: bulk-copy the metadata the producer needs to issue item I's gathers (the
 // caller has fenced generic accesses to the slot against the async proxy)
+template <bool kLsu>
 __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I, uint8_t *meta,
                                            uint64_t *bar) {
   // COPY (bulk path): the item's row runs, or its source rows for a gather4 item.  FOLD and
@@ -273,7 +274,7 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
     bulk_g2s(meta, P.runs + (I.src & ((1ll << kSegShift) - 1)), tx, bar);
     return;
   }
-  const uint32_t tx = (I.op == OP_COPY && !(I.flags & (kItemDirect | kItemLsu)))
+  const uint32_t tx = (I.op == OP_COPY && !(I.flags & (kItemDirect | (kLsu ? kItemLsu : 0))))
                           ? (uint32_t)I.nterms * (uint32_t)sizeof(DevRun)
                           : 0u;
   mbar_expect_tx(bar, tx);
@@ -281,10 +282,11 @@ __device__ __forceinline__ void issue_meta(const ExecParams &P, const DevItem &I
 }
 
 // bytes bulk-copied into the operand area of a stage (gathered rows, or a FOLD's terms window)
+template <bool kLsu>
 __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const DevItem &I) {
   if (I.op == OP_COPY) {
     if (uses_gather4(P, I)) return (uint32_t)((I.rows + 3) / 4 * 4) * (uint32_t)P.row16;
-    if (I.flags & kItemLsu) return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;
+    if (kLsu && (I.flags & kItemLsu)) return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;
     if (!(I.flags & kItemDirect)) return (uint32_t)I.rows * (uint32_t)P.row16;
     return I.src < 0 ? window(~I.src, I.rows, 4).bytes : 0u;  // source-row window only
   }
@@ -296,6 +298,7 @@ __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const Dev
 // producer warp: header, consumer tables and row gathers of data item I (in registers; Ism = its
 // descriptor in shared memory, copied as the stage header) into `st`.  The caller waited for the
 // stage to be free and fenced the consumers' generic reads of it against the async proxy.
+template <bool kLsu>
 __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I,
                                            const DevItem *Ism, uint8_t *st, const uint8_t *meta,
                                            uint64_t *full, int lane, uint32_t item_index,
@@ -313,7 +316,7 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     info[2] = (int32_t)item_index;  // (trace records)
   }
   __syncwarp();  // header and info written before lane 0's arrive publishes the stage
-  if (lane == 0) mbar_expect_tx(full, operand_bytes(P, I) + wtp.bytes + wdst.bytes);
+  if (lane == 0) mbar_expect_tx(full, operand_bytes<kLsu>(P, I) + wtp.bytes + wdst.bytes);
   __syncwarp();
   if (lane == 0) {
     if (wtp.bytes) bulk_g2s(st + kTabTp, P.term_ptr + wtp.a, wtp.bytes, full);
@@ -341,7 +344,7 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
       const Win ws = window(~I.src, I.rows, 4);
       bulk_g2s(ops, P.idx + ws.a, ws.bytes, full);
     }
-  } else if (I.op == OP_COPY && (I.flags & kItemLsu)) {
+  } else if (kLsu && I.op == OP_COPY && (I.flags & kItemLsu)) {
     // consumer cp.async gathers: the source-row window goes after the item's rows
     if (lane == 0 && I.src < 0) {
       const Win ws = window(~I.src, I.rows, 4);
@@ -1018,7 +1021,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     for (uint32_t q = 0; q < (uint32_t)kDescAhead && q < nmine; ++q) req(q);
     for (uint32_t q = 0; q < (uint32_t)kMetaAhead && q < nmine; ++q) {
       const DevItem Iq = desc_ready(q);
-      if (lane == 0) issue_meta(P, Iq, meta_of(q), &metab[q % kMetaSlots]);
+      if (lane == 0) issue_meta<(kMask & kMaskLsu) != 0>(P, Iq, meta_of(q), &metab[q % kMetaSlots]);
     }
     for (; m < nmine; ++m) {
       const DevItem I = desc_ready(m);  // registers: no shared-memory reload per field
@@ -1032,6 +1035,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         P.trace[gidx].sm = smid;
         P.trace[gidx].tag = trace_tag(I, P.groups[I.group].stage, P.groups[I.group].block);
       }
+      if (I.op == OP_READY || I.op == OP_WAIT)  // (their metadata phase completed on the
+        mbar_wait(&metab[m % kMetaSlots], (m / kMetaSlots) & 1u);  // arrive; observe it)
       if (I.op == OP_READY) {
         // my buffers of every layer are free for this call: tell every peer
         if (lane == 0)
@@ -1100,7 +1105,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         if (P.trace && lane == 0) P.trace[gidx].t_ready = globaltimer();
         fence_proxy_async_smem();
         fenced = true;
-        issue_item(P, I, Ism, stages + (size_t)stage * stage_bytes, meta_of(m), &full[stage],
+        issue_item<(kMask & kMaskLsu) != 0>(P, I, Ism, stages + (size_t)stage * stage_bytes,
+                                            meta_of(m), &full[stage],
                    lane, gidx, pol_copy, pol_fold);
         ++k;
         if (sig) {
@@ -1115,7 +1121,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       if (m + kMetaAhead < nmine) {
         const uint32_t q = m + kMetaAhead;
         const DevItem In = desc_ready(q);
-        if (lane == 0) issue_meta(P, In, meta_of(q), &metab[q % kMetaSlots]);
+        if (lane == 0) issue_meta<(kMask & kMaskLsu) != 0>(P, In, meta_of(q), &metab[q % kMetaSlots]);
       }
     }
     if (!ok) {
@@ -1170,7 +1176,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       // the launch's items, so e.g. a forward launch carries no fold code / registers)
       if ((kMask & kMaskCopy) && I.op == OP_COPY && !(I.flags & kItemDirect)) {
         const BufRef DB = P.buf[I.dst_kind][I.dst_rank];
-        if (I.flags & kItemLsu) {  // rows gathered by every consumer thread, then stored as usual
+        if ((kMask & kMaskLsu) && (I.flags & kItemLsu)) {  // rows gathered by every consumer
+                                                            // thread, then stored as usual
           gather_lsu(P, I, const_cast<uint8_t *>(st), tid, T);
           consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
         }
@@ -1253,7 +1260,8 @@ int launch_mask(const ExecParams &p, int grid, int block, cudaStream_t s) {
   return (int)cudaGetLastError();
 }
 
-constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged | kMaskFanout | kMaskTree;
+constexpr int kAll =
+    kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged | kMaskFanout | kMaskTree | kMaskLsu;
 
 }  // namespace
 

@@ -239,7 +239,9 @@ DGCL_HD inline uint32_t trace_tag(const DevItem &I, int stage, int block) {
          (uint32_t)I.dst_rank << 16 | (uint32_t)(stage & 31) << 24 | (uint32_t)(block & 7) << 29;
 }
 constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8, kMaskFanout = 16,
-                  kMaskTree = 32;  // unstaged tree-order FOLD items (their own instance)
+                  kMaskTree = 32,  // unstaged tree-order FOLD items (their own instance)
+                  kMaskLsu = 64;   // COPY items gathered by consumer cp.async (option lsu_gather;
+                                   // only the catch-all instance carries that code)
 
 // A run of `len` rows whose source rows src.. and destination rows dst.. are both consecutive;
 // `pos` is the first row's index inside its item.  One bulk copy moves a run when the pitches

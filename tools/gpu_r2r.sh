@@ -9,7 +9,7 @@ ncu --query-metrics 2>/dev/null | grep -i -E "nvl|nvlrx|nvltx" > gpurun_out/r2r_
 O=gpurun_out/r2r_ab.jsonl; : > $O
 for C in orkut google8 google8_ring reddit; do
   for rep in 1 2; do
-    for L in paper_conf_eurosys_cai0wmcy21_b200/libdgcl.so build/ab/l0u2.so build/ab/l0u4.so; do
+    for L in paper_conf_eurosys_cai0wmcy21_b200/libdgcl.so build/ab/r2o.so build/ab/l0u2.so build/ab/l0u4.so; do
       DGCL_LIBRARY=$PWD/$L timeout 600 python tools/ab_rt.py $C "" | sed "s#^{#{\"lib\": \"$L\", #" >> $O 2>>gpurun_out/r2r_ab.err
     done
   done
