@@ -1035,15 +1035,16 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         P.trace[gidx].sm = smid;
         P.trace[gidx].tag = trace_tag(I, P.groups[I.group].stage, P.groups[I.group].block);
       }
-      if (I.op == OP_READY || I.op == OP_WAIT)  // (their metadata phase completed on the
-        mbar_wait(&metab[m % kMetaSlots], (m / kMetaSlots) & 1u);  // arrive; observe it)
       if (I.op == OP_READY) {
+        // (the item's metadata phase completed on its arrive: observe it, synccheck-clean)
+        mbar_wait(&metab[m % kMetaSlots], (m / kMetaSlots) & 1u);
         // my buffers of every layer are free for this call: tell every peer
         if (lane == 0)
           for (int s = 0; s < P.world; ++s)
             if (s != I.exec_rank)
               st_release(P.flags[s] + kReadyBase + I.exec_rank, P.seq, P.sys_scope);
       } else if (I.op == OP_WAIT) {
+        mbar_wait(&metab[m % kMetaSlots], (m / kMetaSlots) & 1u);
         // forward completion: the launch ends only once every incoming row landed
         if (pend) {
           emit_marker(OP_FLUSH);
