@@ -436,6 +436,7 @@ void build_programs(dgcl_ctx *c) {
           }
           if (it.op == OP_COPY) P.op_mask |= (it.flags & kItemDirect) ? kMaskDirect : kMaskCopy;
           if (it.op == OP_COPY && (it.flags & kItemLsu)) P.op_mask |= kMaskLsu;
+          if (it.op == OP_COPY && it.dst_kind == K_MCAST) P.op_mask |= kMaskMcast;
           if (it.op == OP_FANOUT) P.op_mask |= kMaskFanout;
         }
         P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;

@@ -372,7 +372,7 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
     if (s_abort) return;  // the watchdog fired; the error word is set, leave the launch
     if (kCopy == 3) {  // fold-only instance
       if (I.op == OP_FOLD) fold_rows<V16>(P, I);
-    } else if (I.op == OP_COPY && I.dst_kind == K_MCAST) {
+    } else if (kCopy == 0 && I.op == OP_COPY && I.dst_kind == K_MCAST) {
       copy_rows_mc(P, I);
     } else if (I.op == OP_COPY && (I.flags & kItemAtomic)) {
       copy_rows_atomic(P, I);
@@ -398,7 +398,7 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
       __syncthreads();
       if (threadIdx.x == 0) P.trace[it].t_done = globaltimer();
     }
-    if ((I.flags & kItemSignal) && I.dst_kind == K_MCAST) {  // multicast counter: right away
+    if (kCopy == 0 && (I.flags & kItemSignal) && I.dst_kind == K_MCAST) {  // multicast: at once
       fence_scope(1);
       __syncthreads();
       if (threadIdx.x == 0) mc_publish(P, I.exec_rank, (uint64_t)I.rows);
@@ -486,6 +486,7 @@ int launch_executor(const ExecParams &p, int grid, int block, void *stream) {
   // copy-only: every data item is a COPY (bulk-path or consumer-gather kind: the register path
   // runs both the same way); fold-only: no COPY of any kind and no FANOUT (the kCopy == 3
   // instance runs OP_FOLD items only, so a direct COPY must never reach it)
+  // (multicast and lsu launches take the general instance, kMaskMcast / kMaskLsu)
   const int copies = kMaskCopy | kMaskDirect;
   const int folds = kMaskFold | kMaskStaged | kMaskTree;
   const bool copy_only = p.op_mask != 0 && (p.op_mask & ~copies) == 0;

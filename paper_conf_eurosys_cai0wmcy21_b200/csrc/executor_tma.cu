@@ -1182,7 +1182,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           gather_lsu(P, I, const_cast<uint8_t *>(st), tid, T);
           consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
         }
-        if (I.dst_kind == K_MCAST) {
+        if ((kMask & kMaskMcast) && I.dst_kind == K_MCAST) {
           store_copy_mc(P, I, st, tid, T);
         } else if (I.flags & kItemAtomic) {
           store_copy_atomic(P, I, st, tid, T);
@@ -1261,8 +1261,8 @@ int launch_mask(const ExecParams &p, int grid, int block, cudaStream_t s) {
   return (int)cudaGetLastError();
 }
 
-constexpr int kAll =
-    kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged | kMaskFanout | kMaskTree | kMaskLsu;
+constexpr int kAll = kMaskCopy | kMaskFold | kMaskDirect | kMaskStaged | kMaskFanout | kMaskTree |
+                     kMaskLsu | kMaskMcast;
 
 }  // namespace
 

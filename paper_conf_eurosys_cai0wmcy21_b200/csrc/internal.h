@@ -240,8 +240,9 @@ DGCL_HD inline uint32_t trace_tag(const DevItem &I, int stage, int block) {
 }
 constexpr int32_t kMaskCopy = 1, kMaskFold = 2, kMaskDirect = 4, kMaskStaged = 8, kMaskFanout = 16,
                   kMaskTree = 32,  // unstaged tree-order FOLD items (their own instance)
-                  kMaskLsu = 64;   // COPY items gathered by consumer cp.async (option lsu_gather;
+                  kMaskLsu = 64,   // COPY items gathered by consumer cp.async (option lsu_gather;
                                    // only the catch-all instance carries that code)
+                  kMaskMcast = 128;  // COPY items into the multicast region (likewise)
 
 // A run of `len` rows whose source rows src.. and destination rows dst.. are both consecutive;
 // `pos` is the first row's index inside its item.  One bulk copy moves a run when the pitches
