@@ -27,8 +27,8 @@ using namespace dev;
 
 namespace {
 
-#ifndef DGCL_G4_LANE0
-#define DGCL_G4_LANE0 0  // 0: one gather4 per lane (default); k > 0: lane 0 issues k per step
+#ifndef DGCL_HELPER
+#define DGCL_HELPER 1  // copy launches: a second producer warp issues half of each item's gathers
 #endif
 #ifndef DGCL_FAN_BULK_ROW
 #define DGCL_FAN_BULK_ROW 1024
@@ -218,6 +218,14 @@ __device__ __forceinline__ Win window(int64_t off, int64_t n, int sz) {
   return w;
 }
 
+// named barriers between the producer warp and its helper (ids 1 and 2; __syncthreads is 0)
+__device__ __forceinline__ void named_arrive(int id, int n) {
+  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void named_sync(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
 // COPY item gathered four rows per TMA instruction (tile::gather4 through the launch's tensor map)
 __device__ __forceinline__ bool uses_gather4(const ExecParams &P, const DevItem &I) {
   return (I.flags & kItemGather4) && I.op == OP_COPY && I.src < 0 && I.src_kind < kG4Kinds &&
@@ -295,14 +303,36 @@ __device__ __forceinline__ uint32_t operand_bytes(const ExecParams &P, const Dev
   return window(I.t0, I.nterms, 4).bytes;
 }
 
+// gathers [gb, ge) of a gather4 COPY item, one per lane and round (row indices from its meta slot)
+__device__ __forceinline__ void issue_gather4(const ExecParams &P, const DevItem &I, uint8_t *st,
+                                              const uint8_t *meta, uint64_t *full, int lane, int gb,
+                                              int ge, uint64_t pol) {
+  const uint32_t r16 = (uint32_t)P.row16;
+  uint8_t *ops = st + kStageHdrBytes;
+  const int32_t *sidx = reinterpret_cast<const int32_t *>(meta) +
+                        (int32_t)(~I.src - window(~I.src, I.rows, 4).a);
+  const int32_t base = P.tmap_row_off[I.src_kind][I.exec_rank];
+  const void *tmap = P.tmap[I.src_kind];
+  for (int g = gb + lane; g < ge; g += 32) {
+    const int r = 4 * g, last = I.rows - 1;
+    tma_gather4(ops + (size_t)r * r16, tmap, 0, base + sidx[r], base + sidx[min(r + 1, last)],
+                base + sidx[min(r + 2, last)], base + sidx[min(r + 3, last)], full, pol);
+  }
+}
+
 // producer warp: header, consumer tables and row gathers of data item I (in registers; Ism = its
 // descriptor in shared memory, copied as the stage header) into `st`.  The caller waited for the
 // stage to be free and fenced the consumers' generic reads of it against the async proxy.
-template <bool kLsu>
+// With kHelp, gather4 items are handed to the helper warp through the mailbox mb (stage and
+// meta-slot offsets) after the stage's transaction bytes are armed; the two warps then each issue
+// half of the gathers.
+template <bool kLsu, bool kHelp>
 __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I,
                                            const DevItem *Ism, uint8_t *st, const uint8_t *meta,
                                            uint64_t *full, int lane, uint32_t item_index,
-                                           uint64_t pol_copy, uint64_t pol_fold) {
+                                           uint64_t pol_copy, uint64_t pol_fold, uint32_t *mb,
+                                           bool *mb_busy, const uint8_t *stages_base,
+                                           const uint8_t *metas_base) {
   const uint32_t r16 = (uint32_t)P.row16;
   // consumer tables: term_ptr window (FOLD) and destination rows (when not consecutive)
   Win wtp = {0, 0, 0}, wdst = {0, 0, 0};
@@ -353,36 +383,20 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
   } else if (uses_gather4(P, I)) {
     // four rows per instruction (the last group repeats the item's last row; the stage holds
     // the padding rows, the consumers never store them)
-    const int32_t *sidx = reinterpret_cast<const int32_t *>(meta) +
-                          (int32_t)(~I.src - window(~I.src, I.rows, 4).a);
-    const int32_t base = P.tmap_row_off[I.src_kind][I.exec_rank];
-    const void *tmap = P.tmap[I.src_kind];
     const int ng = (I.rows + 3) / 4;
-#if DGCL_G4_LANE0
-    // variant: lane 0 issues every gather, DGCL_G4_LANE0 per loop iteration (independent
-    // operand registers, so consecutive TMA instructions need not wait for each other's
-    // uniform-register operands)
-    if (lane == 0) {
-      const int last = I.rows - 1;
-      for (int g = 0; g < ng; g += DGCL_G4_LANE0) {
-#pragma unroll
-        for (int j = 0; j < DGCL_G4_LANE0; ++j) {
-          const int r = 4 * (g + j);
-          if (g + j < ng)
-            tma_gather4(ops + (size_t)r * r16, tmap, 0, base + sidx[r],
-                        base + sidx[min(r + 1, last)], base + sidx[min(r + 2, last)],
-                        base + sidx[min(r + 3, last)], full, pol_copy);
-        }
+    const bool hand = kHelp && ng >= 4;  // (the helper takes the upper half of the groups)
+    if (hand) {  // the helper warp takes every other group of 32 (see executor_tma_kernel)
+      if (*mb_busy) named_sync(2, 64);  // (it has read the previous hand-over)
+      if (lane == 0) {
+        mb[0] = (uint32_t)(st - (stages_base));
+        mb[1] = (uint32_t)(meta - metas_base);
+        mb[2] = 0;
       }
+      __syncwarp();
+      named_arrive(1, 64);
+      *mb_busy = true;
     }
-#else
-    for (int g = lane; g < ng; g += 32) {
-      const int r = 4 * g, last = I.rows - 1;
-      tma_gather4(ops + (size_t)r * r16, tmap, 0, base + sidx[r],
-                  base + sidx[min(r + 1, last)], base + sidx[min(r + 2, last)],
-                  base + sidx[min(r + 3, last)], full, pol_copy);
-    }
-#endif
+    issue_gather4(P, I, st, meta, full, lane, 0, hand ? ng / 2 : ng, pol_copy);
   } else if (I.op == OP_COPY) {
     // one bulk copy per run of consecutive source rows when rows are packed (pitch == row16)
     const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
@@ -916,8 +930,17 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   int32_t *s_wait_ok = reinterpret_cast<int32_t *>(dsmem + kPendOff + 1040);
   // producer-private (dynamic claiming): the launch index of the item in each descriptor slot
   uint32_t *s_claim = reinterpret_cast<uint32_t *>(dsmem + kPendOff + 1104);
+  // producer -> helper hand-over: stage offset, meta-slot offset, end flag
+  uint32_t *s_mb = reinterpret_cast<uint32_t *>(dsmem + kPendOff + 1136);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int n_cons_warps = (int)(blockDim.x >> 5) - 1;
+  // copy-only instances: warp 1 helps the producer issue gather4 instructions (the issue loop of
+  // a TMA instruction is serialised per lane: the producer was the bound of the small-row
+  // forwards, profiles/r2k_orkut_fwd_source.md)
+  constexpr bool kHelp = DGCL_HELPER && (kMask & kMaskCopy) &&
+                         !(kMask & (kMaskFold | kMaskStaged | kMaskTree | kMaskFanout | kMaskLsu |
+                                    kMaskMcast | kMaskDirect));
+  constexpr int kProdWarps = kHelp ? 2 : 1;
+  const int n_cons_warps = (int)(blockDim.x >> 5) - kProdWarps;
   // L2 hints (option "l2_policy"): bit 0 data stores evict_first (write-once halo / relay /
   // slot rows), bit 1 COPY / FANOUT source reads evict_last (a row sent to several receivers is
   // read again soon), bit 2 COPY source reads evict_first, bit 3 FOLD operand reads evict_first
@@ -941,7 +964,22 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   }
   __syncthreads();
 
-  if (warp == 0) {
+  if (kHelp && warp == 1) {
+    // ------------------------------- helper warp ---------------------------------------------
+    const uint64_t pol_h = pol_copy;
+    for (;;) {
+      named_sync(1, 64);  // a hand-over (or the end) from the producer
+      const uint32_t so = s_mb[0], mo = s_mb[1], end = s_mb[2];
+      __syncwarp();
+      named_arrive(2, 64);  // mailbox read
+      if (end) break;
+      uint8_t *st = stages + so;
+      const DevItem I = *reinterpret_cast<const DevItem *>(st);
+      fence_proxy_async_smem();
+      issue_gather4(P, I, st, metas + mo, &full[so / stage_bytes], lane, ((I.rows + 3) / 4) / 2,
+                    (I.rows + 3) / 4, pol_h);
+    }
+  } else if (warp == 0) {
     // ------------------------------- producer warp -------------------------------------------
     // item q of this CTA is P.items[blockIdx.x + q * gridDim.x]; its descriptor is bulk-copied
     // into ring slot q % kDescSlots kDescAhead items ahead, its row runs into meta slot
@@ -1000,6 +1038,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     auto known_sources = [&](const DevItem &I) {
       return I.wait_n == 0 || s_wait_ok[I.exec_rank] == I.wait_off;
     };
+    bool mb_busy = false;  // a hand-over to the helper is outstanding (not yet read)
     bool pend = false;  // signalling items issued since the last FLUSH
     int pend_key = -1;  // their counter family: ctr_index(dir, stage, 0)
     auto emit_marker = [&](uint8_t op) {  // header-only stage: FLUSH or END
@@ -1106,9 +1145,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         if (P.trace && lane == 0) P.trace[gidx].t_ready = globaltimer();
         fence_proxy_async_smem();
         fenced = true;
-        issue_item<(kMask & kMaskLsu) != 0>(P, I, Ism, stages + (size_t)stage * stage_bytes,
-                                            meta_of(m), &full[stage],
-                   lane, gidx, pol_copy, pol_fold);
+        issue_item<(kMask & kMaskLsu) != 0, kHelp>(P, I, Ism, stages + (size_t)stage * stage_bytes,
+                                                   meta_of(m), &full[stage], lane, gidx, pol_copy,
+                                                   pol_fold, s_mb, &mb_busy, stages, metas);
         ++k;
         if (sig) {
           pend = true;
@@ -1134,12 +1173,19 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       for (uint32_t q = m; q < m + kMetaAhead && q < nmine; ++q)
         mbar_wait(&metab[q % kMetaSlots], (q / kMetaSlots) & 1u);
     }
+    if (kHelp) {  // release the helper
+      if (mb_busy) named_sync(2, 64);
+      if (lane == 0) s_mb[2] = 1;
+      __syncwarp();
+      named_arrive(1, 64);
+      named_sync(2, 64);
+    }
     // END marker: consumers drain every issued stage, publish pending counts, then stop
     emit_marker(OP_END);
   } else {
     // ------------------------------- consumer warps ------------------------------------------
-    const uint32_t tid = threadIdx.x - 32, T = blockDim.x - 32;
-    const int cw = warp - 1;
+    const uint32_t tid = threadIdx.x - 32 * kProdWarps, T = blockDim.x - 32 * kProdWarps;
+    const int cw = warp - kProdWarps;
     for (uint32_t k = 0;; ++k) {
       uint32_t stage, use;
       ring_pos(k, NS, stage, use);

@@ -1,0 +1,18 @@
+#!/bin/bash
+cd "$(dirname "$0")/.."
+mkdir -p gpurun_out
+make -s all > gpurun_out/build.log 2>&1 || { cat gpurun_out/build.log; exit 1; }
+timeout 1200 python -m pytest tests/test_gpu_exec.py tests/test_gpu_multiproc.py -q -x -k "not full_size" > gpurun_out/r2v_pytest.log 2>&1; tail -2 gpurun_out/r2v_pytest.log
+O=gpurun_out/r2v_ab.jsonl; : > $O
+for C in orkut google8 google2 reddit google8_ring google8_dgx1; do
+  for rep in 1 2; do
+    for L in paper_conf_eurosys_cai0wmcy21_b200/libdgcl.so build/ab/nohelp.so; do
+      DGCL_LIBRARY=$PWD/$L timeout 600 python tools/ab_rt.py $C "" | sed "s#^{#{\"lib\": \"$L\", #" >> $O 2>>gpurun_out/r2v_ab.err
+    done
+  done
+done
+python - <<'P'
+import json
+for l in open("gpurun_out/r2v_ab.jsonl"):
+    d=json.loads(l); print(d["lib"].split("/")[-1].ljust(10), d["config"].ljust(14), d["sets"][0]["ms"])
+P
