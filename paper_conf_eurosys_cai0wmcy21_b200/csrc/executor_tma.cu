@@ -28,7 +28,7 @@ using namespace dev;
 namespace {
 
 #ifndef DGCL_HELPER
-#define DGCL_HELPER 1  // copy launches: a second producer warp issues half of each item's gathers
+#define DGCL_HELPER 1  // copy launches: this many helper warps issue a share of each item's gathers
 #endif
 #ifndef DGCL_FAN_BULK_ROW
 #define DGCL_FAN_BULK_ROW 1024
@@ -384,19 +384,20 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     // four rows per instruction (the last group repeats the item's last row; the stage holds
     // the padding rows, the consumers never store them)
     const int ng = (I.rows + 3) / 4;
-    const bool hand = kHelp && ng >= 4;  // (the helper takes the upper half of the groups)
-    if (hand) {  // the helper warp takes every other group of 32 (see executor_tma_kernel)
-      if (*mb_busy) named_sync(2, 64);  // (it has read the previous hand-over)
+    const bool hand = kHelp && ng >= 4;  // (helper h takes share h + 1 of 1 + DGCL_HELPER)
+    constexpr int kNB = 32 * (1 + (kHelp ? DGCL_HELPER : 0));  // producer + helper threads
+    if (hand) {  // the helper warps take shares of the groups (see executor_tma_kernel)
+      if (*mb_busy) named_sync(2, kNB);  // (they have read the previous hand-over)
       if (lane == 0) {
         mb[0] = (uint32_t)(st - (stages_base));
         mb[1] = (uint32_t)(meta - metas_base);
         mb[2] = 0;
       }
       __syncwarp();
-      named_arrive(1, 64);
+      named_arrive(1, kNB);
       *mb_busy = true;
     }
-    issue_gather4(P, I, st, meta, full, lane, 0, hand ? ng / 2 : ng, pol_copy);
+    issue_gather4(P, I, st, meta, full, lane, 0, hand ? ng / (1 + DGCL_HELPER) : ng, pol_copy);
   } else if (I.op == OP_COPY) {
     // one bulk copy per run of consecutive source rows when rows are packed (pitch == row16)
     const char *sbase = P.buf[I.src_kind][I.exec_rank].ptr;
@@ -939,7 +940,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   constexpr bool kHelp = DGCL_HELPER && (kMask & kMaskCopy) &&
                          !(kMask & (kMaskFold | kMaskStaged | kMaskTree | kMaskFanout | kMaskLsu |
                                     kMaskMcast | kMaskDirect));
-  constexpr int kProdWarps = kHelp ? 2 : 1;
+  constexpr int kProdWarps = kHelp ? 1 + DGCL_HELPER : 1;
   const int n_cons_warps = (int)(blockDim.x >> 5) - kProdWarps;
   // L2 hints (option "l2_policy"): bit 0 data stores evict_first (write-once halo / relay /
   // slot rows), bit 1 COPY / FANOUT source reads evict_last (a row sent to several receivers is
@@ -964,20 +965,22 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   }
   __syncthreads();
 
-  if (kHelp && warp == 1) {
-    // ------------------------------- helper warp ---------------------------------------------
+  if (kHelp && warp >= 1 && warp <= DGCL_HELPER) {
+    // ------------------------------- helper warps --------------------------------------------
+    constexpr int kNB = 32 * (1 + DGCL_HELPER);
     const uint64_t pol_h = pol_copy;
     for (;;) {
-      named_sync(1, 64);  // a hand-over (or the end) from the producer
+      named_sync(1, kNB);  // a hand-over (or the end) from the producer
       const uint32_t so = s_mb[0], mo = s_mb[1], end = s_mb[2];
       __syncwarp();
-      named_arrive(2, 64);  // mailbox read
+      named_arrive(2, kNB);  // mailbox read
       if (end) break;
       uint8_t *st = stages + so;
       const DevItem I = *reinterpret_cast<const DevItem *>(st);
       fence_proxy_async_smem();
-      issue_gather4(P, I, st, metas + mo, &full[so / stage_bytes], lane, ((I.rows + 3) / 4) / 2,
-                    (I.rows + 3) / 4, pol_h);
+      const int ng = (I.rows + 3) / 4;
+      issue_gather4(P, I, st, metas + mo, &full[so / stage_bytes], lane,
+                    ng * warp / (1 + DGCL_HELPER), ng * (warp + 1) / (1 + DGCL_HELPER), pol_h);
     }
   } else if (warp == 0) {
     // ------------------------------- producer warp -------------------------------------------
@@ -1173,12 +1176,13 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       for (uint32_t q = m; q < m + kMetaAhead && q < nmine; ++q)
         mbar_wait(&metab[q % kMetaSlots], (q / kMetaSlots) & 1u);
     }
-    if (kHelp) {  // release the helper
-      if (mb_busy) named_sync(2, 64);
+    if (kHelp) {  // release the helpers
+      constexpr int kNB = 32 * (1 + DGCL_HELPER);
+      if (mb_busy) named_sync(2, kNB);
       if (lane == 0) s_mb[2] = 1;
       __syncwarp();
-      named_arrive(1, 64);
-      named_sync(2, 64);
+      named_arrive(1, kNB);
+      named_sync(2, kNB);
     }
     // END marker: consumers drain every issued stage, publish pending counts, then stop
     emit_marker(OP_END);
