@@ -94,7 +94,6 @@ struct dgcl_ctx {
   // for jobs of <= 4 ranks, else round-robin), 0 round-robin everywhere, k >= 1 batches of k
   int claim_batch = -1;
   bool lsu_gather = false;  // short-run COPY items gathered by consumer cp.async (A/B option)
-  bool spst_fast = true;  // uniform switch: SPST's closed form (parallel) instead of the loop
   int64_t run_bytes = 0;
   bool bulk_store_local = true;   // TMA stores into local HBM (loopback)
   bool bulk_store_peer = false;   // TMA stores into peer memory over NVLink (not yet validated)
@@ -120,6 +119,7 @@ struct dgcl_ctx {
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
   bool hostsim_items = false;         // debug host interpreter: run the work items, not groups
+  bool spst_fast = true;              // uniform switch: SPST's closed form (parallel), not the loop
   int geometry = 0;                   // bulk-copy geometry: 0 auto per program, 1 WIDE, 2 DUAL
   int sm_budget = 0;                  // SMs an executor launch may use (0 = all): the rest stay
                                       // free for kernels overlapping the exchange (NEXT-2)
