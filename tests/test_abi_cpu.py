@@ -370,3 +370,31 @@ def test_uniform_closed_form_equals_spst_loop(m, explicit):
         ctx.destroy()
     assert np.array_equal(plans[0], plans[1]) and costs[0] == costs[1]
     assert np.all(plans[0][:, 3] == 1)
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_random_lowering_host(seed):
+    """Seeded random sweep of the planning + lowering options (ranks, topology, dims, item sizes,
+    geometry, staged folds, reduce form, multicast, fan-out, vertex blocks): the host interpreter
+    of the fused program's work items and groups against the oracle, the plan against the
+    oracle's SPST and invariants."""
+    rng = np.random.RandomState(1000 + seed)
+    m = int(rng.choice([2, 3, 4, 6, 8]))
+    topo = synth.topology.by_name("ring", m) if (m >= 4 and rng.rand() < 0.4) else None
+    opts = {"hostsim_items": int(rng.rand() < 0.7)}
+    for key, vals in (("geometry", [0, 1, 2]), ("stage_fold", [0, 1]),
+                      ("direct_reduce", [0, 1]), ("align_sources", [0, 1]),
+                      ("item_bytes", [1024, 8192, 65536])):
+        opts[key] = int(rng.choice(vals))
+    if topo is None:
+        r = rng.rand()
+        if r < 0.3:
+            opts["multicast"] = int(rng.choice([1, 2]))
+        elif r < 0.5:
+            opts["fanout"] = 1
+    else:
+        opts["pipeline_blocks"] = int(rng.choice([1, 2, 4]))
+    dims = [int(rng.choice([3, 12, 64, 257])) for _ in range(int(rng.randint(1, 3)))]
+    n = int(rng.choice([300, 900, 2000]))
+    g = synth.make_graph(n, 8 * n, m, graph_seed=300 + seed, part_seed=400 + seed)
+    _check_lowering(g, dims, topo, seed=seed, options=opts)

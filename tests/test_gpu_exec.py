@@ -608,3 +608,44 @@ def test_wait_arrival_per_source(flags, opts):
         for (d, s), h in got.items():
             sel = g.part[c.R[d]] == s
             assert _eq(h.cpu().numpy()[sel], Ho[d][sel]), (rep, d, s)
+
+
+def _random_option_case(seed):
+    """A seeded random combination of graph size, ranks, topology, loopback mode, dims and executor
+    options (the option interactions the fixed cases do not enumerate)."""
+    rng = np.random.RandomState(seed)
+    m = int(rng.choice([2, 3, 4, 5, 8]))
+    topo = None
+    if m == 8 and rng.rand() < 0.5:
+        topo = str(rng.choice(["ring", "dgx1_like"]))
+    elif m in (4, 5) and rng.rand() < 0.3:
+        topo = "ring"
+    flags = int(rng.rand() < 0.35)
+    dims = [int(rng.choice([4, 16, 37, 64, 128, 256, 602]))
+            for _ in range(int(rng.randint(1, 3)))]
+    opts = {"small_launch_bytes": int(rng.choice([0, 0, 4 << 20]))}
+    for key, vals in (("tma", [0, 1, 1, 1]), ("geometry", [0, 0, 1, 2]),
+                      ("claim_batch", [-1, 0, 1, 3]), ("stage_fold", [0, 1, 1]),
+                      ("direct_reduce", [0, 1, 1]), ("gather4", [0, 1, 1]),
+                      ("bulk_store", [0, 1, 1]), ("l2_policy", [0, 1, 3]),
+                      ("align_sources", [0, 1])):
+        opts[key] = int(rng.choice(vals))
+    if topo is None and rng.rand() < 0.3:
+        opts["multicast"] = int(rng.choice([1, 2]))
+    elif rng.rand() < 0.2:
+        opts["fanout"] = 1
+    if rng.rand() < 0.2:
+        opts["item_bytes"] = int(rng.choice([2048, 8192]))
+    n = int(rng.choice([800, 3000, 7000]))
+    return m, topo, flags, dims, opts, n
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_random_option_combinations(seed):
+    """Seeded random sweep over executor options, ranks, topologies and loopback modes; every case
+    element by element against the oracle (forward bit-exact, backward bit-exact in tree order, flat
+    order on single-stage plans, R6 bound otherwise, reproducible)."""
+    m, topo, flags, dims, opts, n = _random_option_case(seed)
+    g = synth.make_graph(n, 10 * n, m, graph_seed=100 + seed, part_seed=200 + seed)
+    t = synth.topology.by_name(topo, m) if topo else None
+    _check_case(Case(g, dims, topo=t, seed=seed, flags=flags, options=opts))
