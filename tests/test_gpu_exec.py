@@ -10,6 +10,8 @@ Every case compares the CUDA path with the oracle element by element on seeded i
 Full-size configs (BASELINE.json) are checked on sampled rows the oracle recomputes one by one
 from the hash-defined inputs, plus properties that hold at any size.
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -640,7 +642,7 @@ def _random_option_case(seed):
     return m, topo, flags, dims, opts, n
 
 
-@pytest.mark.parametrize("seed", range(24))
+@pytest.mark.parametrize("seed", range(int(os.environ.get("DGCL_RANDOM_CASES", "48"))))
 def test_random_option_combinations(seed):
     """Seeded random sweep over executor options, ranks, topologies and loopback modes; every case
     element by element against the oracle (forward bit-exact, backward bit-exact in tree order, flat
