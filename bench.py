@@ -273,6 +273,43 @@ def torch_gather_baseline(w, emb, hg, eg, stream, reps=5):
             "(backward, atomic)", "note": "stock PyTorch on the same B200, same layouts"}
 
 
+def per_rank_loopback(w, emb, hg, eg, stream, topo, reps=10):
+    """Context for the multi-GPU path: the same plan run as one launch per virtual rank on its own
+    stream (DGCL_LOOPBACK_PER_RANK) — every rank's program with the ready handshake, done counters
+    and completion waits of the multi-GPU protocol, sharing this GPU's SMs (each launch gets
+    1/m of them) — against the fused launch the bench times.  Per-launch ms, mean of `reps`."""
+    import torch
+    import paper_conf_eurosys_cai0wmcy21_b200 as D
+    c = w.cfg
+    ctx = D.loopback(c.m, w.g.part, list(c.dims), device=0, flags=D.LOOPBACK_PER_RANK)
+    ctx.build_plan(w.g.req_ptr, w.g.req_ids, seed=0, topology=topo)
+    ctx.register_workspace()
+    out = {}
+
+    def timed(fn):
+        for _ in range(2):
+            fn()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(reps):
+            fn()
+        b.record(stream)
+        torch.cuda.synchronize()
+        return a.elapsed_time(b) / reps
+
+    for l in w.fwd_layers:
+        out["fwd%d_d%d" % (l, c.dims[l])] = timed(lambda: ctx.forward(l, emb[l], stream=stream))
+    for l in w.bwd_layers:
+        e2 = eg[l].clone()
+        out["bwd%d_d%d" % (l, c.dims[l])] = timed(lambda: ctx.backward(l, hg[l], e2, stream=stream))
+    ctx.check()
+    ctx.destroy()
+    return {"ms_per_layer": out, "note": "one launch per virtual rank on its own stream with the "
+            "multi-GPU flag protocol (ready / done / completion waits), on one GPU; context, not "
+            "the bench value"}
+
+
 def run_ours_single(args, w):
     import torch
     import paper_conf_eurosys_cai0wmcy21_b200 as D
@@ -450,6 +487,7 @@ def run_ours_single(args, w):
 
     value = w.step_payload_bytes() / (ms_step * 1e-3) / 1e9
     torch_base = None if args.no_torch_baseline else torch_gather_baseline(w, emb, hg, eg, stream)
+    per_rank = None if args.no_per_rank else per_rank_loopback(w, emb, hg, eg, stream, topo)
     cpu = None
     if not args.no_cpu_baseline:
         gbs, secs, used, thr = oracle_sample(w, emb_h, hg_h, eg_h, budget_s=args.cpu_budget)
@@ -490,6 +528,7 @@ def run_ours_single(args, w):
         "clocks": clocks,
         "plan": dict(info, planner_wall_s=plan_s, graph_gen_s=w.gen_s),
         "torch_gather_baseline": torch_base,
+        "per_rank_loopback": per_rank,
     }
     ctx.destroy()
     return out
@@ -554,6 +593,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-torch-baseline", action="store_true")
+    ap.add_argument("--no-per-rank", action="store_true",
+                    help="N = 1: skip the per-rank loopback context measurement")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-cpu-threads", action="store_true")
     ap.add_argument("--item-bytes", type=int, default=0)

@@ -5,7 +5,7 @@ mkdir -p gpurun_out
 make -s all > gpurun_out/build.log 2>&1 || exit 1
 : > gpurun_out/bench_all.jsonl
 for C in ${CFGS:-tiny reddit google2 google4 google8 orkut google8_dgx1 google8_ring reddit_dgx1}; do
-  timeout 900 python bench.py --config $C --steps ${STEPS:-10} --warmup 3 --e2e-steps 0 --no-cpu-baseline \
+  timeout 900 python bench.py --config $C --steps ${STEPS:-10} --warmup 3 --e2e-steps 0 --no-cpu-baseline --no-per-rank \
      ${EXTRA:-} >> gpurun_out/bench_all.jsonl 2> gpurun_out/bench_$C.err
   echo "$C rc=$?"
 done

@@ -11,7 +11,7 @@ for C in ${CFGS:-tiny reddit google2 google4 google8 orkut google8_dgx1 google8_
   N=$(python -c "import json;d=json.loads(open('gpurun_out/${TAG}_${C}_bench.json').read().splitlines()[-1]);print(len(d['ms_per_layer']))" 2>/dev/null || echo 3)
   timeout 1200 ncu --set full --clock-control none --import-source on -k regex:executor -c $N \
     -o gpurun_out/${TAG}_${C}_prof -f \
-    python bench.py --config $C --steps 1 --warmup 3 --e2e-steps 0 --no-cpu-baseline --no-torch-baseline ${EXTRA:-} \
+    python bench.py --config $C --steps 1 --warmup 3 --e2e-steps 0 --no-cpu-baseline --no-torch-baseline --no-per-rank ${EXTRA:-} \
     > gpurun_out/${TAG}_${C}_prof.log 2>&1
   echo "$C bench+ncu rc=$?"
 done

@@ -10,7 +10,7 @@ tail -1 gpurun_out/${TAG}_smoke.log
 timeout 900 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/${TAG}_launches.csv \
-  python bench.py --steps 3 --warmup 3 --e2e-steps 0 --no-cpu-baseline --no-torch-baseline > gpurun_out/${TAG}_launches_bench.json 2>&1
+  python bench.py --steps 3 --warmup 3 --e2e-steps 0 --no-cpu-baseline --no-torch-baseline --no-per-rank > gpurun_out/${TAG}_launches_bench.json 2>&1
 timeout 900 python bench.py --gpus 2 --share-gpu --config tiny --steps 3 --calls 10 > gpurun_out/${TAG}_bench_n2.json 2> gpurun_out/${TAG}_bench_n2.err
 TAG=$TAG bash tools/ncu_all.sh > gpurun_out/${TAG}_ncu_all.log 2>&1
 python - <<P
