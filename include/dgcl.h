@@ -336,6 +336,19 @@ dgcl_status dgcl_multicast_bind(dgcl_ctx *ctx);
  * result into msg.  DGCL_ECUDA if unsupported. */
 dgcl_status dgcl_debug_multicast_selftest(int32_t cuda_device, int64_t bytes, char *msg,
                                           size_t msg_len);
+/* Verification aid (loopback contexts, host only, no device needed): runs the work items of
+ * (layer, direction) — the fused program, or every virtual rank's program — through the flag
+ * protocol of P:1447-1466 on the host: items in list order, each only once the counters it waits
+ * on reached their targets, signals applied at its end.  Checks that every wait target equals the
+ * rows ever signalled on its counter, that the programs cannot deadlock, that every source row
+ * written in the same launch (halo / relay staging / slots / multicast copy) is read only by an
+ * item that waits on its writer's counter, that no row is written twice, and (forward) that
+ * every halo row is written.  mutate 1..4 checks a deliberately broken copy instead (the
+ * checker's negative tests: 1 an item stops waiting, 2 an item moves before its producers, 3 a
+ * data item repeats, 4 a producer stops signalling).  DGCL_EPLAN with the first violation in msg,
+ * else DGCL_OK. */
+dgcl_status dgcl_debug_check_protocol(dgcl_ctx *ctx, int32_t layer, int32_t direction,
+                                      int32_t mutate, char *msg, size_t msg_len);
 
 /* Number of executor kernel launches issued so far by this context. */
 dgcl_status dgcl_launch_count(dgcl_ctx *ctx, uint64_t *count);

@@ -25,7 +25,7 @@ SYMBOLS = [
     "dgcl_plan_export", "dgcl_set_option", "dgcl_trace_read", "dgcl_device_barrier",
     "dgcl_stream_wait_arrival", "dgcl_multicast_supported", "dgcl_multicast_bytes",
     "dgcl_multicast_open", "dgcl_multicast_add", "dgcl_multicast_bind",
-    "dgcl_debug_multicast_selftest",
+    "dgcl_debug_multicast_selftest", "dgcl_debug_check_protocol",
     "dgcl_launch_count", "dgcl_check",
     "dgcl_last_error",
     "dgcl_strerror", "dgcl_destroy", "dgcl_debug_hostsim_forward", "dgcl_debug_hostsim_backward",
@@ -98,6 +98,7 @@ def lib():
             "dgcl_multicast_add": [P],
             "dgcl_multicast_bind": [P],
             "dgcl_debug_multicast_selftest": [I32, I64, ctypes.c_char_p, SZ],
+            "dgcl_debug_check_protocol": [P, I32, I32, I32, ctypes.c_char_p, SZ],
             "dgcl_launch_count": [P, ctypes.POINTER(U64)],
             "dgcl_check": [P],
             "dgcl_destroy": [P],

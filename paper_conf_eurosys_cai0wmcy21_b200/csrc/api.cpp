@@ -17,6 +17,7 @@
 #include <map>
 #include <new>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include <map>
@@ -115,6 +116,7 @@ struct dgcl_ctx {
   size_t mc_map_bytes = 0;      // granularity-rounded size of the mappings
   bool align_sources = true;          // forward COPY items of one source rank cut at common rows
   int pipeline_blocks = 1;            // relay plans: vertex blocks of the stage chaining
+  int leaf_split = 2;                 // relay plans: leaf deliveries after each stage's forwards
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
@@ -247,7 +249,8 @@ int mc_min_fanout(const dgcl_ctx *c) {
 
 void relower(dgcl_ctx *c) {
   lower_plan(c->rel, c->plan, c->part.data(), c->loc, &c->low, c->pipeline_blocks,
-             c->atomic_backward, c->fanout && !mc_min_fanout(c), mc_min_fanout(c));
+             c->atomic_backward, c->fanout && !mc_min_fanout(c), mc_min_fanout(c),
+             c->leaf_split);
 }
 
 void compute_layout(dgcl_ctx *c) {
@@ -1705,6 +1708,16 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }
+  if (k == "leaf_split") {  // relay plans: 0 off, 1 stages >= 2, 2 every stage (see lower_plan)
+    if (value < 0 || value > 2) return fail(c, DGCL_EINVAL, "leaf_split in 0..2");
+    c->leaf_split = (int)value;
+    if (c->planned) {
+      relower(c);
+      compute_layout(c);
+      build_programs(c);
+    }
+    return DGCL_OK;
+  }
   if (k == "pipeline_blocks") {  // relay plans: stage chaining per vertex block (1..8)
     if (value < 1 || value > kMaxBlocks) return fail(c, DGCL_EINVAL, "pipeline_blocks in 1..%d", kMaxBlocks);
     c->pipeline_blocks = (int)value;
@@ -1905,3 +1918,229 @@ dgcl_status dgcl_debug_hostsim_backward(dgcl_ctx *c, int32_t layer, const float 
 }
 
 }  // extern "C"
+
+// ---- verification aid: the flag protocol of one launch, checked on the host ----
+// Runs the programs of (layer, direction) — the fused loopback program, or every virtual rank's
+// program — as a scheduler would: each program's items in list order, an item only once every
+// counter it waits on has reached its target, signals applied when the item ends.  Reports the
+// first violation: a wait target that differs from the rows ever signalled on its counter, a
+// deadlock (no program can advance), a source row read before it was written or by an item that
+// does not wait on its writer's counter (a race on the GPU), a destination row written twice,
+// or (forward) a halo row never written.  If every program completes here, the executor cannot
+// deadlock either: a CTA takes its items in list order, so the item that ran first here among
+// the unfinished ones has all its waits satisfied and nothing of its own CTA before it.
+dgcl_status dgcl_debug_check_protocol(dgcl_ctx *c, int32_t layer, int32_t direction,
+                                      int32_t mutate, char *msg, size_t msg_len) {
+  if (!c || (direction != DIR_FWD && direction != DIR_BWD)) return DGCL_EINVAL;
+  if (!c->planned) return fail(c, DGCL_ESTATE, "no plan");
+  if (layer < 0 || layer >= c->n_layers) return fail(c, DGCL_EINVAL, "bad layer");
+  if (!c->loopback) return fail(c, DGCL_EINVAL, "loopback contexts only (every rank's program)");
+  const Lowered &L = c->low;
+  const int m = c->world;
+  char buf[512];
+  auto bad = [&](const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    std::vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    if (msg && msg_len) std::snprintf(msg, msg_len, "%s", buf);
+    return fail(c, DGCL_EPLAN, "%s", buf);
+  };
+  std::vector<Program> PP;
+  for (int r = 0; r < c->n_prog_ranks; ++r) PP.push_back(c->progs[c->prog_index(layer, direction, r)]);
+  // the checker's own negative tests: a deliberately broken copy of the programs
+  if (mutate) {
+    Program *pw = nullptr;
+    size_t iw = 0;
+    for (Program &p : PP)
+      for (size_t i = 0; i < p.items.size() && !pw; ++i)
+        if (p.items[i].wait_n > 0 && p.items[i].op != OP_WAIT) {
+          pw = &p;
+          iw = i;
+        }
+    if (!pw && mutate != 3) return fail(c, DGCL_EINVAL, "no waiting item to mutate");
+    if (mutate == 1) {         // a stage-chained item that no longer waits (a race)
+      pw->items[iw].wait_n = 0;
+    } else if (mutate == 2) {  // the same item moved before its producers (a deadlock)
+      const DevItem I = pw->items[iw];
+      pw->items.erase(pw->items.begin() + iw);
+      pw->items.insert(pw->items.begin(), I);
+    } else if (mutate == 3) {  // a data item repeated (a row written twice)
+      bool done = false;
+      for (Program &p : PP)
+        for (size_t i = 0; i < p.items.size() && !done; ++i)
+          if (p.items[i].op == OP_COPY || p.items[i].op == OP_FANOUT || p.items[i].op == OP_FOLD) {
+            p.items.push_back(p.items[i]);
+            done = true;
+          }
+      if (!done) return fail(c, DGCL_EINVAL, "no data item to mutate");
+    } else if (mutate == 4) {  // a producer of a waited counter that no longer signals
+      const int32_t ctr = c->low.waits[pw->items[iw].wait_off].ctr;
+      bool done = false;
+      for (Program &p : PP)
+        for (DevItem &I : p.items)
+          if (!done && (I.flags & kItemSignal) && I.sig_ctr == ctr) {
+            I.flags &= (uint8_t)~kItemSignal;
+            done = true;
+          }
+    } else {
+      return fail(c, DGCL_EINVAL, "mutate in 0..4");
+    }
+  }
+  std::vector<const Program *> P;
+  for (const Program &p : PP) P.push_back(&p);
+  auto key = [](int rank, int64_t ctr) { return (uint64_t)rank * kCtrSpace + (uint64_t)ctr; };
+  // rows of buffer (kind, rank) written in this launch: -2 not yet, -1 by an item that does not
+  // signal, else the writer's counter index (on that rank)
+  constexpr int32_t kUnwritten = -2, kNoSignal = -1;
+  std::vector<std::vector<int32_t>> wr((size_t)K_NKINDS * m);
+  auto rows_of = [&](int kind, int r) -> int64_t {
+    switch (kind) {
+      case K_HALO: return c->rel.n_halo[r];
+      case K_RELAY: return L.n_relay[r];
+      case K_SLOT: return L.n_slot[r];
+      case K_MCUC: return L.mc_total;
+      default: return 0;
+    }
+  };
+  for (int k = 0; k < K_NKINDS; ++k)
+    for (int r = 0; r < m; ++r) wr[(size_t)k * m + r].assign(rows_of(k, r), kUnwritten);
+  auto tracked = [&](int kind) { return kind == K_HALO || kind == K_RELAY || kind == K_SLOT || kind == K_MCUC; };
+  // every (receiver, counter, rows) signal of an item
+  auto signals = [&](const DevItem &I, auto &&emit) {
+    if (!(I.flags & kItemSignal) || I.sig_ctr < 0) return;
+    if (I.op == OP_FANOUT) {
+      int64_t cnt[kMaxRanks] = {0};
+      for (int64_t t = I.t0; t + 1 < I.t0 + I.nterms; t += 2) ++cnt[L.terms[t] >> 28];
+      for (int d = 0; d < m; ++d)
+        if (cnt[d]) emit(d, (int64_t)I.sig_ctr, cnt[d]);
+    } else if (I.dst_kind == K_MCAST) {
+      for (int d = 0; d < m; ++d) emit(d, (int64_t)I.sig_ctr, (int64_t)I.rows);
+    } else {
+      emit((int)I.dst_rank, (int64_t)I.sig_ctr, (int64_t)I.rows);
+    }
+  };
+  std::unordered_map<uint64_t, int64_t> total, val;
+  for (const Program *p : P)
+    for (const DevItem &I : p->items)
+      signals(I, [&](int d, int64_t ctr, int64_t n) { total[key(d, ctr)] += n; });
+  for (size_t pi = 0; pi < P.size(); ++pi)
+    for (size_t i = 0; i < P[pi]->items.size(); ++i) {
+      const DevItem &I = P[pi]->items[i];
+      for (int w = I.wait_off; w < I.wait_off + I.wait_n; ++w) {
+        const auto it = total.find(key(I.exec_rank, L.waits[w].ctr));
+        const int64_t have = it == total.end() ? 0 : it->second;
+        if (have != L.waits[w].amount)
+          return bad("program %zu item %zu (group %d): waits for %lld rows on counter %d of rank %d, "
+                     "%lld are ever signalled", pi, i, I.group, (long long)L.waits[w].amount,
+                     L.waits[w].ctr, I.exec_rank, (long long)have);
+      }
+    }
+  auto waits_ok = [&](const DevItem &I) {
+    for (int w = I.wait_off; w < I.wait_off + I.wait_n; ++w) {
+      const auto it = val.find(key(I.exec_rank, L.waits[w].ctr));
+      if ((it == val.end() ? 0 : it->second) < L.waits[w].amount) return false;
+    }
+    return true;
+  };
+  auto waits_on = [&](const DevItem &I, int32_t ctr) {
+    for (int w = I.wait_off; w < I.wait_off + I.wait_n; ++w)
+      if (L.waits[w].ctr == ctr) return true;
+    return false;
+  };
+  // one source row read / destination row written by item I
+  auto read = [&](const DevItem &I, int kind, int r, int64_t row, size_t pi, size_t i) -> bool {
+    if (!tracked(kind)) return true;
+    auto &v = wr[(size_t)kind * m + r];
+    if (row < 0 || row >= (int64_t)v.size()) {
+      bad("program %zu item %zu (group %d): source row %lld of kind %d rank %d out of range", pi, i,
+          I.group, (long long)row, kind, r);
+      return false;
+    }
+    const int32_t w = v[row];
+    if (w == kUnwritten || w == kNoSignal || r != I.exec_rank || !waits_on(I, w)) {
+      bad("program %zu item %zu (group %d, stage %d): reads row %lld of kind %d rank %d %s", pi, i,
+          I.group, L.groups[I.group].stage, (long long)row, kind, r,
+          w == kUnwritten ? "before it is written"
+          : w == kNoSignal ? "whose writer signals no counter"
+                           : "without waiting on its writer's counter");
+      return false;
+    }
+    return true;
+  };
+  auto write = [&](const DevItem &I, int kind, int r, int64_t row, int32_t ctr, size_t pi,
+                   size_t i) -> bool {
+    if (!tracked(kind)) return true;
+    auto &v = wr[(size_t)kind * m + r];
+    if (row < 0 || row >= (int64_t)v.size() || v[row] != kUnwritten) {
+      bad("program %zu item %zu (group %d): destination row %lld of kind %d rank %d %s", pi, i,
+          I.group, (long long)row, kind, r,
+          row < 0 || row >= (int64_t)v.size() ? "out of range" : "written twice");
+      return false;
+    }
+    v[row] = ctr;
+    return true;
+  };
+  auto run = [&](const DevItem &I, const Program &p, size_t pi, size_t i) -> bool {
+    const int32_t sctr = (I.flags & kItemSignal) ? I.sig_ctr : kNoSignal;
+    if (I.op == OP_COPY) {
+      for (int64_t q = I.tp; q < I.tp + I.nterms; ++q) {
+        const DevRun &R = p.runs[q];
+        for (int64_t j = 0; j < R.len; ++j) {
+          if (!read(I, I.src_kind, I.exec_rank, R.src + j, pi, i)) return false;
+          if (I.dst_kind == K_MCAST) {
+            for (int d = 0; d < m; ++d)
+              if (!write(I, K_MCUC, d, R.dst + j, sctr, pi, i)) return false;
+          } else if (!write(I, I.dst_kind, I.dst_rank, R.dst + j, sctr, pi, i)) {
+            return false;
+          }
+        }
+      }
+    } else if (I.op == OP_FANOUT) {
+      for (int64_t t = I.t0; t + 1 < I.t0 + I.nterms; t += 2) {
+        const uint32_t w = L.terms[t];
+        if (!write(I, (w & kFanRelay) ? K_RELAY : K_HALO, (int)(w >> 28), (int64_t)(w & kFanRowMask),
+                   sctr, pi, i))
+          return false;
+      }
+    } else if (I.op == OP_FOLD) {  // (sources not traced: the parity tests cover the folds)
+      for (int64_t j = 0; j < I.rows; ++j) {
+        const int64_t row = I.dst >= 0 ? I.dst + j : (int64_t)L.idx[~I.dst + j];
+        if (!write(I, I.dst_kind, I.dst_rank, row, sctr, pi, i)) return false;
+      }
+    }
+    signals(I, [&](int d, int64_t ctr, int64_t n) { val[key(d, ctr)] += n; });
+    return true;
+  };
+  std::vector<size_t> cur(P.size(), 0);
+  size_t left = 0;
+  for (const Program *p : P) left += p->items.size();
+  while (left > 0) {
+    bool progress = false;
+    for (size_t pi = 0; pi < P.size(); ++pi) {
+      const auto &items = P[pi]->items;
+      while (cur[pi] < items.size() && waits_ok(items[cur[pi]])) {
+        if (!run(items[cur[pi]], *P[pi], pi, cur[pi])) return DGCL_EPLAN;
+        ++cur[pi];
+        --left;
+        progress = true;
+      }
+    }
+    if (!progress) {
+      for (size_t pi = 0; pi < P.size(); ++pi)
+        if (cur[pi] < P[pi]->items.size()) {
+          const DevItem &I = P[pi]->items[cur[pi]];
+          return bad("deadlock: program %zu item %zu (group %d, stage %d) waits forever", pi,
+                     cur[pi], I.group, L.groups[I.group].stage);
+        }
+    }
+  }
+  if (direction == DIR_FWD)
+    for (int r = 0; r < m; ++r) {
+      const auto &v = wr[(size_t)K_HALO * m + r];
+      for (size_t row = 0; row < v.size(); ++row)
+        if (v[row] == kUnwritten) return bad("halo row %zu of rank %d is never written", row, r);
+    }
+  if (msg && msg_len) std::snprintf(msg, msg_len, "ok: %zu programs, %zu counters", P.size(), total.size());
+  return DGCL_OK;
+}

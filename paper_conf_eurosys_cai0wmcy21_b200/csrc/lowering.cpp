@@ -64,7 +64,7 @@ inline int32_t halo_pos(const Relation &rel, int64_t u, int d) {
 
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
                 const std::vector<int64_t> &loc, Lowered *out, int n_blocks, bool with_atomic,
-                bool with_fanout, int mc_min_fanout) {
+                bool with_fanout, int mc_min_fanout, int leaf_split) {
   auto t0 = std::chrono::steady_clock::now();
   // DGCL_TIMING=1: per-section wall times on stderr (planning at scale, NEXT-4)
   static const bool timing = std::getenv("DGCL_TIMING") != nullptr;
@@ -214,6 +214,33 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     for (int d = 0; d < m; ++d) L.mc_off[d + 1] = L.mc_off[d] + L.mc_rows[d];
   }
   L.mc_total = L.mc_off[m];
+
+  // Leaf split (relay plans): a forward delivery that no later stage forwards (the edge's child
+  // has no children in the tree) is needed only by its receiver, so it need not finish before
+  // the next stage starts.  Such deliveries count on a counter block of their own that no stage
+  // waits on, and their items come after the forwarded deliveries of the same stage: stage k+1's
+  // items wait only for stage k's forwarded rows, and the leaves of stage k fill the time the
+  // slowest CTA's forwarded rows take to land (the stage boundary).  Stage 1 (option 2) by edge,
+  // or by row with fan-out items: one fan-out item stores a row into all its first hops, so the
+  // row is "forwarded" if any of its first hops forwards it.
+  const bool split = leaf_split > 0 && K >= 2 && NB == 1;
+  std::vector<uint8_t> leaf_e;
+  if (split) {
+    L.leaf_block = 1;
+    leaf_e.assign(NE, 0);
+    std::vector<uint8_t> row_feeds(NV, 0);
+    for (int64_t vi = 0; vi < NV; ++vi)
+      for (int64_t e = plan.e_ptr[vi]; e < plan.e_ptr[vi + 1]; ++e)
+        if (plan.e_stage[e] == 1 && kid_eptr[e + 1] > kid_eptr[e]) row_feeds[vi] = 1;
+    // (stage 1 by row only with fan-out items; per-pair COPY groups split by edge)
+    for (int64_t e = 0; e < NE; ++e)
+      leaf_e[e] = plan.e_stage[e] == 1 && leaf_split < 2 ? 0
+                  : plan.e_stage[e] == 1 && with_fanout   ? !row_feeds[e_vidx[e]]
+                                                          : kid_eptr[e + 1] == kid_eptr[e];
+  }
+  auto fwd_block = [&](int64_t e) -> int {
+    return split ? (leaf_e[e] ? L.leaf_block : 0) : blk_of[e_vidx[e]];
+  };
   lap("blocks/child_pos/kinds");
   // ---- forward relay staging rows: contiguous per (receiver c, stage k, sender p, src kind) ----
   std::vector<int64_t> relay_row(NE, -1);
@@ -308,7 +335,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
         dk = K_RELAY;
         drow[e] = relay_row[e];
       }
-      ent[e] = {pack_key_b(k, blk_of[vi], p, c, sk, dk), drow[e], e, vi};
+      ent[e] = {pack_key_b(k, fwd_block(e), p, c, sk, dk), drow[e], e, vi};
     }
     if (L.mc_total > 0) {
       size_t w = 0;
@@ -544,7 +571,9 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     else
       reads_inflight = g.op == OP_FOLD || g.src_kind == K_SLOT;
     if (reads_inflight && g.stage >= 2) {
-      auto w = get_waits(g.dir, g.stage - 1, g.exec_rank, g.block);
+      // (leaf split: every forwarded row arrived on the previous stage's non-leaf counters)
+      auto w = get_waits(g.dir, g.stage - 1, g.exec_rank,
+                         split && g.dir == DIR_FWD ? 0 : g.block);
       g.wait_off = w.first;
       g.wait_n = w.second;
     }
@@ -583,7 +612,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     DevGroup g = base_group(OP_WAIT, DIR_FWD, r, r, K + 1);
     g.wait_off = (int32_t)L.waits.size();
     for (int k = 1; k <= K; ++k)
-      for (int bl = 0; bl < NB; ++bl)
+      for (int bl = 0; bl < (split ? L.leaf_block + 1 : NB); ++bl)
         for (int s = 0; s < m; ++s) {
           const int64_t rows = L.rows(DIR_FWD, k, s, r, bl);
           if (rows > 0) L.waits.push_back({(int32_t)ctr_index(DIR_FWD, k, s, bl), 0, rows});
@@ -671,14 +700,20 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
     for (int64_t u = 0; u < N; ++u) rows_of[part[u]].push_back(u);
     bool fits = true;
     std::vector<std::pair<int, uint32_t>> ds;
+    // (leaf split of stage 1: the owners' forwarded rows first, then their leaf rows; a group
+    // keeps all the owner's rows, the other class's rows without receivers)
+    const int n_cls = split && leaf_split >= 2 ? 2 : 1;
+    for (int cls = 0; cls < n_cls && fits; ++cls)
     for (int p = 0; p < m && fits; ++p) {
       DevGroup g = base_group(OP_FANOUT, DIR_FWD, p, p, 1);
+      const int fblock = n_cls == 2 && cls == 1 ? L.leaf_block : 0;
+      g.block = fblock;
       g.src_kind = K_EMB;
       g.dst_kind = K_HALO;
       g.n_rows = (int64_t)rows_of[p].size();
       g.src_base = 0;
       g.dst_base = 0;
-      g.sig_ctr = (int32_t)ctr_index(DIR_FWD, 1, p);
+      g.sig_ctr = (int32_t)ctr_index(DIR_FWD, 1, p, fblock);
       g.ready_rank = kReadyAll;
       g.term_ptr = (int64_t)L.term_ptr.size();
       const size_t t_begin = L.terms.size();
@@ -689,6 +724,7 @@ void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
           ds.clear();
           for (int64_t e = plan.e_ptr[vi]; e < plan.e_ptr[vi + 1]; ++e) {
             if (plan.e_parent[e] != p) continue;
+            if (n_cls == 2 && fwd_block(e) != fblock) continue;
             const int c = plan.e_child[e];
             const int64_t row = child_pos[e] >= 0 ? child_pos[e] : relay_row[e];
             if (row > (int64_t)kFanRowMask) fits = false;

@@ -84,6 +84,9 @@ struct Lowered {
   // per-rank buffer rows
   std::vector<int64_t> n_halo, n_relay, n_slot;  // [m]
   int n_blocks = 1;  // vertex blocks of the stage chaining (relay plans), see ctr_index
+  // relay plans, leaf split: forward deliveries no later stage forwards count on this block's
+  // counters (nothing waits on them but the forward completion), -1 = no split
+  int leaf_block = -1;
   // rows in: [dir][stage][block][src][dst] flattened
   std::vector<int64_t> rows_sd;
   int64_t &rows_at(int dir, int k, int s, int d, int b) {
@@ -95,6 +98,7 @@ struct Lowered {
   int64_t rows(int dir, int k, int s, int d) const {  // all blocks
     int64_t t = 0;
     for (int b = 0; b < n_blocks; ++b) t += rows(dir, k, s, d, b);
+    if (leaf_block >= n_blocks) t += rows(dir, k, s, d, leaf_block);
     return t;
   }
   int64_t n_relay_edges = 0;
@@ -111,9 +115,13 @@ struct Lowered {
 // (atomic backward, fan-out forward) — only when their option is set (they cost lowering time)
 // mc_min_fanout > 0: multicast the rows of vertices requested by >= that many GPUs
 // (single-stage plans)
+// leaf_split (relay plans, n_blocks = 1): 1 = deliveries of stages >= 2 that no later stage
+// forwards get their own counters and come after the forwarded ones of their stage, 2 = stage 1
+// too (by row: a row any of whose first hops forwards it counts as forwarded)
 void lower_plan(const Relation &rel, const Plan &plan, const int32_t *part,
                 const std::vector<int64_t> &loc, Lowered *out, int n_blocks = 1,
-                bool with_atomic = false, bool with_fanout = false, int mc_min_fanout = 0);
+                bool with_atomic = false, bool with_fanout = false, int mc_min_fanout = 0,
+                int leaf_split = 0);
 
 // Work items for one launch: the groups `gids` (already in stage order, READY / WAIT groups
 // included by the caller) cut into row ranges of about item_bytes gathered bytes and interleaved

@@ -308,6 +308,13 @@ class Context:
         check(lib().dgcl_debug_hostsim_forward(self.handle, layer, emb.ctypes.data,
                                                halo.ctypes.data), self.handle)
 
+    def debug_check_protocol(self, layer, direction=0, mutate=0):
+        """Host check of one launch's flag protocol (dgcl.h); raises DGCLError on a violation."""
+        buf = ctypes.create_string_buffer(512)
+        check(lib().dgcl_debug_check_protocol(self.handle, layer, direction, mutate, buf, 512),
+              self.handle)
+        return buf.value.decode()
+
     def debug_hostsim_backward(self, layer, halo_grad, emb_grad):
         halo_grad = _np(halo_grad, np.float32)
         assert emb_grad.dtype == np.float32 and emb_grad.flags.c_contiguous

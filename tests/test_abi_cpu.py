@@ -398,3 +398,72 @@ def test_random_lowering_host(seed):
     n = int(rng.choice([300, 900, 2000]))
     g = synth.make_graph(n, 8 * n, m, graph_seed=300 + seed, part_seed=400 + seed)
     _check_lowering(g, dims, topo, seed=seed, options=opts)
+
+
+# ---- the flag protocol of the lowered programs, checked on the host ----------------------------
+_PROTO_OPTS = [{"leaf_split": 0}, {"leaf_split": 1}, {"leaf_split": 2}, {"pipeline_blocks": 4},
+               {"fanout": 1}, {"fanout": 1, "leaf_split": 1}, {"direct_reduce": 0},
+               {"stage_fold": 0}, {"geometry": 2}]
+
+
+@pytest.mark.parametrize("topo", ["dgx1_like", "ring", None])
+@pytest.mark.parametrize("per_rank", [0, 1])
+def test_protocol_check(topo, per_rank):
+    """Every lowered program passes the host protocol check (dgcl_debug_check_protocol): wait
+    targets equal the rows signalled on their counters, no deadlock in list order, every row read
+    in the launch it is written is read only after waiting on its writer's counter,
+    each halo row written once.  Relay plans under every stage-chaining variant (leaf split off /
+    stages >= 2 / every stage, vertex blocks, per-pair stage 1, staged backward)."""
+    D = _D()
+    g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
+    flags = D.LOOPBACK_PER_RANK if per_rank else D.LOOPBACK_FUSED
+    opts_list = _PROTO_OPTS + ([{"multicast": 1}, {"multicast": 3}] if topo is None else [])
+    for opts in opts_list:
+        ctx = D.loopback(8, g.part, [40, 3], device=-1, flags=flags)
+        for k, v in opts.items():
+            ctx.set_option(k, v)
+        ctx.build_plan(g.req_ptr, g.req_ids, seed=9,
+                       topology=synth.topology.by_name(topo) if topo else None)
+        for layer in range(2):
+            for d in range(2):
+                assert ctx.debug_check_protocol(layer, d).startswith("ok"), (opts, layer, d)
+
+
+@pytest.mark.parametrize("per_rank", [0, 1])
+def test_protocol_check_rejects(per_rank):
+    """The checker's negative pins: a stage-chained item that stops waiting (race), the same item
+    moved before its producers (deadlock in one list; across per-rank lists it only waits), a
+    repeated data item (row written twice / counter overshoot), a producer that stops signalling
+    (target never reached)."""
+    D = _D()
+    g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
+    flags = D.LOOPBACK_PER_RANK if per_rank else D.LOOPBACK_FUSED
+    for topo in ("dgx1_like", "ring"):
+        ctx = D.loopback(8, g.part, [40], device=-1, flags=flags)
+        ctx.build_plan(g.req_ptr, g.req_ids, seed=9, topology=synth.topology.by_name(topo))
+        assert ctx.debug_check_protocol(0, 0).startswith("ok")
+        for mu, what in ((1, "without waiting|before it is written"), (2, "deadlock"),
+                         (3, "written twice|ever signalled"), (4, "ever signalled")):
+            if mu == 2 and per_rank:
+                assert ctx.debug_check_protocol(0, 0, mu).startswith("ok")
+                continue
+            with pytest.raises(D.DGCLError, match=what):
+                ctx.debug_check_protocol(0, 0, mu)
+        if per_rank:  # staged backward: slot reads chained the same way
+            with pytest.raises(D.DGCLError, match="before it is written|without waiting"):
+                ctx.debug_check_protocol(0, 1, 1)
+
+
+@pytest.mark.parametrize("name", ["google8_ring", "google8_dgx1", "reddit_dgx1", "google8"])
+def test_protocol_check_full_size(name):
+    """The BASELINE configs' programs at full size (fused and per-rank) pass the protocol check."""
+    D = _D()
+    c = synth.get_config(name)
+    g = synth.make_graph(c.n, c.e, c.m, c.graph_seed, c.part_seed, keep_edges=False)
+    topo = synth.topology.by_name(c.topology, c.m) if c.topology != "uniform_nvswitch" else None
+    for flags in (D.LOOPBACK_FUSED, D.LOOPBACK_PER_RANK):
+        ctx = D.loopback(c.m, g.part, list(c.dims), device=-1, flags=flags)
+        ctx.build_plan(g.req_ptr, g.req_ids, seed=0, topology=topo)
+        for layer in range(len(c.dims)):
+            for d in range(2):
+                assert ctx.debug_check_protocol(layer, d).startswith("ok"), (flags, layer, d)

@@ -233,31 +233,39 @@ def test_relay_plans(name, flags, tma, sf):
     _check_case(c)
 
 
-@pytest.mark.parametrize("tma,flags,blocks", [(1, 0, 4), (0, 0, 4), (1, 1, 4), (1, 0, 1)])
-def test_trace_stage_causality(tma, flags, blocks):
+@pytest.mark.parametrize("tma,flags,blocks,leaf", [(1, 0, 4, 2), (0, 0, 4, 2), (1, 1, 4, 2),
+                                                   (1, 0, 1, 0), (1, 0, 1, 2), (1, 1, 1, 2),
+                                                   (0, 1, 1, 1)])
+def test_trace_stage_causality(tma, flags, blocks, leaf):
     """Option "trace": per-item timelines of a relay plan's forward.  Stage chaining on device
     flags means no stage-k item of GPU r passes its waits before every stage-(k-1) item of the
     same vertex block into r has stored its rows; every item is traced once, in
-    order start <= ready <= done; with blocks, later blocks' stage k-1 may still be running."""
+    order start <= ready <= done; with blocks, later blocks' stage k-1 may still be running.
+    Leaf split (one block): the stage-(k-1) rows r forwards are block 0; r's stage-k items wait
+    for those, not for the leaf deliveries (block 1) of stage k-1."""
     D = _D()
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
     c = Case(g, [40], topo=synth.topology.by_name("dgx1_like"), seed=9, flags=flags,
-             options={"tma": tma, "trace": 1, "pipeline_blocks": blocks})
+             options={"tma": tma, "trace": 1, "pipeline_blocks": blocks, "leaf_split": leaf})
     K = c.ctx.plan_info()["n_stages"]
     assert K >= 2
     _check_case(c, bwd=False)
     ranks = range(c.m) if flags == D.LOOPBACK_PER_RANK else [0]
     T = [c.ctx.trace(0, 0, r) for r in ranks]
     T = {k: np.concatenate([t[k] for t in T]) for k in T[0]}
-    data = T["op"] <= 1
+    data = (T["op"] <= 1) | (T["op"] == 6)  # COPY, FOLD, FANOUT
     assert data.sum() > 0 and np.all(T["t_start"][data] > 0)
     assert np.all(T["t_start"][data] <= T["t_ready"][data])
     assert np.all(T["t_ready"][data] <= T["t_done"][data])
+    split = blocks == 1 and leaf > 0
+    if split:
+        assert (T["block"][data] == 1).any()  # leaf deliveries exist on this plan
     for r in range(c.m):
         for k in range(2, K + 1):
             for b in range(8):
                 after = data & (T["exec"] == r) & (T["stage"] == k) & (T["block"] == b)
-                before = data & (T["dst"] == r) & (T["stage"] == k - 1) & (T["block"] == b)
+                before = data & (T["dst"] == r) & (T["stage"] == k - 1) & \
+                    (T["block"] == (0 if split else b))
                 if after.any() and before.any():
                     assert T["t_ready"][after].min() >= T["t_done"][before].max(), (r, k, b)
 
