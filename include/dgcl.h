@@ -221,6 +221,10 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    of a block waits only for stage k-1 of the same block, so consecutive stages
  *                    may overlap; 1 = one done counter per (stage, source) as in §6.1.  Measured
  *                    slower with more blocks on one B200 (smaller groups and items)
+ *   "leaf_split"     relay plans: 1 (default) the deliveries of stages >= 2 that no later stage
+ *                    forwards count on done counters of their own (nothing but the forward
+ *                    completion waits on them) and follow the stage's forwarded rows, so stage k+1
+ *                    starts once stage k's forwarded rows landed; 2 stage 1 too; 0 off
  *   "align_sources"  1 (default): the forward COPY groups that read one rank's embeddings (one per
  *                    receiver) are cut into items at common source rows, so the copies of a row
  *                    to its receivers run close together (L2 reuse; rows <= 1 KB); 0: independent

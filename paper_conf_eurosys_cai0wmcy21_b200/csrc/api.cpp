@@ -116,7 +116,8 @@ struct dgcl_ctx {
   size_t mc_map_bytes = 0;      // granularity-rounded size of the mappings
   bool align_sources = true;          // forward COPY items of one source rank cut at common rows
   int pipeline_blocks = 1;            // relay plans: vertex blocks of the stage chaining
-  int leaf_split = 2;                 // relay plans: leaf deliveries after each stage's forwards
+  int leaf_split = 1;                 // relay plans: leaf deliveries after each stage's forwards
+                                      // (A/B r2ab: 1 best; dgx1_like 0.721 -> 0.694 ms)
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
