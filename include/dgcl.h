@@ -225,6 +225,10 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    forwards count on done counters of their own (nothing but the forward
  *                    completion waits on them) and follow the stage's forwarded rows, so stage k+1
  *                    starts once stage k's forwarded rows landed; 2 stage 1 too; 0 off
+ *   "relay_lead_kb"  relay plans with the leaf split: the forwarded rows of every stage run ahead
+ *                    of the leaves — after stage k's forwarded items come about this many KB of
+ *                    leaf rows (any stage <= k), then stage k+1's forwarded items, the remaining
+ *                    leaves last (default 196608; -1 = stage-major build order)
  *   "align_sources"  1 (default): the forward COPY groups that read one rank's embeddings (one per
  *                    receiver) are cut into items at common source rows, so the copies of a row
  *                    to its receivers run close together (L2 reuse; rows <= 1 KB); 0: independent

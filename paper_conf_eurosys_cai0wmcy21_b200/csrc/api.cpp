@@ -118,6 +118,8 @@ struct dgcl_ctx {
   int pipeline_blocks = 1;            // relay plans: vertex blocks of the stage chaining
   int leaf_split = 1;                 // relay plans: leaf deliveries after each stage's forwards
                                       // (A/B r2ab: 1 best; dgx1_like 0.721 -> 0.694 ms)
+  int64_t relay_lead_kb = 196608;     // relay forwards: leaves between stages' forwarded items
+                                      // (A/B r3c/r3d: ring 0.862 -> 0.853 ms, others neutral)
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
@@ -426,6 +428,8 @@ void build_programs(dgcl_ctx *c) {
         build_items(L, G, row_bytes, lim, !fused || c->signal_all, need, &P.items, &P.runs,
                     c->direct_copy_rows,
                     c->stage_fold ? &P.sterms : nullptr);
+        if (dir == DIR_FWD && c->relay_lead_kb >= 0)
+          lead_relay_items(L, &P.items, row_bytes, c->relay_lead_kb * 1024);
         P.op_mask = 0;
         int64_t fold_rows = 0, fold_terms = 0;
         for (const DevItem &it : P.items) {
@@ -1706,6 +1710,12 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "stage_fold") {  // bulk-copy FOLD operand rows into the stage (bulk-copy executor)
     c->stage_fold = value != 0;
+    if (c->planned) build_programs(c);
+    return DGCL_OK;
+  }
+  if (k == "relay_lead_kb") {  // relay forwards: KB of leaves between stages (-1: build order)
+    if (value < -1 || value > (1 << 30)) return fail(c, DGCL_EINVAL, "relay_lead_kb in -1..2^30");
+    c->relay_lead_kb = value;
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }

@@ -332,6 +332,9 @@ __global__ void __launch_bounds__(512, DGCL_REG_MINB) executor_kernel(const __gr
         for (int s = 0; s < P.world; ++s)
           if (s != I.exec_rank && !((s_ready_ok >> s) & 1u)) may_block = true;
       if (I.wait_n > 0 && s_wait_ok[I.exec_rank] != I.wait_off) may_block = true;
+      // (an item that signals nothing: publish the counts of the signalling items before it)
+      if ((I.op == OP_COPY || I.op == OP_FOLD || I.op == OP_FANOUT) && !(I.flags & kItemSignal))
+        may_block = true;
       s_flush = may_block && s_npend > 0;
     }
     __syncthreads();

@@ -1098,7 +1098,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         if (!ok) break;
       } else if (I.op == OP_COPY || I.op == OP_FOLD || I.op == OP_FANOUT) {
         // Done counts are published in batches (FLUSH markers): before this producer could
-        // block on a wait, and whenever the counter family (direction, stage) changes.
+        // block on a wait, whenever the counter family (direction, stage) changes, and before
+        // an item that signals nothing (relay forwards: a stage's leaves follow its forwarded
+        // rows, whose counts the next stage waits on — holding them back until this CTA blocks
+        // would delay that stage by the whole leaf phase)
         const bool sig = (I.flags & kItemSignal) != 0;
         const int key = sig ? I.sig_ctr - I.exec_rank : -1;
         if (pend) {
@@ -1114,17 +1117,18 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
                   ready = ld_acquire(P.flags[I.exec_rank] + kReadyBase + s, P.sys_scope) >= P.seq;
           }
           ready = __shfl_sync(0xffffffffu, ready, 0);
-          if (!ready || (sig && key != pend_key)) {
+          if (!ready || key != pend_key) {
             emit_marker(OP_FLUSH);
             pend = false;
           }
         }
-        int w = 1;
+        int w = 1, acq = 0;
         if (lane == 0) {
           // sources final (stage chaining) and the destination's buffers free (ready word)
           if (!known_sources(I)) {
             w = wait_item_sources(P, I, 100000 + I.group) ? 1 : 0;
             if (w) s_wait_ok[I.exec_rank] = I.wait_off;
+            acq = 1;
           }
           if (w && P.use_ready && I.ready_rank >= 0 && !((ready_ok >> I.ready_rank) & 1u)) {
             w = wait_geq(P.flags[I.exec_rank] + kReadyBase + I.ready_rank, P.seq, P,
@@ -1140,7 +1144,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
         }
         ok = __shfl_sync(0xffffffffu, w, 0) != 0;
         if (!ok) break;
-        if (I.wait_n > 0) fence_proxy_async_global();  // acquired peers' rows -> bulk reads
+        // acquired peers' rows -> bulk reads (a wait list found satisfied earlier was fenced then:
+        // this warp's later bulk reads follow that fence in program order)
+        if (__shfl_sync(0xffffffffu, acq, 0)) fence_proxy_async_global();
         mbar_wait(&metab[m % kMetaSlots], (m / kMetaSlots) & 1u);
         uint32_t stage, use;
         ring_pos(k, NS, stage, use);

@@ -21,6 +21,7 @@
 #include <functional>
 #include <chrono>
 #include <cstring>
+#include <deque>
 #include <map>
 #include <tuple>
 
@@ -1244,6 +1245,58 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
     }
     i = j;
   }
+}
+
+}  // namespace dgcl
+
+namespace dgcl {
+
+// Relay forwards with the leaf split (see lower_plan): the forwarded rows form the critical
+// chain stage 1 -> 2 -> ... -> K (stage k+1's forwarded items wait on stage k's), the leaves
+// feed nothing.  Build order is stage-major, so stage k+1's forwarded items were claimed only
+// after all of stage k's leaves, and then waited for the stage-k drain.  Here the chain goes
+// first: after stage k's forwarded items come about `lead_bytes` of leaves (any stage <= k: all
+// runnable by then) to cover the drain, then stage k+1's forwarded items; the remaining leaves
+// last.  Every item still follows the items it waits on (deadlock-free in list order).
+void lead_relay_items(const Lowered &low, std::vector<DevItem> *items, int64_t row_bytes,
+                      int64_t lead_bytes) {
+  if (low.leaf_block < 0 || lead_bytes < 0 || items->empty()) return;
+  const int64_t row16 = (row_bytes + 15) / 16 * 16;
+  std::vector<DevItem> head, tail;
+  std::vector<std::vector<DevItem>> chain(kMaxStages + 1), leaves(kMaxStages + 1);
+  int K = 0;
+  for (const DevItem &it : *items) {
+    if (it.op == OP_READY) {
+      head.push_back(it);
+      continue;
+    }
+    if (it.op == OP_WAIT) {
+      tail.push_back(it);
+      continue;
+    }
+    const DevGroup &g = low.groups[it.group];
+    if (g.dir != DIR_FWD || g.stage < 1 || g.stage > kMaxStages) return;  // (not a relay forward)
+    K = std::max(K, (int)g.stage);
+    (g.block == low.leaf_block ? leaves : chain)[g.stage].push_back(it);
+  }
+  std::vector<DevItem> out = head;
+  std::deque<DevItem> pool;
+  for (int k = 1; k <= K; ++k) {
+    out.insert(out.end(), chain[k].begin(), chain[k].end());
+    pool.insert(pool.end(), leaves[k].begin(), leaves[k].end());
+    bool more = false;  // forwarded rows in a later stage
+    for (int j = k + 1; j <= K && !more; ++j) more = !chain[j].empty();
+    if (!more) continue;
+    int64_t b = 0;
+    while (!pool.empty() && b < lead_bytes) {
+      b += (int64_t)pool.front().rows * row16;
+      out.push_back(pool.front());
+      pool.pop_front();
+    }
+  }
+  out.insert(out.end(), pool.begin(), pool.end());
+  out.insert(out.end(), tail.begin(), tail.end());
+  if (out.size() == items->size()) items->swap(out);
 }
 
 }  // namespace dgcl

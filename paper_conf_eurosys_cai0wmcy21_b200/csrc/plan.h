@@ -146,4 +146,10 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
                  std::vector<DevItem> *items, std::vector<DevRun> *runs,
                  int64_t direct_copy_rows = 0, std::vector<uint32_t> *sterms = nullptr);
 
+// Relay forwards with the leaf split: reorder a launch's items so the forwarded rows of every
+// stage run ahead of the leaves, with about lead_bytes of leaves between consecutive stages'
+// forwarded items (< 0: keep the build order)
+void lead_relay_items(const Lowered &low, std::vector<DevItem> *items, int64_t row_bytes,
+                      int64_t lead_bytes);
+
 }  // namespace dgcl

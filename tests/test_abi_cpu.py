@@ -403,7 +403,9 @@ def test_random_lowering_host(seed):
 # ---- the flag protocol of the lowered programs, checked on the host ----------------------------
 _PROTO_OPTS = [{"leaf_split": 0}, {"leaf_split": 1}, {"leaf_split": 2}, {"pipeline_blocks": 4},
                {"fanout": 1}, {"fanout": 1, "leaf_split": 1}, {"direct_reduce": 0},
-               {"stage_fold": 0}, {"geometry": 2}]
+               {"stage_fold": 0}, {"geometry": 2}, {"relay_lead_kb": -1}, {"relay_lead_kb": 0},
+               {"relay_lead_kb": 1}, {"leaf_split": 2, "relay_lead_kb": 1},
+               {"leaf_split": 2, "fanout": 1, "relay_lead_kb": 2}]
 
 
 @pytest.mark.parametrize("topo", ["dgx1_like", "ring", None])
