@@ -119,7 +119,7 @@ struct dgcl_ctx {
   int leaf_split = 1;                 // relay plans: leaf deliveries after each stage's forwards
                                       // (A/B r2ab: 1 best; dgx1_like 0.721 -> 0.694 ms)
   int64_t relay_lead_kb = 196608;     // relay forwards: leaves between stages' forwarded items
-                                      // (A/B r3c/r3d: ring 0.862 -> 0.853 ms, others neutral)
+                                      // (A/B r2sc/r2sd: ring 0.862 -> 0.853 ms, others neutral)
   int64_t direct_copy_rows = 0;       // COPY items with shorter average runs: consumer gathers
   bool use_gather4 = true;            // TMA gather4 for short-run embedding gathers
   bool stage_fold = true;             // FOLD operand rows bulk-copied into the stage
