@@ -229,6 +229,10 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    of the leaves — after stage k's forwarded items come about this many KB of
  *                    leaf rows (any stage <= k), then stage k+1's forwarded items, the remaining
  *                    leaves last (default 196608; -1 = stage-major build order)
+ *   "owner_major"    fused loopback: 1 (default) the forward COPY items of one owner's groups (its
+ *                    embeddings to each receiver) run together, owner after owner — the write
+ *                    front is a few long runs of halo rows and the owner's rows stay in L2 for
+ *                    its receivers; 0: chunk c of every (owner, receiver) group together
  *   "align_sources"  1 (default): the forward COPY groups that read one rank's embeddings (one per
  *                    receiver) are cut into items at common source rows, so the copies of a row
  *                    to its receivers run close together (L2 reuse; rows <= 1 KB); 0: independent

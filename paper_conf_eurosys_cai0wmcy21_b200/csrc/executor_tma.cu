@@ -30,11 +30,26 @@ namespace {
 #ifndef DGCL_HELPER
 #define DGCL_HELPER 1  // copy launches: this many helper warps issue a share of each item's gathers
 #endif
+// diagnostic builds (tools/build_variant.sh): DGCL_DIAG_NO_GATHER — COPY items store whatever the
+// stage holds (no row gathers); DGCL_DIAG_NO_STORE — COPY items gather but store nothing
+#ifndef DGCL_DIAG_NO_GATHER
+#define DGCL_DIAG_NO_GATHER 0
+#endif
+#ifndef DGCL_DIAG_NO_STORE
+#define DGCL_DIAG_NO_STORE 0
+#endif
 #ifndef DGCL_FAN_BULK_ROW
 #define DGCL_FAN_BULK_ROW 1024
 #endif
 #ifndef DGCL_STORE_SPLIT
-#define DGCL_STORE_SPLIT 15  // every consumer warp stores its share (measured best, Reddit)
+#define DGCL_STORE_SPLIT 4  // bulk stores per COPY stage (A/B r2sg/r2sh; 15 rotating before)
+#endif
+// DGCL_STORE_FIXED 1: the same consumer warps store every stage, so each of them has one bulk
+// store in flight and a CTA writes at most kStoreSplit runs at a time; HBM writes fewer, longer
+// runs (tools/store_bench.cu: one 60-KB store stream per SM 7.06 TB/s, 15 concurrent 4-KB pieces
+// 6.26 TB/s); 0: warps rotate per stage
+#ifndef DGCL_STORE_FIXED
+#define DGCL_STORE_FIXED 1
 #endif
 constexpr int kStoreSplit = DGCL_STORE_SPLIT;  // bulk stores per COPY item (<= consumer warps)
 constexpr int kFanBulkRowBytes = DGCL_FAN_BULK_ROW;  // fan-out rows stored by bulk stores
@@ -346,13 +361,16 @@ __device__ __forceinline__ void issue_item(const ExecParams &P, const DevItem &I
     info[2] = (int32_t)item_index;  // (trace records)
   }
   __syncwarp();  // header and info written before lane 0's arrive publishes the stage
-  if (lane == 0) mbar_expect_tx(full, operand_bytes<kLsu>(P, I) + wtp.bytes + wdst.bytes);
+  const bool diag_ng = DGCL_DIAG_NO_GATHER && I.op == OP_COPY;
+  if (lane == 0)
+    mbar_expect_tx(full, (diag_ng ? 0u : operand_bytes<kLsu>(P, I)) + wtp.bytes + wdst.bytes);
   __syncwarp();
   if (lane == 0) {
     if (wtp.bytes) bulk_g2s(st + kTabTp, P.term_ptr + wtp.a, wtp.bytes, full);
     if (wdst.bytes) bulk_g2s(st + kTabDst, P.idx + wdst.a, wdst.bytes, full);
   }
   uint8_t *ops = st + kStageHdrBytes;
+  if (diag_ng) return;
   if (I.op == OP_FANOUT) {
     // consecutive source rows: one bulk copy (packed rows), then the destination words
     const BufRef S = P.buf[I.src_kind][I.exec_rank];
@@ -1238,16 +1256,18 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           gather_lsu(P, I, const_cast<uint8_t *>(st), tid, T);
           consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
         }
-        if ((kMask & kMaskMcast) && I.dst_kind == K_MCAST) {
+        if (DGCL_DIAG_NO_STORE) {
+        } else if ((kMask & kMaskMcast) && I.dst_kind == K_MCAST) {
           store_copy_mc(P, I, st, tid, T);
         } else if (I.flags & kItemAtomic) {
           store_copy_atomic(P, I, st, tid, T);
         } else if (P.bulk_store && I.dst >= 0 && DB.pitch == (int64_t)P.row16) {
           // consecutive packed destination rows: kStoreSplit bulk (TMA) stores move the item,
-          // issued by consumer warps (k * kStoreSplit + j) % n_cons_warps, so the stores of
-          // several stages overlap while the other warps move on
+          // issued by consumer warps 0 .. kStoreSplit-1 (DGCL_STORE_FIXED; else rotating
+          // (k * kStoreSplit + j) % n_cons_warps); the other warps move on
           const int split = kStoreSplit < n_cons_warps ? kStoreSplit : n_cons_warps;
-          const int first = (int)((k * (uint32_t)split) % (uint32_t)n_cons_warps);
+          const int first =
+              DGCL_STORE_FIXED ? 0 : (int)((k * (uint32_t)split) % (uint32_t)n_cons_warps);
           const int j = (cw - first + n_cons_warps) % n_cons_warps;
           if (j < split && lane == 0) {
             const int64_t lo = (int64_t)I.rows * j / split;

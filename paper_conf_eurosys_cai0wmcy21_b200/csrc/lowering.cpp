@@ -1156,9 +1156,25 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       }
       max_chunks = std::max(max_chunks, b.size() - 1);
     }
-    // interleave the chunks of the groups of this stage (all peers / sources busy at once)
+    // interleave the chunks of the groups of this stage (all peers / sources busy at once); with
+    // lim.owner_major the forward COPY groups of one executing rank (one owner's embeddings to
+    // each of its receivers, adjacent in [i, j)) are interleaved among themselves and the ranks
+    // follow each other: the launch's write front is a few long runs of halo rows instead of one
+    // chunk of every (owner, receiver) pair, and the owner's rows stay in L2 for its receivers
+    std::vector<std::pair<size_t, size_t>> spans;  // [qb, qe) interleaved together
+    for (size_t qb = i; qb < j;) {
+      size_t qe = qb + 1;
+      const DevGroup &gb = low.groups[gids[qb]];
+      const bool om = lim.owner_major && gb.op == OP_COPY && gb.dir == DIR_FWD;
+      while (qe < j && (!om || (low.groups[gids[qe]].exec_rank == gb.exec_rank &&
+                                low.groups[gids[qe]].op == OP_COPY)))
+        ++qe;
+      spans.push_back({qb, qe});
+      qb = qe;
+    }
+    for (const auto &sp : spans)
     for (size_t c = 0; c < max_chunks; ++c) {
-      for (size_t q = i; q < j; ++q) {
+      for (size_t q = sp.first; q < sp.second; ++q) {
         const DevGroup &g = low.groups[gids[q]];
         const std::vector<int32_t> &b = bounds[q - i];
         if (c + 1 >= b.size()) continue;

@@ -384,7 +384,8 @@ def test_random_lowering_host(seed):
     opts = {"hostsim_items": int(rng.rand() < 0.7)}
     for key, vals in (("geometry", [0, 1, 2]), ("stage_fold", [0, 1]),
                       ("direct_reduce", [0, 1]), ("align_sources", [0, 1]),
-                      ("item_bytes", [1024, 8192, 65536])):
+                      ("item_bytes", [1024, 8192, 65536]), ("owner_major", [0, 1]),
+                      ("relay_lead_kb", [-1, 0, 1, 196608])):
         opts[key] = int(rng.choice(vals))
     if topo is None:
         r = rng.rand()
@@ -405,7 +406,7 @@ _PROTO_OPTS = [{"leaf_split": 0}, {"leaf_split": 1}, {"leaf_split": 2}, {"pipeli
                {"fanout": 1}, {"fanout": 1, "leaf_split": 1}, {"direct_reduce": 0},
                {"stage_fold": 0}, {"geometry": 2}, {"relay_lead_kb": -1}, {"relay_lead_kb": 0},
                {"relay_lead_kb": 1}, {"leaf_split": 2, "relay_lead_kb": 1},
-               {"leaf_split": 2, "fanout": 1, "relay_lead_kb": 2}]
+               {"leaf_split": 2, "fanout": 1, "relay_lead_kb": 2}, {"owner_major": 1}]
 
 
 @pytest.mark.parametrize("topo", ["dgx1_like", "ring", None])
