@@ -48,6 +48,9 @@ namespace {
 // store in flight and a CTA writes at most kStoreSplit runs at a time; HBM writes fewer, longer
 // runs (tools/store_bench.cu: one 60-KB store stream per SM 7.06 TB/s, 15 concurrent 4-KB pieces
 // 6.26 TB/s); 0: warps rotate per stage
+#ifndef DGCL_STG_SHARE
+#define DGCL_STG_SHARE 0  // percent of a bulk-store COPY stage stored with STG instead (A/B)
+#endif
 #ifndef DGCL_STORE_FIXED
 #define DGCL_STORE_FIXED 1
 #endif
@@ -1269,14 +1272,31 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
           const int first =
               DGCL_STORE_FIXED ? 0 : (int)((k * (uint32_t)split) % (uint32_t)n_cons_warps);
           const int j = (cw - first + n_cons_warps) % n_cons_warps;
+          // (DGCL_STG_SHARE > 0: the last share of the rows is stored by the other consumer warps
+          // with LDS + STG, off the TMA unit)
+          const int64_t rows_tma =
+              DGCL_STG_SHARE && n_cons_warps > split ? (int64_t)I.rows * (100 - DGCL_STG_SHARE) / 100
+                                                     : (int64_t)I.rows;
           if (j < split && lane == 0) {
-            const int64_t lo = (int64_t)I.rows * j / split;
-            const int64_t hi = (int64_t)I.rows * (j + 1) / split;
+            const int64_t lo = rows_tma * j / split;
+            const int64_t hi = rows_tma * (j + 1) / split;
             if (hi > lo) {
               s2g(DB.ptr + (I.dst + lo) * DB.pitch, st + kStageHdrBytes + lo * P.row16,
                   (uint32_t)((hi - lo) * P.row16), pol_st);
               bulk_commit();
               bulk_wait_read();  // the stage may be reused once the bulk store has read it
+            }
+          } else if (DGCL_STG_SHARE && j >= split && rows_tma < I.rows) {
+            const uint32_t nch = (uint32_t)P.n_chunks;
+            const uint32_t t2 = (uint32_t)(j - split) * 32 + lane;
+            const uint32_t T2 = (uint32_t)(n_cons_warps - split) * 32;
+            const uint32_t e_end = (uint32_t)I.rows * nch;
+            char *d0 = DB.ptr + I.dst * DB.pitch;
+            const uint8_t *ops = st + kStageHdrBytes;
+            for (uint32_t e = (uint32_t)rows_tma * nch + t2; e < e_end; e += T2) {
+              const uint32_t r = fdiv(e, P);
+              const uint32_t col = e - r * nch;
+              st_v4(d0 + (int64_t)r * DB.pitch + col * 16, lds_v4(ops + r * P.row16 + col * 16));
             }
           }
         } else {
