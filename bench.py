@@ -374,12 +374,18 @@ def run_ours_single(args, w):
     evs = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)]
             for _ in names] for _ in range(K)]
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    launches0 = ctx.launch_count()
+    # per-launch durations: K steps with an event pair around every launch; then the step
+    # itself: K steps back to back with events only at the two ends (an event between two
+    # launches delays the second one's start by a few us, ~1 % of a step)
     torch.cuda.synchronize()
     tw0 = time.time()
-    e0.record(stream)
     for k in range(K):
         step(evs[k])
+    torch.cuda.synchronize()
+    launches0 = ctx.launch_count()
+    e0.record(stream)
+    for k in range(K):
+        step()
     e1.record(stream)
     torch.cuda.synchronize()
     tw1 = time.time()
