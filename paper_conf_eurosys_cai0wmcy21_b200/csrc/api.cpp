@@ -118,7 +118,7 @@ struct dgcl_ctx {
   int pipeline_blocks = 1;            // relay plans: vertex blocks of the stage chaining
   int leaf_split = 1;                 // relay plans: leaf deliveries after each stage's forwards
                                       // (A/B r2ab: 1 best; dgx1_like 0.721 -> 0.694 ms)
-  bool owner_major = true;            // fused loopback forwards: one owner's groups at a time
+  int owner_major = 1;                // fused loopback forwards: one owner's groups at a time
                                       // (A/B r2sh: Reddit fwd602 -1 %, Com-Orkut -2.5 %,
                                       // Web-Google dgx1_like -6 %)
   int64_t relay_lead_kb = 196608;     // relay forwards: leaves between stages' forwarded items
@@ -428,7 +428,7 @@ void build_programs(dgcl_ctx *c) {
                                      (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm);
         lim.align_sources = c->align_sources;
         lim.lsu_gather = c->lsu_gather && c->use_tma;
-        lim.owner_major = c->owner_major && fused;
+        lim.owner_major = fused ? c->owner_major : 0;
         build_items(L, G, row_bytes, lim, !fused || c->signal_all, need, &P.items, &P.runs,
                     c->direct_copy_rows,
                     c->stage_fold ? &P.sterms : nullptr);
@@ -1718,7 +1718,8 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
     return DGCL_OK;
   }
   if (k == "owner_major") {  // fused loopback forwards: items of one owner's groups at a time
-    c->owner_major = value != 0;
+    if (value < 0 || value > 2) return fail(c, DGCL_EINVAL, "owner_major in 0..2");
+    c->owner_major = (int)value;
     if (c->planned) build_programs(c);
     return DGCL_OK;
   }

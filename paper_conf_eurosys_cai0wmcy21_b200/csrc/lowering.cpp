@@ -1166,7 +1166,9 @@ void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t r
       size_t qe = qb + 1;
       const DevGroup &gb = low.groups[gids[qb]];
       const bool om = lim.owner_major && gb.op == OP_COPY && gb.dir == DIR_FWD;
-      while (qe < j && (!om || (low.groups[gids[qe]].exec_rank == gb.exec_rank &&
+      // (owner_major 2: every forward COPY group on its own — one write run at a time)
+      while (qe < j && (!om || (lim.owner_major == 1 &&
+                                low.groups[gids[qe]].exec_rank == gb.exec_rank &&
                                 low.groups[gids[qe]].op == OP_COPY)))
         ++qe;
       spans.push_back({qb, qe});

@@ -139,7 +139,8 @@ struct ItemLimits {
   int64_t min_items;      // COPY items per stage to aim for (co-resident CTAs; 0 = no spreading)
   bool align_sources = true;  // forward COPY groups of one source rank cut at common source rows
   bool lsu_gather = false;    // short-run COPY items gathered by the consumers (kItemLsu)
-  bool owner_major = false;   // forward COPY items: one executing rank's groups at a time
+  int owner_major = 0;        // forward COPY items: 1 one executing rank's groups at a time,
+                              // 2 one group at a time
 };
 ItemLimits item_limits(const TmaGeometry &g, int64_t item_bytes, int64_t min_items = 0);
 void build_items(const Lowered &low, const std::vector<int32_t> &gids, int64_t row_bytes,

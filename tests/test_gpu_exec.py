@@ -166,6 +166,8 @@ def test_tiny_config_bit_exact(small):
     (8, {"direct_reduce": 0, "item_bytes": 4096}),
     (8, {"geometry": 1}), (8, {"geometry": 2}), (4, {"geometry": 2, "direct_reduce": 0}),
     (3, {"geometry": 1, "stage_fold": 0}),
+    # item order of fused forwards: chunk-major / group-major (default owner-major)
+    (8, {"owner_major": 0}), (8, {"owner_major": 2}), (4, {"owner_major": 2, "align_sources": 0}),
     (8, {"fanout": 1}), (4, {"fanout": 1, "tma": 0}), (8, {"fanout": 1, "geometry": 2}),
     (3, {"fanout": 1, "bulk_store": 0}), (4, {"fanout": 1, "geometry": 1}),
     # NVSwitch multicast of high-fan-out rows, emulated on one GPU (one store per virtual rank's
@@ -211,13 +213,19 @@ def test_per_rank_flag_protocol(m, fanout, mc):
                                                ("ring", 0, 1, 5), ("dgx1_like", 1, 1, 6),
                                                ("ring", 1, 0, 6), ("ring", 0, 1, 7),
                                                ("dgx1_like", 0, 1, 7), ("ring", 1, 1, 7),
-                                               ("dgx1_like", 0, 0, 7)])
+                                               ("dgx1_like", 0, 0, 7), ("ring", 0, 1, 8),
+                                               ("dgx1_like", 1, 1, 8), ("ring", 0, 1, 9),
+                                               ("dgx1_like", 0, 0, 9), ("ring", 1, 1, 9),
+                                               ("dgx1_like", 0, 1, 10), ("ring", 0, 1, 11),
+                                               ("ring", 0, 1, 12)])
 def test_relay_plans(name, flags, tma, sf):
     """sf: stage_fold 0/1; 2, 3 = stage_fold with the DUAL / WIDE geometry forced; 4 = fan-out
     stage 1 (first hops into halos and relay staging, done counts per receiver); 5, 6 = one /
     eight vertex blocks in the stage chaining (default 1); 7 = the staged reversed-plan backward
     (direct_reduce = 0: pushes into slots stage by stage, the multi-GPU form) instead of the
-    loopback tree-order programs."""
+    loopback tree-order programs; 8 / 9 = the relay item order off (relay_lead_kb -1) / with a
+    1-KB lead (forwarded rows of the next stage right behind a few leaves); 10 = no leaf split;
+    11 / 12 = chunk-major / group-major stage 1 (owner_major 0 / 2)."""
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
     opts = {"tma": tma, "stage_fold": min(sf, 1)}
     if sf in (2, 3):
@@ -228,6 +236,12 @@ def test_relay_plans(name, flags, tma, sf):
         opts["pipeline_blocks"] = 1 if sf == 5 else 8
     if sf == 7:
         opts["direct_reduce"] = 0
+    if sf in (8, 9):
+        opts["relay_lead_kb"] = -1 if sf == 8 else 1
+    if sf == 10:
+        opts["leaf_split"] = 0
+    if sf in (11, 12):
+        opts["owner_major"] = 0 if sf == 11 else 2
     c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags, options=opts)
     assert c.ctx.plan_info()["n_stages"] >= 2
     _check_case(c)
@@ -647,6 +661,10 @@ def _random_option_case(seed):
     if rng.rand() < 0.2:
         opts["item_bytes"] = int(rng.choice([2048, 8192]))
     n = int(rng.choice([800, 3000, 7000]))
+    # (drawn last: the earlier draws, hence the earlier cases, are unchanged)
+    for key, vals in (("owner_major", [0, 1, 1, 2]), ("relay_lead_kb", [-1, 0, 1, 196608]),
+                      ("leaf_split", [0, 1, 1, 2])):
+        opts[key] = int(rng.choice(vals))
     return m, topo, flags, dims, opts, n
 
 

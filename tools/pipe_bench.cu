@@ -5,6 +5,8 @@
 //                    warps bulk-store it (the executor's scheme)
 //   mode 1 tma/stg : same loads, every consumer thread LDS + STG
 //   mode 2 ldg/stg : no shared memory, every thread LDG.128 x4 -> STG.128 x4
+//   mode 3 fan-out : a chunk is bulk-loaded once and bulk-stored to `split` destination regions
+//                    (one consumer warp each), as a fan-out of one owner's rows to its receivers
 // build: nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a tools/pipe_bench.cu -o build/pipe_bench
 #include <cstdio>
 #include <cstdint>
@@ -34,7 +36,7 @@ __global__ void __launch_bounds__(256) pipe(const char *src, size_t src_bytes, c
   uint64_t *full = reinterpret_cast<uint64_t *>(sm), *empty = full + 8;
   uint8_t *stg = sm + 128;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, ncw = (blockDim.x >> 5) - 1;
-  const size_t nch = total / chunk, G = gridDim.x;
+  const size_t nch = (kMode == 3 ? total / split : total) / chunk, G = gridDim.x;
   const size_t nsrc = src_bytes / chunk;
   if (kMode == 2) {
     for (size_t c = blockIdx.x; c < nch; c += G) {
@@ -83,7 +85,16 @@ __global__ void __launch_bounds__(256) pipe(const char *src, size_t src_bytes, c
     const uint32_t s = i % S, use = i / S;
     uint8_t *st = stg + (size_t)s * chunk;
     mb_wait(&full[s], use & 1);
-    if (kMode == 1) {
+    if (kMode == 3) {
+      if (cw < split && lane == 0) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(
+                         dst + (size_t)cw * nch * chunk + c * chunk),
+                     "r"(sa(st)), "r"(chunk) : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+      }
+    } else if (kMode == 1) {
       for (int o = tid * 16; o < chunk; o += T * 16)
         *reinterpret_cast<int4 *>(dst + c * chunk + o) = *reinterpret_cast<const int4 *>(st + o);
     } else if (cw < split && lane == 0) {
@@ -130,6 +141,8 @@ int main() {
            src_bytes >> 20, chunk, S, split, total / (best * 1e6),
            (src_bytes >= total ? 2.0 : 1.0) * total / (best * 1e6), e ? cudaGetErrorString(e) : "");
   };
+  for (int S : {2, 3})
+    for (int fan : {4, 7}) run("fan-out", pipe<3>, total, 61440, S, fan);
   for (size_t sb : {(size_t)48 << 20, total}) {
     run("ldg/stg", pipe<2>, sb, 61440, 0, 0, 1);
     run("ldg/stg", pipe<2>, sb, 61440, 0, 0, 8);
