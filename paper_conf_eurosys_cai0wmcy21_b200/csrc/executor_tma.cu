@@ -48,6 +48,11 @@ namespace {
 // store in flight and a CTA writes at most kStoreSplit runs at a time; HBM writes fewer, longer
 // runs (tools/store_bench.cu: one 60-KB store stream per SM 7.06 TB/s, 15 concurrent 4-KB pieces
 // 6.26 TB/s); 0: warps rotate per stage
+#ifndef DGCL_ROW_BULK
+#define DGCL_ROW_BULK 1024  // > 0: COPY rows of >= this many bytes to scattered destinations
+                            // (relay stages) go out as one bulk store per row; 0: consumer STG
+                            // (A/B r2so: relay forwards 1-1.5 % faster)
+#endif
 #ifndef DGCL_STG_SHARE
 #define DGCL_STG_SHARE 0  // percent of a bulk-store COPY stage stored with STG instead (A/B)
 #endif
@@ -1298,6 +1303,19 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
               const uint32_t col = e - r * nch;
               st_v4(d0 + (int64_t)r * DB.pitch + col * 16, lds_v4(ops + r * P.row16 + col * 16));
             }
+          }
+        } else if (DGCL_ROW_BULK && P.bulk_store && I.dst < 0 && DB.pitch == (int64_t)P.row16 &&
+                   P.row16 >= DGCL_ROW_BULK) {
+          // scattered destination rows (relay stages): one bulk store per row, rows spread over
+          // the consumer threads
+          const int32_t *tab = reinterpret_cast<const int32_t *>(st + kTabDst) +
+                               reinterpret_cast<const int32_t *>(st + kHdrInfo)[1];
+          for (uint32_t r = tid; r < (uint32_t)I.rows; r += T)
+            s2g(DB.ptr + (int64_t)tab[r] * DB.pitch, st + kStageHdrBytes + r * P.row16,
+                (uint32_t)P.row16, pol_st);
+          if (tid < (uint32_t)I.rows) {
+            bulk_commit();
+            bulk_wait_read();
           }
         } else {
           store_copy(P, I, st, tid, T);
