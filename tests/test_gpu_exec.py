@@ -217,7 +217,8 @@ def test_per_rank_flag_protocol(m, fanout, mc):
                                                ("dgx1_like", 1, 1, 8), ("ring", 0, 1, 9),
                                                ("dgx1_like", 0, 0, 9), ("ring", 1, 1, 9),
                                                ("dgx1_like", 0, 1, 10), ("ring", 0, 1, 11),
-                                               ("ring", 0, 1, 12)])
+                                               ("ring", 0, 1, 12), ("ring", 0, 1, 13),
+                                               ("dgx1_like", 1, 1, 13)])
 def test_relay_plans(name, flags, tma, sf):
     """sf: stage_fold 0/1; 2, 3 = stage_fold with the DUAL / WIDE geometry forced; 4 = fan-out
     stage 1 (first hops into halos and relay staging, done counts per receiver); 5, 6 = one /
@@ -225,7 +226,8 @@ def test_relay_plans(name, flags, tma, sf):
     (direct_reduce = 0: pushes into slots stage by stage, the multi-GPU form) instead of the
     loopback tree-order programs; 8 / 9 = the relay item order off (relay_lead_kb -1) / with a
     1-KB lead (forwarded rows of the next stage right behind a few leaves); 10 = no leaf split;
-    11 / 12 = chunk-major / group-major stage 1 (owner_major 0 / 2)."""
+    11 / 12 = chunk-major / group-major stage 1 (owner_major 0 / 2); 13 = dims 256 / 602 (rows
+    >= 1 KB: relay stages store scattered rows with one bulk store per row)."""
     g = synth.make_graph(4000, 20000, 8, graph_seed=5, part_seed=6)
     opts = {"tma": tma, "stage_fold": min(sf, 1)}
     if sf in (2, 3):
@@ -242,7 +244,8 @@ def test_relay_plans(name, flags, tma, sf):
         opts["leaf_split"] = 0
     if sf in (11, 12):
         opts["owner_major"] = 0 if sf == 11 else 2
-    c = Case(g, [40, 3], topo=synth.topology.by_name(name), seed=9, flags=flags, options=opts)
+    dims = [256, 602] if sf == 13 else [40, 3]
+    c = Case(g, dims, topo=synth.topology.by_name(name), seed=9, flags=flags, options=opts)
     assert c.ctx.plan_info()["n_stages"] >= 2
     _check_case(c)
 
