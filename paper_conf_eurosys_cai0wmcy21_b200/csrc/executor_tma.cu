@@ -106,8 +106,30 @@ __device__ __forceinline__ bool mbar_test(uint64_t *b, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
+#ifndef DGCL_WAIT_HINT
+#define DGCL_WAIT_HINT 0  // ns: try_wait suspend-time hint of the spin waits (0: none)
+#endif
+#ifndef DGCL_WAIT_SLEEP
+#define DGCL_WAIT_SLEEP 0  // ns: nanosleep between failed try_waits (0: none)
+#endif
+__device__ __forceinline__ bool mbar_test_hint(uint64_t *b, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n"
+      " selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(smem_u32(b)), "r"(parity), "r"((uint32_t)DGCL_WAIT_HINT)
+      : "memory");
+  return ok != 0;
+}
 __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+  if (DGCL_WAIT_HINT) {
+    while (!mbar_test_hint(b, parity)) {
+    }
+    return;
+  }
   while (!mbar_test(b, parity)) {
+    if (DGCL_WAIT_SLEEP) __nanosleep(DGCL_WAIT_SLEEP);
   }
 }
 __device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t bytes,
