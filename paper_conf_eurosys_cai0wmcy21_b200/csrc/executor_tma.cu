@@ -1251,12 +1251,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       const uint8_t *st = stages + (size_t)stage * stage_bytes;
       const DevItem I = *reinterpret_cast<const DevItem *>(st);
       if (I.op == OP_END || I.op == OP_FLUSH) {
-        // publish the rows stored since the last flush: every thread's stores (and this warp's
-        // bulk stores) are visible system-wide before one release-add per (source, receiver)
-        if (lane == 0) {
-          bulk_wait_all();
-          fence_proxy_async_global();
-        }
+        // publish the rows stored since the last flush: every thread's stores and bulk stores
+        // are visible system-wide before one release-add per (source, receiver).  (Every thread
+        // waits for its own bulk groups: per-row, fan-out and atomic stores are issued by any
+        // consumer lane, not only lane 0; the wait is a no-op for a thread with none pending.)
+        bulk_wait_all();
+        fence_proxy_async_global();
         fence_scope(P.sys_scope);
         consumer_barrier(&s_bar_count, &s_bar_gen, (unsigned)n_cons_warps, lane);
         // (strided: there are fewer consumer threads than (source, receiver) entries)
@@ -1370,7 +1370,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // this warp is done reading the stage
     }
-    if (lane == 0) bulk_wait_all();  // bulk stores complete before the CTA retires
+    bulk_wait_all();  // every thread's bulk stores complete before the CTA retires
   }
 }
 

@@ -29,7 +29,7 @@ __device__ __forceinline__ uint64_t pol_ef() {
 
 template <int kMode>  // 0 tma, 1 stg, 2 lds, 3 mix
 __global__ void __launch_bounds__(512, 1) store_kernel(char *out, size_t total, int chunk, int split,
-                                                        int depth, int hint) {
+                                                        int depth, int hint, int off) {
   extern __shared__ __align__(128) uint8_t sm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nw = blockDim.x >> 5;
@@ -38,10 +38,10 @@ __global__ void __launch_bounds__(512, 1) store_kernel(char *out, size_t total, 
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncthreads();
   const uint64_t pol = hint ? pol_ef() : 0;
-  const size_t nchunks = total / chunk;
+  const size_t nchunks = total / chunk - 1;
   int inflight = 0;
   for (size_t c = blockIdx.x; c < nchunks; c += gridDim.x) {
-    char *dst = out + c * chunk;
+    char *dst = out + c * chunk + off;
     const bool tma_w = kMode == 0 || (kMode == 3 && warp < split);
     if (tma_w) {
       const int parts = kMode == 0 ? split : split;
@@ -88,12 +88,12 @@ int main(int argc, char **argv) {
   cudaEvent_t a, b;
   cudaEventCreate(&a);
   cudaEventCreate(&b);
-  auto run = [&](const char *name, auto kern, int chunk, int split, int depth, int hint, int ctas) {
+  auto run = [&](const char *name, auto kern, int chunk, int split, int depth, int hint, int ctas, int off = 0) {
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     float best = 1e9f;
     for (int rep = 0; rep < 6; ++rep) {
       cudaEventRecord(a);
-      kern<<<sms * ctas, 512, chunk, 0>>>(out, total, chunk, split, depth, hint);
+      kern<<<sms * ctas, 512, chunk, 0>>>(out, total, chunk, split, depth, hint, off);
       cudaEventRecord(b);
       cudaEventSynchronize(b);
       float ms;
@@ -101,9 +101,18 @@ int main(int argc, char **argv) {
       if (rep > 0 && ms < best) best = ms;
     }
     cudaError_t e = cudaGetLastError();
-    printf("%-4s chunk %6d split %2d depth %d hint %d ctas/SM %d: %7.0f GB/s %s\n", name, chunk,
-           split, depth, hint, ctas, total / (best * 1e6), e ? cudaGetErrorString(e) : "");
+    printf("%-4s chunk %6d split %2d depth %d hint %d ctas/SM %d off %3d: %7.0f GB/s %s\n", name,
+           chunk, split, depth, hint, ctas, off, (total - chunk) / (best * 1e6),
+           e ? cudaGetErrorString(e) : "");
   };
+  if (argc > 1) {  // alignment study: chunk = 25 rows of a 2416-B pitch, start offsets
+    for (int off : {0, 16, 32, 64, 128})
+      for (int split : {1, 4})
+        run("tma", store_kernel<0>, 60400, split, 1, 1, 1, off);
+    for (int off : {0, 16})
+      run("stg", store_kernel<1>, 60400, 0, 1, 1, 1, off);
+    return 0;
+  }
   for (int hint = 0; hint < 2; ++hint) {
     run("stg", store_kernel<1>, 61440, 0, 1, hint, 1);
     run("lds", store_kernel<2>, 61440, 0, 1, hint, 1);
