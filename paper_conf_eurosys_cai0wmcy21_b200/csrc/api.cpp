@@ -494,7 +494,14 @@ void build_programs(dgcl_ctx *c) {
         // (relay forwards chained on flags now run DUAL too: 1.08 -> 1.01 ms on the Web-Google
         // ring plan, 0.83 -> 0.81 dgx1_like, no bimodality with device-scope flags, A/B r2j/r2k)
         (void)waits;
-        if ((copy_only && ops > 0 && bytes >= 8192 * ops) || (P.op_mask & (kMaskFold | kMaskTree)))
+        if (std::getenv("DGCL_DEBUG_GEO"))
+          std::fprintf(stderr, "geo: layer %d dir %d rank %d copy_only %d ops %lld bytes %lld per op %.0f\n",
+                       l, dir, r, (int)copy_only, (long long)ops, (long long)bytes,
+                       ops ? (double)bytes / ops : 0.0);
+        // (copy launches need >= 28 KB per bulk operation for WIDE since the fixed store warps:
+        // Reddit fwd602 33.5 KB / op 0.714 WIDE vs 0.804 DUAL, fwd256 24.5 KB / op 0.317 vs 0.311,
+        // A/B r2sj; 8 KB before)
+        if ((copy_only && ops > 0 && bytes >= 28672 * ops) || (P.op_mask & (kMaskFold | kMaskTree)))
           build(P, r, 0);
       }
       // per-rank loopback: the ranks' launches run concurrently on one device and their CTAs wait
