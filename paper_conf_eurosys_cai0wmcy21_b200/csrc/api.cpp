@@ -49,6 +49,7 @@ struct Program {
   TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
   mutable uint64_t claims = 0;  // dynamic item claiming: the counter's value before the next launch
   bool relay_fwd = false;       // a forward program with stage chaining (waits on counters)
+  bool simple_copy = false;     // COPY items only, no waits / signals / gather4, <= 240 rows each
 };
 
 }  // namespace
@@ -118,6 +119,7 @@ struct dgcl_ctx {
   int pipeline_blocks = 1;            // relay plans: vertex blocks of the stage chaining
   int leaf_split = 1;                 // relay plans: leaf deliveries after each stage's forwards
                                       // (A/B r2ab: 1 best; dgx1_like 0.721 -> 0.694 ms)
+  bool dual_producer = true;          // simple copy launches: two producer warps (any time)
   int owner_major = 1;                // fused loopback forwards: one owner's groups at a time
                                       // (A/B r2sh: Reddit fwd602 -1 %, Com-Orkut -2.5 %,
                                       // Web-Google dgx1_like -6 %)
@@ -452,6 +454,14 @@ void build_programs(dgcl_ctx *c) {
           if (it.op == OP_FANOUT) P.op_mask |= kMaskFanout;
         }
         P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
+        // dual producers (executor_tma.cu) need plain copies whose runs fit half a meta slot
+        P.simple_copy = !P.items.empty();
+        for (const DevItem &it : P.items)
+          if (it.op != OP_COPY || it.wait_n > 0 || (it.flags & (kItemSignal | kItemGather4 |
+                                                                  kItemDirect | kItemLsu |
+                                                                  kItemAtomic)) ||
+              it.dst_kind == K_MCAST || it.rows > 240 || it.nterms > 240)
+            P.simple_copy = false;
         P.relay_fwd = false;
         for (const DevItem &it : P.items)
           if (it.dir == DIR_FWD && it.op == OP_COPY && it.wait_n > 0) P.relay_fwd = true;
@@ -883,6 +893,10 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
       Pp.claim_batch = cb;
       claimed = (uint64_t)cb * ((uint64_t)(Pp.n_items + cb - 1) / cb + (uint64_t)grid);
     }
+    // two producer warps for simple copy launches on the WIDE geometry (option dual_producer)
+    Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy && pg.geo == 0 &&
+                    Pp.op_mask == kMaskCopy && !Pp.claim && !Pp.trace && Pp.gather4_mask == 0)
+                       ? 1 : 0;
     const int rc = launch_executor(Pp, grid, block, st);
     if (rc == 0) pg.claims += claimed;  // (a launch that never ran added nothing on the device)
     return rc;
@@ -1679,6 +1693,10 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "host_async") {  // host-buffer calls return once queued (see dgcl_forward_host)
     c->host_async = value != 0;
+    return DGCL_OK;
+  }
+  if (k == "dual_producer") {  // simple copy launches: two producer warps (any time)
+    c->dual_producer = value != 0;
     return DGCL_OK;
   }
   if (k == "hostsim_items") {  // verification aid: the host interpreter runs the work items

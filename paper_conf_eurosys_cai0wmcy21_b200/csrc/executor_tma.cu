@@ -72,7 +72,14 @@ static_assert(kDescAhead > kMetaAhead && kDescAhead < kDescSlots && kMetaAhead <
               "prefetch distances");
 // shared-memory carve-up (internal.h, tma_smem_bytes): offsets depend on the launch geometry
 constexpr size_t kMetaOff = 256;     // after the mbarriers (full, empty, meta, desc)
-static_assert((2 * kMaxTmaStages + kMetaSlots + kDescSlots) * 8 <= 256, "mbarrier region");
+// dual-producer mode (ExecParams::dual_prod): 2 producer warps, each with half of the descriptor
+// ring and the metadata region cut into kDualMetaSlots half-size slots per producer
+constexpr int kDualMetaSlots = 4;
+constexpr int kDualDescAhead = 3, kDualMetaAhead = 2;  // (a descriptor lands before its runs are asked for)
+constexpr int kMetaBarriers = 2 * kDualMetaSlots;  // (single mode uses the first kMetaSlots)
+static_assert((2 * kMaxTmaStages + kMetaBarriers + kDescSlots) * 8 <= 256, "mbarrier region");
+static_assert(kDescSlots == 2 * 4 && kDualDescAhead < 4 && kDualMetaAhead < kDualMetaSlots,
+              "dual-producer rings");
 static_assert(kMetaSlots * 8 * 64 <= 4 * 8 * 1024 && kDescSlots == 8, "layout of tma_smem_bytes");
 constexpr size_t kSmemMax = tma_smem_bytes(kGeoWide);
 
@@ -963,7 +970,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   uint64_t *full = reinterpret_cast<uint64_t *>(dsmem);
   uint64_t *empty = full + kMaxTmaStages;
   uint64_t *metab = empty + kMaxTmaStages;
-  uint64_t *descb = metab + kMetaSlots;
+  uint64_t *descb = metab + kMetaBarriers;
   uint8_t *metas = dsmem + kMetaOff;
   DevItem *descs = reinterpret_cast<DevItem *>(dsmem + kDescOff);
   uint8_t *stages = dsmem + kStageOff;
@@ -1007,13 +1014,84 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], n_cons_warps);
     }
-    for (int s = 0; s < kMetaSlots; ++s) mbar_init(&metab[s], 1);
+    for (int s = 0; s < kMetaBarriers; ++s) mbar_init(&metab[s], 1);
     for (int s = 0; s < kDescSlots; ++s) mbar_init(&descb[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
 
-  if (kHelp && warp >= 1 && warp <= DGCL_HELPER) {
+  if (kHelp && P.dual_prod && warp <= 1) {
+    // --------------------- dual producers (simple copy launches) -----------------------------
+    // A launch of plain COPY items — no waits, no signals, no gather4, no tracing, round-robin
+    // items (the host sets dual_prod only then) — has no FLUSH markers, so item m of this CTA
+    // simply takes stage use k = m.  Warps 0 and 1 then split the items (m = w, w + 2, ...),
+    // each with its own descriptor slots [4w, 4w + 4) and metadata slots (half-size), and issue
+    // their items' bulk copies independently; the consumers still take the stages in k order.
+    // (ncu r2sk: on the Reddit dim-602 forward one producer warp was busy ~100 % of the time,
+    // ~450 dependent instructions per item — the launch's bound.)
+    const int pw = warp;
+    const uint32_t G = gridDim.x;
+    const uint32_t nmine =
+        blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
+    const size_t mb2 = meta_bytes / 2;
+    auto item_of = [&](uint32_t j) { return (uint32_t)pw + 2u * j; };  // my j-th item
+    auto dslot = [&](uint32_t j) { return (uint32_t)(4 * pw) + (j & 3u); };
+    auto mslot = [&](uint32_t j) { return (uint32_t)(kDualMetaSlots * pw) + (j % kDualMetaSlots); };
+    auto req_desc = [&](uint32_t j) {  // lane 0
+      const uint32_t sl = dslot(j);
+      mbar_expect_tx(&descb[sl], (uint32_t)sizeof(DevItem));
+      bulk_g2s(descs + sl, P.items + blockIdx.x + (uint64_t)item_of(j) * G, (uint32_t)sizeof(DevItem),
+               &descb[sl]);
+    };
+    auto desc_wait = [&](uint32_t j) -> const DevItem & {
+      mbar_wait(&descb[dslot(j)], (j >> 2) & 1u);
+      return descs[dslot(j)];
+    };
+    auto meta_at = [&](uint32_t j) { return metas + (size_t)mslot(j) * mb2; };
+    auto meta_req = [&](uint32_t j) {  // lane 0, descriptor j ready
+      issue_meta<false>(P, descs[dslot(j)], meta_at(j), &metab[mslot(j)]);
+    };
+    uint32_t nj = 0;  // my items
+    while (item_of(nj) < nmine) ++nj;
+    fence_proxy_async_smem();
+    if (lane == 0)
+      for (uint32_t j = 0; j < (uint32_t)kDualDescAhead && j < nj; ++j) req_desc(j);
+    for (uint32_t j = 0; j < (uint32_t)kDualMetaAhead && j < nj; ++j) {
+      desc_wait(j);
+      if (lane == 0) meta_req(j);
+    }
+    bool dummy = false;
+    for (uint32_t j = 0; j < nj; ++j) {
+      const uint32_t m = item_of(j);
+      const DevItem I = desc_wait(j);
+      mbar_wait(&metab[mslot(j)], (j / kDualMetaSlots) & 1u);
+      uint32_t stage, use;
+      ring_pos(m, NS, stage, use);
+      if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
+      fence_proxy_async_smem();
+      issue_item<false, false>(P, I, &descs[dslot(j)], stages + (size_t)stage * stage_bytes,
+                               meta_at(j), &full[stage], lane, blockIdx.x + m * G, pol_copy,
+                               pol_fold, s_mb, &dummy, stages, metas);
+      __syncwarp();
+      // prefetch (the fence above covers the slots read so far)
+      if (lane == 0 && j + kDualDescAhead < nj) req_desc(j + kDualDescAhead);
+      if (j + kDualMetaAhead < nj) {
+        desc_wait(j + kDualMetaAhead);
+        if (lane == 0) meta_req(j + kDualMetaAhead);
+      }
+      __syncwarp();
+    }
+    if ((nmine & 1u) == (uint32_t)pw) {  // END at stage use nmine, after every item
+      uint32_t stage, use;
+      ring_pos(nmine, NS, stage, use);
+      if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
+      if (lane == 0) {
+        reinterpret_cast<DevItem *>(stages + (size_t)stage * stage_bytes)->op = OP_END;
+        mbar_arrive(&full[stage]);
+      }
+      __syncwarp();
+    }
+  } else if (kHelp && warp >= 1 && warp <= DGCL_HELPER) {
     // ------------------------------- helper warps --------------------------------------------
     constexpr int kNB = 32 * (1 + DGCL_HELPER);
     const uint64_t pol_h = pol_copy;
