@@ -230,8 +230,8 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *                    leaf rows (any stage <= k), then stage k+1's forwarded items, the remaining
  *                    leaves last (default 196608; -1 = stage-major build order)
  *   "dual_producer"  1 (default): launches of plain copies (no waits, no signals, no gather4,
- *                    WIDE geometry, round-robin items) run two producer warps that split the
- *                    items; 0: one producer (any time)
+ *                    round-robin items) run two producer warps per CTA that split the items;
+ *                    0: one producer (any time)
  *   "owner_major"    fused loopback: 1 (default) the forward COPY items of one owner's groups (its
  *                    embeddings to each receiver) run together, owner after owner — the write
  *                    front is a few long runs of halo rows and the owner's rows stay in L2 for

@@ -49,7 +49,8 @@ struct Program {
   TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
   mutable uint64_t claims = 0;  // dynamic item claiming: the counter's value before the next launch
   bool relay_fwd = false;       // a forward program with stage chaining (waits on counters)
-  bool simple_copy = false;     // COPY items only, no waits / signals / gather4, <= 240 rows each
+  bool simple_copy = false;     // COPY items only, no waits / signals / gather4
+  int max_runs = 0;             // most row runs of one COPY item (metadata slot bytes / 16)
 };
 
 }  // namespace
@@ -456,12 +457,15 @@ void build_programs(dgcl_ctx *c) {
         P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
         // dual producers (executor_tma.cu) need plain copies whose runs fit half a meta slot
         P.simple_copy = !P.items.empty();
-        for (const DevItem &it : P.items)
+        P.max_runs = 0;
+        for (const DevItem &it : P.items) {
           if (it.op != OP_COPY || it.wait_n > 0 || (it.flags & (kItemSignal | kItemGather4 |
                                                                   kItemDirect | kItemLsu |
                                                                   kItemAtomic)) ||
-              it.dst_kind == K_MCAST || it.rows > 240 || it.nterms > 240)
+              it.dst_kind == K_MCAST)
             P.simple_copy = false;
+          if (it.op == OP_COPY) P.max_runs = std::max(P.max_runs, (int)it.nterms);
+        }
         P.relay_fwd = false;
         for (const DevItem &it : P.items)
           if (it.dir == DIR_FWD && it.op == OP_COPY && it.wait_n > 0) P.relay_fwd = true;
@@ -894,7 +898,9 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
       claimed = (uint64_t)cb * ((uint64_t)(Pp.n_items + cb - 1) / cb + (uint64_t)grid);
     }
     // two producer warps for simple copy launches on the WIDE geometry (option dual_producer)
-    Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy && pg.geo == 0 &&
+    // (each producer's metadata slots are half size: an item's runs must fit meta_bytes / 2)
+    Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy &&
+                    (int64_t)pg.max_runs * (int64_t)sizeof(DevRun) <= Pp.meta_bytes / 2 &&
                     Pp.op_mask == kMaskCopy && !Pp.claim && !Pp.trace && Pp.gather4_mask == 0)
                        ? 1 : 0;
     const int rc = launch_executor(Pp, grid, block, st);

@@ -220,8 +220,8 @@ struct alignas(64) ExecParams {
   uint64_t *mc_flags;
   uint64_t *mcuc_flags[kMaxRanks];
   int32_t mc_emulate;
-  // 1: a simple copy launch (COPY items only: no waits, no signals, no gather4, items of <= 240
-  // rows, round-robin, WIDE geometry, copy-only instance) runs two producer warps
+  // 1: a simple copy launch (COPY items only: no waits, no signals, no gather4, every item's
+  // runs within half a metadata slot, round-robin, copy-only instance) runs two producer warps
   int32_t dual_prod;
 };
 

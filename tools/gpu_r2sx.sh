@@ -1,0 +1,13 @@
+#!/bin/bash
+cd "$(dirname "$0")/.."
+mkdir -p gpurun_out
+make -s all > gpurun_out/build.log 2>&1 || { cat gpurun_out/build.log; exit 1; }
+timeout 900 python -m pytest tests/test_gpu_exec.py -q -x -k "uniform or tiny or random_option" > gpurun_out/r2sx_pytest.log 2>&1; tail -2 gpurun_out/r2sx_pytest.log
+O=gpurun_out/r2sx_ab.txt; : > $O
+for rep in 1 2; do
+  timeout 300 python tools/ab_rt.py reddit "dual_producer=0" "dual_producer=1" 2>>gpurun_out/r2sx_ab.err | python -c "
+import json,sys
+d=json.loads(sys.stdin.read())
+for s in d['sets']: print('reddit', s['opts'], s['ms'])" >> $O
+done
+cat $O
