@@ -49,8 +49,8 @@ struct Program {
   TraceRec *d_trace = nullptr;  // option "trace": per-item timeline of the last launch
   mutable uint64_t claims = 0;  // dynamic item claiming: the counter's value before the next launch
   bool relay_fwd = false;       // a forward program with stage chaining (waits on counters)
-  bool simple_copy = false;     // COPY items only, no waits / signals / gather4
-  int max_runs = 0;             // most row runs of one COPY item (metadata slot bytes / 16)
+  bool simple_copy = false;     // COPY items only, no waits / signals
+  int64_t max_meta = 0;         // largest producer metadata of one COPY item (runs / row window)
 };
 
 }  // namespace
@@ -457,14 +457,16 @@ void build_programs(dgcl_ctx *c) {
         P.fold_wide = fold_rows > 0 && fold_terms >= 4 * fold_rows;
         // dual producers (executor_tma.cu) need plain copies whose runs fit half a meta slot
         P.simple_copy = !P.items.empty();
-        P.max_runs = 0;
+        P.max_meta = 0;
         for (const DevItem &it : P.items) {
-          if (it.op != OP_COPY || it.wait_n > 0 || (it.flags & (kItemSignal | kItemGather4 |
-                                                                  kItemDirect | kItemLsu |
-                                                                  kItemAtomic)) ||
+          if (it.op != OP_COPY || it.wait_n > 0 ||
+              (it.flags & (kItemSignal | kItemDirect | kItemLsu | kItemAtomic)) ||
               it.dst_kind == K_MCAST)
             P.simple_copy = false;
-          if (it.op == OP_COPY) P.max_runs = std::max(P.max_runs, (int)it.nterms);
+          if (it.op == OP_COPY)  // runs (16 B each), or a gather4 item's 16-B-aligned row window
+            P.max_meta = std::max<int64_t>(P.max_meta, (it.flags & kItemGather4)
+                                                           ? (int64_t)it.rows * 4 + 32
+                                                           : (int64_t)it.nterms * 16);
         }
         P.relay_fwd = false;
         for (const DevItem &it : P.items)
@@ -899,9 +901,12 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     }
     // two producer warps for simple copy launches on the WIDE geometry (option dual_producer)
     // (each producer's metadata slots are half size: an item's runs must fit meta_bytes / 2)
+    // (DUAL-geometry launches of bulk-copy runs only — already two producers per SM — gain
+    // nothing: Reddit fwd256 0.311 -> 0.312 / 0.318 -> 0.322, A/B r2sx / r2sz; WIDE and gather4
+    // launches do: fwd602 0.718 -> 0.695, Web-Google-8 0.437 -> 0.428)
     Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy &&
-                    (int64_t)pg.max_runs * (int64_t)sizeof(DevRun) <= Pp.meta_bytes / 2 &&
-                    Pp.op_mask == kMaskCopy && !Pp.claim && !Pp.trace && Pp.gather4_mask == 0)
+                    (pg.geo == 0 || pg.g4_kinds != 0) && pg.max_meta <= Pp.meta_bytes / 2 &&
+                    Pp.op_mask == kMaskCopy && !Pp.claim && !Pp.trace)
                        ? 1 : 0;
     const int rc = launch_executor(Pp, grid, block, st);
     if (rc == 0) pg.claims += claimed;  // (a launch that never ran added nothing on the device)

@@ -1022,11 +1022,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
 
   if (kHelp && P.dual_prod && warp <= 1) {
     // --------------------- dual producers (simple copy launches) -----------------------------
-    // A launch of plain COPY items — no waits, no signals, no gather4, no tracing, round-robin
-    // items (the host sets dual_prod only then) — has no FLUSH markers, so item m of this CTA
+    // A launch of plain COPY items — no waits, no signals, no tracing, round-robin items (the
+    // host sets dual_prod only then) — has no FLUSH markers, so item m of this CTA
     // simply takes stage use k = m.  Warps 0 and 1 then split the items (m = w, w + 2, ...),
     // each with its own descriptor slots [4w, 4w + 4) and metadata slots (half-size), and issue
-    // their items' bulk copies independently; the consumers still take the stages in k order.
+    // their items' bulk copies / gather4s independently (no helper hand-over); the consumers
+    // still take the stages in k order.
     // (ncu r2sk: on the Reddit dim-602 forward one producer warp was busy ~100 % of the time,
     // ~450 dependent instructions per item — the launch's bound.)
     const int pw = warp;

@@ -220,8 +220,9 @@ struct alignas(64) ExecParams {
   uint64_t *mc_flags;
   uint64_t *mcuc_flags[kMaxRanks];
   int32_t mc_emulate;
-  // 1: a simple copy launch (COPY items only: no waits, no signals, no gather4, every item's
-  // runs within half a metadata slot, round-robin, copy-only instance) runs two producer warps
+  // 1: a simple copy launch (COPY items only: no waits, no signals, every item's runs or row
+  // window within half a metadata slot, round-robin, copy-only instance) runs two producer warps
+  // (gather4 items are issued by their own producer, without the helper hand-over)
   int32_t dual_prod;
 };
 
