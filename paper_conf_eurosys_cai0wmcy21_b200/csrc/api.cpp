@@ -459,7 +459,7 @@ void build_programs(dgcl_ctx *c) {
         P.simple_copy = !P.items.empty();
         P.max_meta = 0;
         for (const DevItem &it : P.items) {
-          if (it.op != OP_COPY || it.wait_n > 0 ||
+          if ((it.op != OP_COPY && it.op != OP_FOLD) || it.wait_n > 0 ||
               (it.flags & (kItemSignal | kItemDirect | kItemLsu | kItemAtomic)) ||
               it.dst_kind == K_MCAST)
             P.simple_copy = false;
@@ -467,6 +467,8 @@ void build_programs(dgcl_ctx *c) {
             P.max_meta = std::max<int64_t>(P.max_meta, (it.flags & kItemGather4)
                                                            ? (int64_t)it.rows * 4 + 32
                                                            : (int64_t)it.nterms * 16);
+          else if (it.op == OP_FOLD && (it.flags & kItemStaged))  // its segments
+            P.max_meta = std::max<int64_t>(P.max_meta, (int64_t)(it.src >> kSegShift) * 16);
         }
         P.relay_fwd = false;
         for (const DevItem &it : P.items)
@@ -904,9 +906,13 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     // (DUAL-geometry launches of bulk-copy runs only — already two producers per SM — gain
     // nothing: Reddit fwd256 0.311 -> 0.312 / 0.318 -> 0.322, A/B r2sx / r2sz; WIDE and gather4
     // launches do: fwd602 0.718 -> 0.695, Web-Google-8 0.437 -> 0.428)
-    Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy &&
-                    (pg.geo == 0 || pg.g4_kinds != 0) && pg.max_meta <= Pp.meta_bytes / 2 &&
-                    Pp.op_mask == kMaskCopy && !Pp.claim && !Pp.trace)
+    // staged folds (fused in-place / tree-order backward): the producer bounds them too (ncu
+    // r2tb: ~600 dependent instructions per item)
+    const bool dual_copy = Pp.op_mask == kMaskCopy && (pg.geo == 0 || pg.g4_kinds != 0);
+    const bool dual_fold = Pp.op_mask == kMaskStaged || Pp.op_mask == (kMaskTree | kMaskStaged);
+    Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy && (dual_copy || dual_fold) &&
+                    pg.max_meta <= Pp.meta_bytes / 2 && !Pp.claim && !Pp.trace &&
+                    block >= 4 * 32)
                        ? 1 : 0;
     const int rc = launch_executor(Pp, grid, block, st);
     if (rc == 0) pg.claims += claimed;  // (a launch that never ran added nothing on the device)

@@ -996,7 +996,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
                          !(kMask & (kMaskFold | kMaskStaged | kMaskTree | kMaskFanout | kMaskLsu |
                                     kMaskMcast | kMaskDirect));
   constexpr int kProdWarps = kHelp ? 1 + DGCL_HELPER : 1;
-  const int n_cons_warps = (int)(blockDim.x >> 5) - kProdWarps;
+  // dual producers (P.dual_prod): copy-only instances use the helper warp, staged-fold instances
+  // take warp 1 from the consumers
+  constexpr bool kDualCap =
+      kHelp || kMask == kMaskStaged || kMask == (kMaskTree | kMaskStaged);
+  const int prod_warps = (kDualCap && P.dual_prod) ? 2 : kProdWarps;
+  const int n_cons_warps = (int)(blockDim.x >> 5) - prod_warps;
   // L2 hints (option "l2_policy"): bit 0 data stores evict_first (write-once halo / relay /
   // slot rows), bit 1 COPY / FANOUT source reads evict_last (a row sent to several receivers is
   // read again soon), bit 2 COPY source reads evict_first, bit 3 FOLD operand reads evict_first
@@ -1020,10 +1025,11 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   }
   __syncthreads();
 
-  if (kHelp && P.dual_prod && warp <= 1) {
+  if (kDualCap && P.dual_prod && warp <= 1) {
     // --------------------- dual producers (simple copy launches) -----------------------------
-    // A launch of plain COPY items — no waits, no signals, no tracing, round-robin items (the
-    // host sets dual_prod only then) — has no FLUSH markers, so item m of this CTA
+    // A launch of plain COPY items or staged FOLD items — no waits, no signals, no tracing,
+    // round-robin items (the host sets dual_prod only then) — has no FLUSH markers, so item m
+    // of this CTA
     // simply takes stage use k = m.  Warps 0 and 1 then split the items (m = w, w + 2, ...),
     // each with its own descriptor slots [4w, 4w + 4) and metadata slots (half-size), and issue
     // their items' bulk copies / gather4s independently (no helper hand-over); the consumers
@@ -1321,8 +1327,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     emit_marker(OP_END);
   } else {
     // ------------------------------- consumer warps ------------------------------------------
-    const uint32_t tid = threadIdx.x - 32 * kProdWarps, T = blockDim.x - 32 * kProdWarps;
-    const int cw = warp - kProdWarps;
+    const uint32_t tid = threadIdx.x - 32 * prod_warps, T = blockDim.x - 32 * prod_warps;
+    const int cw = warp - prod_warps;
     for (uint32_t k = 0;; ++k) {
       uint32_t stage, use;
       ring_pos(k, NS, stage, use);
