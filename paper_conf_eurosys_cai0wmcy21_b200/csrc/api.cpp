@@ -120,7 +120,10 @@ struct dgcl_ctx {
   int pipeline_blocks = 1;            // relay plans: vertex blocks of the stage chaining
   int leaf_split = 1;                 // relay plans: leaf deliveries after each stage's forwards
                                       // (A/B r2ab: 1 best; dgx1_like 0.721 -> 0.694 ms)
-  bool dual_producer = true;          // simple copy launches: two producer warps (any time)
+#ifndef DGCL_DUAL_PRODUCER_DEFAULT
+#define DGCL_DUAL_PRODUCER_DEFAULT 1  // (build-time A/B of the sustained bench)
+#endif
+  bool dual_producer = DGCL_DUAL_PRODUCER_DEFAULT;  // simple launches: two producer warps
   int owner_major = 1;                // fused loopback forwards: one owner's groups at a time
                                       // (A/B r2sh: Reddit fwd602 -1 %, Com-Orkut -2.5 %,
                                       // Web-Google dgx1_like -6 %)
