@@ -274,7 +274,7 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "host_async"     0 (default) / 1: dgcl_forward_host / dgcl_backward_host return before the
  *                    device->host copy completes (any time)
  *   "geometry"       bulk-copy launch geometry: 0 (default) auto per launch, 1 WIDE (1 CTA per
- *                    SM, 3 x 64 KB stages), 2 DUAL (2 CTAs per SM, 2 x 47 KB stages)
+ *                    SM, 4 x 48 KB stages), 2 DUAL (2 CTAs per SM, 2 x 47 KB stages)
  *   "bulk_store", "bulk_store_peer"  TMA stores for packed contiguous destinations in local HBM
  *                    (default 1) / peer memory (default 0)
  * Options other than "timeout_ms", "debug_skip_rank" and "host_async" must be set before

@@ -7,7 +7,7 @@
 // four scattered rows), and the "send" is a bulk (TMA) store or a coalesced 16-B store stream from
 // shared memory to the destination rows (a peer's halo over NVLink 5, or local HBM).
 //
-// Per CTA (one per SM, 512 threads, 3 x 64 KB stages, descriptor ring, 4 x 8 KB run windows):
+// Per CTA (WIDE: one per SM, 4 x 48 KB stages; DUAL: two per SM, 2 x 47 KB; descriptor ring, run windows):
 //   warp 0 (producer) walks the CTA's items in order with a metadata pipeline — descriptors
 //     bulk-copied 6 items ahead, row runs / source rows 3 items ahead — so no dependent global
 //     load is on its critical path.  Per data item it resolves the source waits (stage chaining)
@@ -83,9 +83,9 @@ static_assert(kDescSlots == 2 * 4 && kDualDescAhead < 4 && kDualMetaAhead < kDua
 static_assert(kMetaSlots * 8 * 64 <= 4 * 8 * 1024 && kDescSlots == 8, "layout of tma_smem_bytes");
 constexpr size_t kSmemMax = tma_smem_bytes(kGeoWide);
 
-// k-th stage use of a ring of ns (2 or 3) stages: slot and use count without a division
+// k-th stage use of a ring of ns (2, 3 or 4) stages: slot and use count without a division
 __device__ __forceinline__ void ring_pos(uint32_t k, uint32_t ns, uint32_t &slot, uint32_t &use) {
-  use = ns == 2 ? (k >> 1) : (__umulhi(k, 0xAAAAAAABu) >> 1);
+  use = ns == 2 ? (k >> 1) : ns == 4 ? (k >> 2) : (__umulhi(k, 0xAAAAAAABu) >> 1);
   slot = k - use * ns;
 }
 

@@ -263,7 +263,7 @@ struct DevRun {
 // and one stage = [0,64) item header | [64,128) info | [128,2176) term_ptr window (FOLD) |
 //   [2176,4096) destination-row window | [4096, stage_bytes) operand rows + staged terms.
 // Two geometries, chosen per launch (per program) by the host:
-//   WIDE: 1 CTA per SM, 3 x 64 KB stages — large items; best for long row runs of big rows
+//   WIDE: 1 CTA per SM, 4 x 48 KB stages — large items; best for long row runs of big rows
 //         (write-dominated forward of Reddit-shaped rows: 0.94 vs 0.75 of HBM peak)
 //   DUAL: 2 CTAs per SM, 2 x 47 KB stages — two producer warps per SM; best when the producer's
 //         per-item work dominates (short runs, staged folds: backward 0.70 -> 0.95-1.0 of peak)
@@ -271,7 +271,11 @@ struct DevRun {
 struct TmaGeometry {
   int32_t stages, stage_bytes, meta_bytes, threads, ctas_per_sm, max_item_rows;
 };
-constexpr TmaGeometry kGeoWide = {3, 64 * 1024, 8 * 1024, 256, 1, 464};
+#ifndef DGCL_WIDE_STAGES  // (build-time A/B of the WIDE geometry; 3 x 64 KB until the dual
+#define DGCL_WIDE_STAGES 4  //  producers: 4 x 48 KB then won, Reddit fwd602 0.696 -> 0.685, r2tf)
+#define DGCL_WIDE_STAGE_KB 48
+#endif
+constexpr TmaGeometry kGeoWide = {DGCL_WIDE_STAGES, DGCL_WIDE_STAGE_KB * 1024, 8 * 1024, 256, 1, 464};
 #ifndef DGCL_DUAL_STAGES  // (build-time A/B of the DUAL geometry, tools/build_variant.sh)
 #define DGCL_DUAL_STAGES 2
 #define DGCL_DUAL_STAGE_KB 47
@@ -282,7 +286,7 @@ constexpr TmaGeometry kGeoDual = {DGCL_DUAL_STAGES, DGCL_DUAL_STAGE_KB * 1024,
                                   DGCL_DUAL_META_KB * 1024, 256, DGCL_DUAL_CTAS,
                                   DGCL_DUAL_META_KB * 1024 / 16 < 240 ? DGCL_DUAL_META_KB * 1024 / 16
                                                                        : 240};
-constexpr int kMaxTmaStages = 3;
+constexpr int kMaxTmaStages = 4;
 constexpr int kStageHdrBytes = 4096;
 constexpr int kTmaBufBytes = kGeoWide.stage_bytes;          // largest stage
 constexpr int kTmaOperandBytes = kTmaBufBytes - kStageHdrBytes;
