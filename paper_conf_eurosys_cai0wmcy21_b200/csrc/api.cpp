@@ -514,15 +514,19 @@ void build_programs(dgcl_ctx *c) {
         const bool copy_only = (P.op_mask & ~(kMaskCopy | kMaskFanout)) == 0;
         // (relay forwards chained on flags now run DUAL too: 1.08 -> 1.01 ms on the Web-Google
         // ring plan, 0.83 -> 0.81 dgx1_like, no bimodality with device-scope flags, A/B r2j/r2k)
-        (void)waits;
         if (std::getenv("DGCL_DEBUG_GEO"))
           std::fprintf(stderr, "geo: layer %d dir %d rank %d copy_only %d ops %lld bytes %lld per op %.0f\n",
                        l, dir, r, (int)copy_only, (long long)ops, (long long)bytes,
                        ops ? (double)bytes / ops : 0.0);
-        // (copy launches need >= 28 KB per bulk operation for WIDE since the fixed store warps:
-        // Reddit fwd602 33.5 KB / op 0.714 WIDE vs 0.804 DUAL, fwd256 24.5 KB / op 0.317 vs 0.311,
-        // A/B r2sj; 8 KB before)
-        if ((copy_only && ops > 0 && bytes >= 28672 * ops) || (P.op_mask & (kMaskFold | kMaskTree)))
+        // (copy launches without waits or signals — two producers, 4 x 48 KB stages — run WIDE from 3.5 KB
+        // per bulk operation: Web-Google-8 forward 4.1 KB / op 0.425 DUAL vs 0.419 WIDE,
+        // Web-Google-2 0.186 vs 0.182, Reddit fwd256 0.313 vs 0.311, Com-Orkut 2.8 KB / op 1.43
+        // vs 1.53, A/B r2tg; with waits / signals (relay forwards, per-rank programs: one
+        // producer) from 28 KB, r2sj)
+        bool sigs = false;
+        for (const DevItem &it : P.items) sigs = sigs || (it.flags & kItemSignal);
+        const int64_t wide_op = (waits || sigs) ? 28672 : 3584;
+        if ((copy_only && ops > 0 && bytes >= wide_op * ops) || (P.op_mask & (kMaskFold | kMaskTree)))
           build(P, r, 0);
       }
       // per-rank loopback: the ranks' launches run concurrently on one device and their CTAs wait
