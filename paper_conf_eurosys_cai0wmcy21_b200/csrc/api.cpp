@@ -523,9 +523,13 @@ void build_programs(dgcl_ctx *c) {
         // Web-Google-2 0.186 vs 0.182, Reddit fwd256 0.313 vs 0.311, Com-Orkut 2.8 KB / op 1.43
         // vs 1.53, A/B r2tg; with waits / signals (relay forwards, per-rank programs: one
         // producer) from 28 KB, r2sj)
+        // (the launch gets dual producers only without waits, signals and item claims: claims
+        // are on for jobs of <= 4 ranks by default — Web-Google-4 forward on WIDE with claims,
+        // one producer: 0.414 ms vs 0.292 DUAL, r2th)
         bool sigs = false;
         for (const DevItem &it : P.items) sigs = sigs || (it.flags & kItemSignal);
-        const int64_t wide_op = (waits || sigs) ? 28672 : 3584;
+        const bool claims = c->claim_batch > 0 || (c->claim_batch < 0 && m <= 4);
+        const int64_t wide_op = (waits || sigs || claims) ? 28672 : 3584;
         if ((copy_only && ops > 0 && bytes >= wide_op * ops) || (P.op_mask & (kMaskFold | kMaskTree)))
           build(P, r, 0);
       }

@@ -1,0 +1,15 @@
+#!/bin/bash
+# 2- / 4-way jobs on WIDE: claims (single producer) vs round-robin (dual producers)
+cd "$(dirname "$0")/.."
+mkdir -p gpurun_out
+make -s all > gpurun_out/build.log 2>&1 || { cat gpurun_out/build.log; exit 1; }
+O=gpurun_out/r2th_ab.txt; : > $O
+for rep in 1 2; do
+for cfg in google2 google4 google8; do
+  timeout 300 python tools/ab_rt.py $cfg "" "claim_batch=0" "claim_batch=2" 2>>gpurun_out/r2th_ab.err | python -c "
+import json,sys
+d=json.loads(sys.stdin.read())
+for s in d['sets']: print('$cfg'.ljust(8), s['opts'], s['ms'])" >> $O
+done
+done
+cat $O
