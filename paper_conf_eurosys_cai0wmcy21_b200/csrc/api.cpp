@@ -923,7 +923,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     const bool dual_fold = Pp.op_mask == kMaskStaged || Pp.op_mask == (kMaskTree | kMaskStaged);
     Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy && (dual_copy || dual_fold) &&
                     pg.max_meta <= Pp.meta_bytes / 2 && !Pp.claim && !Pp.trace &&
-                    block >= 4 * 32)
+                    !Pp.use_ready && block >= 4 * 32)
                        ? 1 : 0;
     const int rc = launch_executor(Pp, grid, block, st);
     if (rc == 0) pg.claims += claimed;  // (a launch that never ran added nothing on the device)
