@@ -232,6 +232,9 @@ dgcl_status dgcl_plan_export(dgcl_ctx *ctx, int64_t *n_edges, int64_t *u, int32_
  *   "dual_producer"  1 (default): launches of plain copies (no waits, no signals, no gather4,
  *                    round-robin items) run two producer warps per CTA that split the items;
  *                    0: one producer (any time)
+ *   "dual_claims"    1 (default): dual producers also for launches whose items are claimed
+ *                    dynamically (each producer claims its own batches; stage uses from a shared
+ *                    counter); 0: such launches keep one producer (any time)
  *   "owner_major"    fused loopback: 1 (default) the forward COPY items of one owner's groups (its
  *                    embeddings to each receiver) run together, owner after owner — the write
  *                    front is a few long runs of halo rows and the owner's rows stay in L2 for

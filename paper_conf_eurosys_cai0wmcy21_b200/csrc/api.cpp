@@ -124,6 +124,10 @@ struct dgcl_ctx {
 #define DGCL_DUAL_PRODUCER_DEFAULT 1  // (build-time A/B of the sustained bench)
 #endif
   bool dual_producer = DGCL_DUAL_PRODUCER_DEFAULT;  // simple launches: two producer warps
+#ifndef DGCL_DUAL_CLAIMS_DEFAULT
+#define DGCL_DUAL_CLAIMS_DEFAULT 1  // (A/B r2tk: Web-Google-4 forward on WIDE 0.416 -> 0.293 ms)
+#endif
+  bool dual_claims = DGCL_DUAL_CLAIMS_DEFAULT;  // ... also when their items are claimed dynamically
   int owner_major = 1;                // fused loopback forwards: one owner's groups at a time
                                       // (A/B r2sh: Reddit fwd602 -1 %, Com-Orkut -2.5 %,
                                       // Web-Google dgx1_like -6 %)
@@ -523,12 +527,13 @@ void build_programs(dgcl_ctx *c) {
         // Web-Google-2 0.186 vs 0.182, Reddit fwd256 0.313 vs 0.311, Com-Orkut 2.8 KB / op 1.43
         // vs 1.53, A/B r2tg; with waits / signals (relay forwards, per-rank programs: one
         // producer) from 28 KB, r2sj)
-        // (the launch gets dual producers only without waits, signals and item claims: claims
-        // are on for jobs of <= 4 ranks by default — Web-Google-4 forward on WIDE with claims,
-        // one producer: 0.414 ms vs 0.292 DUAL, r2th)
+        // (the launch gets dual producers only without waits and signals, and with claims only
+        // under option dual_claims (default on) — Web-Google-4 forward on WIDE with claims and
+        // one producer: 0.414 ms vs 0.292 DUAL, r2th; with dual producers 0.2925, r2tk)
         bool sigs = false;
         for (const DevItem &it : P.items) sigs = sigs || (it.flags & kItemSignal);
-        const bool claims = c->claim_batch > 0 || (c->claim_batch < 0 && m <= 4);
+        const bool claims = (c->claim_batch > 0 || (c->claim_batch < 0 && m <= 4)) &&
+                            !(c->dual_producer && c->dual_claims);
         const int64_t wide_op = (waits || sigs || claims) ? 28672 : 3584;
         if ((copy_only && ops > 0 && bytes >= wide_op * ops) || (P.op_mask & (kMaskFold | kMaskTree)))
           build(P, r, 0);
@@ -922,9 +927,12 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     const bool dual_copy = Pp.op_mask == kMaskCopy && (pg.geo == 0 || pg.g4_kinds != 0);
     const bool dual_fold = Pp.op_mask == kMaskStaged || Pp.op_mask == (kMaskTree | kMaskStaged);
     Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy && (dual_copy || dual_fold) &&
-                    pg.max_meta <= Pp.meta_bytes / 2 && !Pp.claim && !Pp.trace &&
-                    !Pp.use_ready && block >= 4 * 32)
+                    pg.max_meta <= Pp.meta_bytes / 2 && (!Pp.claim || c->dual_claims) &&
+                    !Pp.trace && !Pp.use_ready && block >= 4 * 32)
                        ? 1 : 0;
+    // (with claims each of the two producers ends with one failing claim)
+    if (Pp.claim && Pp.dual_prod)
+      claimed = (uint64_t)cb * ((uint64_t)(Pp.n_items + cb - 1) / cb + 2 * (uint64_t)grid);
     const int rc = launch_executor(Pp, grid, block, st);
     if (rc == 0) pg.claims += claimed;  // (a launch that never ran added nothing on the device)
     return rc;
@@ -1725,6 +1733,10 @@ dgcl_status dgcl_set_option(dgcl_ctx *c, const char *key, int64_t value) {
   }
   if (k == "dual_producer") {  // simple copy launches: two producer warps (any time)
     c->dual_producer = value != 0;
+    return DGCL_OK;
+  }
+  if (k == "dual_claims") {  // dual producers also for launches with dynamic claims (any time)
+    c->dual_claims = value != 0;
     return DGCL_OK;
   }
   if (k == "hostsim_items") {  // verification aid: the host interpreter runs the work items

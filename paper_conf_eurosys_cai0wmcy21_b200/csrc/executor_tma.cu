@@ -1011,6 +1011,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
   const uint64_t pol_fold = (lp & 8) ? policy_evict_first() : 0;
   for (int i = threadIdx.x; i < kMaxRanks * kMaxRanks; i += blockDim.x) s_pend[i] = 0;
   if (threadIdx.x == 0) {
+    s_mb[0] = 0;  // (dual producers with claims: next stage use, finished producers)
+    s_mb[1] = 0;
     s_pend_base = 0;
     s_bar_count = 0;
     s_bar_gen = 0;
@@ -1036,19 +1038,41 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     // still take the stages in k order.
     // (ncu r2sk: on the Reddit dim-602 forward one producer warp was busy ~100 % of the time,
     // ~450 dependent instructions per item — the launch's bound.)
+    // With dynamic claiming (P.claim) the producers claim their own batches and take stage uses
+    // from a shared counter (s_mb[0]; the helper mailbox is unused here), so item order and
+    // stage order need not agree; the second producer to run out of items emits END (s_mb[1]).
     const int pw = warp;
     const uint32_t G = gridDim.x;
-    const uint32_t nmine =
-        blockIdx.x < (uint32_t)P.n_items ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G : 0;
+    const bool claims = P.claim != nullptr;
+    const uint32_t nmine = claims ? 0xffffffffu
+                           : blockIdx.x < (uint32_t)P.n_items
+                               ? ((uint32_t)P.n_items - blockIdx.x + G - 1) / G
+                               : 0;
     const size_t mb2 = meta_bytes / 2;
-    auto item_of = [&](uint32_t j) { return (uint32_t)pw + 2u * j; };  // my j-th item
     auto dslot = [&](uint32_t j) { return (uint32_t)(4 * pw) + (j & 3u); };
     auto mslot = [&](uint32_t j) { return (uint32_t)(kDualMetaSlots * pw) + (j % kDualMetaSlots); };
-    auto req_desc = [&](uint32_t j) {  // lane 0
+    uint64_t bnext = 0;
+    uint32_t bleft = 0;
+    auto req_desc = [&](uint32_t j) -> bool {  // lane 0: my j-th item (claims: false = none left)
       const uint32_t sl = dslot(j);
+      uint64_t idx;
+      if (claims) {
+        if (bleft == 0) {
+          const uint64_t b0 = atomicAdd(reinterpret_cast<unsigned long long *>(P.claim),
+                                        (unsigned long long)P.claim_batch) - P.claim_base;
+          if (b0 >= (uint64_t)P.n_items) return false;
+          bnext = b0;
+          bleft = (uint32_t)min((uint64_t)P.claim_batch, (uint64_t)P.n_items - b0);
+        }
+        idx = bnext++;
+        --bleft;
+      } else {
+        idx = blockIdx.x + (uint64_t)((uint32_t)pw + 2u * j) * G;
+      }
+      s_claim[sl] = (uint32_t)idx;
       mbar_expect_tx(&descb[sl], (uint32_t)sizeof(DevItem));
-      bulk_g2s(descs + sl, P.items + blockIdx.x + (uint64_t)item_of(j) * G, (uint32_t)sizeof(DevItem),
-               &descb[sl]);
+      bulk_g2s(descs + sl, P.items + idx, (uint32_t)sizeof(DevItem), &descb[sl]);
+      return true;
     };
     auto desc_wait = [&](uint32_t j) -> const DevItem & {
       mbar_wait(&descb[dslot(j)], (j >> 2) & 1u);
@@ -1058,39 +1082,68 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
     auto meta_req = [&](uint32_t j) {  // lane 0, descriptor j ready
       issue_meta<false>(P, descs[dslot(j)], meta_at(j), &metab[mslot(j)]);
     };
-    uint32_t nj = 0;  // my items
-    while (item_of(nj) < nmine) ++nj;
+    // my items: round-robin m = pw, pw + 2, ... < nmine; claims: until a claim fails
+    uint32_t nj = 0;
+    if (!claims)
+      while ((uint32_t)pw + 2u * nj < nmine) ++nj;
+    else
+      nj = 0xffffffffu;
+    auto request = [&](uint32_t j) {  // warp-collective: request my j-th item (claims: learn the end)
+      int ok = 1;
+      if (lane == 0) ok = req_desc(j) ? 1 : 0;
+      ok = __shfl_sync(0xffffffffu, ok, 0);
+      if (!ok && j < nj) nj = j;
+    };
     fence_proxy_async_smem();
-    if (lane == 0)
-      for (uint32_t j = 0; j < (uint32_t)kDualDescAhead && j < nj; ++j) req_desc(j);
+    for (uint32_t j = 0; j < (uint32_t)kDualDescAhead && j < nj; ++j) request(j);
     for (uint32_t j = 0; j < (uint32_t)kDualMetaAhead && j < nj; ++j) {
       desc_wait(j);
       if (lane == 0) meta_req(j);
     }
     bool dummy = false;
     for (uint32_t j = 0; j < nj; ++j) {
-      const uint32_t m = item_of(j);
       const DevItem I = desc_wait(j);
       mbar_wait(&metab[mslot(j)], (j / kDualMetaSlots) & 1u);
+      uint32_t k = (uint32_t)pw + 2u * j;  // stage use (round-robin: my item's position)
+      if (claims) {
+        if (lane == 0) k = atomicAdd(&s_mb[0], 1u);
+        k = __shfl_sync(0xffffffffu, k, 0);
+      }
       uint32_t stage, use;
-      ring_pos(m, NS, stage, use);
+      ring_pos(k, NS, stage, use);
       if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
       fence_proxy_async_smem();
       issue_item<false, false>(P, I, &descs[dslot(j)], stages + (size_t)stage * stage_bytes,
-                               meta_at(j), &full[stage], lane, blockIdx.x + m * G, pol_copy,
+                               meta_at(j), &full[stage], lane, s_claim[dslot(j)], pol_copy,
                                pol_fold, s_mb, &dummy, stages, metas);
       __syncwarp();
       // prefetch (the fence above covers the slots read so far)
-      if (lane == 0 && j + kDualDescAhead < nj) req_desc(j + kDualDescAhead);
+      if (j + kDualDescAhead < nj) request(j + kDualDescAhead);
       if (j + kDualMetaAhead < nj) {
         desc_wait(j + kDualMetaAhead);
         if (lane == 0) meta_req(j + kDualMetaAhead);
       }
       __syncwarp();
     }
-    if ((nmine & 1u) == (uint32_t)pw) {  // END at stage use nmine, after every item
+    // END after every item: round-robin at stage use nmine (by the producer whose turn it is);
+    // claims: the second producer to finish takes the next stage use
+    bool emit = false;
+    uint32_t kend = nmine;
+    if (claims) {
+      int last = 0;
+      if (lane == 0 && atomicAdd(&s_mb[1], 1u) == 1u) {
+        last = 1;
+        kend = atomicAdd(&s_mb[0], 1u);
+      }
+      last = __shfl_sync(0xffffffffu, last, 0);
+      kend = __shfl_sync(0xffffffffu, kend, 0);
+      emit = last != 0;
+    } else {
+      emit = (nmine & 1u) == (uint32_t)pw;
+    }
+    if (emit) {
       uint32_t stage, use;
-      ring_pos(nmine, NS, stage, use);
+      ring_pos(kend, NS, stage, use);
       if (use > 0) mbar_wait(&empty[stage], (use - 1) & 1u);
       if (lane == 0) {
         reinterpret_cast<DevItem *>(stages + (size_t)stage * stage_bytes)->op = OP_END;
