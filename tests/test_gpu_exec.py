@@ -169,6 +169,9 @@ def test_tiny_config_bit_exact(small):
     # two producer warps (simple copy launches on the WIDE geometry) and one
     (8, {"geometry": 1, "gather4": 0}), (3, {"geometry": 1, "gather4": 0, "item_bytes": 4096}),
     (8, {"geometry": 1, "gather4": 0, "dual_producer": 0}),
+    # dual producers with dynamic claims (each claims its own batches)
+    (4, {"geometry": 1, "claim_batch": 2}), (8, {"claim_batch": 3, "item_bytes": 4096}),
+    (2, {"geometry": 1, "claim_batch": 1, "dual_claims": 0}),
     # item order of fused forwards: chunk-major / group-major (default owner-major)
     (8, {"owner_major": 0}), (8, {"owner_major": 2}), (4, {"owner_major": 2, "align_sources": 0}),
     (8, {"fanout": 1}), (4, {"fanout": 1, "tma": 0}), (8, {"fanout": 1, "geometry": 2}),
@@ -669,7 +672,8 @@ def _random_option_case(seed):
     n = int(rng.choice([800, 3000, 7000]))
     # (drawn last: the earlier draws, hence the earlier cases, are unchanged)
     for key, vals in (("owner_major", [0, 1, 1, 2]), ("relay_lead_kb", [-1, 0, 1, 196608]),
-                      ("leaf_split", [0, 1, 1, 2]), ("dual_producer", [0, 1, 1])):
+                      ("leaf_split", [0, 1, 1, 2]), ("dual_producer", [0, 1, 1]),
+                      ("dual_claims", [0, 1, 1])):
         opts[key] = int(rng.choice(vals))
     return m, topo, flags, dims, opts, n
 
