@@ -14,10 +14,12 @@
 //     and the destination's ready word, claims a stage, writes the item header, arms the stage's
 //     "full" mbarrier with the byte count and issues the row gathers plus the consumers' tables;
 //     before it could block on a wait it inserts a FLUSH marker so pending done counts go out;
-//   warps 1-15 (consumers) take stages in order: store (COPY) or fold-and-store (FOLD), count the
+//   (launches without waits or signals: warps 0 and 1 are two producers splitting the items —
+//    ExecParams::dual_prod; copy launches otherwise use warp 1 as a gather4 helper)
+//   the other warps (consumers) take stages in order: store (COPY) or fold-and-store (FOLD), count the
 //     item's rows in shared memory (published at FLUSH / END: fence.sys, then one
 //     red.release.sys per (source, receiver)) and release the stage.  An END header stops them.
-// Up to 3 x 60 KB of gathers are in flight per SM, hiding HBM / NVLink latency without registers.
+// Up to ~180 KB of gathers are in flight per SM, hiding HBM / NVLink latency without registers.
 
 #include "device_common.cuh"
 
