@@ -467,7 +467,16 @@ class GraphAllgather:
             class _F(torch.autograd.Function):
                 @staticmethod
                 def forward(fctx, emb_, dctx_, layer_):
-                    halo = dctx_.forward(layer_, emb_)
+                    # rows whose pitch or base is not 16-B aligned (e.g. a contiguous [n, 602]
+                    # tensor) are laid out at the library pitch first, so the launch takes the
+                    # bulk-copy executor (the 4-byte register path serves them at ~0.4 of peak)
+                    p = dctx_.pitch(layer_)
+                    src = emb_
+                    if emb_.dim() == 2 and ((emb_.stride(0) * 4) % 16 or emb_.data_ptr() % 16 or
+                                            emb_.stride(1) != 1):
+                        src = torch.zeros(emb_.shape[0], p, dtype=emb_.dtype, device=emb_.device)
+                        src[:, :emb_.shape[1]] = emb_
+                    halo = dctx_.forward(layer_, src)
                     fctx.dctx = dctx_
                     fctx.layer = layer_
                     fctx.n = emb_.shape[0]

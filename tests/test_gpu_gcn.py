@@ -21,6 +21,20 @@ def test_gcn_partitions_match_full_graph():
         assert v < 1e-5, (k, v)
 
 
+def test_gcn_unaligned_dims_match_full_graph():
+    """The same with feature dims that are not multiples of 4 floats (contiguous [n, 602] / [n, 7]
+    activations: graph_allgather lays them out at the library pitch, bulk-copy executor)."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(__file__)), "examples"))
+    import gcn_loopback
+    errs, launches = gcn_loopback.run(dims=(602, 7), out_dim=3)
+    assert launches >= 4
+    for k, v in errs.items():
+        assert v < 1e-5, (k, v)
+
+
 def test_gcn_aggregation_overlapped_with_exchange():
     """NEXT-2: the aggregation's local part runs on a second stream while the executor (with
     sm_budget) moves the halo; each (receiver, source) block waits on its arrival counter
