@@ -42,7 +42,7 @@ struct Program {
   size_t dev_off = 0;  // offset (in items) into the device item pool
   int op_mask = 0;     // kMaskCopy / kMaskFold / kMaskDirect / kMaskStaged items present
   bool fold_wide = false;  // FOLD rows average >= 4 terms
-  int geo = 0;             // bulk-copy launch geometry: 0 = kGeoWide, 1 = kGeoDual
+  int geo = 0;             // bulk-copy launch geometry: 0 = kGeoWide, 1 = kGeoDual, 2 = kGeoWide3
   int64_t bytes = 0;       // operand rows moved (rows x 16-B-rounded row, + fold terms)
   int g4_kinds = 0;        // source kinds of its gather4 items (tensor maps the launch needs)
   bool tree = false;       // carries tree-order FOLD programs (kTermRankTree)
@@ -434,8 +434,8 @@ void build_programs(dgcl_ctx *c) {
         const std::vector<int32_t> &G = fan ? gids_fan[r] : gids[r];
         const std::vector<uint8_t> need = needed_counters(L, G);
         P.geo = geo;
-        ItemLimits lim = item_limits(geo ? kGeoDual : kGeoWide, c->item_bytes,
-                                     (int64_t)c->sm_count * (geo ? kGeoDual : kGeoWide).ctas_per_sm);
+        ItemLimits lim = item_limits(geometry_of(geo), c->item_bytes,
+                                     (int64_t)c->sm_count * geometry_of(geo).ctas_per_sm);
         lim.align_sources = c->align_sources;
         lim.lsu_gather = c->lsu_gather && c->use_tma;
         lim.owner_major = fused ? c->owner_major : 0;
@@ -495,8 +495,21 @@ void build_programs(dgcl_ctx *c) {
       };
       for (int r = 0; r < c->n_prog_ranks; ++r) {
         Program &P = c->progs[c->prog_index(l, dir, r)];
+        // WIDE: 4 x 48 KB stages for launches that get two producers, 3 x 64 KB (WIDE3) for
+        // launches that keep one (waits, signals, READY / WAIT items)
+        auto build_wide = [&](Program &Q, int rr) {
+          build(Q, rr, 0);
+          bool one = false;
+          for (const DevItem &it : Q.items)
+            one = one || it.wait_n > 0 || (it.flags & kItemSignal) || it.op == OP_READY ||
+                  it.op == OP_WAIT;
+          if (one) build(Q, rr, 2);
+        };
         if (c->geometry) {
-          build(P, r, c->geometry - 1);
+          if (c->geometry == 1)
+            build_wide(P, r);
+          else
+            build(P, r, c->geometry - 1);
           continue;
         }
         // auto: DUAL (two producer warps per SM) unless the launch is bulk-copy friendly —
@@ -536,7 +549,7 @@ void build_programs(dgcl_ctx *c) {
                             !(c->dual_producer && c->dual_claims);
         const int64_t wide_op = (waits || sigs || claims) ? 28672 : 3584;
         if ((copy_only && ops > 0 && bytes >= wide_op * ops) || (P.op_mask & (kMaskFold | kMaskTree)))
-          build(P, r, 0);
+          build_wide(P, r);
       }
       // per-rank loopback: the ranks' launches run concurrently on one device and their CTAs wait
       // on each other's flags, so together they must be co-resident.  A WIDE CTA (one per SM by
@@ -575,8 +588,8 @@ dgcl_status upload(dgcl_ctx *c, T **dptr, const std::vector<T> &v) {
 // launches with many terms per row, 512 otherwise — and the user's "threads" option wins
 int tma_block(const dgcl_ctx *c, const Program &pg) {
   if (c->threads_set) return c->threads;
-  const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
-  if (pg.geo == 0 && (pg.op_mask & (kMaskFold | kMaskTree)))
+  const TmaGeometry &G = geometry_of(pg.geo);
+  if (pg.geo != 1 && (pg.op_mask & (kMaskFold | kMaskTree)))
     return pg.op_mask == kMaskFold && pg.fold_wide && !pg.tree ? 1024 : 512;
   return G.threads;
 }
@@ -878,7 +891,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     Pp.fold_wide = pg.fold_wide ? 1 : 0;
     Pp.n_items = (int32_t)pg.items.size();
     Pp.trace = pg.d_trace;
-    const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
+    const TmaGeometry &G = geometry_of(pg.geo);
     const int tblock = tma_block(c, pg);
     const auto occ = c->tma_ctas.find({pg.geo, tblock, occ_mask(c, pg)});
     const int tctas = occ == c->tma_ctas.end() ? 0 : occ->second;
@@ -924,7 +937,7 @@ dgcl_status launch(dgcl_ctx *c, int layer, int dir, const float *in, int64_t in_
     // launches do: fwd602 0.718 -> 0.695, Web-Google-8 0.437 -> 0.428)
     // staged folds (fused in-place / tree-order backward): the producer bounds them too (ncu
     // r2tb: ~600 dependent instructions per item)
-    const bool dual_copy = Pp.op_mask == kMaskCopy && (pg.geo == 0 || pg.g4_kinds != 0);
+    const bool dual_copy = Pp.op_mask == kMaskCopy && (pg.geo != 1 || pg.g4_kinds != 0);
     const bool dual_fold = Pp.op_mask == kMaskStaged || Pp.op_mask == (kMaskTree | kMaskStaged);
     Pp.dual_prod = (c->dual_producer && Pp.use_tma && pg.simple_copy && (dual_copy || dual_fold) &&
                     pg.max_meta <= Pp.meta_bytes / 2 && (!Pp.claim || c->dual_claims) &&
@@ -1157,7 +1170,7 @@ dgcl_status dgcl_register_workspace(dgcl_ctx *c, void *dev, size_t bytes) {
     const int block = tma_block(c, pg);
     const int mk = occ_mask(c, pg);
     if (c->tma_ctas.count({pg.geo, block, mk})) continue;
-    const TmaGeometry &G = pg.geo ? kGeoDual : kGeoWide;
+    const TmaGeometry &G = geometry_of(pg.geo);
     int n = 0;
     e = executor_tma_occupancy(mk, block, tma_smem_bytes(G), &n);
     if (e != 0) return fail(c, DGCL_ECUDA, "occupancy query failed");

@@ -83,7 +83,8 @@ static_assert((2 * kMaxTmaStages + kMetaBarriers + kDescSlots) * 8 <= 256, "mbar
 static_assert(kDescSlots == 2 * 4 && kDualDescAhead < 4 && kDualMetaAhead < kDualMetaSlots,
               "dual-producer rings");
 static_assert(kMetaSlots * 8 * 64 <= 4 * 8 * 1024 && kDescSlots == 8, "layout of tma_smem_bytes");
-constexpr size_t kSmemMax = tma_smem_bytes(kGeoWide);
+constexpr size_t kSmemMax = tma_smem_bytes(kGeoWide) > tma_smem_bytes(kGeoWide3)
+                                ? tma_smem_bytes(kGeoWide) : tma_smem_bytes(kGeoWide3);
 
 // k-th stage use of a ring of ns (2, 3 or 4) stages: slot and use count without a division
 __device__ __forceinline__ void ring_pos(uint32_t k, uint32_t ns, uint32_t &slot, uint32_t &use) {

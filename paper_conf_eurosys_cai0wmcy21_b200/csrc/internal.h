@@ -276,6 +276,10 @@ struct TmaGeometry {
 #define DGCL_WIDE_STAGE_KB 48
 #endif
 constexpr TmaGeometry kGeoWide = {DGCL_WIDE_STAGES, DGCL_WIDE_STAGE_KB * 1024, 8 * 1024, 256, 1, 464};
+// WIDE with 3 x 64 KB stages for launches that keep one producer (waits / signals: relay and
+// per-rank programs) — larger items, less producer work per byte (per-rank Reddit fwd602: 4 x 48
+// KB 1.13 ms vs 3 x 64 KB 0.82)
+constexpr TmaGeometry kGeoWide3 = {3, 64 * 1024, 8 * 1024, 256, 1, 464};
 #ifndef DGCL_DUAL_STAGES  // (build-time A/B of the DUAL geometry, tools/build_variant.sh)
 #define DGCL_DUAL_STAGES 2
 #define DGCL_DUAL_STAGE_KB 47
@@ -288,12 +292,17 @@ constexpr TmaGeometry kGeoDual = {DGCL_DUAL_STAGES, DGCL_DUAL_STAGE_KB * 1024,
                                                                        : 240};
 constexpr int kMaxTmaStages = 4;
 constexpr int kStageHdrBytes = 4096;
-constexpr int kTmaBufBytes = kGeoWide.stage_bytes;          // largest stage
+constexpr int kTmaBufBytes = kGeoWide3.stage_bytes;         // largest stage
 constexpr int kTmaOperandBytes = kTmaBufBytes - kStageHdrBytes;
 constexpr size_t tma_smem_bytes(const TmaGeometry &g) {
   return 256 + 4 * (size_t)g.meta_bytes + 8 * 64 + (size_t)g.stages * g.stage_bytes + 1152;
 }
 static_assert(tma_smem_bytes(kGeoWide) <= 227 * 1024, "WIDE: one CTA per SM");
+static_assert(tma_smem_bytes(kGeoWide3) <= 227 * 1024, "WIDE3: one CTA per SM");
+static_assert(kGeoWide.stage_bytes <= kGeoWide3.stage_bytes && kGeoDual.stage_bytes <= kGeoWide3.stage_bytes,
+              "kTmaBufBytes is the largest stage");
+// launch geometry by index: 0 WIDE (4 x 48 KB, dual-producer launches), 1 DUAL, 2 WIDE3
+inline const TmaGeometry &geometry_of(int g) { return g == 1 ? kGeoDual : g == 2 ? kGeoWide3 : kGeoWide; }
 static_assert(tma_smem_bytes(kGeoDual) * DGCL_DUAL_CTAS <= 227 * 1024, "DUAL: CTAs per SM");
 static_assert(kGeoWide.max_item_rows * 16 <= kGeoWide.meta_bytes &&
                   kGeoDual.max_item_rows * 16 <= kGeoDual.meta_bytes,
