@@ -86,9 +86,9 @@ static_assert(kMetaSlots * 8 * 64 <= 4 * 8 * 1024 && kDescSlots == 8, "layout of
 constexpr size_t kSmemMax = tma_smem_bytes(kGeoWide) > tma_smem_bytes(kGeoWide3)
                                 ? tma_smem_bytes(kGeoWide) : tma_smem_bytes(kGeoWide3);
 
-// k-th stage use of a ring of ns stages: slot and use count (no division for 2, 3 or 4)
+// k-th stage use of a ring of ns (2, 3 or 4) stages: slot and use count without a division
 __device__ __forceinline__ void ring_pos(uint32_t k, uint32_t ns, uint32_t &slot, uint32_t &use) {
-  use = ns == 2 ? (k >> 1) : ns == 4 ? (k >> 2) : ns == 3 ? (__umulhi(k, 0xAAAAAAABu) >> 1) : k / ns;
+  use = ns == 2 ? (k >> 1) : ns == 4 ? (k >> 2) : (__umulhi(k, 0xAAAAAAABu) >> 1);
   slot = k - use * ns;
 }
 

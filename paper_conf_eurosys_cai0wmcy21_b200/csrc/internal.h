@@ -290,10 +290,7 @@ constexpr TmaGeometry kGeoDual = {DGCL_DUAL_STAGES, DGCL_DUAL_STAGE_KB * 1024,
                                   DGCL_DUAL_META_KB * 1024, 256, DGCL_DUAL_CTAS,
                                   DGCL_DUAL_META_KB * 1024 / 16 < 240 ? DGCL_DUAL_META_KB * 1024 / 16
                                                                        : 240};
-#ifndef DGCL_MAX_TMA_STAGES
-#define DGCL_MAX_TMA_STAGES 4
-#endif
-constexpr int kMaxTmaStages = DGCL_MAX_TMA_STAGES;
+constexpr int kMaxTmaStages = 4;
 constexpr int kStageHdrBytes = 4096;
 constexpr int kTmaBufBytes = kGeoWide3.stage_bytes;         // largest stage
 constexpr int kTmaOperandBytes = kTmaBufBytes - kStageHdrBytes;
